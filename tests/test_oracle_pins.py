@@ -1,0 +1,385 @@
+"""Pins of the CPU oracle against what the paper and mathematics fix (-m "not gpu").
+
+Each test names the passage it follows.  None of them compares the oracle with itself:
+the expected values are the paper's printed examples (tests/golden/, cited), closed forms
+(tests/closed_forms.py), invariants that hold for every permutation, published known-answer
+vectors, numpy routines, or brute force over all inputs of tiny size.
+"""
+import itertools
+import math
+from fractions import Fraction
+
+import numpy as np
+import pytest
+
+from closed_forms import (CYCLIC_TRANSVERSALS_ODD, balls_in_bins_cdf, expectation, pmf_from_cdf,
+                          random_access_cdf, variance)
+from conftest import golden
+
+pytestmark = pytest.mark.filterwarnings("ignore::DeprecationWarning")
+
+
+def _rows(path):
+    return [ln.split() for ln in open(path) if ln.strip() and not ln.startswith("#")]
+
+
+# ---------------------------------------------------------------- O1/O2 Philox
+def test_philox_known_answers(oracle):
+    for r in _rows(golden("philox_kat.txt")):
+        v = [int(x, 16) for x in r]
+        out = oracle.philox4x32_10(v[0:4], v[4:6])
+        assert [int(x) for x in out] == v[6:10]
+
+
+def test_word_counter_contract(oracle):
+    # O2: word t of domain d for trial n is component t&3 of Philox(ctr=(n_lo,n_hi,t>>2,d), key)
+    seed, n = 0x0123456789ABCDEF, 0xFEDCBA9876543210
+    for d in (0, 1, 2):
+        for t in (0, 1, 2, 3, 4, 7, 30, 31):
+            ctr = [n & 0xFFFFFFFF, n >> 32, t >> 2, d]
+            key = [seed & 0xFFFFFFFF, seed >> 32]
+            assert oracle.word(seed, n, d, t) == int(oracle.philox4x32_10(ctr, key)[t & 3])
+
+
+# ---------------------------------------------------------------- O3 permutation
+@pytest.mark.parametrize("w", [2, 3, 5, 16, 32, 33, 64, 256])
+def test_perm_is_permutation(oracle, w):
+    for n in range(50):
+        p = oracle.perm(7, n, w)
+        assert sorted(p.tolist()) == list(range(w))
+
+
+def test_perm_uniform_chi2_w4(oracle):
+    # P:L959-962 §IV: P is selected from all w! permutations uniformly at random.
+    N = 48000
+    counts = {}
+    for n in range(N):
+        key = tuple(oracle.perm(11, n, 4).tolist())
+        counts[key] = counts.get(key, 0) + 1
+    assert len(counts) == 24
+    exp = N / 24
+    chi2 = sum((c - exp) ** 2 / exp for c in counts.values())
+    assert chi2 < 49.7  # chi^2_{23} 0.999 quantile
+
+
+def test_perm_durstenfeld_first_swap(oracle):
+    # O3 step k = w-1 swaps a[w-1] with a[j], j = floor(word(0,0)*w / 2^32)
+    seed, n, w = 3, 9, 32
+    u = oracle.word(seed, n, 0, 0)
+    j = (u * w) >> 32
+    a = list(range(w))
+    a[w - 1], a[j] = a[j], a[w - 1]
+    # later steps never touch position w-1 again
+    assert int(oracle.perm(seed, n, w)[w - 1]) == a[w - 1]
+
+
+# ---------------------------------------------------------------- O4/O5
+def test_ras_shifts_range_and_uniformity(oracle):
+    w, N = 32, 4000
+    cnt = np.zeros(w)
+    for n in range(N):
+        r = oracle.ras_shifts(5, n, w)
+        assert r.max() < w
+        np.add.at(cnt, r.astype(np.int64), 1)
+    exp = N * w / w
+    chi2 = ((cnt - exp) ** 2 / exp).sum()
+    assert chi2 < 61.1  # chi^2_{31} 0.999
+
+
+def test_random_cells_range(oracle):
+    for w in (2, 7, 32, 256):
+        rows, cols = oracle.random_cells(9, 4, w)
+        assert rows.max() < w and cols.max() < w
+
+
+# ---------------------------------------------------------------- O6/O11 layouts
+def test_fig6_rap_layout(oracle):
+    rows = _rows(golden("fig6_rap_layout.txt"))
+    w = int(rows[0][1])
+    P = [int(x) for x in rows[1][1:]]
+    expect = np.array([[int(x) for x in r] for r in rows[2:]], dtype=np.uint32)
+    logical = np.arange(w * w, dtype=np.uint32).reshape(w, w)
+    assert np.array_equal(oracle.rap_layout(P, logical), expect)
+    # the same mapping through the address function: value v=(i,j) sits at address i*w+(j+P[i])%w
+    for i in range(w):
+        for j in range(w):
+            a = oracle.address(oracle.RAP, w, i, j, P)
+            assert expect.reshape(-1)[a] == i * w + j
+
+
+def test_fig6_worked_entry(oracle):
+    # with P=(2,0,3,1), a[2][1] is mapped to a[2][(1+3) mod 4] = a[2][0]
+    assert oracle.address(oracle.RAP, 4, 2, 1, [2, 0, 3, 1]) == 2 * 4 + 0
+
+
+def test_banks_are_address_mod_w(oracle):
+    # cell m[i] is in bank i mod w; a[i][j] (RAW) is in bank j
+    w = 8
+    for i in range(w):
+        for j in range(w):
+            assert oracle.address(oracle.RAW, w, i, j) % w == j
+            assert oracle.address(oracle.PAD, w, i, j) % w == (i + j) % w
+            assert oracle.address(oracle.XOR, w, i, j) % w == i ^ j
+
+
+# ---------------------------------------------------------------- O8 congestion
+def test_fig2_congestion_rules(oracle):
+    # (1) distinct banks -> 1; (2) all to one bank -> 4; (3) one address -> merged -> 1
+    w = 4
+    assert oracle.congestion(w, [0, 1, 2, 3], [1, 2, 3, 0], oracle.RAW) == 1
+    assert oracle.congestion(w, [0, 1, 2, 3], [2, 2, 2, 2], oracle.RAW) == 4
+    assert oracle.congestion(w, [1, 1, 1, 1], [2, 2, 2, 2], oracle.RAW) == 1
+
+
+def test_fig3_dmm_example(oracle):
+    rows = _rows(golden("fig3_dmm.txt"))
+    w = int(rows[0][1])
+    cong = []
+    for r in rows[1:3]:
+        addrs = [int(x) for x in r[2:6]]
+        c = oracle.congestion(w, [a // w for a in addrs], [a % w for a in addrs], oracle.RAW)
+        assert c == int(r[7])
+        cong.append(c)
+    assert sum(cong) == int(rows[3][1])
+    lat, t = int(rows[4][1]), int(rows[4][3])
+    assert oracle.dmm_time(cong, lat) == t
+
+
+def test_lemma1_dmm_times(oracle):
+    # P:L774-785 §III: contiguous access of a w x w matrix by w warps takes w + l - 1 time
+    # units; stride access w^2 + l - 1 (RAW).
+    for w in (4, 8, 32):
+        l = 5
+        contig = [oracle.congestion(w, [i] * w, list(range(w)), oracle.RAW) for i in range(w)]
+        stride = [oracle.congestion(w, list(range(w)), [i] * w, oracle.RAW) for i in range(w)]
+        assert oracle.dmm_time(contig, l) == w + l - 1
+        assert oracle.dmm_time(stride, l) == w * w + l - 1
+
+
+def test_fig4_diagonal_pattern(oracle):
+    rows = _rows(golden("fig4_diagonal.txt"))
+    w = int(rows[0][1])
+    grid = np.array([[int(x) for x in r] for r in rows[1:]])
+    # warp W(0) = threads 0..w-1 touches cells where grid < w: they must be O7's (t, t)
+    r0, c0 = oracle.pattern_cells(oracle.DIAGONAL, oracle.RAW, w)
+    for t in range(w):
+        assert grid[r0[t], c0[t]] == t
+    # RAW diagonal is conflict-free for every warp of Fig.4
+    for i in range(w):
+        cells = [(r, c) for r in range(w) for c in range(w) if i * w <= grid[r, c] < (i + 1) * w]
+        assert oracle.congestion(w, [r for r, _ in cells], [c for _, c in cells], oracle.RAW) == 1
+
+
+@pytest.mark.parametrize("w", [2, 3, 4, 5, 6, 7])
+def test_theorem2_contiguous_stride_one_for_every_perm(oracle, w):
+    # Theorem 2 special case: RAP contiguous & stride congestion
+    # is exactly 1 for EVERY permutation P.
+    for P in itertools.permutations(range(w)):
+        for i in range(w):
+            assert oracle.congestion(w, [i] * w, list(range(w)), oracle.RAP, P) == 1
+            assert oracle.congestion(w, list(range(w)), [i] * w, oracle.RAP, P) == 1
+
+
+def test_raw_facts(oracle):
+    # RAW contiguous 1, stride w, diagonal 1; malicious same-bank = w
+    for w in (4, 16, 32, 64):
+        for pat, expect in ((oracle.CONTIGUOUS, 1), (oracle.STRIDE, w), (oracle.DIAGONAL, 1),
+                            (oracle.MALICIOUS, w)):
+            r, c = oracle.pattern_cells(pat, oracle.RAW, w)
+            assert oracle.congestion(w, r, c, oracle.RAW) == expect
+
+
+def test_deterministic_baselines_have_malicious_sets(oracle):
+    # DESIGN.md finding: +1 padding is w-way on the anti-diagonal, XOR on the diagonal
+    w = 32
+    for s in (oracle.PAD, oracle.XOR):
+        r, c = oracle.pattern_cells(oracle.MALICIOUS, s, w)
+        assert oracle.congestion(w, r, c, s) == w
+        for pat in (oracle.CONTIGUOUS, oracle.STRIDE):
+            r, c = oracle.pattern_cells(pat, s, w)
+            assert oracle.congestion(w, r, c, s) == 1
+
+
+@pytest.mark.parametrize("w", [2, 3, 4, 5, 6])
+def test_ras_stride_exact_by_enumeration(oracle, w):
+    # Enumerate all w^w RAS shift vectors: the exact expected stride congestion must equal the
+    # balls-into-bins closed form (r_i independent uniform).
+    rows, cols = list(range(w)), [0] * w
+    hist = [0] * (w + 1)
+    for r in itertools.product(range(w), repeat=w):
+        hist[oracle.congestion(w, rows, cols, oracle.RAS, r)] += 1
+    pmf = pmf_from_cdf(balls_in_bins_cdf, w)
+    assert [Fraction(h, w ** w) for h in hist] == pmf
+
+
+@pytest.mark.parametrize("w", [2, 3])
+def test_random_access_exact_by_enumeration(oracle, w):
+    # All (w^2)^w ordered draws with replacement: exact PMF = closed form, for every scheme
+    # ("all three implementations have the same congestion" for random access).
+    cells = [(i, j) for i in range(w) for j in range(w)]
+    pmf = pmf_from_cdf(random_access_cdf, w)
+    P = list(range(w))[::-1]
+    rshift = [1 % w] * w
+    for scheme, shift in ((oracle.RAW, None), (oracle.RAS, rshift), (oracle.RAP, P),
+                          (oracle.PAD, None)):
+        hist = [0] * (w + 1)
+        for draw in itertools.product(cells, repeat=w):
+            hist[oracle.congestion(w, [a for a, _ in draw], [b for _, b in draw], scheme, shift)] += 1
+        assert [Fraction(h, (w * w) ** w) for h in hist] == pmf
+
+
+@pytest.mark.parametrize("w", [3, 4, 5, 6, 7])
+def test_rap_diagonal_pair_collisions_and_transversals(oracle, w):
+    # P:L1437-1446 §V: two requests to distinct rows and columns share a bank with
+    # probability 1/(w-1) under RAP (1/w under RAS).  Over all w! permutations the mean
+    # number of colliding pairs of the diagonal access is therefore C(w,2)/(w-1) = w/2.
+    pairs = Fraction(0)
+    hist = [0] * (w + 1)
+    perms = list(itertools.permutations(range(w)))
+    for P in perms:
+        banks = [oracle.address(oracle.RAP, w, t, t, P) % w for t in range(w)]
+        pairs += sum(1 for a, b in itertools.combinations(banks, 2) if a == b)
+        hist[oracle.congestion(w, list(range(w)), list(range(w)), oracle.RAP, P)] += 1
+    assert pairs / len(perms) == Fraction(w, 2)
+    # congestion 1 <=> (t + P[t]) mod w distinct <=> a transversal of the cyclic Latin square
+    assert hist[1] == (CYCLIC_TRANSVERSALS_ODD[w] if w % 2 else 0)
+    # congestion w <=> t + P[t] constant mod w: exactly w permutations; w-1 is impossible
+    assert hist[w] == w and hist[w - 1] == 0
+
+
+def test_ras_pair_collision(oracle):
+    w = 4
+    pairs = Fraction(0)
+    for r in itertools.product(range(w), repeat=w):
+        banks = [oracle.address(oracle.RAS, w, t, t, r) % w for t in range(w)]
+        pairs += sum(1 for a, b in itertools.combinations(banks, 2) if a == b)
+    assert pairs / w ** w == Fraction(math.comb(w, 2), w)
+
+
+# ---------------------------------------------------------------- O9 sweep
+def _E(h):
+    h = np.asarray(h, dtype=np.float64)
+    c = np.arange(h.shape[-1])
+    n = h.sum(-1)
+    mu = (h * c).sum(-1) / n
+    sd = np.sqrt((h * (c - mu[..., None]) ** 2).sum(-1) / n)
+    return mu, sd, n
+
+
+def test_sweep_exact_small_w_against_enumeration(oracle):
+    # the sweep's FY sampling: MC expectation of RAP diagonal at w=5 against the exact value
+    # over all 5! permutations (brute force).  Theorem 2 invariants hold on every trial.
+    w, N = 5, 200000
+    h = oracle.sweep(w, ["contiguous", "stride", "diagonal"], ["rap"], 1, 0, N)
+    assert h[0, 0, 1] == N and h[1, 0, 1] == N
+    exact = Fraction(0)
+    for P in itertools.permutations(range(w)):
+        exact += oracle.congestion(w, list(range(w)), list(range(w)), oracle.RAP, P)
+    exact /= math.factorial(w)
+    mu, sd, n = _E(h[2, 0])
+    assert abs(mu - float(exact)) < 3.29 * sd / math.sqrt(n)
+
+
+def test_sweep_w32_anchor_353(oracle):
+    # The paper's "3.53 at w=32" (Tab.II) binds to RAS
+    # stride/diagonal/malicious (reading i).  Closed form 3.532941; 99% CI.
+    w, N = 32, 400000
+    h = oracle.sweep(w, ["stride", "diagonal", "random", "malicious"], ["raw", "ras", "rap"], 2, 0, N)
+    pmf = pmf_from_cdf(balls_in_bins_cdf, w)
+    E_ras = float(expectation(pmf))
+    sd_ras = float(variance(pmf)) ** 0.5
+    ci = 2.576 * sd_ras / math.sqrt(N)
+    for pi in (0, 1, 3):                     # stride, diagonal, malicious under RAS
+        mu, _, _ = _E(h[pi, 1])
+        assert abs(mu - E_ras) < ci
+        assert round(mu, 2) == 3.53
+    # RAW stride = 32 deterministically, RAP stride = 1 on every trial (Theorem 2)
+    assert h[0, 0, 32] == N and h[0, 2, 1] == N
+    # random access: closed form 3.435408 for every scheme (Tab.II 3.44)
+    pmf_r = pmf_from_cdf(random_access_cdf, w)
+    E_r, sd_r = float(expectation(pmf_r)), float(variance(pmf_r)) ** 0.5
+    for si in range(3):
+        mu, _, _ = _E(h[2, si])
+        assert abs(mu - E_r) < 2.576 * sd_r / math.sqrt(N)
+    # RAP diagonal rounds to Table II's 3.61; malicious(RAP) is the diagonal, trial for trial
+    mu, sd, n = _E(h[1, 2])
+    assert abs(mu - 3.61) < 0.005 + 2.576 * sd / math.sqrt(n)
+    assert np.array_equal(h[1, 2], h[3, 2])
+    assert np.array_equal(h[0, 1], h[3, 1])
+
+
+def test_sweep_w32_chi2_against_exact_pmf(oracle):
+    w, N = 32, 200000
+    h = oracle.sweep(w, ["stride", "random"], ["ras"], 3, 0, N)
+    for row, cdf in ((h[0, 0], balls_in_bins_cdf), (h[1, 0], random_access_cdf)):
+        pmf = [float(p) for p in pmf_from_cdf(cdf, w)]
+        # pool tail bins with expected count < 5
+        obs, exp = [], []
+        o_acc = e_acc = 0.0
+        for c in range(w + 1):
+            o_acc += float(row[c]); e_acc += N * pmf[c]
+            if e_acc >= 5:
+                obs.append(o_acc); exp.append(e_acc); o_acc = e_acc = 0.0
+        obs[-1] += o_acc; exp[-1] += e_acc
+        chi2 = sum((o - e) ** 2 / e for o, e in zip(obs, exp))
+        assert chi2 < 27.9  # chi^2 with <= 9 dof, 0.999 quantile
+
+
+TABLE2_N = {16: 200000, 32: 200000, 64: 60000, 128: 15000, 256: 4000}
+
+
+@pytest.mark.parametrize("w", [16, 32, 64, 128, 256])
+def test_table2_reproduced(oracle, w):
+    # Every Table II entry within rounding (±0.005) + 99% MC interval.
+    col = [16, 32, 64, 128, 256].index(w)
+    table = {(r[0], r[1]): float(r[2 + col]) for r in _rows(golden("table2.txt"))}
+    pats = ["contiguous", "stride", "diagonal", "random"]
+    schs = ["raw", "ras", "rap"]
+    h = oracle.sweep(w, pats, schs, 4, 0, TABLE2_N[w])
+    for pi, p in enumerate(pats):
+        for si, s in enumerate(schs):
+            mu, sd, n = _E(h[pi, si])
+            tol = 0.005 + 2.576 * sd / math.sqrt(n) + 1e-12
+            assert abs(mu - table[(p, s)]) <= tol, (p, s, mu, table[(p, s)])
+
+
+def test_sweep_is_additive_over_trial_ranges(oracle):
+    # O9 with counter-based draws: any split of [first, first+N) sums to the same histogram.
+    a = oracle.sweep(32, ["random", "diagonal"], ["ras", "rap"], 9, 1000, 3000, threads=1)
+    b = oracle.sweep(32, ["random", "diagonal"], ["ras", "rap"], 9, 1000, 1234, threads=3)
+    b += oracle.sweep(32, ["random", "diagonal"], ["ras", "rap"], 9, 2234, 1766, threads=2)
+    assert np.array_equal(a, b)
+
+
+# ---------------------------------------------------------------- O10 transpose
+def test_fig5_transpose(oracle):
+    rows = _rows(golden("fig5_transpose.txt"))
+    w = int(rows[0][1])
+    i = [r[0] for r in rows].index("in")
+    o = [r[0] for r in rows].index("out")
+    A = np.array([[int(x) for x in r] for r in rows[i + 1:i + 1 + w]], dtype=np.float64)
+    B = np.array([[int(x) for x in r] for r in rows[o + 1:o + 1 + w]], dtype=np.float64)
+    assert np.array_equal(oracle.transpose(A), B)
+
+
+@pytest.mark.parametrize("dtype", [np.uint32, np.uint64, np.float32, np.float64, np.uint8, np.uint16])
+def test_transpose_matches_numpy_and_is_involution(oracle, dtype):
+    rng = np.random.default_rng(0)
+    for shape in ((1, 1), (1, 37), (33, 65), (64, 32), (100, 3)):
+        bits = rng.integers(0, 2 ** 63, size=shape, dtype=np.uint64)
+        A = bits.astype(np.dtype(dtype).newbyteorder("=").str.replace("f", "u")).view(dtype) \
+            if np.dtype(dtype).kind == "f" else bits.astype(dtype)
+        T = oracle.transpose(A)
+        assert T.tobytes() == np.ascontiguousarray(A.T).tobytes()
+        assert oracle.transpose(T).tobytes() == A.tobytes()
+
+
+def test_transpose_strided_source(oracle):
+    big = np.arange(40 * 50, dtype=np.uint32).reshape(40, 50)
+    sub = big[3:20, 5:42]
+    assert np.array_equal(oracle.transpose(sub), sub.T)
+
+
+def test_transpose_empty(oracle):
+    A = np.zeros((0, 5), dtype=np.uint32)
+    assert oracle.transpose(A).shape == (5, 0)
