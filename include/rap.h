@@ -1,0 +1,140 @@
+/*
+ * rap.h -- C ABI of librap.so, the B200 (sm_100a) hot path of the Random Address
+ * Permute-Shift (RAP) technique of Nakano, Matsumae and Ito (ICPPW 2014).
+ *
+ * Citations "P:L<a>-<b>" are line numbers in the paper text plus the section,
+ * figure or table.  The problem statement these calls follow (§II):
+ *   - the Discrete Memory Machine (DMM) has w memory banks; address a is in bank a mod w;
+ *   - a warp of w threads issues w requests at once; identical addresses are merged;
+ *   - the congestion of the access is the maximum number of distinct requests destined
+ *     for one bank.
+ * RAP stores element a[i][j] of a w x w matrix at a[i][(j + P[i]) mod w] for a permutation
+ * P drawn uniformly from all w! permutations (§IV, Fig.6); RAS is the same with
+ * independent shifts r[i]; RAW is the plain row-major layout.
+ *
+ * Conventions (all entry points):
+ *   - Ownership: the caller owns every buffer.  Pointers named d_* (and src/dst of
+ *     rap_transpose) are DEVICE pointers on the current CUDA device.  The library keeps no
+ *     allocation and no mutable global state; calls are thread-safe.
+ *   - Asynchrony: device work is enqueued on `stream` (a cudaStream_t passed as void*;
+ *     NULL = the legacy default stream) and returns immediately; results are valid once
+ *     the stream is synchronised.
+ *   - Errors: argument errors are detected on the host BEFORE anything is enqueued and
+ *     returned as RAP_ERR_INVALID_ARG / RAP_ERR_UNSUPPORTED / RAP_ERR_ALIAS; a failed
+ *     launch returns RAP_ERR_CUDA.  No exception crosses the ABI.  There is no CPU
+ *     fallback: every computation runs in the library's CUDA kernels.
+ *   - Random numbers (paper: "selected uniformly at random"; the contract is
+ *     this library's, reading vi): Philox4x32-10 with key = (seed_lo, seed_hi);
+ *     word t of domain d for index n is Philox(ctr = (n_lo, n_hi, t>>2, d), key)[t & 3].
+ *     Domain 0 feeds the permutation (Durstenfeld: for k = w-1..1, j = floor(word(0,w-1-k)
+ *     * (k+1) / 2^32), swap a[k], a[j]); domain 1 the RAS shifts r[i] = floor(word(1,i) *
+ *     w / 2^32); domain 2 the random-access cells cell_t = floor(word(2,t) * w*w / 2^32).
+ */
+#ifndef RAP_H_
+#define RAP_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define RAP_ABI_VERSION 1
+#define RAP_MAX_W 32
+
+typedef enum {
+    RAP_OK = 0,
+    RAP_ERR_INVALID_ARG = 1,  /* a size, pointer, enum or mask is out of range          */
+    RAP_ERR_UNSUPPORTED = 2,  /* valid request this build does not implement             */
+    RAP_ERR_ALIAS = 3,        /* src and dst of an out-of-place transpose overlap        */
+    RAP_ERR_CUDA = 4          /* a CUDA runtime call or kernel launch failed             */
+} rap_status_t;
+
+/* Shared-memory tile layouts of rap_transpose (a 32 x 32 tile, row i of the input tile). */
+typedef enum {
+    RAP_LAYOUT_RAW = 0,  /* a[i][j] at [i][j]                   (RAW CRSW)   */
+    RAP_LAYOUT_PAD = 1,  /* a[i][j] at [i][j] of a [32][33] array   (+1 padding baseline) */
+    RAP_LAYOUT_XOR = 2,  /* a[i][j] at [i][j xor i]                 (XOR-swizzle baseline)*/
+    RAP_LAYOUT_RAS = 3,  /* a[i][j] at [i][(j + r[i]) mod 32]          */
+    RAP_LAYOUT_RAP = 4   /* a[i][j] at [i][(j + P[i]) mod 32]        */
+} rap_layout_t;
+
+/* Address maps of the DMM congestion evaluator (physical address of logical cell (i,j)). */
+typedef enum {
+    RAP_SCHEME_RAW = 0,  /* i*w + j                                                      */
+    RAP_SCHEME_RAS = 1,  /* i*w + (j + r[i]) mod w                                       */
+    RAP_SCHEME_RAP = 2,  /* i*w + (j + P[i]) mod w                                       */
+    RAP_SCHEME_PAD = 3,  /* i*(w+1) + j                                                  */
+    RAP_SCHEME_XOR = 4   /* i*w + (j xor i); w must be a power of two                    */
+} rap_scheme_t;
+
+/* Warp access patterns of the sweep; lane t = 0..w-1 (§III). */
+typedef enum {
+    RAP_PAT_CONTIGUOUS = 0,  /* (0, t)                                                    */
+    RAP_PAT_STRIDE = 1,      /* (t, 0)                                                    */
+    RAP_PAT_DIAGONAL = 2,    /* (t, t)       Fig.4 warp W(0): a[(0+t) mod w][t]           */
+    RAP_PAT_RANDOM = 3,      /* w cells i.i.d. uniform with replacement (domain 2)        */
+    RAP_PAT_MALICIOUS = 4    /* scheme-aware worst case: RAW,RAS -> (t,0); RAP,XOR ->     */
+                             /* (t,t); PAD -> (t,(w-t) mod w)       (reading iii)*/
+} rap_pattern_t;
+
+int rap_abi_version(void);
+const char *rap_status_str(rap_status_t s);
+
+/* T0 -- permutations P_n = perm(seed, n, w) for n = first_index .. first_index+count-1
+ * (§IV).  d_perm_out: device uint8_t[count][w]; row k holds P_{first_index+k}.
+ * 2 <= w <= 32.  count == 0 is a no-op. */
+rap_status_t rap_perm_gen(uint64_t seed, uint64_t first_index, uint64_t count, uint32_t w,
+                          uint8_t *d_perm_out, void *stream);
+
+/* T1-T3 -- out-of-place transpose staged through 32 x 32 shared-memory tiles in `layout`
+ * (§III; RAP layout P:L1005-1023 §IV, RAP CRSW listing P:L1515-1546 §VI):
+ *     dst[c * ld_dst + r] = src[r * ld_src + c]   for 0 <= r < rows, 0 <= c < cols.
+ * src, dst: device pointers, row-major with leading dimensions ld_src >= cols and
+ * ld_dst >= rows (elements).  elem_bytes in {4, 8}: a raw bit copy (float32/float64 NaN
+ * payloads, -0, subnormals are preserved).  The tile layout changes only where an element
+ * sits in shared memory, never the result.  RAP uses P = perm(seed, 0, 32), RAS uses
+ * r = shifts(seed, 0, 32); seed is ignored by RAW/PAD/XOR.  rows == 0 or cols == 0 is a
+ * no-op.  Overlapping src/dst -> RAP_ERR_ALIAS.  16-byte aligned src with ld_src a
+ * multiple of 16/elem_bytes takes 128-bit loads; anything else takes 32/64-bit loads
+ * (still on the GPU). */
+rap_status_t rap_transpose(const void *src, void *dst, int64_t rows, int64_t cols,
+                           int64_t ld_src, int64_t ld_dst, uint32_t elem_bytes,
+                           rap_layout_t layout, uint64_t seed, void *stream);
+
+/* C3 -- the DMM congestion evaluator itself (§II), batched: warp k issues the w
+ * requests to logical cells (d_rows[k*w + t], d_cols[k*w + t]) of a w x w matrix laid out
+ * by `scheme` with per-warp shift vector d_shift[k*w .. k*w+w-1] (P for RAP, r for RAS;
+ * may be NULL for RAW/PAD/XOR).  d_congestion_out[k] = max over banks of the number of
+ * distinct addresses destined for the bank (1..w).  Cells and shifts must be < w; a warp
+ * with any out-of-range cell or shift gets congestion 0 (an error marker, never a valid
+ * congestion).  n_warps == 0 is a no-op. */
+rap_status_t rap_congestion(uint32_t w, uint64_t n_warps, const uint32_t *d_rows,
+                            const uint32_t *d_cols, rap_scheme_t scheme, const uint32_t *d_shift,
+                            uint32_t *d_congestion_out, void *stream);
+
+/* C1-C4 -- Monte-Carlo sweep (Tab.II P:L1567-1577 §V): for every trial n in
+ * [first_trial, first_trial + n_trials) draw P_n, r_n and the random cells from the counter
+ * contract, evaluate each selected (pattern, scheme) and count the congestion.
+ * d_hist: device uint64_t[npat][nsch][w+1] where npat = popcount(pattern_mask) and
+ * nsch = popcount(scheme_mask), patterns/schemes in enum order; ACCUMULATED (+=), so the
+ * caller zeroes it once and may split a run into any chunks (bit-identical sums).
+ * Masks are bit sets of rap_pattern_t / rap_scheme_t (1..31).  XOR needs w = 2^k. */
+rap_status_t rap_congestion_sweep(uint32_t w, uint32_t pattern_mask, uint32_t scheme_mask,
+                                  uint64_t seed, uint64_t first_trial, uint64_t n_trials,
+                                  uint64_t *d_hist, void *stream);
+
+/* C3 over user traces: d_cells: device uint32_t[n_warps][w], cell = row*w + col < w*w.
+ * Every trace warp is evaluated under every trial's P_n / r_n, n in [first_trial,
+ * first_trial + n_trials).  d_hist: device uint64_t[nsch][w+1], ACCUMULATED (+=);
+ * each scheme row gains n_warps * n_trials counts.  Bin 0 counts trace warps holding a
+ * cell >= w*w (invalid input; valid congestions are 1..w). */
+rap_status_t rap_congestion_trace(uint32_t w, uint64_t n_warps, const uint32_t *d_cells,
+                                  uint32_t scheme_mask, uint64_t seed, uint64_t first_trial,
+                                  uint64_t n_trials, uint64_t *d_hist, void *stream);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* RAP_H_ */

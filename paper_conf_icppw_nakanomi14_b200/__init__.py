@@ -1,0 +1,193 @@
+"""RAP (Random Address Permute-Shift, Nakano-Matsumae-Ito, ICPPW 2014) on B200.
+
+Thin Python binding over ``librap.so`` (C ABI: ``include/rap.h``).  Every step of the hot
+path runs in the library's sm_100a kernels; this module only marshals torch tensors (device
+memory), the current CUDA stream and the enums.  There is no CPU fallback: calling with a
+CPU tensor, or without the built library, raises.
+
+Functions keep the C names without the ``rap_`` prefix:
+  perm_gen, transpose, congestion, congestion_sweep, congestion_trace.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import torch
+
+from . import build as _build
+
+__all__ = ["perm_gen", "transpose", "congestion", "congestion_sweep", "congestion_trace",
+           "LAYOUTS", "SCHEMES", "PATTERNS", "RapError", "lib", "library_path"]
+
+LAYOUTS = {"raw": 0, "pad": 1, "xor": 2, "ras": 3, "rap": 4}
+SCHEMES = {"raw": 0, "ras": 1, "rap": 2, "pad": 3, "xor": 4}
+PATTERNS = {"contiguous": 0, "stride": 1, "diagonal": 2, "random": 3, "malicious": 4}
+STATUS = {0: "RAP_OK", 1: "RAP_ERR_INVALID_ARG", 2: "RAP_ERR_UNSUPPORTED", 3: "RAP_ERR_ALIAS",
+          4: "RAP_ERR_CUDA"}
+
+
+class RapError(RuntimeError):
+    def __init__(self, status: int, what: str):
+        super().__init__(f"{what}: {STATUS.get(status, status)}")
+        self.status = status
+
+
+_lib = None
+
+
+def library_path() -> str:
+    return _build.LIB
+
+
+def lib():
+    """Load librap.so (built in-tree by ``__graft_entry__.build()``); raise if it is missing."""
+    global _lib
+    if _lib is None:
+        path = _build.LIB
+        if not os.path.exists(path):
+            raise ImportError(f"{path} is missing: run `python -c 'import __graft_entry__ as g; "
+                              "g.build()'` (no CPU fallback exists)")
+        L = ctypes.CDLL(path)
+        u8p, u32p, u64p, vp = (ctypes.c_void_p,) * 4
+        i32, u32, u64, i64 = ctypes.c_int, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_int64
+        L.rap_abi_version.restype = i32
+        L.rap_status_str.argtypes = [i32]
+        L.rap_status_str.restype = ctypes.c_char_p
+        L.rap_perm_gen.argtypes = [u64, u64, u64, u32, u8p, vp]
+        L.rap_transpose.argtypes = [vp, vp, i64, i64, i64, i64, u32, i32, u64, vp]
+        L.rap_congestion.argtypes = [u32, u64, u32p, u32p, i32, u32p, u32p, vp]
+        L.rap_congestion_sweep.argtypes = [u32, u32, u32, u64, u64, u64, u64p, vp]
+        L.rap_congestion_trace.argtypes = [u32, u64, u32p, u32, u64, u64, u64, u64p, vp]
+        for f in ("rap_perm_gen", "rap_transpose", "rap_congestion", "rap_congestion_sweep",
+                  "rap_congestion_trace"):
+            getattr(L, f).restype = i32
+        if L.rap_abi_version() != 1:
+            raise ImportError("librap.so ABI version mismatch")
+        _lib = L
+    return _lib
+
+
+def _stream(t: torch.Tensor):
+    return ctypes.c_void_p(torch.cuda.current_stream(t.device).cuda_stream)
+
+
+def _need_cuda(*ts):
+    for t in ts:
+        if t is not None and not t.is_cuda:
+            raise ValueError("RAP kernels run on the GPU only: pass CUDA tensors (no CPU fallback)")
+
+
+def _check(rc: int, what: str):
+    if rc != 0:
+        raise RapError(rc, what)
+
+
+def _mask(sel, table) -> int:
+    if isinstance(sel, int):
+        return sel
+    m = 0
+    for x in sel:
+        m |= 1 << (table[x] if isinstance(x, str) else int(x))
+    return m
+
+
+def perm_gen(seed: int, count: int, w: int = 32, first_index: int = 0,
+             device="cuda", out: torch.Tensor | None = None) -> torch.Tensor:
+    """Permutations P_n = perm(seed, n, w), n = first_index .. +count-1 -> uint8 [count, w]."""
+    if out is None:
+        out = torch.empty((count, w), dtype=torch.uint8, device=device)
+    _need_cuda(out)
+    assert out.dtype == torch.uint8 and out.is_contiguous() and out.numel() == count * w
+    with torch.cuda.device(out.device):
+        _check(lib().rap_perm_gen(seed, first_index, count, w, ctypes.c_void_p(out.data_ptr()),
+                                  _stream(out)), "rap_perm_gen")
+    return out
+
+
+def transpose(x: torch.Tensor, layout: str = "rap", seed: int = 0,
+              out: torch.Tensor | None = None) -> torch.Tensor:
+    """out[c, r] = x[r, c] (bit copy) via 32x32 shared-memory tiles in `layout`.
+
+    x: 2-D CUDA tensor with 4- or 8-byte elements and unit inner stride.  out (optional):
+    [cols, rows] tensor of the same dtype, unit inner stride, not overlapping x.
+    """
+    _need_cuda(x, out)
+    if x.dim() != 2:
+        raise ValueError("transpose expects a 2-D tensor")
+    eb = x.element_size()
+    if eb not in (4, 8):
+        raise ValueError("transpose supports 4- and 8-byte elements")
+    rows, cols = x.shape
+    if x.stride(1) != 1 and rows * cols > 0:
+        x = x.contiguous()
+    if out is None:
+        out = torch.empty((cols, rows), dtype=x.dtype, device=x.device)
+    if out.shape != (cols, rows) or out.dtype != x.dtype or (out.stride(1) != 1 and rows * cols):
+        raise ValueError("out must be a [cols, rows] tensor of x's dtype with unit inner stride")
+    ld_src = x.stride(0) if rows > 1 else max(cols, 1)
+    ld_dst = out.stride(0) if cols > 1 else max(rows, 1)
+    with torch.cuda.device(x.device):
+        _check(lib().rap_transpose(ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(out.data_ptr()),
+                                   rows, cols, ld_src, ld_dst, eb, LAYOUTS[layout], seed,
+                                   _stream(x)), "rap_transpose")
+    return out
+
+
+def congestion(rows: torch.Tensor, cols: torch.Tensor, scheme: str = "rap",
+               shift: torch.Tensor | None = None, w: int | None = None,
+               out: torch.Tensor | None = None) -> torch.Tensor:
+    """DMM congestion of n warps: rows/cols/shift int32 or uint32 CUDA [n, w] -> uint32 [n]."""
+    _need_cuda(rows, cols, shift, out)
+    n, ww = rows.shape
+    w = ww if w is None else w
+    assert ww == w and cols.shape == rows.shape
+    for t in (rows, cols) + ((shift,) if shift is not None else ()):
+        assert t.dtype in (torch.int32, torch.uint32) and t.is_contiguous()
+    if shift is not None:
+        assert shift.shape == rows.shape
+    if out is None:
+        out = torch.empty(n, dtype=torch.uint32, device=rows.device)
+    with torch.cuda.device(rows.device):
+        _check(lib().rap_congestion(w, n, ctypes.c_void_p(rows.data_ptr()),
+                                    ctypes.c_void_p(cols.data_ptr()), SCHEMES[scheme],
+                                    ctypes.c_void_p(shift.data_ptr() if shift is not None else 0),
+                                    ctypes.c_void_p(out.data_ptr()), _stream(rows)),
+               "rap_congestion")
+    return out
+
+
+def congestion_sweep(n_trials: int, seed: int, w: int = 32, patterns=("contiguous", "stride",
+                     "diagonal", "random", "malicious"), schemes=("raw", "ras", "rap"),
+                     first_trial: int = 0, out: torch.Tensor | None = None,
+                     device="cuda") -> torch.Tensor:
+    """Monte-Carlo congestion histogram int64 [npat, nsch, w+1], ACCUMULATED into `out`."""
+    pm, sm = _mask(patterns, PATTERNS), _mask(schemes, SCHEMES)
+    shape = (bin(pm).count("1"), bin(sm).count("1"), w + 1)
+    if out is None:
+        out = torch.zeros(shape, dtype=torch.int64, device=device)
+    _need_cuda(out)
+    assert tuple(out.shape) == shape and out.dtype == torch.int64 and out.is_contiguous()
+    with torch.cuda.device(out.device):
+        _check(lib().rap_congestion_sweep(w, pm, sm, seed, first_trial, n_trials,
+                                          ctypes.c_void_p(out.data_ptr()), _stream(out)),
+               "rap_congestion_sweep")
+    return out
+
+
+def congestion_trace(cells: torch.Tensor, n_trials: int, seed: int, schemes=("raw", "ras", "rap"),
+                     first_trial: int = 0, out: torch.Tensor | None = None) -> torch.Tensor:
+    """cells int32/uint32 CUDA [n_warps, w] (row*w+col) -> int64 [nsch, w+1] (accumulated)."""
+    _need_cuda(cells, out)
+    n, w = cells.shape
+    assert cells.dtype in (torch.int32, torch.uint32) and cells.is_contiguous()
+    sm = _mask(schemes, SCHEMES)
+    shape = (bin(sm).count("1"), w + 1)
+    if out is None:
+        out = torch.zeros(shape, dtype=torch.int64, device=cells.device)
+    assert tuple(out.shape) == shape and out.dtype == torch.int64 and out.is_contiguous()
+    with torch.cuda.device(cells.device):
+        _check(lib().rap_congestion_trace(w, n, ctypes.c_void_p(cells.data_ptr()), sm, seed,
+                                          first_trial, n_trials, ctypes.c_void_p(out.data_ptr()),
+                                          _stream(cells)), "rap_congestion_trace")
+    return out

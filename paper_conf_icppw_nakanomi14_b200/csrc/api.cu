@@ -1,0 +1,124 @@
+// api.cu -- the extern "C" boundary of librap.so (include/rap.h): argument validation on the
+// host, then one enqueue of the corresponding kernel launcher.  No computation of the method
+// happens here; there is no CPU fallback.
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "../../include/rap.h"
+#include "rap_internal.h"
+
+namespace {
+
+rap_status_t from_cuda(cudaError_t e) { return e == cudaSuccess ? RAP_OK : RAP_ERR_CUDA; }
+
+bool is_pow2(uint32_t w) { return w && !(w & (w - 1)); }
+
+// product of two non-negative int64 without overflow -> false on overflow
+bool mul_ok(int64_t a, int64_t b, int64_t *out) {
+    if (a < 0 || b < 0) return false;
+    if (a != 0 && b > INT64_MAX / a) return false;
+    *out = a * b;
+    return true;
+}
+
+// byte extent [first, last) touched by a row-major matrix with leading dimension ld
+bool extent(uintptr_t base, int64_t rows, int64_t cols, int64_t ld, uint32_t eb, uintptr_t *lo,
+            uintptr_t *hi) {
+    int64_t span;
+    if (!mul_ok(rows - 1, ld, &span)) return false;
+    if (span > INT64_MAX - cols) return false;
+    span += cols;
+    int64_t bytes;
+    if (!mul_ok(span, (int64_t)eb, &bytes)) return false;
+    *lo = base;
+    *hi = base + (uintptr_t)bytes;
+    return *hi >= *lo;
+}
+
+}  // namespace
+
+extern "C" {
+
+int rap_abi_version(void) { return RAP_ABI_VERSION; }
+
+const char *rap_status_str(rap_status_t s) {
+    switch (s) {
+    case RAP_OK: return "RAP_OK";
+    case RAP_ERR_INVALID_ARG: return "RAP_ERR_INVALID_ARG: argument out of range";
+    case RAP_ERR_UNSUPPORTED: return "RAP_ERR_UNSUPPORTED: request not implemented";
+    case RAP_ERR_ALIAS: return "RAP_ERR_ALIAS: src and dst overlap (transpose is out-of-place)";
+    case RAP_ERR_CUDA: return "RAP_ERR_CUDA: CUDA runtime or launch failure";
+    }
+    return "RAP_ERR_UNKNOWN";
+}
+
+rap_status_t rap_perm_gen(uint64_t seed, uint64_t first_index, uint64_t count, uint32_t w,
+                          uint8_t *d_perm_out, void *stream) {
+    if (w < 2 || w > RAP_MAX_W) return RAP_ERR_INVALID_ARG;
+    if (count == 0) return RAP_OK;
+    if (!d_perm_out || count > (UINT64_MAX / w)) return RAP_ERR_INVALID_ARG;
+    return from_cuda(rapk::launch_perm_gen(seed, first_index, count, w, d_perm_out,
+                                           (cudaStream_t)stream));
+}
+
+rap_status_t rap_transpose(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
+                           int64_t ld_dst, uint32_t elem_bytes, rap_layout_t layout, uint64_t seed,
+                           void *stream) {
+    if (elem_bytes != 4 && elem_bytes != 8) return RAP_ERR_INVALID_ARG;
+    if ((int)layout < RAP_LAYOUT_RAW || (int)layout > RAP_LAYOUT_RAP) return RAP_ERR_INVALID_ARG;
+    if (rows < 0 || cols < 0) return RAP_ERR_INVALID_ARG;
+    if (rows == 0 || cols == 0) return RAP_OK;
+    if (!src || !dst) return RAP_ERR_INVALID_ARG;
+    if (ld_src < cols || ld_dst < rows) return RAP_ERR_INVALID_ARG;
+    if ((uintptr_t)src % elem_bytes || (uintptr_t)dst % elem_bytes) return RAP_ERR_INVALID_ARG;
+    uintptr_t s_lo, s_hi, d_lo, d_hi;
+    if (!extent((uintptr_t)src, rows, cols, ld_src, elem_bytes, &s_lo, &s_hi) ||
+        !extent((uintptr_t)dst, cols, rows, ld_dst, elem_bytes, &d_lo, &d_hi))
+        return RAP_ERR_INVALID_ARG;
+    if (s_lo < d_hi && d_lo < s_hi) return RAP_ERR_ALIAS;
+    return from_cuda(rapk::launch_transpose(src, dst, rows, cols, ld_src, ld_dst, elem_bytes,
+                                            (int)layout, seed, (cudaStream_t)stream));
+}
+
+rap_status_t rap_congestion(uint32_t w, uint64_t n_warps, const uint32_t *d_rows,
+                            const uint32_t *d_cols, rap_scheme_t scheme, const uint32_t *d_shift,
+                            uint32_t *d_congestion_out, void *stream) {
+    if (w < 2 || w > RAP_MAX_W) return RAP_ERR_INVALID_ARG;
+    if ((int)scheme < RAP_SCHEME_RAW || (int)scheme > RAP_SCHEME_XOR) return RAP_ERR_INVALID_ARG;
+    if (scheme == RAP_SCHEME_XOR && !is_pow2(w)) return RAP_ERR_INVALID_ARG;
+    if (n_warps == 0) return RAP_OK;
+    if (!d_rows || !d_cols || !d_congestion_out) return RAP_ERR_INVALID_ARG;
+    if ((scheme == RAP_SCHEME_RAS || scheme == RAP_SCHEME_RAP) && !d_shift) return RAP_ERR_INVALID_ARG;
+    if (n_warps > UINT64_MAX / w) return RAP_ERR_INVALID_ARG;
+    const uint32_t *shift = (scheme == RAP_SCHEME_RAS || scheme == RAP_SCHEME_RAP) ? d_shift : nullptr;
+    return from_cuda(rapk::launch_congestion(w, n_warps, d_rows, d_cols, (int)scheme, shift,
+                                             d_congestion_out, (cudaStream_t)stream));
+}
+
+rap_status_t rap_congestion_sweep(uint32_t w, uint32_t pattern_mask, uint32_t scheme_mask,
+                                  uint64_t seed, uint64_t first_trial, uint64_t n_trials,
+                                  uint64_t *d_hist, void *stream) {
+    if (w < 2 || w > RAP_MAX_W) return RAP_ERR_INVALID_ARG;
+    if (pattern_mask == 0 || pattern_mask > 31u || scheme_mask == 0 || scheme_mask > 31u)
+        return RAP_ERR_INVALID_ARG;
+    if (((scheme_mask >> RAP_SCHEME_XOR) & 1u) && !is_pow2(w)) return RAP_ERR_INVALID_ARG;
+    if (n_trials == 0) return RAP_OK;
+    if (!d_hist) return RAP_ERR_INVALID_ARG;
+    return from_cuda(rapk::launch_sweep(w, pattern_mask, scheme_mask, seed, first_trial, n_trials,
+                                        d_hist, (cudaStream_t)stream));
+}
+
+rap_status_t rap_congestion_trace(uint32_t w, uint64_t n_warps, const uint32_t *d_cells,
+                                  uint32_t scheme_mask, uint64_t seed, uint64_t first_trial,
+                                  uint64_t n_trials, uint64_t *d_hist, void *stream) {
+    if (w < 2 || w > RAP_MAX_W) return RAP_ERR_INVALID_ARG;
+    if (scheme_mask == 0 || scheme_mask > 31u) return RAP_ERR_INVALID_ARG;
+    if (((scheme_mask >> RAP_SCHEME_XOR) & 1u) && !is_pow2(w)) return RAP_ERR_INVALID_ARG;
+    if (n_warps == 0 || n_trials == 0) return RAP_OK;
+    if (!d_cells || !d_hist) return RAP_ERR_INVALID_ARG;
+    if (n_warps > UINT64_MAX / w) return RAP_ERR_INVALID_ARG;
+    return from_cuda(rapk::launch_trace(w, n_warps, d_cells, scheme_mask, seed, first_trial,
+                                        n_trials, d_hist, (cudaStream_t)stream));
+}
+
+}  // extern "C"

@@ -1,0 +1,28 @@
+// rap_internal.h -- launcher declarations shared by the kernel translation units and the
+// C-ABI layer (api.cu).  Not part of the public ABI (include/rap.h).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "../../include/rap.h"
+
+namespace rapk {
+
+cudaError_t launch_transpose(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
+                             int64_t ld_dst, uint32_t elem_bytes, int layout, uint64_t seed,
+                             cudaStream_t st);
+
+cudaError_t launch_perm_gen(uint64_t seed, uint64_t first, uint64_t count, uint32_t w, uint8_t *out,
+                            cudaStream_t st);
+
+cudaError_t launch_congestion(uint32_t w, uint64_t n_warps, const uint32_t *rows, const uint32_t *cols,
+                              int scheme, const uint32_t *shift, uint32_t *out, cudaStream_t st);
+
+cudaError_t launch_sweep(uint32_t w, uint32_t pattern_mask, uint32_t scheme_mask, uint64_t seed,
+                         uint64_t first, uint64_t n_trials, uint64_t *hist, cudaStream_t st);
+
+cudaError_t launch_trace(uint32_t w, uint64_t n_warps, const uint32_t *cells, uint32_t scheme_mask,
+                         uint64_t seed, uint64_t first, uint64_t n_trials, uint64_t *hist,
+                         cudaStream_t st);
+
+}  // namespace rapk

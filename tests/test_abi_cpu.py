@@ -1,0 +1,122 @@
+"""Host-side checks of the C ABI that need no GPU (-m "not gpu").
+
+librap.so must load, export every function include/rap.h declares, validate arguments
+BEFORE touching CUDA, and -- with no GPU present -- fail with RAP_ERR_CUDA instead of
+computing anything on the CPU (there is no CPU fallback).
+"""
+import ctypes
+import os
+import re
+
+import pytest
+import torch
+
+from conftest import ROOT
+
+import paper_conf_icppw_nakanomi14_b200 as rap
+from paper_conf_icppw_nakanomi14_b200 import build as rbuild
+
+OK, INVALID, UNSUPPORTED, ALIAS, CUDA = 0, 1, 2, 3, 4
+
+
+@pytest.fixture(scope="module")
+def L():
+    rbuild.build()
+    return rap.lib()
+
+
+def header_functions():
+    src = open(os.path.join(ROOT, "include", "rap.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(rap_[a-z_]+)\s*\(", src)))
+
+
+def test_exports_every_declared_symbol(L):
+    names = header_functions()
+    assert {"rap_perm_gen", "rap_transpose", "rap_congestion", "rap_congestion_sweep",
+            "rap_congestion_trace", "rap_status_str", "rap_abi_version"} <= set(names)
+    for n in names:
+        assert hasattr(L, n), n
+    assert L.rap_abi_version() == 1
+
+
+def test_status_strings(L):
+    for s in range(5):
+        assert L.rap_status_str(s).decode().startswith("RAP_")
+
+
+P = ctypes.c_void_p
+
+
+def test_transpose_validation(L):
+    a, b = P(0x10000000), P(0x20000000)
+    s = P(0)
+    assert L.rap_transpose(a, b, 4, 4, 4, 4, 3, 4, 0, s) == INVALID      # elem_bytes
+    assert L.rap_transpose(a, b, 4, 4, 4, 4, 4, 9, 0, s) == INVALID      # layout
+    assert L.rap_transpose(a, b, -1, 4, 4, 4, 4, 4, 0, s) == INVALID     # rows < 0
+    assert L.rap_transpose(a, b, 4, 8, 4, 4, 4, 4, 0, s) == INVALID      # ld_src < cols
+    assert L.rap_transpose(a, b, 8, 4, 4, 4, 4, 4, 0, s) == INVALID      # ld_dst < rows
+    assert L.rap_transpose(P(0), b, 4, 4, 4, 4, 4, 4, 0, s) == INVALID   # null
+    assert L.rap_transpose(P(0x10000002), b, 4, 4, 4, 4, 4, 4, 0, s) == INVALID  # misaligned
+    assert L.rap_transpose(a, P(0x10000020), 4, 4, 4, 4, 4, 4, 0, s) == ALIAS
+    assert L.rap_transpose(a, b, 0, 4, 4, 4, 4, 4, 0, s) == OK          # empty: no-op
+    assert L.rap_transpose(a, b, 1 << 62, 1 << 62, 1 << 62, 1 << 62, 8, 4, 0, s) == INVALID
+
+
+@pytest.mark.skipif(torch.cuda.is_available(), reason="checks the no-GPU behaviour")
+def test_valid_calls_fail_loudly_without_gpu(L):
+    # a well-formed request reaches CUDA and fails there: nothing is computed on the host
+    a, b = P(0x10000000), P(0x20000000)
+    assert L.rap_transpose(a, b, 64, 64, 64, 64, 4, 4, 0, P(0)) == CUDA
+    assert L.rap_congestion_sweep(32, 31, 7, 1, 0, 1000, P(0x30000000), P(0)) == CUDA
+    assert L.rap_perm_gen(1, 0, 10, 32, P(0x30000000), P(0)) == CUDA
+
+
+def test_sweep_validation(L):
+    h, s = P(0x30000000), P(0)
+    assert L.rap_congestion_sweep(1, 31, 7, 1, 0, 10, h, s) == INVALID    # w < 2
+    assert L.rap_congestion_sweep(33, 31, 7, 1, 0, 10, h, s) == INVALID   # w > 32
+    assert L.rap_congestion_sweep(32, 0, 7, 1, 0, 10, h, s) == INVALID    # empty pattern mask
+    assert L.rap_congestion_sweep(32, 32, 7, 1, 0, 10, h, s) == INVALID   # unknown pattern
+    assert L.rap_congestion_sweep(32, 31, 64, 1, 0, 10, h, s) == INVALID  # unknown scheme
+    assert L.rap_congestion_sweep(24, 31, 16, 1, 0, 10, h, s) == INVALID  # XOR needs 2^k
+    assert L.rap_congestion_sweep(32, 31, 7, 1, 0, 10, P(0), s) == INVALID
+    assert L.rap_congestion_sweep(32, 31, 7, 1, 0, 0, P(0), s) == OK      # no trials: no-op
+
+
+def test_congestion_trace_perm_validation(L):
+    d, s = P(0x30000000), P(0)
+    assert L.rap_congestion(1, 4, d, d, 2, d, d, s) == INVALID
+    assert L.rap_congestion(32, 4, d, d, 7, d, d, s) == INVALID
+    assert L.rap_congestion(32, 4, d, d, 2, P(0), d, s) == INVALID        # RAP needs shifts
+    assert L.rap_congestion(12, 4, d, d, 4, None, d, s) == INVALID        # XOR needs 2^k
+    assert L.rap_congestion(32, 0, d, d, 2, d, d, s) == OK
+    assert L.rap_congestion_trace(32, 4, d, 0, 1, 0, 5, d, s) == INVALID
+    assert L.rap_congestion_trace(32, 4, P(0), 7, 1, 0, 5, d, s) == INVALID
+    assert L.rap_congestion_trace(32, 0, d, 7, 1, 0, 5, d, s) == OK
+    assert L.rap_perm_gen(1, 0, 4, 33, d, s) == INVALID
+    assert L.rap_perm_gen(1, 0, 4, 1, d, s) == INVALID
+    assert L.rap_perm_gen(1, 0, 4, 32, P(0), s) == INVALID
+    assert L.rap_perm_gen(1, 0, 0, 32, P(0), s) == OK
+
+
+def test_python_binding_refuses_cpu_tensors(L):
+    x = torch.zeros(8, 8)
+    with pytest.raises(ValueError):
+        rap.transpose(x)
+    with pytest.raises(ValueError):
+        rap.congestion_sweep(10, 1, out=torch.zeros(5, 3, 33, dtype=torch.int64))
+
+
+def test_product_does_not_import_oracle():
+    # the product package and the oracle share no code and never import each other
+    pkg = os.path.join(ROOT, "paper_conf_icppw_nakanomi14_b200")
+    for dirpath, _, files in os.walk(pkg):
+        for f in files:
+            if f.endswith((".py", ".cu", ".cuh", ".h", ".cpp")):
+                txt = open(os.path.join(dirpath, f)).read()
+                assert "oracle" not in re.sub(r"(#|//).*", "", txt).lower().replace("oracle/", ""), f
+    for f in os.listdir(os.path.join(ROOT, "oracle")):
+        if f.endswith((".py", ".c")):
+            txt = open(os.path.join(ROOT, "oracle", f)).read()
+            assert "import paper_conf" not in txt and "csrc" not in txt and "rap.h" not in txt, f

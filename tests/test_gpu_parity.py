@@ -1,0 +1,253 @@
+"""GPU parity: the CUDA path (through the C ABI / binding) against the CPU oracle (-m gpu).
+
+Integer and bit work, so every comparison is bit-exact: transposed bytes (as uint32/uint64
+views, including NaN payloads, -0, Inf, subnormals), permutations, per-warp congestions and
+per-seed u64 histograms.
+"""
+import itertools
+import math
+
+import numpy as np
+import pytest
+import torch
+
+import workloads
+from closed_forms import balls_in_bins_cdf, expectation, pmf_from_cdf, random_access_cdf, variance
+
+pytestmark = pytest.mark.gpu
+
+LAYOUT_NAMES = ["raw", "pad", "xor", "ras", "rap"]
+ALL_PAT = ["contiguous", "stride", "diagonal", "random", "malicious"]
+ALL_SCH = ["raw", "ras", "rap", "pad", "xor"]
+
+
+@pytest.fixture(scope="module")
+def rap():
+    import __graft_entry__
+    __graft_entry__.build()
+    import paper_conf_icppw_nakanomi14_b200 as r
+    assert torch.cuda.is_available(), "GPU tests need a CUDA device"
+    return r
+
+
+def bits(t):
+    return workloads.as_bits_numpy(t)
+
+
+# ------------------------------------------------------------------ T0 permutations
+@pytest.mark.parametrize("w", [2, 3, 5, 16, 31, 32])
+def test_perm_gen_matches_oracle(rap, oracle, w):
+    first, count = 12345678901, 3000
+    P = rap.perm_gen(seed=77, count=count, w=w, first_index=first).cpu().numpy()
+    for k in range(0, count, 7):
+        assert np.array_equal(P[k], oracle.perm(77, first + k, w).astype(np.uint8)), k
+    assert all(sorted(row) == list(range(w)) for row in P.tolist())
+
+
+# ------------------------------------------------------------------ T1-T3 transpose
+SHAPES = [(1, 1), (1, 100), (100, 1), (32, 32), (33, 65), (64, 32), (257, 129), (1000, 3), (5, 1000),
+          (96, 4096)]
+
+
+@pytest.mark.parametrize("layout", LAYOUT_NAMES)
+@pytest.mark.parametrize("dtype", [torch.float32, torch.float64])
+def test_transpose_shapes(rap, oracle, layout, dtype):
+    for i, (r, c) in enumerate(SHAPES):
+        x = workloads.random_bits(r, c, dtype, seed=i)
+        y = rap.transpose(x.cuda(), layout=layout, seed=i + 11)
+        torch.cuda.synchronize()
+        assert y.shape == (c, r)
+        assert np.array_equal(bits(y), oracle.transpose(bits(x))), (layout, r, c)
+
+
+@pytest.mark.parametrize("layout", ["rap", "raw", "xor"])
+@pytest.mark.parametrize("dtype", [torch.float32, torch.float64])
+def test_transpose_strided_and_misaligned(rap, oracle, layout, dtype):
+    # row pitch ld_src > cols (vector path when 16B-aligned), an odd column offset (scalar
+    # path), and an output with row pitch ld_dst > rows
+    big = workloads.random_bits(300, 260, dtype, seed=3)
+    for (r0, c0, r1, c1) in [(0, 0, 300, 256), (3, 4, 291, 250), (1, 1, 200, 77), (2, 3, 35, 40)]:
+        xs = big.cuda()[r0:r1, c0:c1]
+        out_big = torch.zeros((c1 - c0, (r1 - r0) + 9), dtype=dtype, device="cuda")
+        out = out_big[:, 5:5 + (r1 - r0)]
+        rap.transpose(xs, layout=layout, seed=1, out=out)
+        torch.cuda.synchronize()
+        assert np.array_equal(bits(out), oracle.transpose(bits(big[r0:r1, c0:c1])))
+        assert not bits(out_big[:, :5]).any() and not bits(out_big[:, 5 + (r1 - r0):]).any()
+
+
+def test_transpose_empty_and_alias(rap):
+    x = torch.zeros((0, 7), device="cuda")
+    assert rap.transpose(x).shape == (7, 0)
+    buf = torch.zeros(64 * 64 * 2, device="cuda")
+    with pytest.raises(rap.RapError):
+        rap.transpose(buf[:4096].view(64, 64), out=buf[2048:2048 + 4096].view(64, 64))
+
+
+def test_transpose_result_independent_of_seed(rap):
+    x = workloads.random_bits(200, 300, torch.float32, seed=9).cuda()
+    ref = rap.transpose(x, layout="raw")
+    for s in (0, 1, 2, 2 ** 63 + 5):
+        assert torch.equal(rap.transpose(x, layout="rap", seed=s).view(torch.int32), ref.view(torch.int32))
+
+
+def _band_check(oracle, x_dev, y_dev, n_bands=6, band=48, seed=0):
+    """Full-size check on sampled row bands: the oracle transposes each band of x."""
+    rows, cols = x_dev.shape
+    rng = np.random.default_rng(seed)
+    starts = sorted(set([0, rows - band] + rng.integers(0, rows - band, n_bands).tolist()))
+    for r0 in starts:
+        xb = bits(x_dev[r0:r0 + band])
+        yb = bits(y_dev[:, r0:r0 + band])
+        assert np.array_equal(yb, oracle.transpose(xb)), r0
+
+
+@pytest.mark.parametrize("layout", LAYOUT_NAMES)
+def test_transpose_cfg3_8192_f32(rap, oracle, layout):
+    # BASELINE cfg3 at full size, in the launch configuration bench.py times
+    x = workloads.random_bits(8192, 8192, torch.float32, seed=0, device="cuda")
+    y = rap.transpose(x, layout=layout, seed=0)
+    torch.cuda.synchronize()
+    if layout == "rap":
+        assert np.array_equal(bits(y), oracle.transpose(bits(x), threads=oracle.max_threads()))
+    else:
+        _band_check(oracle, x, y, seed=1)
+    # property at any size: transposing twice is the identity (bit-exact)
+    z = rap.transpose(y, layout=layout, seed=1)
+    assert torch.equal(z.view(torch.int32), x.view(torch.int32))
+
+
+def test_transpose_cfg4_16384_f64(rap, oracle):
+    x = workloads.random_bits(16384, 16384, torch.float64, seed=0, device="cuda")
+    y = rap.transpose(x, layout="rap", seed=0)
+    torch.cuda.synchronize()
+    _band_check(oracle, x, y, n_bands=4, band=40, seed=2)
+    del x
+    # column bands too (output rows)
+    xs = workloads.random_bits(16384, 16384, torch.float64, seed=0, device="cuda")
+    for c0 in (0, 7777, 16384 - 33):
+        assert np.array_equal(bits(y[c0:c0 + 33]), oracle.transpose(bits(xs[:, c0:c0 + 33])))
+
+
+def test_transpose_cfg1_tile(rap, oracle):
+    for seed in (0, 1, 2):
+        x = workloads.random_bits(32, 32, torch.float32, seed=seed)
+        y = rap.transpose(x.cuda(), layout="rap", seed=seed)
+        torch.cuda.synchronize()
+        assert np.array_equal(bits(y), oracle.transpose(bits(x)))
+
+
+# ------------------------------------------------------------------ C3 batched evaluator
+@pytest.mark.parametrize("w", [2, 4, 7, 16, 32])
+def test_congestion_batched_matches_oracle(rap, oracle, w):
+    rng = np.random.default_rng(w)
+    n = 400
+    rows = rng.integers(0, w, (n, w))
+    cols = rng.integers(0, w, (n, w))
+    # duplicates and structured warps
+    rows[::5] = rows[::5, :1]
+    cols[::7] = cols[::7, :1]
+    rows[1::9], cols[1::9] = np.arange(w), np.arange(w)
+    shift = np.stack([rng.permutation(w) for _ in range(n)])
+    schemes = ["raw", "ras", "rap", "pad"] + (["xor"] if w & (w - 1) == 0 else [])
+    t = lambda a: torch.from_numpy(a.astype(np.int32)).cuda()
+    for s in schemes:
+        got = rap.congestion(t(rows), t(cols), s, shift=t(shift)).cpu().numpy()
+        for k in range(n):
+            sh = shift[k] if s in ("ras", "rap") else None
+            assert got[k] == oracle.congestion(w, rows[k], cols[k], oracle.SCHEMES[s], sh), (s, k)
+
+
+def test_congestion_out_of_range_marks_zero(rap):
+    rows = torch.zeros((2, 32), dtype=torch.int32, device="cuda")
+    cols = torch.arange(32, dtype=torch.int32, device="cuda").repeat(2, 1)
+    cols[1, 5] = 40
+    got = rap.congestion(rows, cols, "raw").cpu().tolist()
+    assert got == [1, 0]
+
+
+# ------------------------------------------------------------------ C1-C4 sweep
+@pytest.mark.parametrize("seed", [1, 2, 3])
+def test_sweep_bit_exact_w32(rap, oracle, seed):
+    N = 1_000_000
+    g = rap.congestion_sweep(N, seed=seed, w=32, patterns=ALL_PAT, schemes=ALL_SCH)
+    o = oracle.sweep(32, ALL_PAT, ALL_SCH, seed, 0, N)
+    assert np.array_equal(g.cpu().numpy().astype(np.uint64), o)
+
+
+@pytest.mark.parametrize("w", [2, 3, 7, 16, 31])
+def test_sweep_bit_exact_other_w(rap, oracle, w):
+    N = 100_000
+    sch = ["raw", "ras", "rap", "pad"] + (["xor"] if w & (w - 1) == 0 else [])
+    g = rap.congestion_sweep(N, seed=5, w=w, patterns=ALL_PAT, schemes=sch, first_trial=2 ** 33 + 17)
+    o = oracle.sweep(w, ALL_PAT, sch, 5, 2 ** 33 + 17, N)
+    assert np.array_equal(g.cpu().numpy().astype(np.uint64), o)
+
+
+def test_sweep_masks_and_chunks(rap, oracle):
+    N = 200_000
+    for pats, schs in ((["random"], ["rap"]), (["stride", "malicious"], ["ras", "xor"]),
+                       (["diagonal"], ["raw", "pad"])):
+        g = rap.congestion_sweep(N, seed=8, patterns=pats, schemes=schs, first_trial=99)
+        o = oracle.sweep(32, pats, schs, 8, 99, N)
+        assert np.array_equal(g.cpu().numpy().astype(np.uint64), o)
+    # accumulation: arbitrary chunks sum to the one-shot histogram
+    one = rap.congestion_sweep(N, seed=4)
+    acc = torch.zeros_like(one)
+    for a, b in ((0, 1), (1, 77777), (77777, 150001), (150001, N)):
+        rap.congestion_sweep(b - a, seed=4, first_trial=a, out=acc)
+    assert torch.equal(one, acc)
+
+
+def test_sweep_full_size_1e9(rap, oracle):
+    # BASELINE cfg2 at full size: 10^9 trials, w=32.  Properties that hold at any size plus
+    # a sampled sub-range recomputed by the oracle.
+    N = 10 ** 9
+    h = rap.congestion_sweep(N, seed=1, patterns=ALL_PAT, schemes=["raw", "ras", "rap"]).cpu().numpy()
+    assert (h.sum(-1) == N).all()
+    assert h[0, :, 1].tolist() == [N, N, N]          # contiguous: 1 under every scheme
+    assert h[1, 0, 32] == N and h[1, 2, 1] == N      # stride: RAW 32, RAP 1 (Theorem 2)
+    assert h[2, 0, 1] == N                           # diagonal RAW 1
+    assert np.array_equal(h[1, 1], h[4, 1]) and np.array_equal(h[2, 2], h[4, 2])
+    c = np.arange(33)
+    pmf = pmf_from_cdf(balls_in_bins_cdf, 32)
+    E, sd = float(expectation(pmf)), float(variance(pmf)) ** 0.5
+    mu = (h[1, 1] * c).sum() / N
+    assert abs(mu - E) < 2.576 * sd / math.sqrt(N)   # ~3.53, 99% CI
+    pmf_r = pmf_from_cdf(random_access_cdf, 32)
+    Er, sdr = float(expectation(pmf_r)), float(variance(pmf_r)) ** 0.5
+    for s in range(3):
+        assert abs((h[3, s] * c).sum() / N - Er) < 2.576 * sdr / math.sqrt(N)
+    mu_rap = (h[2, 2] * c).sum() / N
+    assert round(mu_rap, 2) == 3.61                  # Table II RAP diagonal
+    # sampled sub-range of the same run: bit-exact against the oracle
+    first = 987_654_321
+    g = rap.congestion_sweep(200_000, seed=1, first_trial=first)
+    o = oracle.sweep(32, ALL_PAT, ["raw", "ras", "rap"], 1, first, 200_000)
+    assert np.array_equal(g.cpu().numpy().astype(np.uint64), o)
+
+
+# ------------------------------------------------------------------ trace evaluator
+def test_trace_matches_oracle(rap, oracle):
+    w, n_trials, first = 32, 40, 1000
+    cells = workloads.trace_cells(30, w, seed=4)
+    g = rap.congestion_trace(cells.cuda(), n_trials, seed=6, schemes=ALL_SCH, first_trial=first)
+    expect = np.zeros((5, w + 1), dtype=np.uint64)
+    cl = cells.numpy()
+    for n in range(first, first + n_trials):
+        P, r = oracle.perm(6, n, w), oracle.ras_shifts(6, n, w)
+        for k in range(cl.shape[0]):
+            rows, cols = cl[k] // w, cl[k] % w
+            for si, s in enumerate(ALL_SCH):
+                sh = {"ras": r, "rap": P}.get(s)
+                expect[si, oracle.congestion(w, rows, cols, oracle.SCHEMES[s], sh)] += 1
+    assert np.array_equal(g.cpu().numpy().astype(np.uint64), expect)
+
+
+def test_trace_small_w_and_invalid(rap, oracle):
+    w = 8
+    cells = workloads.trace_cells(13, w, seed=1)
+    cells[3, 2] = w * w + 5                          # invalid -> bin 0
+    g = rap.congestion_trace(cells.cuda(), 7, seed=2, schemes=["rap", "raw"]).cpu().numpy()
+    assert g[:, 0].tolist() == [7, 7]
+    assert (g.sum(-1) == 13 * 7).all()
