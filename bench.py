@@ -46,6 +46,7 @@ def parse():
                    choices=["default", "sweep", "cfg4", "tile", "layouts", "dist"])
     p.add_argument("--sweep-trials", type=int, default=1 << 24)
     p.add_argument("--layout", default="rap")
+    p.add_argument("--sweep-algo", default="default", choices=["default", "match"])
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu", action="store_true")
     return p.parse_args()
@@ -245,7 +246,7 @@ def main():
             if do_t:
                 rap.transpose(x, layout=lay, seed=0, out=y)
             if do_s:
-                rap.congestion_sweep(S, seed=1, first_trial=trial0, out=hist)
+                rap.congestion_sweep(S, seed=1, first_trial=trial0, out=hist, algo=args.sweep_algo)
                 trial0 += S
         torch.cuda.synchronize()
         hist.zero_()
@@ -264,7 +265,7 @@ def main():
                 e[1].record(stream)
                 e[2].record(stream)
                 if do_s:
-                    rap.congestion_sweep(S, seed=1, first_trial=trial0, out=hist)
+                    rap.congestion_sweep(S, seed=1, first_trial=trial0, out=hist, algo=args.sweep_algo)
                     trial0 += S
                     launches += 1
                 e[3].record(stream)

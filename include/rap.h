@@ -124,6 +124,19 @@ rap_status_t rap_congestion_sweep(uint32_t w, uint32_t pattern_mask, uint32_t sc
                                   uint64_t seed, uint64_t first_trial, uint64_t n_trials,
                                   uint64_t *d_hist, void *stream);
 
+/* Kernel designs of the sweep (identical histograms):
+ *   RAP_SWEEP_DEFAULT  lane-mode bit-sliced Fisher-Yates (one trial per lane, no shuffles)
+ *                      + ballot bank histogram in warp mode;
+ *   RAP_SWEEP_MATCH    one warp per trial, shuffle Fisher-Yates + __match_any_sync histogram
+ *                      (kept as the measured ablation). */
+typedef enum { RAP_SWEEP_DEFAULT = 0, RAP_SWEEP_MATCH = 1 } rap_sweep_algo_t;
+
+/* rap_congestion_sweep with an explicit kernel design; algo outside rap_sweep_algo_t ->
+ * RAP_ERR_INVALID_ARG.  rap_congestion_sweep(...) == rap_congestion_sweep_algo(..., 0, ...). */
+rap_status_t rap_congestion_sweep_algo(uint32_t w, uint32_t pattern_mask, uint32_t scheme_mask,
+                                       uint64_t seed, uint64_t first_trial, uint64_t n_trials,
+                                       uint64_t *d_hist, uint32_t algo, void *stream);
+
 /* C3 over user traces: d_cells: device uint32_t[n_warps][w], cell = row*w + col < w*w.
  * Every trace warp is evaluated under every trial's P_n / r_n, n in [first_trial,
  * first_trial + n_trials).  d_hist: device uint64_t[nsch][w+1], ACCUMULATED (+=);

@@ -22,6 +22,7 @@ __all__ = ["perm_gen", "transpose", "congestion", "congestion_sweep", "congestio
 
 LAYOUTS = {"raw": 0, "pad": 1, "xor": 2, "ras": 3, "rap": 4}
 SCHEMES = {"raw": 0, "ras": 1, "rap": 2, "pad": 3, "xor": 4}
+SWEEP_ALGOS = {"default": 0, "match": 1}
 PATTERNS = {"contiguous": 0, "stride": 1, "diagonal": 2, "random": 3, "malicious": 4}
 STATUS = {0: "RAP_OK", 1: "RAP_ERR_INVALID_ARG", 2: "RAP_ERR_UNSUPPORTED", 3: "RAP_ERR_ALIAS",
           4: "RAP_ERR_CUDA"}
@@ -58,9 +59,10 @@ def lib():
         L.rap_transpose.argtypes = [vp, vp, i64, i64, i64, i64, u32, i32, u64, vp]
         L.rap_congestion.argtypes = [u32, u64, u32p, u32p, i32, u32p, u32p, vp]
         L.rap_congestion_sweep.argtypes = [u32, u32, u32, u64, u64, u64, u64p, vp]
+        L.rap_congestion_sweep_algo.argtypes = [u32, u32, u32, u64, u64, u64, u64p, u32, vp]
         L.rap_congestion_trace.argtypes = [u32, u64, u32p, u32, u64, u64, u64, u64p, vp]
         for f in ("rap_perm_gen", "rap_transpose", "rap_congestion", "rap_congestion_sweep",
-                  "rap_congestion_trace"):
+                  "rap_congestion_sweep_algo", "rap_congestion_trace"):
             getattr(L, f).restype = i32
         if L.rap_abi_version() != 1:
             raise ImportError("librap.so ABI version mismatch")
@@ -160,8 +162,12 @@ def congestion(rows: torch.Tensor, cols: torch.Tensor, scheme: str = "rap",
 def congestion_sweep(n_trials: int, seed: int, w: int = 32, patterns=("contiguous", "stride",
                      "diagonal", "random", "malicious"), schemes=("raw", "ras", "rap"),
                      first_trial: int = 0, out: torch.Tensor | None = None,
-                     device="cuda") -> torch.Tensor:
-    """Monte-Carlo congestion histogram int64 [npat, nsch, w+1], ACCUMULATED into `out`."""
+                     device="cuda", algo: str = "default") -> torch.Tensor:
+    """Monte-Carlo congestion histogram int64 [npat, nsch, w+1], ACCUMULATED into `out`.
+
+    algo: "default" (bit-sliced lane-mode Fisher-Yates + ballot histogram) or "match"
+    (warp shuffle Fisher-Yates + __match_any_sync, the measured ablation); identical results.
+    """
     pm, sm = _mask(patterns, PATTERNS), _mask(schemes, SCHEMES)
     shape = (bin(pm).count("1"), bin(sm).count("1"), w + 1)
     if out is None:
@@ -169,9 +175,9 @@ def congestion_sweep(n_trials: int, seed: int, w: int = 32, patterns=("contiguou
     _need_cuda(out)
     assert tuple(out.shape) == shape and out.dtype == torch.int64 and out.is_contiguous()
     with torch.cuda.device(out.device):
-        _check(lib().rap_congestion_sweep(w, pm, sm, seed, first_trial, n_trials,
-                                          ctypes.c_void_p(out.data_ptr()), _stream(out)),
-               "rap_congestion_sweep")
+        _check(lib().rap_congestion_sweep_algo(w, pm, sm, seed, first_trial, n_trials,
+                                               ctypes.c_void_p(out.data_ptr()), SWEEP_ALGOS[algo],
+                                               _stream(out)), "rap_congestion_sweep")
     return out
 
 

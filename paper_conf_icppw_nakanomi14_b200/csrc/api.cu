@@ -76,6 +76,8 @@ rap_status_t rap_transpose(const void *src, void *dst, int64_t rows, int64_t col
         !extent((uintptr_t)dst, cols, rows, ld_dst, elem_bytes, &d_lo, &d_hi))
         return RAP_ERR_INVALID_ARG;
     if (s_lo < d_hi && d_lo < s_hi) return RAP_ERR_ALIAS;
+    // 32 x 32 tiles are indexed with 32-bit counters: up to 2^31 tiles (2^41 elements)
+    if (((rows + 31) / 32) * ((cols + 31) / 32) >= (int64_t(1) << 31)) return RAP_ERR_UNSUPPORTED;
     return from_cuda(rapk::launch_transpose(src, dst, rows, cols, ld_src, ld_dst, elem_bytes,
                                             (int)layout, seed, (cudaStream_t)stream));
 }
@@ -95,17 +97,26 @@ rap_status_t rap_congestion(uint32_t w, uint64_t n_warps, const uint32_t *d_rows
                                              d_congestion_out, (cudaStream_t)stream));
 }
 
-rap_status_t rap_congestion_sweep(uint32_t w, uint32_t pattern_mask, uint32_t scheme_mask,
-                                  uint64_t seed, uint64_t first_trial, uint64_t n_trials,
-                                  uint64_t *d_hist, void *stream) {
+rap_status_t rap_congestion_sweep_algo(uint32_t w, uint32_t pattern_mask, uint32_t scheme_mask,
+                                       uint64_t seed, uint64_t first_trial, uint64_t n_trials,
+                                       uint64_t *d_hist, uint32_t algo, void *stream) {
     if (w < 2 || w > RAP_MAX_W) return RAP_ERR_INVALID_ARG;
     if (pattern_mask == 0 || pattern_mask > 31u || scheme_mask == 0 || scheme_mask > 31u)
         return RAP_ERR_INVALID_ARG;
     if (((scheme_mask >> RAP_SCHEME_XOR) & 1u) && !is_pow2(w)) return RAP_ERR_INVALID_ARG;
+    if (algo > RAP_SWEEP_MATCH) return RAP_ERR_INVALID_ARG;
     if (n_trials == 0) return RAP_OK;
     if (!d_hist) return RAP_ERR_INVALID_ARG;
-    return from_cuda(rapk::launch_sweep(w, pattern_mask, scheme_mask, seed, first_trial, n_trials,
-                                        d_hist, (cudaStream_t)stream));
+    auto launch = algo == RAP_SWEEP_MATCH ? rapk::launch_sweep_match : rapk::launch_sweep;
+    return from_cuda(launch(w, pattern_mask, scheme_mask, seed, first_trial, n_trials, d_hist,
+                            (cudaStream_t)stream));
+}
+
+rap_status_t rap_congestion_sweep(uint32_t w, uint32_t pattern_mask, uint32_t scheme_mask,
+                                  uint64_t seed, uint64_t first_trial, uint64_t n_trials,
+                                  uint64_t *d_hist, void *stream) {
+    return rap_congestion_sweep_algo(w, pattern_mask, scheme_mask, seed, first_trial, n_trials,
+                                     d_hist, RAP_SWEEP_DEFAULT, stream);
 }
 
 rap_status_t rap_congestion_trace(uint32_t w, uint64_t n_warps, const uint32_t *d_cells,

@@ -22,40 +22,77 @@ constexpr int kSweepWarps = 8;
 constexpr int kMaxEval = 25;                 // 5 patterns x 5 schemes
 constexpr int kMaxBins = kMaxEval * (RAP_MAX_W + 1);
 
-// Congestion of the warp access in which active lane t (< w) requests logical cell
-// (row, col) of a w x w matrix stored by `scheme`.  P / r: lane i holds P[i] / r[i].
-template <int W>
-__device__ __forceinline__ uint32_t warp_congestion(uint32_t row, uint32_t col, int scheme, uint32_t P,
-                                                    uint32_t r, uint32_t lane, uint32_t w_rt,
-                                                    bool dedupe) {
-    const uint32_t w = W ? (uint32_t)W : w_rt;
-    const bool active = lane < w;
-    uint32_t addr, bank;
+// ---------------------------------------------------------------------------------------
+// Congestion by bit-sliced ballots (default).  Each lane v counts the requests to bank v:
+// with B_k = ballot(bit k of bank), the lanes whose bank equals v are AND_k (v_k ? B_k : ~B_k);
+// popc of that (restricted to the counted lanes) is the load of bank v, and the congestion is
+// the warp maximum (__reduce_max_sync).  Five VOTE + five LOP3 + POPC + REDUX per access.
+struct LaneSel {
+    uint32_t nsel[5];        // bit k of lane ? 0 : ~0
+    __device__ __forceinline__ explicit LaneSel(uint32_t lane) {
+#pragma unroll
+        for (int k = 0; k < 5; ++k) nsel[k] = ((lane >> k) & 1u) ? 0u : 0xffffffffu;
+    }
+};
+
+__device__ __forceinline__ uint32_t max_bank_load(uint32_t bank, uint32_t counted, const LaneSel &ls) {
+    uint32_t m = counted;
+#pragma unroll
+    for (int k = 0; k < 5; ++k) m &= __ballot_sync(kFull, (bank >> k) & 1u) ^ ls.nsel[k];
+    return __reduce_max_sync(kFull, __popc(m));
+}
+
+// Merged requests: lanes of `active` that carry the first occurrence of their
+// 10-bit key (the logical cell row*32 + col; every address map is injective on cells).
+__device__ __forceinline__ uint32_t first_occurrences(uint32_t key, uint32_t active, uint32_t lane) {
+    uint32_t same = active;
+#pragma unroll
+    for (int k = 0; k < 10; ++k) {
+        const uint32_t b = __ballot_sync(kFull, (key >> k) & 1u);
+        same &= ((key >> k) & 1u) ? b : ~b;
+    }
+    const bool leader = (same & ((1u << lane) - 1u)) == 0u;
+    return __ballot_sync(kFull, leader) & active;
+}
+
+// Bank of logical cell (row, col) under `scheme`; sh = shift of that row (r[row] or P[row]).
+__device__ __forceinline__ uint32_t bank_of(int scheme, uint32_t row, uint32_t col, uint32_t sh, uint32_t w) {
     switch (scheme) {
     case RAP_SCHEME_RAS:
-    case RAP_SCHEME_RAP: {
-        const uint32_t sh = __shfl_sync(kFull, scheme == RAP_SCHEME_RAP ? P : r, row & 31u);
-        uint32_t pc = col + sh;
-        pc = (pc >= w) ? pc - w : pc;                    // (col + shift[row]) mod w
-        bank = pc;
-        addr = row * w + pc;
-        break;
+    case RAP_SCHEME_RAP: { const uint32_t b = col + sh; return b >= w ? b - w : b; }
+    case RAP_SCHEME_PAD: { const uint32_t b = row + col; return b >= w ? b - w : b; }
+    case RAP_SCHEME_XOR: return col ^ row;
+    default: return col;
     }
-    case RAP_SCHEME_PAD: {
-        uint32_t b = row + col;
-        bank = (b >= w) ? b - w : b;                     // (row*(w+1) + col) mod w
-        addr = row * (w + 1) + col;
-        break;
-    }
-    case RAP_SCHEME_XOR:
-        bank = col ^ row;
-        addr = row * w + bank;
-        break;
-    default:                                             // RAW
-        bank = col;
-        addr = row * w + col;
-        break;
-    }
+}
+
+// Generic evaluator: lane t (< w) requests (row, col); P / r: lane i holds P[i] / r[i].
+__device__ __forceinline__ uint32_t warp_congestion(uint32_t row, uint32_t col, int scheme, uint32_t P,
+                                                    uint32_t r, uint32_t lane, uint32_t w,
+                                                    const LaneSel &ls) {
+    const uint32_t active = (w >= 32) ? kFull : ((1u << w) - 1u);
+    uint32_t sh = 0;
+    if (scheme == RAP_SCHEME_RAS || scheme == RAP_SCHEME_RAP)
+        sh = __shfl_sync(kFull, scheme == RAP_SCHEME_RAP ? P : r, row & 31u);
+    const uint32_t bank = bank_of(scheme, row, col, sh, w);
+    const uint32_t counted = first_occurrences(row * 32u + col, active, lane);
+    return max_bank_load(bank, counted, ls);
+}
+
+// ---------------------------------------------------------------------------------------
+// Ablation variant (the north-star sketch): __match_any_sync on the address to merge, then
+// popc(__match_any_sync(bank)).  Bit-identical results; kept to measure the design choice.
+template <int W>
+__device__ __forceinline__ uint32_t warp_congestion_match(uint32_t row, uint32_t col, int scheme, uint32_t P,
+                                                          uint32_t r, uint32_t lane, uint32_t w_rt,
+                                                          bool dedupe) {
+    const uint32_t w = W ? (uint32_t)W : w_rt;
+    const bool active = lane < w;
+    uint32_t sh = 0;
+    if (scheme == RAP_SCHEME_RAS || scheme == RAP_SCHEME_RAP)
+        sh = __shfl_sync(kFull, scheme == RAP_SCHEME_RAP ? P : r, row & 31u);
+    const uint32_t bank = bank_of(scheme, row, col, sh, w);
+    const uint32_t addr = row * 32u + col;
     uint32_t key = bank;
     if (dedupe) {                                        // merge identical addresses
         const uint32_t same = __match_any_sync(kFull, active ? addr : (0x40000000u | lane));
@@ -94,11 +131,190 @@ __device__ __forceinline__ void flush_hist(uint32_t (*sh)[kMaxBins], int nwarps,
     }
 }
 
-// ------------------------------------------------------------------ C1-C4 sweep
+// ------------------------------------------------------------------ C1-C4 sweep (default)
+// Two phases per batch of 32 trials, per warp:
+//  lane mode  (lane L <-> trial n0+L): the lane draws its own Philox words (C1), runs the
+//             whole Durstenfeld shuffle on a bit-sliced permutation held in 5 registers --
+//             plane k has bit i = bit k of a[i], so a swap a[k] <-> a[j] is a few shifts and
+//             XORs per plane, no shuffles (C2) -- and stores its RAS shifts and random cells
+//             into a [32][33] shared-memory transpose buffer (+1 padding: the lane-mode write
+//             and the warp-mode read are both conflict-free).
+//  warp mode  (lane t <-> DMM thread t of trial n0+m, m = 0..31): broadcast trial m's planes
+//             (5 shuffles), unpack P[t]; read r[t] and cell t from shared memory; evaluate
+//             every selected (pattern, scheme) with the ballot evaluator (C3); lane e counts
+//             evaluation e in the CTA histogram (C4).
+constexpr int kSweepWarpsV2 = 4;
+
 template <int W>
-__global__ void __launch_bounds__(kSweepWarps * 32)
+__device__ __forceinline__ void swap_planes(uint32_t (&pl)[5], uint32_t k, uint32_t j) {
+#pragma unroll
+    for (int b = 0; b < 5; ++b) {
+        const uint32_t d = ((pl[b] >> j) ^ (pl[b] >> k)) & 1u;
+        pl[b] ^= (d << j) | (d << k);
+    }
+}
+
+// C1+C2 in lane mode: P_n = perm(seed, n, w) as bit planes.
+template <int W>
+__device__ __forceinline__ void lane_perm_planes(uint64_t seed, uint64_t n, uint32_t w_rt, uint32_t (&pl)[5]) {
+    const uint32_t w = W ? (uint32_t)W : w_rt;
+    pl[0] = 0xAAAAAAAAu; pl[1] = 0xCCCCCCCCu; pl[2] = 0xF0F0F0F0u; pl[3] = 0xFF00FF00u; pl[4] = 0xFFFF0000u;
+    if (W) {
+#pragma unroll
+        for (int blk = 0; blk < (W ? (W + 2) / 4 : 1); ++blk) {
+            const uint4 c = philox_block(seed, n, kDomainFY, blk);
+            const uint32_t u[4] = {c.x, c.y, c.z, c.w};
+#pragma unroll
+            for (int i = 0; i < 4; ++i) {
+                const int t = 4 * blk + i;
+                if (t >= W - 1) break;
+                const uint32_t k = (uint32_t)(W - 1 - t);
+                swap_planes<W>(pl, k, mulshift(u[i], k + 1));
+            }
+        }
+    } else {
+        for (uint32_t blk = 0; 4 * blk + 1 < w; ++blk) {
+            const uint4 c = philox_block(seed, n, kDomainFY, blk);
+            const uint32_t u[4] = {c.x, c.y, c.z, c.w};
+#pragma unroll
+            for (int i = 0; i < 4; ++i) {
+                const uint32_t t = 4 * blk + i;
+                if (t + 1 < w) {
+                    const uint32_t k = w - 1 - t;
+                    swap_planes<0>(pl, k, mulshift(u[i], k + 1));
+                }
+            }
+        }
+    }
+}
+
+__device__ __forceinline__ uint32_t plane_value(const uint32_t (&q)[5], uint32_t i) {
+    uint32_t v = 0;
+#pragma unroll
+    for (int b = 0; b < 5; ++b) v |= ((q[b] >> i) & 1u) << b;
+    return v;
+}
+
+template <int W>
+__global__ void __launch_bounds__(kSweepWarpsV2 * 32)
 sweep_kernel(uint32_t w_rt, uint32_t pmask, uint32_t smask, uint64_t seed, uint64_t first,
              uint64_t n_trials, uint64_t *__restrict__ hist) {
+    const uint32_t w = W ? (uint32_t)W : w_rt;
+    __shared__ uint32_t sh_hist[kMaxBins];
+    __shared__ uint32_t sh_tr[kSweepWarpsV2][32 * 33];
+    const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
+    const uint32_t npat = __popc(pmask), nsch = __popc(smask);
+    const uint32_t nbins = npat * nsch * (w + 1);
+    for (uint32_t b = threadIdx.x; b < nbins; b += blockDim.x) sh_hist[b] = 0;
+    __syncthreads();
+
+    const LaneSel ls(lane);
+    const uint32_t active = (w >= 32) ? kFull : ((1u << w) - 1u);
+    const bool any_random = (pmask >> RAP_PAT_RANDOM) & 1u;
+    const bool need_r = ((smask >> RAP_SCHEME_RAS) & 1u) != 0u;
+    uint32_t *tr = sh_tr[warp];
+
+    const uint64_t nbatch = (n_trials + 31) / 32;
+    const uint64_t stride = (uint64_t)gridDim.x * kSweepWarpsV2;
+    for (uint64_t bt = (uint64_t)blockIdx.x * kSweepWarpsV2 + warp; bt < nbatch; bt += stride) {
+        const uint64_t n0 = first + bt * 32;
+        const uint32_t nvalid = (uint32_t)min((uint64_t)32, n_trials - bt * 32);
+        // ---- lane mode: trial n0 + lane
+        uint32_t pl[5];
+        lane_perm_planes<W>(seed, n0 + lane, w, pl);
+        if (need_r || any_random) {
+#pragma unroll
+            for (int blk = 0; blk < 8; ++blk) {
+                if (!W && 4u * blk >= w) break;
+                const uint4 cr = need_r ? philox_block(seed, n0 + lane, kDomainRAS, blk) : make_uint4(0, 0, 0, 0);
+                const uint4 cc = any_random ? philox_block(seed, n0 + lane, kDomainRandom, blk) : make_uint4(0, 0, 0, 0);
+                const uint32_t ur[4] = {cr.x, cr.y, cr.z, cr.w};
+                const uint32_t uc[4] = {cc.x, cc.y, cc.z, cc.w};
+#pragma unroll
+                for (int i = 0; i < 4; ++i) {
+                    const uint32_t t = 4 * blk + i;
+                    if (W || t < w)
+                        tr[t * 33 + lane] = (mulshift(ur[i], w) << 10) | mulshift(uc[i], w * w);
+                }
+            }
+        }
+        __syncwarp();
+        // ---- warp mode: lane t is DMM thread t of trial n0 + m
+        for (uint32_t m = 0; m < nvalid; ++m) {
+            uint32_t q[5];
+#pragma unroll
+            for (int b = 0; b < 5; ++b) q[b] = __shfl_sync(kFull, pl[b], m);
+            const uint32_t Pt = plane_value(q, lane);          // P[t]
+            const uint32_t P0 = plane_value(q, 0);             // P[0] (uniform)
+            const uint32_t packed = (W || lane < w) ? tr[lane * 33 + m] : 0u;
+            const uint32_t rt = packed >> 10;                  // r[t]
+            const uint32_t r0 = __shfl_sync(kFull, rt, 0);
+            uint32_t rrow = 0, rcol = 0, Pr = 0, rr = 0, leaders = active;
+            if (any_random) {
+                const uint32_t cell = packed & 1023u;
+                if (W == 32) { rrow = cell >> 5; rcol = cell & 31u; }
+                else { rrow = cell / w; rcol = cell - rrow * w; }
+                Pr = plane_value(q, rrow);                     // P[row_t]
+                rr = __shfl_sync(kFull, rt, rrow);             // r[row_t]
+                leaders = first_occurrences(rrow * 32u + rcol, active, lane);
+            }
+            uint32_t mine = 0, e = 0;
+            uint32_t c_stride[5] = {0, 0, 0, 0, 0}, c_diag[5] = {0, 0, 0, 0, 0};
+#pragma unroll
+            for (int p = 0; p < 5; ++p) {
+                if (!((pmask >> p) & 1u)) continue;
+#pragma unroll
+                for (int s = 0; s < 5; ++s) {
+                    if (!((smask >> s) & 1u)) continue;
+                    uint32_t c;
+                    // malicious (reading iii) is the stride set under RAW/RAS and the diagonal
+                    // set under RAP/XOR: the same access, so its evaluation is reused
+                    if (p == RAP_PAT_MALICIOUS && (s == RAP_SCHEME_RAW || s == RAP_SCHEME_RAS) &&
+                        ((pmask >> RAP_PAT_STRIDE) & 1u)) {
+                        c = c_stride[s];
+                    } else if (p == RAP_PAT_MALICIOUS && (s == RAP_SCHEME_RAP || s == RAP_SCHEME_XOR) &&
+                               ((pmask >> RAP_PAT_DIAGONAL) & 1u)) {
+                        c = c_diag[s];
+                    } else {
+                        uint32_t row, col, shP, shR;
+                        switch (p) {
+                        case RAP_PAT_CONTIGUOUS: row = 0; col = lane; shP = P0; shR = r0; break;
+                        case RAP_PAT_STRIDE: row = lane; col = 0; shP = Pt; shR = rt; break;
+                        case RAP_PAT_DIAGONAL: row = lane; col = lane; shP = Pt; shR = rt; break;
+                        case RAP_PAT_RANDOM: row = rrow; col = rcol; shP = Pr; shR = rr; break;
+                        default:
+                            row = lane; shP = Pt; shR = rt;
+                            if (s == RAP_SCHEME_RAW || s == RAP_SCHEME_RAS) col = 0;
+                            else if (s == RAP_SCHEME_PAD) col = (lane == 0) ? 0u : w - lane;
+                            else col = lane;
+                            break;
+                        }
+                        const uint32_t sh = (s == RAP_SCHEME_RAP) ? shP : shR;
+                        const uint32_t bank = bank_of(s, row, col, sh, w);
+                        c = max_bank_load(bank, p == RAP_PAT_RANDOM ? leaders : active, ls);
+                    }
+                    if (p == RAP_PAT_STRIDE) c_stride[s] = c;
+                    if (p == RAP_PAT_DIAGONAL) c_diag[s] = c;
+                    mine = (lane == e) ? c : mine;
+                    ++e;
+                }
+            }
+            if (lane < e) atomicAdd(&sh_hist[lane * (w + 1) + mine], 1u);
+        }
+        __syncwarp();
+    }
+    __syncthreads();
+    for (uint32_t b = threadIdx.x; b < nbins; b += blockDim.x)
+        if (sh_hist[b]) atomicAdd((unsigned long long *)(hist + b), (unsigned long long)sh_hist[b]);
+}
+
+// ------------------------------------------------------------------ C1-C4 sweep (ablation)
+// The north-star sketch, kept as a measured alternative: one warp per trial, Philox blocks
+// spread over lanes, warp Fisher-Yates by __shfl_sync, __match_any_sync histogram.
+template <int W>
+__global__ void __launch_bounds__(kSweepWarps * 32)
+sweep_match_kernel(uint32_t w_rt, uint32_t pmask, uint32_t smask, uint64_t seed, uint64_t first,
+                   uint64_t n_trials, uint64_t *__restrict__ hist) {
     const uint32_t w = W ? (uint32_t)W : w_rt;
     __shared__ uint32_t sh_hist[kSweepWarps][kMaxBins];
     __shared__ __align__(16) uint32_t sh_words[kSweepWarps][4 * 32];
@@ -112,7 +328,6 @@ sweep_kernel(uint32_t w_rt, uint32_t pmask, uint32_t smask, uint64_t seed, uint6
     const uint64_t stride = (uint64_t)gridDim.x * kSweepWarps;
     for (uint64_t i = (uint64_t)blockIdx.x * kSweepWarps + warp; i < n_trials; i += stride) {
         const uint64_t n = first + i;
-        // C1: lane L computes Philox block (L & 7) of domain (L >> 3): 24 useful blocks
         const uint4 blk = philox_block(seed, n, lane >> 3, lane & 7u);
         *reinterpret_cast<uint4 *>(&sh_words[warp][4 * lane]) = blk;   // word(d,t) at [32d + t]
         __syncwarp();
@@ -120,7 +335,6 @@ sweep_kernel(uint32_t w_rt, uint32_t pmask, uint32_t smask, uint64_t seed, uint6
         const uint32_t u_ras = sh_words[warp][32 + lane];
         const uint32_t u_rnd = sh_words[warp][64 + lane];
         __syncwarp();
-        // C2: warp Fisher-Yates; RAS shifts; random cells
         const uint32_t P = warp_fisher_yates<W>(u_fy, lane, w);
         const uint32_t r = mulshift(u_ras, w);
         uint32_t rrow = 0, rcol = 0;
@@ -129,7 +343,6 @@ sweep_kernel(uint32_t w_rt, uint32_t pmask, uint32_t smask, uint64_t seed, uint6
             if (W == 32) { rrow = cell >> 5; rcol = cell & 31u; }
             else { rrow = cell / w; rcol = cell - rrow * w; }
         }
-        // C3: every selected (pattern, scheme); lane e keeps evaluation e's congestion
         uint32_t mine = 0, e = 0;
 #pragma unroll
         for (int p = 0; p < 5; ++p) {
@@ -139,12 +352,11 @@ sweep_kernel(uint32_t w_rt, uint32_t pmask, uint32_t smask, uint64_t seed, uint6
                 if (!((smask >> s) & 1u)) continue;
                 uint32_t row, col;
                 pattern_cell(p, s, lane, w, rrow, rcol, row, col);
-                const uint32_t c = warp_congestion<W>(row, col, s, P, r, lane, w, p == RAP_PAT_RANDOM);
+                const uint32_t c = warp_congestion_match<W>(row, col, s, P, r, lane, w, p == RAP_PAT_RANDOM);
                 mine = (lane == e) ? c : mine;
                 ++e;
             }
         }
-        // C4: count
         if (lane < e) sh_hist[warp][lane * (w + 1) + mine] += 1;
     }
     flush_hist(sh_hist, kSweepWarps, nbins, hist);
@@ -162,6 +374,7 @@ trace_kernel(uint32_t w, uint64_t n_warps, const uint32_t *__restrict__ cells, u
     const uint32_t nbins = nsch * (w + 1);
     for (uint32_t b = lane; b < nbins; b += 32) sh_hist[warp][b] = 0;
     __syncwarp();
+    const LaneSel ls(lane);
     const bool need_p = (smask >> RAP_SCHEME_RAP) & 1u, need_r = (smask >> RAP_SCHEME_RAS) & 1u;
     const uint64_t nchunks = (n_warps + kTraceChunk - 1) / kTraceChunk;
     const uint64_t nitems = n_trials * nchunks;
@@ -181,7 +394,7 @@ trace_kernel(uint32_t w, uint64_t n_warps, const uint32_t *__restrict__ cells, u
 #pragma unroll
             for (int s = 0; s < 5; ++s) {
                 if (!((smask >> s) & 1u)) continue;
-                const uint32_t c = warp_congestion<0>(row, col, s, P, r, lane, w, true);
+                const uint32_t c = warp_congestion(row, col, s, P, r, lane, w, ls);
                 mine = (lane == e) ? (bad ? 0u : c) : mine;
                 ++e;
             }
@@ -197,6 +410,7 @@ congestion_kernel(uint32_t w, uint64_t n_warps, const uint32_t *__restrict__ row
                   const uint32_t *__restrict__ cols, int scheme, const uint32_t *__restrict__ shift,
                   uint32_t *__restrict__ out) {
     const uint32_t lane = threadIdx.x & 31u;
+    const LaneSel ls(lane);
     const uint64_t stride = (uint64_t)gridDim.x * (blockDim.x >> 5);
     for (uint64_t k = (uint64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); k < n_warps;
          k += stride) {
@@ -205,9 +419,9 @@ congestion_kernel(uint32_t w, uint64_t n_warps, const uint32_t *__restrict__ row
         const uint32_t col = active ? cols[k * w + lane] : 0u;
         const uint32_t sh = (active && shift) ? shift[k * w + lane] : 0u;
         const bool bad = active && (row >= w || col >= w || sh >= w);
-        const uint32_t c = warp_congestion<0>(active ? row % w : 0u, active ? col % w : 0u, scheme,
-                                              sh % w, sh % w, lane, w, true);
         const bool any_bad = __any_sync(kFull, bad);
+        const uint32_t c = warp_congestion(any_bad ? 0u : row, any_bad ? 0u : col, scheme,
+                                           any_bad ? 0u : sh, any_bad ? 0u : sh, lane, w, ls);
         if (lane == 0) out[k] = any_bad ? 0u : c;
     }
 }
@@ -244,28 +458,34 @@ static int clamp_grid(uint64_t items, int per_cta, int cap) {
     return (int)(want < (uint64_t)cap ? (want ? want : 1) : (uint64_t)cap);
 }
 
+template <typename K>
+static void run_sweep(K kernel, int warps_per_cta, uint64_t trials_per_item, uint32_t w, uint32_t pmask,
+                      uint32_t smask, uint64_t seed, uint64_t first, uint64_t n_trials, uint64_t *hist,
+                      cudaStream_t st) {
+    const int threads = warps_per_cta * 32;
+    const uint64_t items = (n_trials + trials_per_item - 1) / trials_per_item;
+    const int grid = clamp_grid(items, warps_per_cta, resident_ctas(kernel, threads));
+    // u32 shared counters: keep the trials counted by one CTA below 2^31 per launch
+    const uint64_t chunk = (uint64_t)grid * (1ull << 31);
+    for (uint64_t done = 0; done < n_trials; done += chunk) {
+        const uint64_t cnt = (n_trials - done < chunk) ? n_trials - done : chunk;
+        kernel<<<grid, threads, 0, st>>>(w, pmask, smask, seed, first + done, cnt, hist);
+    }
+}
+
 cudaError_t launch_sweep(uint32_t w, uint32_t pmask, uint32_t smask, uint64_t seed, uint64_t first,
                          uint64_t n_trials, uint64_t *hist, cudaStream_t st) {
     if (n_trials == 0) return cudaSuccess;
-    const int threads = kSweepWarps * 32;
-    if (w == 32) {
-        auto k = sweep_kernel<32>;
-        const int grid = clamp_grid(n_trials, kSweepWarps, resident_ctas(k, threads));
-        // per-warp u32 counters: keep trials per warp below 2^31 by chunking the range
-        const uint64_t chunk = (uint64_t)grid * kSweepWarps * (1ull << 31);
-        for (uint64_t done = 0; done < n_trials; done += chunk) {
-            const uint64_t cnt = (n_trials - done < chunk) ? n_trials - done : chunk;
-            k<<<grid, threads, 0, st>>>(w, pmask, smask, seed, first + done, cnt, hist);
-        }
-    } else {
-        auto k = sweep_kernel<0>;
-        const int grid = clamp_grid(n_trials, kSweepWarps, resident_ctas(k, threads));
-        const uint64_t chunk = (uint64_t)grid * kSweepWarps * (1ull << 31);
-        for (uint64_t done = 0; done < n_trials; done += chunk) {
-            const uint64_t cnt = (n_trials - done < chunk) ? n_trials - done : chunk;
-            k<<<grid, threads, 0, st>>>(w, pmask, smask, seed, first + done, cnt, hist);
-        }
-    }
+    if (w == 32) run_sweep(sweep_kernel<32>, kSweepWarpsV2, 32, w, pmask, smask, seed, first, n_trials, hist, st);
+    else run_sweep(sweep_kernel<0>, kSweepWarpsV2, 32, w, pmask, smask, seed, first, n_trials, hist, st);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_sweep_match(uint32_t w, uint32_t pmask, uint32_t smask, uint64_t seed, uint64_t first,
+                               uint64_t n_trials, uint64_t *hist, cudaStream_t st) {
+    if (n_trials == 0) return cudaSuccess;
+    if (w == 32) run_sweep(sweep_match_kernel<32>, kSweepWarps, 1, w, pmask, smask, seed, first, n_trials, hist, st);
+    else run_sweep(sweep_match_kernel<0>, kSweepWarps, 1, w, pmask, smask, seed, first, n_trials, hist, st);
     return cudaGetLastError();
 }
 

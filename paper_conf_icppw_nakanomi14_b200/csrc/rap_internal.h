@@ -8,6 +8,19 @@
 
 namespace rapk {
 
+// Launch-shape knobs of the transpose (defaults chosen by tools/tune_transpose.cu on B200).
+struct TransposeTuning {
+    uint32_t group = 0;   // tile-rows per traversal group (0 = row-major tile order)
+    int minb = 2;         // __launch_bounds__ min blocks per SM (register budget)
+};
+constexpr uint32_t kDefaultGroup32 = 0, kDefaultGroup64 = 0;
+constexpr int kDefaultMinB32 = 1, kDefaultMinB64 = 1;
+TransposeTuning default_tuning(uint32_t elem_bytes);
+
+cudaError_t launch_transpose_tuned(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
+                                   int64_t ld_dst, uint32_t elem_bytes, int layout, uint64_t seed,
+                                   const TransposeTuning &tu, cudaStream_t st);
+
 cudaError_t launch_transpose(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
                              int64_t ld_dst, uint32_t elem_bytes, int layout, uint64_t seed,
                              cudaStream_t st);
@@ -20,6 +33,9 @@ cudaError_t launch_congestion(uint32_t w, uint64_t n_warps, const uint32_t *rows
 
 cudaError_t launch_sweep(uint32_t w, uint32_t pattern_mask, uint32_t scheme_mask, uint64_t seed,
                          uint64_t first, uint64_t n_trials, uint64_t *hist, cudaStream_t st);
+
+cudaError_t launch_sweep_match(uint32_t w, uint32_t pattern_mask, uint32_t scheme_mask, uint64_t seed,
+                               uint64_t first, uint64_t n_trials, uint64_t *hist, cudaStream_t st);
 
 cudaError_t launch_trace(uint32_t w, uint64_t n_warps, const uint32_t *cells, uint32_t scheme_mask,
                          uint64_t seed, uint64_t first, uint64_t n_trials, uint64_t *hist,

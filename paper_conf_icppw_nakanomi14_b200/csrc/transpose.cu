@@ -78,14 +78,33 @@ __device__ __forceinline__ void tile_rows(uint32_t *scratch, uint64_t seed, uint
     }
 }
 
+// Tile t -> (ti, tj).  Tiles are walked in groups of `group` tile-rows, column by column
+// inside a group, so the ~#warps tiles in flight at any moment form a roughly square block:
+// both the input rows they read and the output rows they write are long contiguous runs
+// (DRAM page locality on both sides).  group == 0: plain row-major tile order.
+__device__ __forceinline__ void tile_coords(uint32_t t, uint32_t tiles_r, uint32_t tiles_c, uint32_t group,
+                                            uint32_t &ti, uint32_t &tj) {
+    if (group == 0) {
+        ti = t / tiles_c;
+        tj = t - ti * tiles_c;
+        return;
+    }
+    const uint32_t per = group * tiles_c;
+    const uint32_t g = t / per, rem = t - g * per;
+    const uint32_t base = g * group;
+    const uint32_t nrows = min(group, tiles_r - base);
+    tj = rem / nrows;
+    ti = base + (rem - tj * nrows);
+}
+
 // ------------------------------------------------------------------ 32-bit elements
 constexpr int kWarps32 = 8;
 
-template <int L, bool VEC>
-__global__ void __launch_bounds__(kWarps32 * 32)
+template <int L, bool VEC, int MINB>
+__global__ void __launch_bounds__(kWarps32 * 32, MINB)
 transpose_b32_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, int64_t rows,
-                     int64_t cols, int64_t ld_src, int64_t ld_dst, uint64_t seed, int64_t tiles_c,
-                     int64_t ntiles) {
+                     int64_t cols, int64_t ld_src, int64_t ld_dst, uint64_t seed, uint32_t tiles_r,
+                     uint32_t tiles_c, uint32_t ntiles, uint32_t group) {
     constexpr int S = Tile<L>::S;
     __shared__ __align__(16) uint32_t smem[kWarps32][32 * S];
     const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
@@ -95,13 +114,14 @@ transpose_b32_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ ds
     tile_rows<L, 8>(tile, seed, lane, sh_lane, row_g, sh_g);
     const uint32_t q = lane & 7u;              // 16-byte chunk of the row
 
-    const int64_t stride = (int64_t)gridDim.x * kWarps32;
-    int64_t t = (int64_t)blockIdx.x * kWarps32 + warp;
+    const uint32_t stride = gridDim.x * kWarps32;
+    uint32_t t = blockIdx.x * kWarps32 + warp;
     uint4 v[8];
 
-    auto load = [&](int64_t tt) {
-        const int64_t ti = tt / tiles_c, tj = tt - ti * tiles_c;
-        const int64_t r0 = ti * 32, c0 = tj * 32;
+    auto load = [&](uint32_t tt) {
+        uint32_t ti, tj;
+        tile_coords(tt, tiles_r, tiles_c, group, ti, tj);
+        const int64_t r0 = (int64_t)ti * 32, c0 = (int64_t)tj * 32;
         const bool full = (r0 + 32 <= rows) && (c0 + 32 <= cols);
         if (VEC && full) {
 #pragma unroll
@@ -134,13 +154,14 @@ transpose_b32_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ ds
             rowp[phys_col<L>(row_g[g], 4 * q + 3, sh_g[g])] = v[g].w;
         }
         __syncwarp();
-        const int64_t cur = t;
+        const uint32_t cur = t;
         t += stride;
         if (t < ntiles) load(t);               // T3: next tile in flight while draining
 
         // T2: stride (column-wise) read of the tile, coalesced row writes of the output
-        const int64_t ti = cur / tiles_c, tj = cur - ti * tiles_c;
-        const int64_t r0 = ti * 32, c0 = tj * 32;
+        uint32_t ti, tj;
+        tile_coords(cur, tiles_r, tiles_c, group, ti, tj);
+        const int64_t r0 = (int64_t)ti * 32, c0 = (int64_t)tj * 32;
         const uint32_t *myrow = tile + lane * S;
         uint32_t *out = dst + c0 * ld_dst + r0 + lane;
         if ((r0 + 32 <= rows) && (c0 + 32 <= cols)) {
@@ -160,11 +181,11 @@ transpose_b32_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ ds
 // ------------------------------------------------------------------ 64-bit elements
 constexpr int kWarps64 = 4;
 
-template <int L, bool VEC>
-__global__ void __launch_bounds__(kWarps64 * 32)
+template <int L, bool VEC, int MINB>
+__global__ void __launch_bounds__(kWarps64 * 32, MINB)
 transpose_b64_kernel(const uint64_t *__restrict__ src, uint64_t *__restrict__ dst, int64_t rows,
-                     int64_t cols, int64_t ld_src, int64_t ld_dst, uint64_t seed, int64_t tiles_c,
-                     int64_t ntiles) {
+                     int64_t cols, int64_t ld_src, int64_t ld_dst, uint64_t seed, uint32_t tiles_r,
+                     uint32_t tiles_c, uint32_t ntiles, uint32_t group) {
     constexpr int S = Tile<L>::S;
     __shared__ __align__(16) uint32_t smem[kWarps64][2][32 * S];   // [warp][lo/hi plane]
     const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
@@ -175,13 +196,14 @@ transpose_b64_kernel(const uint64_t *__restrict__ src, uint64_t *__restrict__ ds
     tile_rows<L, 16>(lo_plane, seed, lane, sh_lane, row_g, sh_g);
     const uint32_t q = lane & 15u;             // 16-byte chunk = elements 2q, 2q+1
 
-    const int64_t stride = (int64_t)gridDim.x * kWarps64;
-    int64_t t = (int64_t)blockIdx.x * kWarps64 + warp;
+    const uint32_t stride = gridDim.x * kWarps64;
+    uint32_t t = blockIdx.x * kWarps64 + warp;
     uint4 v[16];
 
-    auto load = [&](int64_t tt) {
-        const int64_t ti = tt / tiles_c, tj = tt - ti * tiles_c;
-        const int64_t r0 = ti * 32, c0 = tj * 32;
+    auto load = [&](uint32_t tt) {
+        uint32_t ti, tj;
+        tile_coords(tt, tiles_r, tiles_c, group, ti, tj);
+        const int64_t r0 = (int64_t)ti * 32, c0 = (int64_t)tj * 32;
         const bool full = (r0 + 32 <= rows) && (c0 + 32 <= cols);
         if (VEC && full) {
 #pragma unroll
@@ -213,12 +235,13 @@ transpose_b64_kernel(const uint64_t *__restrict__ src, uint64_t *__restrict__ ds
             hi_plane[p1] = v[g].w;
         }
         __syncwarp();
-        const int64_t cur = t;
+        const uint32_t cur = t;
         t += stride;
         if (t < ntiles) load(t);
 
-        const int64_t ti = cur / tiles_c, tj = cur - ti * tiles_c;
-        const int64_t r0 = ti * 32, c0 = tj * 32;
+        uint32_t ti, tj;
+        tile_coords(cur, tiles_r, tiles_c, group, ti, tj);
+        const int64_t r0 = (int64_t)ti * 32, c0 = (int64_t)tj * 32;
         const uint32_t *mylo = lo_plane + lane * S;
         const uint32_t *myhi = hi_plane + lane * S;
         uint64_t *out = dst + c0 * ld_dst + r0 + lane;
@@ -256,37 +279,63 @@ static int grid_for(K kernel, int threads, int64_t ntiles, int warps_per_cta) {
     return (int)(want < cap ? want : cap);
 }
 
-template <int L, bool VEC>
+TransposeTuning default_tuning(uint32_t elem_bytes) {
+    TransposeTuning t;
+    t.group = elem_bytes == 4 ? kDefaultGroup32 : kDefaultGroup64;
+    t.minb = elem_bytes == 4 ? kDefaultMinB32 : kDefaultMinB64;
+    return t;
+}
+
+template <int L, bool VEC, int MINB>
 static cudaError_t launch_b32(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
-                              int64_t ld_dst, uint64_t seed, cudaStream_t st) {
-    const int64_t tiles_r = (rows + 31) / 32, tiles_c = (cols + 31) / 32;
-    const int64_t ntiles = tiles_r * tiles_c;
-    auto k = transpose_b32_kernel<L, VEC>;
+                              int64_t ld_dst, uint64_t seed, uint32_t group, cudaStream_t st) {
+    const uint32_t tiles_r = (uint32_t)((rows + 31) / 32), tiles_c = (uint32_t)((cols + 31) / 32);
+    const uint32_t ntiles = tiles_r * tiles_c;
+    auto k = transpose_b32_kernel<L, VEC, MINB>;
     const int grid = grid_for(k, kWarps32 * 32, ntiles, kWarps32);
     k<<<grid, kWarps32 * 32, 0, st>>>((const uint32_t *)src, (uint32_t *)dst, rows, cols, ld_src,
-                                      ld_dst, seed, tiles_c, ntiles);
+                                      ld_dst, seed, tiles_r, tiles_c, ntiles, group);
+    return cudaGetLastError();
+}
+
+template <int L, bool VEC, int MINB>
+static cudaError_t launch_b64(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
+                              int64_t ld_dst, uint64_t seed, uint32_t group, cudaStream_t st) {
+    const uint32_t tiles_r = (uint32_t)((rows + 31) / 32), tiles_c = (uint32_t)((cols + 31) / 32);
+    const uint32_t ntiles = tiles_r * tiles_c;
+    auto k = transpose_b64_kernel<L, VEC, MINB>;
+    const int grid = grid_for(k, kWarps64 * 32, ntiles, kWarps64);
+    k<<<grid, kWarps64 * 32, 0, st>>>((const uint64_t *)src, (uint64_t *)dst, rows, cols, ld_src,
+                                      ld_dst, seed, tiles_r, tiles_c, ntiles, group);
     return cudaGetLastError();
 }
 
 template <int L, bool VEC>
-static cudaError_t launch_b64(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
-                              int64_t ld_dst, uint64_t seed, cudaStream_t st) {
-    const int64_t tiles_r = (rows + 31) / 32, tiles_c = (cols + 31) / 32;
-    const int64_t ntiles = tiles_r * tiles_c;
-    auto k = transpose_b64_kernel<L, VEC>;
-    const int grid = grid_for(k, kWarps64 * 32, ntiles, kWarps64);
-    k<<<grid, kWarps64 * 32, 0, st>>>((const uint64_t *)src, (uint64_t *)dst, rows, cols, ld_src,
-                                      ld_dst, seed, tiles_c, ntiles);
-    return cudaGetLastError();
+static cudaError_t launch_minb(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
+                               int64_t ld_dst, uint32_t eb, uint64_t seed, const TransposeTuning &tu,
+                               cudaStream_t st) {
+    if (eb == 4) {
+        switch (tu.minb) {
+        case 1: return launch_b32<L, VEC, 1>(src, dst, rows, cols, ld_src, ld_dst, seed, tu.group, st);
+        case 3: return launch_b32<L, VEC, 3>(src, dst, rows, cols, ld_src, ld_dst, seed, tu.group, st);
+        case 4: return launch_b32<L, VEC, 4>(src, dst, rows, cols, ld_src, ld_dst, seed, tu.group, st);
+        default: return launch_b32<L, VEC, 2>(src, dst, rows, cols, ld_src, ld_dst, seed, tu.group, st);
+        }
+    }
+    switch (tu.minb) {
+    case 1: return launch_b64<L, VEC, 1>(src, dst, rows, cols, ld_src, ld_dst, seed, tu.group, st);
+    case 3: return launch_b64<L, VEC, 3>(src, dst, rows, cols, ld_src, ld_dst, seed, tu.group, st);
+    case 4: return launch_b64<L, VEC, 4>(src, dst, rows, cols, ld_src, ld_dst, seed, tu.group, st);
+    default: return launch_b64<L, VEC, 2>(src, dst, rows, cols, ld_src, ld_dst, seed, tu.group, st);
+    }
 }
 
 template <bool VEC>
 static cudaError_t dispatch(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
-                            int64_t ld_dst, uint32_t eb, int layout, uint64_t seed, cudaStream_t st) {
-#define RAPK_CASE(LAY)                                                                           \
-    case LAY:                                                                                    \
-        return eb == 4 ? launch_b32<LAY, VEC>(src, dst, rows, cols, ld_src, ld_dst, seed, st)    \
-                       : launch_b64<LAY, VEC>(src, dst, rows, cols, ld_src, ld_dst, seed, st);
+                            int64_t ld_dst, uint32_t eb, int layout, uint64_t seed,
+                            const TransposeTuning &tu, cudaStream_t st) {
+#define RAPK_CASE(LAY) \
+    case LAY: return launch_minb<LAY, VEC>(src, dst, rows, cols, ld_src, ld_dst, eb, seed, tu, st);
     switch (layout) {
         RAPK_CASE(RAP_LAYOUT_RAW)
         RAPK_CASE(RAP_LAYOUT_PAD)
@@ -298,12 +347,19 @@ static cudaError_t dispatch(const void *src, void *dst, int64_t rows, int64_t co
     return cudaErrorInvalidValue;
 }
 
+cudaError_t launch_transpose_tuned(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
+                                   int64_t ld_dst, uint32_t elem_bytes, int layout, uint64_t seed,
+                                   const TransposeTuning &tu, cudaStream_t st) {
+    const bool vec = ((uintptr_t)src % 16 == 0) && ((ld_src * elem_bytes) % 16 == 0);
+    return vec ? dispatch<true>(src, dst, rows, cols, ld_src, ld_dst, elem_bytes, layout, seed, tu, st)
+               : dispatch<false>(src, dst, rows, cols, ld_src, ld_dst, elem_bytes, layout, seed, tu, st);
+}
+
 cudaError_t launch_transpose(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
                              int64_t ld_dst, uint32_t elem_bytes, int layout, uint64_t seed,
                              cudaStream_t st) {
-    const bool vec = ((uintptr_t)src % 16 == 0) && ((ld_src * elem_bytes) % 16 == 0);
-    return vec ? dispatch<true>(src, dst, rows, cols, ld_src, ld_dst, elem_bytes, layout, seed, st)
-               : dispatch<false>(src, dst, rows, cols, ld_src, ld_dst, elem_bytes, layout, seed, st);
+    return launch_transpose_tuned(src, dst, rows, cols, ld_src, ld_dst, elem_bytes, layout, seed,
+                                  default_tuning(elem_bytes), st);
 }
 
 }  // namespace rapk

@@ -82,6 +82,11 @@ def test_sweep_validation(L):
     assert L.rap_congestion_sweep(24, 31, 16, 1, 0, 10, h, s) == INVALID  # XOR needs 2^k
     assert L.rap_congestion_sweep(32, 31, 7, 1, 0, 10, P(0), s) == INVALID
     assert L.rap_congestion_sweep(32, 31, 7, 1, 0, 0, P(0), s) == OK      # no trials: no-op
+    L.rap_congestion_sweep_algo.argtypes = [ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32,
+                                            ctypes.c_uint64, ctypes.c_uint64, ctypes.c_uint64,
+                                            ctypes.c_void_p, ctypes.c_uint32, ctypes.c_void_p]
+    assert L.rap_congestion_sweep_algo(32, 31, 7, 1, 0, 10, h, 2, s) == INVALID   # unknown algo
+    assert L.rap_congestion_sweep_algo(32, 31, 7, 1, 0, 0, h, 1, s) == OK
 
 
 def test_congestion_trace_perm_validation(L):

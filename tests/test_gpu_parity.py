@@ -175,13 +175,25 @@ def test_sweep_bit_exact_w32(rap, oracle, seed):
     assert np.array_equal(g.cpu().numpy().astype(np.uint64), o)
 
 
-@pytest.mark.parametrize("w", [2, 3, 7, 16, 31])
-def test_sweep_bit_exact_other_w(rap, oracle, w):
-    N = 100_000
+@pytest.mark.parametrize("algo", ["default", "match"])
+@pytest.mark.parametrize("w", [2, 3, 7, 16, 31, 32])
+def test_sweep_bit_exact_other_w(rap, oracle, w, algo):
+    N = 100_003
     sch = ["raw", "ras", "rap", "pad"] + (["xor"] if w & (w - 1) == 0 else [])
-    g = rap.congestion_sweep(N, seed=5, w=w, patterns=ALL_PAT, schemes=sch, first_trial=2 ** 33 + 17)
+    g = rap.congestion_sweep(N, seed=5, w=w, patterns=ALL_PAT, schemes=sch, first_trial=2 ** 33 + 17,
+                             algo=algo)
     o = oracle.sweep(w, ALL_PAT, sch, 5, 2 ** 33 + 17, N)
     assert np.array_equal(g.cpu().numpy().astype(np.uint64), o)
+
+
+def test_sweep_algos_agree_tiny_ranges(rap, oracle):
+    # ragged batches: n_trials not a multiple of 32, single trials, odd first_trial
+    for first, n in ((0, 1), (5, 31), (31, 33), (1000, 65), (2 ** 40 + 3, 97)):
+        a = rap.congestion_sweep(n, seed=12, first_trial=first, algo="default")
+        b = rap.congestion_sweep(n, seed=12, first_trial=first, algo="match")
+        o = oracle.sweep(32, ALL_PAT, ["raw", "ras", "rap"], 12, first, n)
+        assert torch.equal(a, b)
+        assert np.array_equal(a.cpu().numpy().astype(np.uint64), o)
 
 
 def test_sweep_masks_and_chunks(rap, oracle):
