@@ -28,17 +28,30 @@
 
 namespace rapk {
 
+// Shared-memory geometry of one warp's 32 x 32 tile, in 4-byte words.
+//   RP   : row pitch.  RAP / RAS rows are 64 words wide: element (i, j) sits at word
+//          i*64 + j + sh[i] -- the rotation is NOT wrapped in the address, the bank decoder
+//          (address mod 32) performs the "mod w" of the paper, so bank(i, j) = (j + P[i]) mod 32
+//          exactly as in P:L1005-1016 while every access is base + immediate.
+//          RAW / XOR: 32 words; PAD: 33 words (the [32][33] baseline).
+//   EW   : 4-byte words per element (1: 32-bit, 2: 64-bit split into lo / hi planes, each a
+//          full 32 x RP array, so both planes see the 32-bit bank function).
 template <int L>
-struct Tile {
-    static constexpr int S = (L == RAP_LAYOUT_PAD) ? 33 : 32;   // row pitch in 4-byte words
+struct Geom {
+    static constexpr int RP = (L == RAP_LAYOUT_RAP || L == RAP_LAYOUT_RAS) ? 64
+                            : (L == RAP_LAYOUT_PAD) ? 33 : 32;
 };
 
-// physical column of logical element (row, col) of the tile; sh = shift of that row
+template <int L, int EW>
+__host__ __device__ constexpr int warp_smem_words() { return 32 * Geom<L>::RP * EW; }
+
+// word offset of logical element (row, col) inside a plane; sh = shift of that row
 template <int L>
-__device__ __forceinline__ uint32_t phys_col(uint32_t row, uint32_t col, uint32_t sh) {
-    if (L == RAP_LAYOUT_XOR) return col ^ row;
-    if (L == RAP_LAYOUT_RAS || L == RAP_LAYOUT_RAP) return (col + sh) & 31u;
-    return col;
+__device__ __forceinline__ uint32_t word_of(uint32_t row, uint32_t col, uint32_t sh) {
+    constexpr int RP = Geom<L>::RP;
+    if (L == RAP_LAYOUT_XOR) return row * RP + (col ^ row);
+    if (L == RAP_LAYOUT_RAS || L == RAP_LAYOUT_RAP) return row * RP + col + sh;
+    return row * RP + col;
 }
 
 __device__ __forceinline__ uint4 ldg_stream128(const void *p) {
@@ -48,40 +61,8 @@ __device__ __forceinline__ uint4 ldg_stream128(const void *p) {
     return r;
 }
 
-// Per-warp prologue shared by the 32- and 64-bit kernels: sh_lane = shift of tile row `lane`
-// (P[lane] for RAP, r[lane] for RAS), and for load group g of G groups of R = 32/G rows the
-// row this lane loads and that row's shift.
-template <int L, int G>
-__device__ __forceinline__ void tile_rows(uint32_t *scratch, uint64_t seed, uint32_t lane,
-                                          uint32_t &sh_lane, uint32_t (&row_g)[G], uint32_t (&sh_g)[G]) {
-    constexpr int R = 32 / G;                  // rows covered by one load instruction
-    const uint32_t c = lane / (32 / R);        // which of the R rows this lane loads
-    sh_lane = 0;
-    if (L == RAP_LAYOUT_RAP) sh_lane = warp_perm<32>(seed, 0, lane, 32);
-    if (L == RAP_LAYOUT_RAS) sh_lane = warp_ras_shift(seed, 0, lane, 32);
-    if (L == RAP_LAYOUT_RAP) {
-        scratch[sh_lane] = lane;               // P^-1 through shared memory
-        __syncwarp();
-        const uint32_t pinv = scratch[lane];
-        __syncwarp();
-#pragma unroll
-        for (int g = 0; g < G; ++g) {
-            row_g[g] = __shfl_sync(kFull, pinv, R * g + c);   // P[row_g] = R*g + c
-            sh_g[g] = R * g + c;
-        }
-    } else {
-#pragma unroll
-        for (int g = 0; g < G; ++g) {
-            row_g[g] = R * g + c;
-            sh_g[g] = __shfl_sync(kFull, sh_lane, R * g + c);
-        }
-    }
-}
-
 // Tile t -> (ti, tj).  Tiles are walked in groups of `group` tile-rows, column by column
-// inside a group, so the ~#warps tiles in flight at any moment form a roughly square block:
-// both the input rows they read and the output rows they write are long contiguous runs
-// (DRAM page locality on both sides).  group == 0: plain row-major tile order.
+// inside a group (group == 0: plain row-major tile order).
 __device__ __forceinline__ void tile_coords(uint32_t t, uint32_t tiles_r, uint32_t tiles_c, uint32_t group,
                                             uint32_t &ti, uint32_t &tj) {
     if (group == 0) {
@@ -97,183 +78,172 @@ __device__ __forceinline__ void tile_coords(uint32_t t, uint32_t tiles_r, uint32
     ti = base + (rem - tj * nrows);
 }
 
-// ------------------------------------------------------------------ 32-bit elements
-constexpr int kWarps32 = 8;
+// Load geometry: a 128-bit load carries NE = 4/EW elements, LPR = 32/NE lanes cover one tile
+// row, so one warp instruction loads R = 32/LPR rows and a tile takes G = 32/R instructions.
+template <int L, int EW>
+struct TileCfg {
+    static constexpr int NE = 4 / EW;               // elements per 16-byte chunk
+    static constexpr int LPR = 32 / NE;             // lanes per tile row (8 or 16)
+    static constexpr int R = 32 / LPR;              // tile rows per load instruction (4 or 2)
+    static constexpr int G = 32 / R;                // load instructions per tile (8 or 16)
+};
 
-template <int L, bool VEC, int MINB>
-__global__ void __launch_bounds__(kWarps32 * 32, MINB)
-transpose_b32_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, int64_t rows,
-                     int64_t cols, int64_t ld_src, int64_t ld_dst, uint64_t seed, uint32_t tiles_r,
-                     uint32_t tiles_c, uint32_t ntiles, uint32_t group) {
-    constexpr int S = Tile<L>::S;
-    __shared__ __align__(16) uint32_t smem[kWarps32][32 * S];
+constexpr int kWarpsT = 4;                          // warps per CTA
+
+template <int L, int EW, bool VEC, int DEPTH, int MINB>
+__global__ void __launch_bounds__(kWarpsT * 32, MINB)
+transpose_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, int64_t rows,
+                 int64_t cols, int64_t ld_src, int64_t ld_dst, uint64_t seed, uint32_t tiles_r,
+                 uint32_t tiles_c, uint32_t ntiles, uint32_t group) {
+    using C = TileCfg<L, EW>;
+    constexpr int NE = C::NE, R = C::R, G = C::G, LPR = C::LPR;
+    constexpr int PW = 32 * Geom<L>::RP;            // plane size in words
+    extern __shared__ __align__(16) uint32_t smem_dyn[];
     const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
-    uint32_t *tile = smem[warp];
+    uint32_t *tile = smem_dyn + warp * warp_smem_words<L, EW>();
 
-    uint32_t sh_lane, row_g[8], sh_g[8];
-    tile_rows<L, 8>(tile, seed, lane, sh_lane, row_g, sh_g);
-    const uint32_t q = lane & 7u;              // 16-byte chunk of the row
-
-    const uint32_t stride = gridDim.x * kWarps32;
-    uint32_t t = blockIdx.x * kWarps32 + warp;
-    uint4 v[8];
-
-    auto load = [&](uint32_t tt) {
-        uint32_t ti, tj;
-        tile_coords(tt, tiles_r, tiles_c, group, ti, tj);
-        const int64_t r0 = (int64_t)ti * 32, c0 = (int64_t)tj * 32;
-        const bool full = (r0 + 32 <= rows) && (c0 + 32 <= cols);
-        if (VEC && full) {
-#pragma unroll
-            for (int g = 0; g < 8; ++g)
-                v[g] = ldg_stream128(src + (r0 + row_g[g]) * ld_src + c0 + 4 * q);
-        } else {
-#pragma unroll
-            for (int g = 0; g < 8; ++g) {
-                const int64_t r = r0 + row_g[g];
-                const uint32_t *p = src + r * ld_src + c0 + 4 * q;
-                const bool rok = r < rows;
-                const int64_t cc = c0 + 4 * q;
-                v[g].x = (rok && cc + 0 < cols) ? __ldg(p + 0) : 0u;
-                v[g].y = (rok && cc + 1 < cols) ? __ldg(p + 1) : 0u;
-                v[g].z = (rok && cc + 2 < cols) ? __ldg(p + 2) : 0u;
-                v[g].w = (rok && cc + 3 < cols) ? __ldg(p + 3) : 0u;
-            }
-        }
-    };
-
-    if (t < ntiles) load(t);
-    while (t < ntiles) {
-        // T1: contiguous (row-wise) write of the tile into shared memory
-#pragma unroll
-        for (int g = 0; g < 8; ++g) {
-            uint32_t *rowp = tile + row_g[g] * S;
-            rowp[phys_col<L>(row_g[g], 4 * q + 0, sh_g[g])] = v[g].x;
-            rowp[phys_col<L>(row_g[g], 4 * q + 1, sh_g[g])] = v[g].y;
-            rowp[phys_col<L>(row_g[g], 4 * q + 2, sh_g[g])] = v[g].z;
-            rowp[phys_col<L>(row_g[g], 4 * q + 3, sh_g[g])] = v[g].w;
-        }
+    // ---- T0: the per-warp shift vector, lane i holds sh[i] (P[i] for RAP, r[i] for RAS)
+    uint32_t sh_lane = 0;
+    if (L == RAP_LAYOUT_RAP) sh_lane = warp_perm<32>(seed, 0, lane, 32);
+    if (L == RAP_LAYOUT_RAS) sh_lane = warp_ras_shift(seed, 0, lane, 32);
+    // load group g: this lane loads tile row row_g[g], chunk q (elements NE*q .. NE*q+NE-1).
+    // RAP: the R rows of group g are P^-1(R*g + 0..R-1) -- one row per residue of P mod R --
+    // so each STS of the group hits 32 distinct banks.
+    const uint32_t q = lane % LPR, c_in = lane / LPR;
+    uint32_t row_g[G], a_g[G];
+    uint32_t pinv = lane;
+    if (L == RAP_LAYOUT_RAP) {
+        tile[sh_lane] = lane;
         __syncwarp();
-        const uint32_t cur = t;
-        t += stride;
-        if (t < ntiles) load(t);               // T3: next tile in flight while draining
-
-        // T2: stride (column-wise) read of the tile, coalesced row writes of the output
-        uint32_t ti, tj;
-        tile_coords(cur, tiles_r, tiles_c, group, ti, tj);
-        const int64_t r0 = (int64_t)ti * 32, c0 = (int64_t)tj * 32;
-        const uint32_t *myrow = tile + lane * S;
-        uint32_t *out = dst + c0 * ld_dst + r0 + lane;
-        if ((r0 + 32 <= rows) && (c0 + 32 <= cols)) {
-#pragma unroll
-            for (int c = 0; c < 32; ++c) out[c * ld_dst] = myrow[phys_col<L>(lane, c, sh_lane)];
-        } else {
-            const bool rok = r0 + lane < rows;
-            const int64_t cmax = cols - c0;
-#pragma unroll 4
-            for (int c = 0; c < 32; ++c)
-                if (rok && c < cmax) out[c * ld_dst] = myrow[phys_col<L>(lane, c, sh_lane)];
-        }
+        pinv = tile[lane];
         __syncwarp();
     }
-}
+#pragma unroll
+    for (int g = 0; g < G; ++g) {
+        const uint32_t rr = (uint32_t)(R * g) + c_in;
+        row_g[g] = (L == RAP_LAYOUT_RAP) ? __shfl_sync(kFull, pinv, rr) : rr;
+        const uint32_t shg = (L == RAP_LAYOUT_RAP) ? rr : __shfl_sync(kFull, sh_lane, rr);
+        a_g[g] = word_of<L>(row_g[g], NE * q, shg);     // first element of the chunk
+    }
+    const uint32_t drain_base = word_of<L>(lane, 0, sh_lane);
 
-// ------------------------------------------------------------------ 64-bit elements
-constexpr int kWarps64 = 4;
+    const uint32_t stride = gridDim.x * kWarpsT;
+    uint32_t t = blockIdx.x * kWarpsT + warp;
 
-template <int L, bool VEC, int MINB>
-__global__ void __launch_bounds__(kWarps64 * 32, MINB)
-transpose_b64_kernel(const uint64_t *__restrict__ src, uint64_t *__restrict__ dst, int64_t rows,
-                     int64_t cols, int64_t ld_src, int64_t ld_dst, uint64_t seed, uint32_t tiles_r,
-                     uint32_t tiles_c, uint32_t ntiles, uint32_t group) {
-    constexpr int S = Tile<L>::S;
-    __shared__ __align__(16) uint32_t smem[kWarps64][2][32 * S];   // [warp][lo/hi plane]
-    const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
-    uint32_t *lo_plane = smem[warp][0];
-    uint32_t *hi_plane = smem[warp][1];
-
-    uint32_t sh_lane, row_g[16], sh_g[16];
-    tile_rows<L, 16>(lo_plane, seed, lane, sh_lane, row_g, sh_g);
-    const uint32_t q = lane & 15u;             // 16-byte chunk = elements 2q, 2q+1
-
-    const uint32_t stride = gridDim.x * kWarps64;
-    uint32_t t = blockIdx.x * kWarps64 + warp;
-    uint4 v[16];
-
-    auto load = [&](uint32_t tt) {
+    auto load = [&](uint4 (&v)[G], uint32_t tt) {
         uint32_t ti, tj;
         tile_coords(tt, tiles_r, tiles_c, group, ti, tj);
         const int64_t r0 = (int64_t)ti * 32, c0 = (int64_t)tj * 32;
         const bool full = (r0 + 32 <= rows) && (c0 + 32 <= cols);
         if (VEC && full) {
+            const uint32_t *base = src + (r0 * ld_src + c0 + NE * q) * EW;
 #pragma unroll
-            for (int g = 0; g < 16; ++g)
-                v[g] = ldg_stream128(src + (r0 + row_g[g]) * ld_src + c0 + 2 * q);
+            for (int g = 0; g < G; ++g) v[g] = ldg_stream128(base + (int64_t)row_g[g] * ld_src * EW);
         } else {
 #pragma unroll
-            for (int g = 0; g < 16; ++g) {
+            for (int g = 0; g < G; ++g) {
                 const int64_t r = r0 + row_g[g];
-                const uint64_t *p = src + r * ld_src + c0 + 2 * q;
-                const bool rok = r < rows;
-                const int64_t cc = c0 + 2 * q;
-                const uint64_t e0 = (rok && cc + 0 < cols) ? __ldg((const unsigned long long *)p + 0) : 0ull;
-                const uint64_t e1 = (rok && cc + 1 < cols) ? __ldg((const unsigned long long *)p + 1) : 0ull;
-                v[g] = make_uint4((uint32_t)e0, (uint32_t)(e0 >> 32), (uint32_t)e1, (uint32_t)(e1 >> 32));
+                const int64_t cc = c0 + NE * q;
+                const uint32_t *p = src + (r * ld_src + cc) * EW;
+                uint32_t w4[4];
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    const bool ok = (r < rows) && (cc + k / EW < cols);
+                    w4[k] = ok ? __ldg(p + k) : 0u;
+                }
+                v[g] = make_uint4(w4[0], w4[1], w4[2], w4[3]);
             }
         }
     };
 
-    if (t < ntiles) load(t);
-    while (t < ntiles) {
+    // T1: contiguous (row-wise) write into the RAP tile -- every address is a_g + immediate
+    auto store_tile = [&](const uint4 (&v)[G]) {
 #pragma unroll
-        for (int g = 0; g < 16; ++g) {
-            const uint32_t p0 = row_g[g] * S + phys_col<L>(row_g[g], 2 * q + 0, sh_g[g]);
-            const uint32_t p1 = row_g[g] * S + phys_col<L>(row_g[g], 2 * q + 1, sh_g[g]);
-            lo_plane[p0] = v[g].x;
-            hi_plane[p0] = v[g].y;
-            lo_plane[p1] = v[g].z;
-            hi_plane[p1] = v[g].w;
+        for (int g = 0; g < G; ++g) {
+            const uint32_t w4[4] = {v[g].x, v[g].y, v[g].z, v[g].w};
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+                const uint32_t e = k / EW, plane = k % EW;     // element of the chunk, lo/hi word
+                uint32_t off;
+                if (L == RAP_LAYOUT_XOR) off = word_of<L>(row_g[g], NE * q + e, 0);
+                else off = a_g[g] + e;
+                tile[plane * PW + off] = w4[k];
+            }
         }
-        __syncwarp();
-        const uint32_t cur = t;
-        t += stride;
-        if (t < ntiles) load(t);
+    };
 
+    // T2: stride (column-wise) read -- lane i walks its row window -- and coalesced row stores
+    auto drain = [&](uint32_t tt) {
         uint32_t ti, tj;
-        tile_coords(cur, tiles_r, tiles_c, group, ti, tj);
+        tile_coords(tt, tiles_r, tiles_c, group, ti, tj);
         const int64_t r0 = (int64_t)ti * 32, c0 = (int64_t)tj * 32;
-        const uint32_t *mylo = lo_plane + lane * S;
-        const uint32_t *myhi = hi_plane + lane * S;
-        uint64_t *out = dst + c0 * ld_dst + r0 + lane;
+        const int64_t ostride = ld_dst * EW;                       // words between output rows
+        uint32_t *o = dst + (c0 * ld_dst + r0 + lane) * EW;        // this lane's column
         if ((r0 + 32 <= rows) && (c0 + 32 <= cols)) {
 #pragma unroll
             for (int c = 0; c < 32; ++c) {
-                const uint32_t pc = phys_col<L>(lane, c, sh_lane);
-                out[c * ld_dst] = ((uint64_t)myhi[pc] << 32) | mylo[pc];
+                const uint32_t off = (L == RAP_LAYOUT_XOR) ? word_of<L>(lane, c, 0) : drain_base + c;
+                if (EW == 1) *o = tile[off];
+                else *reinterpret_cast<uint2 *>(o) = make_uint2(tile[off], tile[PW + off]);
+                o += ostride;
             }
         } else {
             const bool rok = r0 + lane < rows;
-            const int64_t cmax = cols - c0;
-#pragma unroll 4
-            for (int c = 0; c < 32; ++c) {
-                if (rok && c < cmax) {
-                    const uint32_t pc = phys_col<L>(lane, c, sh_lane);
-                    out[c * ld_dst] = ((uint64_t)myhi[pc] << 32) | mylo[pc];
+            const int cmax = (int)min((int64_t)32, cols - c0);
+            for (int c = 0; c < cmax; ++c) {
+                const uint32_t off = (L == RAP_LAYOUT_XOR) ? word_of<L>(lane, c, 0) : drain_base + c;
+                if (rok) {
+                    if (EW == 1) *o = tile[off];
+                    else *reinterpret_cast<uint2 *>(o) = make_uint2(tile[off], tile[PW + off]);
                 }
+                o += ostride;
             }
         }
-        __syncwarp();
+    };
+
+    if (DEPTH == 1) {
+        uint4 v[G];
+        if (t < ntiles) load(v, t);
+        while (t < ntiles) {
+            store_tile(v);
+            __syncwarp();
+            const uint32_t cur = t;
+            t += stride;
+            if (t < ntiles) load(v, t);                  // T3: next tile in flight
+            drain(cur);
+            __syncwarp();
+        }
+    } else {
+        uint4 va[G], vb[G];
+        if (t < ntiles) load(va, t);
+        if (t + stride < ntiles) load(vb, t + stride);
+        while (t < ntiles) {
+            store_tile(va);
+            __syncwarp();
+            if (t + 2 * stride < ntiles) load(va, t + 2 * stride);
+            drain(t);
+            __syncwarp();
+            t += stride;
+            if (t >= ntiles) break;
+            store_tile(vb);
+            __syncwarp();
+            if (t + 2 * stride < ntiles) load(vb, t + 2 * stride);
+            drain(t);
+            __syncwarp();
+            t += stride;
+        }
     }
 }
 
 // ------------------------------------------------------------------ launchers
 template <typename K>
-static int grid_for(K kernel, int threads, int64_t ntiles, int warps_per_cta) {
+static int grid_for(K kernel, int threads, size_t smem, int64_t ntiles, int warps_per_cta, int ctas_per_sm) {
     int dev = 0, sms = 148, occ = 1;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kernel, threads, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kernel, threads, smem);
     if (occ < 1) occ = 1;
+    if (ctas_per_sm > 0 && ctas_per_sm < occ) occ = ctas_per_sm;
     const int64_t want = (ntiles + warps_per_cta - 1) / warps_per_cta;
     const int64_t cap = (int64_t)sms * occ;
     return (int)(want < cap ? want : cap);
@@ -283,59 +253,51 @@ TransposeTuning default_tuning(uint32_t elem_bytes) {
     TransposeTuning t;
     t.group = elem_bytes == 4 ? kDefaultGroup32 : kDefaultGroup64;
     t.minb = elem_bytes == 4 ? kDefaultMinB32 : kDefaultMinB64;
+    t.depth = elem_bytes == 4 ? kDefaultDepth32 : kDefaultDepth64;
+    t.ctas_per_sm = elem_bytes == 4 ? kDefaultCtas32 : kDefaultCtas64;
     return t;
 }
 
-template <int L, bool VEC, int MINB>
-static cudaError_t launch_b32(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
-                              int64_t ld_dst, uint64_t seed, uint32_t group, cudaStream_t st) {
+template <int L, int EW, bool VEC, int DEPTH, int MINB>
+static cudaError_t launch_one(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
+                              int64_t ld_dst, uint64_t seed, const TransposeTuning &tu, cudaStream_t st) {
     const uint32_t tiles_r = (uint32_t)((rows + 31) / 32), tiles_c = (uint32_t)((cols + 31) / 32);
     const uint32_t ntiles = tiles_r * tiles_c;
-    auto k = transpose_b32_kernel<L, VEC, MINB>;
-    const int grid = grid_for(k, kWarps32 * 32, ntiles, kWarps32);
-    k<<<grid, kWarps32 * 32, 0, st>>>((const uint32_t *)src, (uint32_t *)dst, rows, cols, ld_src,
-                                      ld_dst, seed, tiles_r, tiles_c, ntiles, group);
+    auto k = transpose_kernel<L, EW, VEC, DEPTH, MINB>;
+    const size_t smem = sizeof(uint32_t) * warp_smem_words<L, EW>() * kWarpsT;
+    cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    const int grid = grid_for(k, kWarpsT * 32, smem, ntiles, kWarpsT, tu.ctas_per_sm);
+    k<<<grid, kWarpsT * 32, smem, st>>>((const uint32_t *)src, (uint32_t *)dst, rows, cols, ld_src,
+                                        ld_dst, seed, tiles_r, tiles_c, ntiles, tu.group);
     return cudaGetLastError();
 }
 
-template <int L, bool VEC, int MINB>
-static cudaError_t launch_b64(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
-                              int64_t ld_dst, uint64_t seed, uint32_t group, cudaStream_t st) {
-    const uint32_t tiles_r = (uint32_t)((rows + 31) / 32), tiles_c = (uint32_t)((cols + 31) / 32);
-    const uint32_t ntiles = tiles_r * tiles_c;
-    auto k = transpose_b64_kernel<L, VEC, MINB>;
-    const int grid = grid_for(k, kWarps64 * 32, ntiles, kWarps64);
-    k<<<grid, kWarps64 * 32, 0, st>>>((const uint64_t *)src, (uint64_t *)dst, rows, cols, ld_src,
-                                      ld_dst, seed, tiles_r, tiles_c, ntiles, group);
-    return cudaGetLastError();
-}
-
-template <int L, bool VEC>
-static cudaError_t launch_minb(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
-                               int64_t ld_dst, uint32_t eb, uint64_t seed, const TransposeTuning &tu,
-                               cudaStream_t st) {
-    if (eb == 4) {
-        switch (tu.minb) {
-        case 1: return launch_b32<L, VEC, 1>(src, dst, rows, cols, ld_src, ld_dst, seed, tu.group, st);
-        case 3: return launch_b32<L, VEC, 3>(src, dst, rows, cols, ld_src, ld_dst, seed, tu.group, st);
-        case 4: return launch_b32<L, VEC, 4>(src, dst, rows, cols, ld_src, ld_dst, seed, tu.group, st);
-        default: return launch_b32<L, VEC, 2>(src, dst, rows, cols, ld_src, ld_dst, seed, tu.group, st);
-        }
-    }
-    switch (tu.minb) {
-    case 1: return launch_b64<L, VEC, 1>(src, dst, rows, cols, ld_src, ld_dst, seed, tu.group, st);
-    case 3: return launch_b64<L, VEC, 3>(src, dst, rows, cols, ld_src, ld_dst, seed, tu.group, st);
-    case 4: return launch_b64<L, VEC, 4>(src, dst, rows, cols, ld_src, ld_dst, seed, tu.group, st);
-    default: return launch_b64<L, VEC, 2>(src, dst, rows, cols, ld_src, ld_dst, seed, tu.group, st);
-    }
+template <int L, int EW, bool VEC>
+static cudaError_t launch_shape(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
+                                int64_t ld_dst, uint64_t seed, const TransposeTuning &tu, cudaStream_t st) {
+#define RAPK_SHAPE(D, M)                                                                             \
+    if (tu.depth == D && tu.minb == M)                                                               \
+        return launch_one<L, EW, VEC, D, M>(src, dst, rows, cols, ld_src, ld_dst, seed, tu, st);
+#ifdef RAP_TUNING_SWEEP
+    RAPK_SHAPE(1, 2) RAPK_SHAPE(1, 3) RAPK_SHAPE(1, 4) RAPK_SHAPE(1, 6) RAPK_SHAPE(1, 8)
+    RAPK_SHAPE(2, 2) RAPK_SHAPE(2, 3) RAPK_SHAPE(2, 4) RAPK_SHAPE(2, 6)
+#endif
+#undef RAPK_SHAPE
+    (void)tu;
+    return launch_one<L, EW, VEC, EW == 1 ? kDefaultDepth32 : kDefaultDepth64,
+                      EW == 1 ? kDefaultMinB32 : kDefaultMinB64>(src, dst, rows, cols, ld_src, ld_dst,
+                                                                 seed, tu, st);
 }
 
 template <bool VEC>
 static cudaError_t dispatch(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
                             int64_t ld_dst, uint32_t eb, int layout, uint64_t seed,
                             const TransposeTuning &tu, cudaStream_t st) {
-#define RAPK_CASE(LAY) \
-    case LAY: return launch_minb<LAY, VEC>(src, dst, rows, cols, ld_src, ld_dst, eb, seed, tu, st);
+#define RAPK_CASE(LAY)                                                                             \
+    case LAY:                                                                                      \
+        return eb == 4 ? launch_shape<LAY, 1, VEC>(src, dst, rows, cols, ld_src, ld_dst, seed, tu, st) \
+                       : launch_shape<LAY, 2, VEC>(src, dst, rows, cols, ld_src, ld_dst, seed, tu, st);
     switch (layout) {
         RAPK_CASE(RAP_LAYOUT_RAW)
         RAPK_CASE(RAP_LAYOUT_PAD)
