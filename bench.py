@@ -1,22 +1,23 @@
 """bench.py -- RAP hot path on B200: one JSON line per run (driver contract).
 
 A step is one pass of the whole hot path over one batch of synthetic input:
-  T0-T3  RAP transpose of the BASELINE cfg3 matrix (8192 x 8192 float32, out-of-place,
-         inputs 256 MiB > 126 MB L2, so no flush is needed between steps), and
-  C1-C4  one batch of the cfg2 congestion sweep (w = 32, all 5 patterns x RAW/RAS/RAP;
-         --sweep-trials per step, counter-based so batches are disjoint trial ranges).
-`value` is the headline transpose throughput in GB/s: algorithmic bytes (read once + write
-once) / the transpose kernels' device time inside the timed steps (CUDA events on the
-launching stream).  The sweep is reported beside it as trials/s (`sweep`).
+  T0-T3  RAP transpose of the BASELINE cfg3 matrix (8192 x 8192 float32, out-of-place; input
+         and output are 256 MiB each, larger than the 126 MB L2, so no flush between steps),
+  C1-C4  one batch of the cfg2 congestion sweep (w = 32, 5 patterns x RAW/RAS/RAP,
+         --sweep-trials per rank per step; counter-based, so batches are disjoint trial ranges
+         that continue across steps), and on N > 1 ranks the NCCL all-reduce of the histogram.
+`value` is the headline transpose throughput (GB/s, whole job): algorithmic bytes (read once +
+write once) of all ranks / the transpose device time inside the timed steps (CUDA events on
+the launching stream, max over ranks).  The sweep is reported beside it (`sweep`).
 
---workload picks another config as the timed step: sweep (cfg2 only), cfg4 (16384^2
-float64), tile (cfg1 32x32), layouts (cfg3 under raw/pad/xor/ras/rap), dist (cfg5,
-row-block-sharded 32768^2 with NCCL all-to-all; needs torchrun).
---impl reference times the CPU oracle (the only reference this paper has) on a bounded
-sample of the same workload, on the host cores.
+--workload picks another timed step: sweep (cfg2 only; value = trials/s), cfg4 (16384^2
+float64 transpose), tile (cfg1 32 x 32), layouts (cfg3 under raw/pad/xor/ras/rap; value =
+RAP), dist (cfg5: 32768^2 float32 row-block-sharded over the ranks, NCCL all-to-all).
+--impl reference times the CPU oracle (the only reference this paper has: it publishes no
+code) on a bounded sample of the same workload on the host cores; rank 0 only.
 
-N > 1 (torchrun): every rank transposes its own cfg3 matrix (replicas; weak scaling) and
-sweeps a disjoint trial range; the histograms are all-reduced over NCCL once per step.
+N > 1 (torchrun, one process per GPU): every rank transposes its own cfg3 matrix (replicas,
+weak scaling) and sweeps its own trial batch; `dist` shards one matrix (strong scaling).
 """
 from __future__ import annotations
 
@@ -34,6 +35,7 @@ sys.path.insert(0, ROOT)
 METRIC = "RAP transpose GB/s vs HBM peak; smem wavefronts/request; congestion trials/s"
 ALL_PAT = ["contiguous", "stride", "diagonal", "random", "malicious"]
 SCH = ["raw", "ras", "rap"]
+NVLINK_GBS = 770.0   # measured peer copy per direction (B200_PROFILING.md); 900 nominal
 
 
 def parse():
@@ -45,41 +47,44 @@ def parse():
     p.add_argument("--workload", default="default",
                    choices=["default", "sweep", "cfg4", "tile", "layouts", "dist"])
     p.add_argument("--sweep-trials", type=int, default=1 << 24)
-    p.add_argument("--layout", default="rap")
     p.add_argument("--sweep-algo", default="default", choices=["default", "match"])
+    p.add_argument("--layout", default="rap")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu", action="store_true")
     return p.parse_args()
+
+
+def dist_env():
+    return (int(os.environ.get("WORLD_SIZE", "1")), int(os.environ.get("RANK", "0")),
+            int(os.environ.get("LOCAL_RANK", "0")))
 
 
 def load_peaks():
     path = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(path):
         d = json.load(open(path))
-        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, torch copy_)"
-    return 6650.0, "fallback (B200_PROFILING.md: 6.65 TB/s)"
+        return float(d["hbm_gbs"]), "measured: MEASURED_PEAKS.json hbm_gbs (torch copy_, 2 GiB)"
+    return 6650.0, "fallback: B200_PROFILING.md 6.65 TB/s"
 
 
-def load_traffic(kernel_key: str):
-    """dram bytes per launch from the committed ncu --set full summary, if present."""
+def load_profile(kernel_key: str):
+    """Per-launch DRAM bytes and smem wavefronts/request from the committed ncu summary."""
     path = os.path.join(ROOT, "profiles", "ncu_summary.json")
     if not os.path.exists(path):
         return None
-    d = json.load(open(path))
-    k = d.get("kernels", {}).get(kernel_key)
-    return None if k is None else k.get("dram_bytes_per_launch")
+    return json.load(open(path)).get("kernels", {}).get(kernel_key)
 
 
 class Clocks:
-    """nvidia-smi sampler running during the timed region."""
+    """nvidia-smi sampler running during the timed region (start before, stop after)."""
 
     FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
               "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
               "clocks_event_reasons.sw_power_cap")
+    NAMES = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
 
     def __init__(self, index: int):
-        self.index = index
-        self.proc = None
+        self.index, self.proc, self.result = index, None, None
 
     def __enter__(self):
         try:
@@ -87,9 +92,9 @@ class Clocks:
                 ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
                  "--format=csv,noheader,nounits", "-lms", "50"],
                 stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            time.sleep(0.15)
         except OSError:
             self.proc = None
-        time.sleep(0.15)
         return self
 
     def __exit__(self, *a):
@@ -100,7 +105,6 @@ class Clocks:
         self.proc.terminate()
         out, _ = self.proc.communicate(timeout=10)
         sm, mx, reasons = [], [], set()
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
         for ln in out.strip().splitlines():
             f = [x.strip() for x in ln.split(",")]
             if len(f) < 7:
@@ -110,7 +114,7 @@ class Clocks:
                 mx.append(float(f[1]))
             except ValueError:
                 continue
-            for n, v in zip(names, f[3:7]):
+            for n, v in zip(self.NAMES, f[3:7]):
                 if v.lower().startswith("active"):
                     reasons.add(n)
         self.result = {"sm_mhz": statistics.median(sm) if sm else None,
@@ -118,20 +122,12 @@ class Clocks:
                        "samples": len(sm)}
 
 
-def dist_env():
-    ws = int(os.environ.get("WORLD_SIZE", "1"))
-    rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
-    return ws, rank, local
-
-
 # ---------------------------------------------------------------------------- reference arm
 def run_reference(args):
-    """The CPU oracle timed on the host cores on a bounded sample of the workload."""
-    ws, rank, _ = dist_env()
-    if ws > 1 and rank != 0:
+    """The CPU oracle, as it stands, on the host cores, on a bounded sample of the workload."""
+    world, rank, _ = dist_env()
+    if world > 1 and rank != 0:
         return
-    import numpy as np
     import torch
 
     import oracle
@@ -141,38 +137,39 @@ def run_reference(args):
         n = 20000
         unit, what = "trials/s", f"{n} trials of the w=32 sweep (5 patterns x RAW/RAS/RAP) per step"
         fn = lambda k: oracle.sweep(32, ALL_PAT, SCH, 1, k * n, n, threads=threads)
-        work = n
+        work, cfg = n, {"workload": "cfg2 w=32 congestion sweep (oracle sample)"}
     else:
-        rows, cols, dt = (16384, 16384, torch.float64) if args.workload == "cfg4" else (8192, 8192, torch.float32)
-        band = 512
+        rows, cols, dt = {"cfg4": (16384, 16384, torch.float64), "dist": (32768, 32768, torch.float32),
+                          "tile": (32, 32, torch.float32)}.get(args.workload, (8192, 8192, torch.float32))
+        band = min(rows, 512)
         x = workloads.as_bits_numpy(workloads.random_bits(band, cols, dt, seed=0))
         unit = "GB/s"
-        what = f"{band} x {cols} row band of the {rows}x{cols} {dt} matrix per step (oracle naive transpose)"
+        what = f"{band} x {cols} row band of the {rows}x{cols} {str(dt)[6:]} matrix per step, naive oracle transpose"
         fn = lambda k: oracle.transpose(x, threads=threads)
         work = 2 * x.nbytes / 1e9
+        cfg = {"workload": f"{rows}x{cols} {str(dt)[6:]} transpose (oracle sample)", "rows": rows, "cols": cols}
     for k in range(args.warmup):
         fn(k)
     t0 = time.perf_counter()
     for k in range(args.steps):
         fn(args.warmup + k)
-    dt_s = time.perf_counter() - t0
-    value = work * args.steps / dt_s
-    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": unit, "n_gpus": ws,
-            "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt_s / args.steps * 1e3,
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
-            "data": "synthetic",
-            "config": {"workload": args.workload if args.workload != "default" else "cfg3 8192x8192 float32 transpose"},
+    el = time.perf_counter() - t0
+    value = work * args.steps / el
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": unit, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": el / args.steps * 1e3,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "dtype": "u64" if args.workload == "cfg4" else "u32", "data": "synthetic", "config": cfg,
             "cpu_baseline": {"value": value, "unit": unit, "cores": threads, "kind": "oracle", "sample": what},
             "e2e": {"value": value, "unit": unit, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
 
-# ---------------------------------------------------------------------------- our arm
+# ---------------------------------------------------------------------------- helpers
 def cpu_baseline_transpose(rows, cols, dt):
     import oracle
     import workloads
     threads = oracle.max_threads()
-    band = 1024
+    band = min(rows, 1024)
     x = workloads.as_bits_numpy(workloads.random_bits(band, cols, dt, seed=0))
     oracle.transpose(x, threads=threads)
     reps, t0 = 0, time.perf_counter()
@@ -197,171 +194,240 @@ def cpu_baseline_sweep():
             "sample": f"{n * reps} trials of the w=32 sweep (5 patterns x RAW/RAS/RAP) in {el:.1f} s"}
 
 
+def reduce_over_ranks(x: float, world: int, dev, op: str) -> float:
+    if world == 1:
+        return x
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor([x], dtype=torch.float64, device=dev)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX if op == "max" else dist.ReduceOp.SUM)
+    return float(t.item())
+
+
+# ---------------------------------------------------------------------------- our arm
 def main():
     args = parse()
     if args.impl == "reference":
         return run_reference(args)
-    if args.gpus > 1 or args.workload == "dist":
-        from paper_conf_icppw_nakanomi14_b200 import bench_dist
-        return bench_dist.main(args)
+    import numpy as np
     import torch
+    import torch.distributed as dist
 
     import __graft_entry__
     __graft_entry__.build()
     import paper_conf_icppw_nakanomi14_b200 as rap
+    from paper_conf_icppw_nakanomi14_b200 import dist as rdist
     import workloads
 
-    dev = torch.device("cuda", 0)
+    world, rank, local = dist_env()
+    dev = torch.device("cuda", local)
     torch.cuda.set_device(dev)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
     stream = torch.cuda.current_stream()
     peak, peak_src = load_peaks()
+    wl = args.workload
+    barrier = (lambda: dist.barrier()) if world > 1 else (lambda: None)
+    rmax = lambda v: reduce_over_ranks(v, world, dev, "max")
 
-    if args.workload == "cfg4":
+    # ---------------- workload setup
+    if wl == "cfg4":
         rows = cols = 16384
-        dt, dname, layouts = torch.float64, "u64", [args.layout]
-    elif args.workload == "tile":
+        dt = torch.float64
+    elif wl == "tile":
         rows = cols = 32
-        dt, dname, layouts = torch.float32, "u32", [args.layout]
+        dt = torch.float32
+    elif wl == "dist":
+        rows, cols = 32768 // world, 32768
+        dt = torch.float32
     else:
         rows = cols = 8192
-        dt, dname, layouts = torch.float32, "u32", [args.layout]
-    if args.workload == "layouts":
-        layouts = ["raw", "pad", "xor", "ras", "rap"]
-    do_t = args.workload != "sweep"
-    do_s = args.workload in ("default", "sweep")
+        dt = torch.float32
+    do_t = wl != "sweep"
+    do_s = wl in ("default", "sweep")
+    layouts = ["raw", "pad", "xor", "ras", "rap"] if wl == "layouts" else [args.layout]
     eb = torch.empty((), dtype=dt).element_size()
-    nbytes = 2 * rows * cols * eb
-
-    x = workloads.random_bits(rows, cols, dt, seed=0, device=dev) if do_t else None
-    y = torch.empty((cols, rows), dtype=dt, device=dev) if do_t else None
-    hist = torch.zeros((5, 3, 33), dtype=torch.int64, device=dev)
+    nbytes = 2 * rows * cols * eb                     # per rank per step
+    x = workloads.random_bits(rows, cols, dt, seed=rank, device=dev) if do_t else None
+    y = None
+    if do_t:
+        y = torch.empty((rows, cols) if wl == "dist" else (cols, rows), dtype=dt, device=dev)
+    work = {}
     S = args.sweep_trials
+    hist = torch.zeros((5, 3, 33), dtype=torch.int64, device=dev)
+
+    def step_transpose(lay):
+        if wl == "dist":
+            rdist.transpose_sharded(x, layout=lay, seed=0, out=y, work=work)
+            return 1 if world == 1 else 2          # local transpose (+ unpack)
+        rap.transpose(x, layout=lay, seed=0, out=y)
+        return 1
+
+    def step_sweep(k):
+        # this rank's batch of the global trial sequence: step k covers trials
+        # [k*S*world, (k+1)*S*world), rank r the r-th slice of it
+        rap.congestion_sweep(S, seed=1, first_trial=(k * world + rank) * S, out=hist, algo=args.sweep_algo)
+        if world > 1:
+            dist.all_reduce(hist)
+        return 1
 
     results = {}
     for lay in layouts:
-        launches = 0
-        ev = []
-        trial0 = 0
         for k in range(args.warmup):
             if do_t:
-                rap.transpose(x, layout=lay, seed=0, out=y)
+                step_transpose(lay)
             if do_s:
-                rap.congestion_sweep(S, seed=1, first_trial=trial0, out=hist, algo=args.sweep_algo)
-                trial0 += S
+                step_sweep(k)
         torch.cuda.synchronize()
         hist.zero_()
-        trial0 = 0
-        with Clocks(0) as clk:
+        launches, ev = 0, []
+        barrier()
+        torch.cuda.synchronize()
+        with Clocks(local) as clk:
             start = torch.cuda.Event(enable_timing=True)
             end = torch.cuda.Event(enable_timing=True)
-            torch.cuda.synchronize()
             start.record(stream)
             for k in range(args.steps):
                 e = [torch.cuda.Event(enable_timing=True) for _ in range(4)]
                 e[0].record(stream)
                 if do_t:
-                    rap.transpose(x, layout=lay, seed=0, out=y)
-                    launches += 1
+                    launches += step_transpose(lay)
                 e[1].record(stream)
                 e[2].record(stream)
                 if do_s:
-                    rap.congestion_sweep(S, seed=1, first_trial=trial0, out=hist, algo=args.sweep_algo)
-                    trial0 += S
-                    launches += 1
+                    launches += step_sweep(k)
                 e[3].record(stream)
                 ev.append(e)
             end.record(stream)
             torch.cuda.synchronize()
-        total_ms = start.elapsed_time(end)
+            barrier()
         t_ms = [e[0].elapsed_time(e[1]) for e in ev]
         s_ms = [e[2].elapsed_time(e[3]) for e in ev]
-        results[lay] = dict(total_ms=total_ms, t_ms=t_ms, s_ms=s_ms, clocks=clk.result, launches=launches)
+        results[lay] = dict(total_ms=rmax(start.elapsed_time(end)), t_sum=rmax(sum(t_ms)), t_ms=t_ms,
+                            s_sum=rmax(sum(s_ms)), s_ms=s_ms, clocks=clk.result, launches=launches)
 
-    lay = args.layout if args.workload != "layouts" else "rap"
+    lay = "rap" if wl == "layouts" else args.layout
     r = results[lay]
-    line = {"metric": METRIC, "n_gpus": 1, "steps": args.steps, "warmup": args.warmup,
-            "ms_per_step": r["total_ms"] / args.steps, "higher_is_better": True, "scaling": "weak",
-            "vs_baseline": None, "dtype": dname, "data": "synthetic"}
+    line = {"metric": METRIC, "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": r["total_ms"] / args.steps, "higher_is_better": True,
+            "scaling": "strong" if wl == "dist" else "weak", "vs_baseline": None,
+            "dtype": "u64" if eb == 8 else "u32", "data": "synthetic (seeded random bit patterns)"}
     if do_t:
-        avg_t = sum(r["t_ms"]) / len(r["t_ms"])
-        gbs = nbytes / (avg_t * 1e-3) / 1e9
+        gbs = nbytes * world * args.steps / (r["t_sum"] * 1e-3) / 1e9
+        kern_ms = statistics.median(r["t_ms"])
         line.update(value=gbs, unit="GB/s")
-        line["config"] = {"workload": {"default": "cfg3 8192x8192 float32 RAP transpose + cfg2 w=32 sweep batch",
-                                       "cfg4": "cfg4 16384x16384 float64 RAP transpose",
-                                       "tile": "cfg1 32x32 float32 RAP tile",
-                                       "layouts": "cfg3 8192x8192 float32 transpose, 5 smem layouts"}[args.workload],
-                          "rows": rows, "cols": cols, "elem_bytes": eb, "layout": lay,
-                          "l2": "inputs larger than L2 (no flush)" if nbytes // 2 > 126e6 else "L2-resident (latency case)",
-                          "algorithmic_bytes_per_step": nbytes}
+        desc = {"default": "cfg3 8192x8192 float32 RAP transpose + cfg2 w=32 sweep batch",
+                "cfg4": "cfg4 16384x16384 float64 RAP transpose (two 32-bit RAP planes)",
+                "tile": "cfg1 32x32 float32 RAP tile (latency case)",
+                "layouts": "cfg3 8192x8192 float32 transpose under 5 smem layouts",
+                "dist": f"cfg5 32768x32768 float32 row-block-sharded transpose over {world} GPU(s)"}[wl]
+        line["config"] = {"workload": desc, "rows": rows * (world if wl == "dist" else 1), "cols": cols,
+                          "elem_bytes": eb, "layout": lay,
+                          "parallelism": (f"row blocks + NCCL all-to-all, {world} ranks" if wl == "dist"
+                                          else f"replicas x{world}" if world > 1 else "single GPU"),
+                          "l2": ("inputs larger than L2 (no flush)" if nbytes // 2 > 126e6
+                                 else "input fits in L2 (no flush; latency case)"),
+                          "algorithmic_bytes_per_step_per_rank": nbytes}
+        if do_s:
+            line["config"]["sweep_trials_per_step"] = S * world
         kkey = f"transpose_b{eb * 8}_{lay}"
-        line["roofline"] = {"bound": "hbm", "achieved": gbs, "peak": peak, "unit": "GB/s",
-                            "frac": gbs / peak, "traffic": load_traffic(kkey),
-                            "peak_source": peak_src, "frac_of_8TBs_nominal": gbs / 8000.0,
-                            "kernel": kkey, "kernel_ms_median": statistics.median(r["t_ms"])}
-        if args.workload == "layouts":
-            line["layouts_gbs"] = {l: nbytes / (sum(v["t_ms"]) / len(v["t_ms"]) * 1e-3) / 1e9
+        prof = load_profile(kkey) or {}
+        if wl == "dist" and world > 1:
+            nv = (world - 1) / world * (rows * cols * eb) / (kern_ms * 1e-3) / 1e9
+            line["roofline"] = {"bound": "nvlink", "achieved": nv, "peak": NVLINK_GBS, "unit": "GB/s",
+                                "frac": nv / NVLINK_GBS, "traffic": None,
+                                "peak_source": "B200_PROFILING.md measured peer copy per direction",
+                                "note": "bytes each rank sends over NVLink per step / step time"}
+        else:
+            ach = nbytes / (kern_ms * 1e-3) / 1e9
+            line["roofline"] = {"bound": "hbm", "achieved": ach, "peak": peak, "unit": "GB/s",
+                                "frac": ach / peak, "traffic": prof.get("dram_bytes_per_launch"),
+                                "peak_source": peak_src, "frac_of_8TBs_nominal": ach / 8000.0,
+                                "kernel": kkey, "kernel_ms_median": kern_ms,
+                                "algorithmic_bytes_per_launch": nbytes,
+                                "smem_wavefronts_per_request": prof.get("smem_wavefronts_per_request"),
+                                "profile": prof.get("source")}
+        if wl == "layouts":
+            line["layouts_gbs"] = {l: nbytes * world * args.steps / (v["t_sum"] * 1e-3) / 1e9
                                    for l, v in results.items()}
     if do_s:
-        s_avg = sum(r["s_ms"]) / len(r["s_ms"])
-        tps = S / (s_avg * 1e-3)
+        tps = S * world * args.steps / (r["s_sum"] * 1e-3)
         h = hist.cpu().numpy()
-        import numpy as np
         c = np.arange(33)
         E = lambda a: float((a * c).sum() / a.sum())
-        sweep = {"trials_per_s": tps, "trials_per_step": S, "w": 32,
-                 "E_ras_stride": E(h[1, 1]), "E_rap_diagonal": E(h[2, 2]), "E_random": E(h[3, 2]),
-                 "E_raw_malicious": E(h[4, 0]), "E_rap_stride": E(h[1, 2]),
-                 "kernel_ms_median": statistics.median(r["s_ms"])}
-        line["sweep"] = sweep
+        line["sweep"] = {"trials_per_s": tps, "trials_per_step": S * world, "w": 32, "algo": args.sweep_algo,
+                         "E_ras_stride": E(h[1, 1]), "E_rap_diagonal": E(h[2, 2]), "E_random": E(h[3, 2]),
+                         "E_raw_malicious": E(h[4, 0]), "E_rap_stride": E(h[1, 2]),
+                         "kernel_ms_median": statistics.median(r["s_ms"])}
         if not do_t:
             line.update(value=tps, unit="trials/s",
-                        config={"workload": "cfg2 w=32 congestion sweep", "trials_per_step": S})
-            line["roofline"] = {"bound": "alu", "achieved": None, "peak": None, "unit": "warp-instr/s",
-                                "frac": None, "traffic": None,
-                                "note": "issue-bound; see profiles/ for smsp__issue_active"}
+                        config={"workload": "cfg2 w=32 congestion sweep, 5 patterns x RAW/RAS/RAP",
+                                "trials_per_step": S * world,
+                                "parallelism": (f"trial ranges x{world} + NCCL all-reduce" if world > 1
+                                                else "single GPU")})
+            prof = load_profile("sweep_w32") or {}
+            line["roofline"] = {"bound": "alu", "achieved": prof.get("issue_active_frac"), "peak": 1.0,
+                                "unit": "fraction of issue slots", "frac": prof.get("issue_active_frac"),
+                                "traffic": None, "profile": prof.get("source"),
+                                "note": "issue-bound integer kernel: achieved = smsp__issue_active from ncu"}
     line["clocks"] = r["clocks"]
-    line["gpu_launches"] = r["launches"]
+    line["gpu_launches"] = int(reduce_over_ranks(r["launches"], world, dev, "sum"))
 
-    # ---- e2e: the same step through the public API with host buffers (pinned)
+    # ---------------- e2e through the public API with pinned host buffers
+    K = max(3, min(args.steps, 20))
     if not args.no_e2e and do_t:
         hx = x.cpu().pin_memory()
-        hy = torch.empty((cols, rows), dtype=dt).pin_memory()
-        hh = torch.empty_like(hist, device="cpu").pin_memory()
+        hy = torch.empty(tuple(y.shape), dtype=dt).pin_memory()
         dx = torch.empty_like(x)
-        for k in range(2):
+
+        def e2e_step():
             dx.copy_(hx, non_blocking=True)
-            rap.transpose(dx, layout=lay, seed=0, out=y)
+            if wl == "dist":
+                rdist.transpose_sharded(dx, layout=lay, seed=0, out=y, work=work)
+            else:
+                rap.transpose(dx, layout=lay, seed=0, out=y)
             hy.copy_(y, non_blocking=True)
+
+        for _ in range(2):
+            e2e_step()
         torch.cuda.synchronize()
-        K = max(3, min(args.steps, 20))
+        barrier()
+        st = torch.cuda.Event(enable_timing=True)
+        en = torch.cuda.Event(enable_timing=True)
+        st.record(stream)
+        for _ in range(K):
+            e2e_step()
+        en.record(stream)
+        torch.cuda.synchronize()
+        ms = rmax(st.elapsed_time(en)) / K
+        bd = torch.int32 if eb == 4 else torch.int64
+        assert torch.equal(hy.view(bd), y.cpu().view(bd)), "e2e result differs from the device result"
+        line["e2e"] = {"value": nbytes * world / (ms * 1e-3) / 1e9, "unit": "GB/s",
+                       "h2d_bytes_per_step": hx.numel() * eb * world, "d2h_bytes_per_step": hy.numel() * eb * world,
+                       "ms_per_step": ms, "steps": K,
+                       "note": "pinned host matrix -> H2D -> transpose (public API) -> D2H of the result"}
+    elif not args.no_e2e and do_s:
+        hh = torch.empty_like(hist, device="cpu").pin_memory()
         st = torch.cuda.Event(enable_timing=True)
         en = torch.cuda.Event(enable_timing=True)
         st.record(stream)
         for k in range(K):
-            dx.copy_(hx, non_blocking=True)
-            rap.transpose(dx, layout=lay, seed=0, out=y)
-            hy.copy_(y, non_blocking=True)
-            if do_s:
-                rap.congestion_sweep(S, seed=1, first_trial=k * S, out=hist)
-                hh.copy_(hist, non_blocking=True)
+            step_sweep(k)
+            hh.copy_(hist, non_blocking=True)
         en.record(stream)
         torch.cuda.synchronize()
-        ms = st.elapsed_time(en) / K
-        line["e2e"] = {"value": nbytes / (ms * 1e-3) / 1e9, "unit": "GB/s",
-                       "h2d_bytes_per_step": hx.numel() * eb,
-                       "d2h_bytes_per_step": hy.numel() * eb + (hh.numel() * 8 if do_s else 0),
-                       "ms_per_step": ms, "steps": K,
-                       "note": "pinned host in -> H2D -> rap.transpose -> D2H (+ sweep batch, histogram D2H)"}
-        bd = torch.int32 if eb == 4 else torch.int64
-        assert torch.equal(hy.view(bd), y.cpu().view(bd)), "e2e result differs from the device result"
-    if not args.no_cpu:
-        if do_t:
-            line["cpu_baseline"] = cpu_baseline_transpose(rows, cols, dt)
-        else:
-            line["cpu_baseline"] = cpu_baseline_sweep()
+        ms = rmax(st.elapsed_time(en)) / K
+        line["e2e"] = {"value": S * world / (ms * 1e-3), "unit": "trials/s", "h2d_bytes_per_step": 0,
+                       "d2h_bytes_per_step": hh.numel() * 8, "ms_per_step": ms, "steps": K,
+                       "note": "sweep batch through the public API + D2H of the histogram (inputs are counters)"}
+    if rank == 0 and not args.no_cpu and world == 1:
+        line["cpu_baseline"] = cpu_baseline_transpose(rows, cols, dt) if do_t else cpu_baseline_sweep()
         if do_s and do_t:
             line["sweep"]["cpu_baseline"] = cpu_baseline_sweep()
-    print(json.dumps(line), flush=True)
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
 
 
 if __name__ == "__main__":

@@ -146,6 +146,17 @@ rap_status_t rap_congestion_trace(uint32_t w, uint64_t n_warps, const uint32_t *
                                   uint32_t scheme_mask, uint64_t seed, uint64_t first_trial,
                                   uint64_t n_trials, uint64_t *d_hist, void *stream);
 
+/* T4 -- block unpack after the all-to-all of the row-block-sharded transpose (BASELINE cfg5;
+ * not in the paper, which has one w x w matrix).  Rank g of G holds rows gM..(g+1)M of the
+ * N x N matrix A (N = G*M); rap_transpose of that M x N shard gives N x M whose row block s is
+ * the M x M block destined for rank s; after the exchange the receive buffer holds, for every
+ * source s, recv[s] = (A[sM:(s+1)M, gM:(g+1)M])^T (M x M, contiguous, source order).  This call
+ * places it:  d_out[x * ld_out + s*M + a] = d_recv[(s*M + x) * M + a]  (0 <= s < G, x, a < M),
+ * i.e. rows gM..(g+1)M of A^T.  Device pointers; ld_out >= G*M; raw bit copy of elem_bytes in
+ * {4, 8}; overlapping buffers -> RAP_ERR_ALIAS; G == 0 or M == 0 is a no-op. */
+rap_status_t rap_unpack_blocks(const void *d_recv, void *d_out, int64_t G, int64_t M, int64_t ld_out,
+                               uint32_t elem_bytes, void *stream);
+
 #ifdef __cplusplus
 }
 #endif

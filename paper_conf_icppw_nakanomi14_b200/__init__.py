@@ -17,7 +17,7 @@ import torch
 
 from . import build as _build
 
-__all__ = ["perm_gen", "transpose", "congestion", "congestion_sweep", "congestion_trace",
+__all__ = ["perm_gen", "transpose", "congestion", "congestion_sweep", "congestion_trace", "unpack_blocks",
            "LAYOUTS", "SCHEMES", "PATTERNS", "RapError", "lib", "library_path"]
 
 LAYOUTS = {"raw": 0, "pad": 1, "xor": 2, "ras": 3, "rap": 4}
@@ -61,8 +61,9 @@ def lib():
         L.rap_congestion_sweep.argtypes = [u32, u32, u32, u64, u64, u64, u64p, vp]
         L.rap_congestion_sweep_algo.argtypes = [u32, u32, u32, u64, u64, u64, u64p, u32, vp]
         L.rap_congestion_trace.argtypes = [u32, u64, u32p, u32, u64, u64, u64, u64p, vp]
+        L.rap_unpack_blocks.argtypes = [vp, vp, i64, i64, i64, u32, vp]
         for f in ("rap_perm_gen", "rap_transpose", "rap_congestion", "rap_congestion_sweep",
-                  "rap_congestion_sweep_algo", "rap_congestion_trace"):
+                  "rap_congestion_sweep_algo", "rap_congestion_trace", "rap_unpack_blocks"):
             getattr(L, f).restype = i32
         if L.rap_abi_version() != 1:
             raise ImportError("librap.so ABI version mismatch")
@@ -196,4 +197,21 @@ def congestion_trace(cells: torch.Tensor, n_trials: int, seed: int, schemes=("ra
         _check(lib().rap_congestion_trace(w, n, ctypes.c_void_p(cells.data_ptr()), sm, seed,
                                           first_trial, n_trials, ctypes.c_void_p(out.data_ptr()),
                                           _stream(cells)), "rap_congestion_trace")
+    return out
+
+
+def unpack_blocks(recv: torch.Tensor, out: torch.Tensor, G: int) -> torch.Tensor:
+    """After the all-to-all of the sharded transpose: out[x, s*M + a] = recv[s*M + x, a].
+
+    recv: CUDA [G*M, M] (source-ordered M x M blocks); out: CUDA [M, >= G*M] with unit inner stride.
+    """
+    _need_cuda(recv, out)
+    GM, M = recv.shape
+    assert GM == G * M and recv.is_contiguous() and out.dtype == recv.dtype
+    assert out.shape[0] == M and out.shape[1] >= G * M and out.stride(1) == 1
+    eb = recv.element_size()
+    with torch.cuda.device(recv.device):
+        _check(lib().rap_unpack_blocks(ctypes.c_void_p(recv.data_ptr()), ctypes.c_void_p(out.data_ptr()),
+                                       G, M, out.stride(0) if M > 1 else G * M, eb, _stream(recv)),
+               "rap_unpack_blocks")
     return out

@@ -132,4 +132,23 @@ rap_status_t rap_congestion_trace(uint32_t w, uint64_t n_warps, const uint32_t *
                                         n_trials, d_hist, (cudaStream_t)stream));
 }
 
+rap_status_t rap_unpack_blocks(const void *d_recv, void *d_out, int64_t G, int64_t M, int64_t ld_out,
+                               uint32_t elem_bytes, void *stream) {
+    if (elem_bytes != 4 && elem_bytes != 8) return RAP_ERR_INVALID_ARG;
+    if (G < 0 || M < 0) return RAP_ERR_INVALID_ARG;
+    if (G == 0 || M == 0) return RAP_OK;
+    int64_t width;
+    if (!mul_ok(G, M, &width) || ld_out < width) return RAP_ERR_INVALID_ARG;
+    if (!d_recv || !d_out) return RAP_ERR_INVALID_ARG;
+    if ((uintptr_t)d_recv % elem_bytes || (uintptr_t)d_out % elem_bytes) return RAP_ERR_INVALID_ARG;
+    uintptr_t r_lo, r_hi, o_lo, o_hi;
+    int64_t rrows;
+    if (!mul_ok(G, M, &rrows)) return RAP_ERR_INVALID_ARG;
+    if (!extent((uintptr_t)d_recv, rrows, M, M, elem_bytes, &r_lo, &r_hi) ||
+        !extent((uintptr_t)d_out, M, width, ld_out, elem_bytes, &o_lo, &o_hi))
+        return RAP_ERR_INVALID_ARG;
+    if (r_lo < o_hi && o_lo < r_hi) return RAP_ERR_ALIAS;
+    return from_cuda(rapk::launch_unpack_blocks(d_recv, d_out, G, M, ld_out, elem_bytes, (cudaStream_t)stream));
+}
+
 }  // extern "C"

@@ -1,0 +1,52 @@
+// exchange.cu -- step T4 of the RAP hot path (BASELINE cfg5): the block unpack that follows the
+// NCCL all-to-all of the row-block-sharded transpose.  After rank g has transposed its M x N
+// row block (rap_transpose) and exchanged the M x M blocks, block s of the receive buffer is
+// (A[sM:(s+1)M, gM:(g+1)M])^T and belongs at columns sM..(s+1)M of the rank's output rows:
+//     out[x * ld_out + s*M + a] = recv[(s*M + x) * M + a],   0 <= s < G, 0 <= x, a < M.
+// A bandwidth-bound copy: 128-bit loads and stores when M and the pointers allow, one warp per
+// 512-byte run, persistent grid.
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "rap_internal.h"
+
+namespace rapk {
+
+// V = vector type; each block has M rows of Mv vectors; ld_v = output row pitch in vectors
+template <typename V>
+__global__ void __launch_bounds__(256) unpack_blocks_kernel(const V *__restrict__ recv, V *__restrict__ out,
+                                                            int64_t G, int64_t M, int64_t Mv, int64_t ld_v) {
+    // work item = one vector of the receive buffer, in receive order (coalesced reads)
+    const int64_t total = G * M * Mv;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t a = i % Mv;
+        const int64_t row = i / Mv;         // s*M + x
+        const int64_t s = row / M, x = row - s * M;
+        out[x * ld_v + s * Mv + a] = recv[i];
+    }
+}
+
+cudaError_t launch_unpack_blocks(const void *recv, void *out, int64_t G, int64_t M, int64_t ld_out,
+                                 uint32_t elem_bytes, cudaStream_t st) {
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const int grid = sms * 8;
+    const int64_t vb = 16;
+    const bool v16 = ((uintptr_t)recv % 16 == 0) && ((uintptr_t)out % 16 == 0) &&
+                     ((M * elem_bytes) % vb == 0) && ((ld_out * elem_bytes) % vb == 0);
+    if (v16) {
+        const int64_t k = vb / elem_bytes;
+        unpack_blocks_kernel<uint4><<<grid, 256, 0, st>>>((const uint4 *)recv, (uint4 *)out, G, M, M / k,
+                                                          ld_out / k);
+    } else if (elem_bytes == 8) {
+        unpack_blocks_kernel<uint64_t><<<grid, 256, 0, st>>>((const uint64_t *)recv, (uint64_t *)out, G, M, M,
+                                                             ld_out);
+    } else {
+        unpack_blocks_kernel<uint32_t><<<grid, 256, 0, st>>>((const uint32_t *)recv, (uint32_t *)out, G, M, M,
+                                                             ld_out);
+    }
+    return cudaGetLastError();
+}
+
+}  // namespace rapk

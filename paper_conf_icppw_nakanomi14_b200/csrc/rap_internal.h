@@ -46,4 +46,7 @@ cudaError_t launch_trace(uint32_t w, uint64_t n_warps, const uint32_t *cells, ui
                          uint64_t seed, uint64_t first, uint64_t n_trials, uint64_t *hist,
                          cudaStream_t st);
 
+cudaError_t launch_unpack_blocks(const void *recv, void *out, int64_t G, int64_t M, int64_t ld_out,
+                                 uint32_t elem_bytes, cudaStream_t st);
+
 }  // namespace rapk

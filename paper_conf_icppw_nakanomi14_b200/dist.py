@@ -1,0 +1,72 @@
+"""Multi-GPU paths of the RAP hot path (one process per GPU, torch.distributed over NCCL).
+
+Only two places shard:
+  * congestion_sweep -- trials are independent (counter-based draws: trial n is a pure function
+    of (seed, n)), so rank g sweeps the g-th contiguous slice of [first, first + N) and ONE
+    all-reduce (SUM, int64) of the histogram combines them.  Integer sums are order-free, so
+    the result is bit-identical to the one-GPU run and to the oracle for any world size.
+  * transpose_sharded -- BASELINE cfg5: A (N x N) is row-block sharded, rank g holding rows
+    gM..(g+1)M (M = N/G).  The local rap_transpose of the M x N shard yields N x M whose row
+    block s is exactly the M x M block rank s needs; one all-to-all exchanges them and
+    rap_unpack_blocks places the received blocks as rows gM..(g+1)M of A^T.
+`local` hooks exist only so the exchange logic can be exercised with the gloo backend on CPU
+(tests pass CPU stand-ins); by default every step is the CUDA library.
+"""
+from __future__ import annotations
+
+import torch
+import torch.distributed as dist
+
+from . import congestion_sweep as _sweep
+from . import transpose as _transpose
+from . import unpack_blocks as _unpack
+
+
+def trial_slice(n_trials: int, rank: int, world: int, first_trial: int = 0):
+    lo = first_trial + n_trials * rank // world
+    hi = first_trial + n_trials * (rank + 1) // world
+    return lo, hi - lo
+
+
+def congestion_sweep(n_trials: int, seed: int, group=None, first_trial: int = 0, local=None, **kw):
+    """All-reduced histogram of [first_trial, first_trial + n_trials) swept across the group."""
+    on = dist.is_initialized()
+    rank, world = (dist.get_rank(group), dist.get_world_size(group)) if on else (0, 1)
+    first, count = trial_slice(n_trials, rank, world, first_trial)
+    fn = local if local is not None else _sweep
+    h = fn(count, seed, first_trial=first, **kw)
+    if world > 1:
+        dist.all_reduce(h, op=dist.ReduceOp.SUM, group=group)
+    return h
+
+
+def transpose_sharded(shard: torch.Tensor, group=None, layout: str = "rap", seed: int = 0,
+                      out: torch.Tensor | None = None, local_transpose=None, local_unpack=None,
+                      work: dict | None = None) -> torch.Tensor:
+    """Rows gM..(g+1)M of A^T from rows gM..(g+1)M of A, for the whole group.
+
+    shard: [M, N] with N = world * M.  Returns out: [M, N].  `work` may carry preallocated
+    "send" / "recv" buffers ([N, M]) so repeated calls allocate nothing.
+    """
+    world = dist.get_world_size(group) if dist.is_initialized() else 1
+    M, N = shard.shape
+    if N != world * M:
+        raise ValueError(f"sharded transpose needs a square matrix: shard {M}x{N}, world {world}")
+    tr = local_transpose if local_transpose is not None else (
+        lambda x, o: _transpose(x, layout=layout, seed=seed, out=o))
+    if out is None:
+        out = torch.empty((M, N), dtype=shard.dtype, device=shard.device)
+    if world == 1:                                    # nothing to exchange: transpose in place
+        tr(shard, out)
+        return out
+    up = local_unpack if local_unpack is not None else (lambda r, o, G: _unpack(r, o, G))
+    work = {} if work is None else work
+    send = work.get("send")
+    if send is None or send.shape != (N, M) or send.dtype != shard.dtype or send.device != shard.device:
+        send = work["send"] = torch.empty((N, M), dtype=shard.dtype, device=shard.device)
+        work["recv"] = torch.empty_like(send)
+    recv = work["recv"]
+    tr(shard, send)                                   # T1-T3: local RAP transpose, M x N -> N x M
+    dist.all_to_all_single(recv, send, group=group)   # T4: M x M blocks, NCCL over NVLink
+    up(recv, out, world)                              # T4: place the blocks
+    return out

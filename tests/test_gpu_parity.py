@@ -263,3 +263,53 @@ def test_trace_small_w_and_invalid(rap, oracle):
     g = rap.congestion_trace(cells.cuda(), 7, seed=2, schemes=["rap", "raw"]).cpu().numpy()
     assert g[:, 0].tolist() == [7, 7]
     assert (g.sum(-1) == 13 * 7).all()
+
+
+# ------------------------------------------------------------------ T4 sharded transpose pieces
+@pytest.mark.parametrize("dtype", [torch.float32, torch.float64])
+@pytest.mark.parametrize("G,M", [(1, 64), (2, 96), (4, 64), (8, 33), (3, 50)])
+def test_sharded_transpose_emulated_on_one_gpu(rap, oracle, dtype, G, M):
+    # G virtual ranks on one device: local rap_transpose per shard, the all-to-all as block
+    # slicing, rap_unpack_blocks per rank; the union must equal the oracle's A^T.
+    N = G * M
+    A = workloads.random_bits(N, N, dtype, seed=G * 100 + M)
+    Ad = A.cuda()
+    sends = [rap.transpose(Ad[g * M:(g + 1) * M].contiguous(), layout="rap", seed=3) for g in range(G)]
+    outs = []
+    for g in range(G):
+        recv = torch.cat([sends[s][g * M:(g + 1) * M] for s in range(G)], 0).contiguous()
+        outs.append(rap.unpack_blocks(recv, torch.empty((M, N), dtype=dtype, device="cuda"), G))
+    got = torch.cat(outs, 0)
+    torch.cuda.synchronize()
+    assert np.array_equal(bits(got), oracle.transpose(bits(A)))
+
+
+def test_unpack_blocks_strided_output(rap):
+    G, M = 3, 40
+    recv = workloads.random_bits(G * M, M, torch.float32, seed=1).cuda()
+    big = torch.zeros((M, G * M + 7), dtype=torch.float32, device="cuda")
+    rap.unpack_blocks(recv, big, G)
+    r = recv.view(torch.int32).view(G, M, M).cpu()
+    b = big.view(torch.int32).cpu()
+    for s in range(G):
+        assert torch.equal(b[:, s * M:(s + 1) * M], r[s])
+    assert not b[:, G * M:].any()
+
+
+def test_dist_world1_nccl(rap, oracle):
+    # the dist entry points under a real NCCL process group of size 1 (the 1-GPU box)
+    import os
+    import torch.distributed as dist
+    from paper_conf_icppw_nakanomi14_b200 import dist as rdist
+    os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+    os.environ.setdefault("MASTER_PORT", "29561")
+    dist.init_process_group("nccl", rank=0, world_size=1)
+    try:
+        h = rdist.congestion_sweep(50_000, seed=2, first_trial=3)
+        o = oracle.sweep(32, ALL_PAT, ["raw", "ras", "rap"], 2, 3, 50_000)
+        assert np.array_equal(h.cpu().numpy().astype(np.uint64), o)
+        A = workloads.random_bits(256, 256, torch.float32, seed=4)
+        out = rdist.transpose_sharded(A.cuda())
+        assert np.array_equal(bits(out), oracle.transpose(bits(A)))
+    finally:
+        dist.destroy_process_group()
