@@ -13,6 +13,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <atomic>
+
 #include "rap_rng.cuh"
 #include "rap_internal.h"
 
@@ -195,11 +197,21 @@ __device__ __forceinline__ uint32_t plane_value(const uint32_t (&q)[5], uint32_t
     return v;
 }
 
+// (x mod w) for x < 2w; a mask when w is a compile-time power of two
 template <int W>
+__device__ __forceinline__ uint32_t mod_w(uint32_t x, uint32_t w) {
+    if (W && !(W & (W - 1))) return x & (uint32_t)(W - 1);
+    return x >= w ? x - w : x;
+}
+
+// PM / SM: pattern / scheme masks fixed at compile time (0 = take the runtime masks), so the
+// common configurations evaluate with no mask tests and constant evaluation slots.
+template <int W, uint32_t PM, uint32_t SM>
 __global__ void __launch_bounds__(kSweepWarpsV2 * 32)
-sweep_kernel(uint32_t w_rt, uint32_t pmask, uint32_t smask, uint64_t seed, uint64_t first,
+sweep_kernel(uint32_t w_rt, uint32_t pmask_rt, uint32_t smask_rt, uint64_t seed, uint64_t first,
              uint64_t n_trials, uint64_t *__restrict__ hist) {
     const uint32_t w = W ? (uint32_t)W : w_rt;
+    const uint32_t pmask = PM ? PM : pmask_rt, smask = SM ? SM : smask_rt;
     __shared__ uint32_t sh_hist[kMaxBins];
     __shared__ uint32_t sh_tr[kSweepWarpsV2][32 * 33];
     const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
@@ -290,7 +302,11 @@ sweep_kernel(uint32_t w_rt, uint32_t pmask, uint32_t smask, uint64_t seed, uint6
                             break;
                         }
                         const uint32_t sh = (s == RAP_SCHEME_RAP) ? shP : shR;
-                        const uint32_t bank = bank_of(s, row, col, sh, w);
+                        uint32_t bank;
+                        if (s == RAP_SCHEME_RAS || s == RAP_SCHEME_RAP) bank = mod_w<W>(col + sh, w);
+                        else if (s == RAP_SCHEME_PAD) bank = mod_w<W>(row + col, w);
+                        else if (s == RAP_SCHEME_XOR) bank = col ^ row;
+                        else bank = col;
                         c = max_bank_load(bank, p == RAP_PAT_RANDOM ? leaders : active, ls);
                     }
                     if (p == RAP_PAT_STRIDE) c_stride[s] = c;
@@ -440,17 +456,29 @@ perm_gen_kernel(uint64_t seed, uint64_t first, uint64_t count, uint32_t w, uint8
 
 // ------------------------------------------------------------------ launchers
 static int sm_count() {
-    int dev = 0, sms = 148;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    static std::atomic<int> cache[kMaxDevices];
+    int dev = 0, sms = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= kMaxDevices) return 148;
+    sms = cache[dev].load(std::memory_order_relaxed);
+    if (sms == 0) {
+        if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || sms <= 0) sms = 148;
+        cache[dev].store(sms, std::memory_order_relaxed);
+    }
     return sms;
 }
 
-template <typename K>
-static int resident_ctas(K kernel, int threads) {
-    int occ = 1;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kernel, threads, 0);
-    return (occ < 1 ? 1 : occ) * sm_count();
+// resident CTAs of `kernel` per device (occupancy query cached per kernel and device)
+template <auto Kernel>
+static int resident_ctas(int threads) {
+    static std::atomic<int> cache[kMaxDevices];
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= kMaxDevices) dev = 0;
+    int occ = cache[dev].load(std::memory_order_relaxed);
+    if (occ == 0) {
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, Kernel, threads, 0) != cudaSuccess || occ < 1) occ = 1;
+        cache[dev].store(occ, std::memory_order_relaxed);
+    }
+    return occ * sm_count();
 }
 
 static int clamp_grid(uint64_t items, int per_cta, int cap) {
@@ -458,34 +486,40 @@ static int clamp_grid(uint64_t items, int per_cta, int cap) {
     return (int)(want < (uint64_t)cap ? (want ? want : 1) : (uint64_t)cap);
 }
 
-template <typename K>
-static void run_sweep(K kernel, int warps_per_cta, uint64_t trials_per_item, uint32_t w, uint32_t pmask,
+template <auto Kernel>
+static void run_sweep(int warps_per_cta, uint64_t trials_per_item, uint32_t w, uint32_t pmask,
                       uint32_t smask, uint64_t seed, uint64_t first, uint64_t n_trials, uint64_t *hist,
                       cudaStream_t st) {
     const int threads = warps_per_cta * 32;
     const uint64_t items = (n_trials + trials_per_item - 1) / trials_per_item;
-    const int grid = clamp_grid(items, warps_per_cta, resident_ctas(kernel, threads));
+    const int grid = clamp_grid(items, warps_per_cta, resident_ctas<Kernel>(threads));
     // u32 shared counters: keep the trials counted by one CTA below 2^31 per launch
     const uint64_t chunk = (uint64_t)grid * (1ull << 31);
     for (uint64_t done = 0; done < n_trials; done += chunk) {
         const uint64_t cnt = (n_trials - done < chunk) ? n_trials - done : chunk;
-        kernel<<<grid, threads, 0, st>>>(w, pmask, smask, seed, first + done, cnt, hist);
+        Kernel<<<grid, threads, 0, st>>>(w, pmask, smask, seed, first + done, cnt, hist);
     }
 }
 
 cudaError_t launch_sweep(uint32_t w, uint32_t pmask, uint32_t smask, uint64_t seed, uint64_t first,
                          uint64_t n_trials, uint64_t *hist, cudaStream_t st) {
     if (n_trials == 0) return cudaSuccess;
-    if (w == 32) run_sweep(sweep_kernel<32>, kSweepWarpsV2, 32, w, pmask, smask, seed, first, n_trials, hist, st);
-    else run_sweep(sweep_kernel<0>, kSweepWarpsV2, 32, w, pmask, smask, seed, first, n_trials, hist, st);
+    if (w == 32 && pmask == 31u && smask == 7u)
+        run_sweep<sweep_kernel<32, 31u, 7u>>(kSweepWarpsV2, 32, w, pmask, smask, seed, first, n_trials, hist, st);
+    else if (w == 32 && pmask == 31u && smask == 31u)
+        run_sweep<sweep_kernel<32, 31u, 31u>>(kSweepWarpsV2, 32, w, pmask, smask, seed, first, n_trials, hist, st);
+    else if (w == 32)
+        run_sweep<sweep_kernel<32, 0u, 0u>>(kSweepWarpsV2, 32, w, pmask, smask, seed, first, n_trials, hist, st);
+    else
+        run_sweep<sweep_kernel<0, 0u, 0u>>(kSweepWarpsV2, 32, w, pmask, smask, seed, first, n_trials, hist, st);
     return cudaGetLastError();
 }
 
 cudaError_t launch_sweep_match(uint32_t w, uint32_t pmask, uint32_t smask, uint64_t seed, uint64_t first,
                                uint64_t n_trials, uint64_t *hist, cudaStream_t st) {
     if (n_trials == 0) return cudaSuccess;
-    if (w == 32) run_sweep(sweep_match_kernel<32>, kSweepWarps, 1, w, pmask, smask, seed, first, n_trials, hist, st);
-    else run_sweep(sweep_match_kernel<0>, kSweepWarps, 1, w, pmask, smask, seed, first, n_trials, hist, st);
+    if (w == 32) run_sweep<sweep_match_kernel<32>>(kSweepWarps, 1, w, pmask, smask, seed, first, n_trials, hist, st);
+    else run_sweep<sweep_match_kernel<0>>(kSweepWarps, 1, w, pmask, smask, seed, first, n_trials, hist, st);
     return cudaGetLastError();
 }
 
@@ -495,7 +529,7 @@ cudaError_t launch_trace(uint32_t w, uint64_t n_warps, const uint32_t *cells, ui
     if (n_trials == 0 || n_warps == 0) return cudaSuccess;
     const int threads = kSweepWarps * 32;
     const uint64_t nchunks = (n_warps + kTraceChunk - 1) / kTraceChunk;
-    const int grid = clamp_grid(n_trials * nchunks, kSweepWarps, resident_ctas(trace_kernel, threads));
+    const int grid = clamp_grid(n_trials * nchunks, kSweepWarps, resident_ctas<trace_kernel>(threads));
     // counts per warp <= items_per_warp * kTraceChunk; chunk the trial range to stay < 2^31
     const uint64_t trials_chunk = ((uint64_t)grid * kSweepWarps * ((1ull << 31) / kTraceChunk)) / nchunks + 1;
     for (uint64_t done = 0; done < n_trials; done += trials_chunk) {
@@ -508,7 +542,7 @@ cudaError_t launch_trace(uint32_t w, uint64_t n_warps, const uint32_t *cells, ui
 cudaError_t launch_congestion(uint32_t w, uint64_t n_warps, const uint32_t *rows, const uint32_t *cols,
                               int scheme, const uint32_t *shift, uint32_t *out, cudaStream_t st) {
     if (n_warps == 0) return cudaSuccess;
-    const int grid = clamp_grid(n_warps, 8, resident_ctas(congestion_kernel, 256));
+    const int grid = clamp_grid(n_warps, 8, resident_ctas<congestion_kernel>(256));
     congestion_kernel<<<grid, 256, 0, st>>>(w, n_warps, rows, cols, scheme, shift, out);
     return cudaGetLastError();
 }
@@ -516,7 +550,7 @@ cudaError_t launch_congestion(uint32_t w, uint64_t n_warps, const uint32_t *rows
 cudaError_t launch_perm_gen(uint64_t seed, uint64_t first, uint64_t count, uint32_t w, uint8_t *out,
                             cudaStream_t st) {
     if (count == 0) return cudaSuccess;
-    const int grid = clamp_grid(count, 8, resident_ctas(perm_gen_kernel, 256));
+    const int grid = clamp_grid(count, 8, resident_ctas<perm_gen_kernel>(256));
     perm_gen_kernel<<<grid, 256, 0, st>>>(seed, first, count, w, out);
     return cudaGetLastError();
 }

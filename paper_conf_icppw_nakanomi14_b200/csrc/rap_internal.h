@@ -8,6 +8,8 @@
 
 namespace rapk {
 
+constexpr int kMaxDevices = 64;
+
 // Launch-shape knobs of the transpose (defaults chosen by tools/tune_transpose.cu on B200).
 struct TransposeTuning {
     uint32_t group = 0;   // tile-rows per traversal group (0 = row-major tile order)

@@ -23,6 +23,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <atomic>
+
 #include "rap_rng.cuh"
 #include "rap_internal.h"
 
@@ -236,17 +238,38 @@ transpose_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, i
 }
 
 // ------------------------------------------------------------------ launchers
+// Host-side launch shape, cached per kernel instantiation and device: the dynamic-smem
+// attribute and the occupancy query run once, so a launch costs one cudaGetDevice + one launch.
+struct ShapeCache {
+    std::atomic<int> occ[kMaxDevices];      // 0 = not yet known
+    std::atomic<int> sms[kMaxDevices];
+};
+
 template <typename K>
-static int grid_for(K kernel, int threads, size_t smem, int64_t ntiles, int warps_per_cta, int ctas_per_sm) {
-    int dev = 0, sms = 148, occ = 1;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kernel, threads, smem);
-    if (occ < 1) occ = 1;
+static cudaError_t grid_for(K kernel, ShapeCache &cache, int threads, size_t smem, int64_t ntiles,
+                            int warps_per_cta, int ctas_per_sm, int *grid_out) {
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    if (dev < 0 || dev >= kMaxDevices) return cudaErrorInvalidDevice;
+    int occ = cache.occ[dev].load(std::memory_order_relaxed);
+    int sms = cache.sms[dev].load(std::memory_order_relaxed);
+    if (occ == 0) {
+        e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e != cudaSuccess) return e;
+        e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        if (e != cudaSuccess) return e;
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kernel, threads, smem);
+        if (e != cudaSuccess) return e;
+        if (occ < 1) occ = 1;
+        cache.sms[dev].store(sms, std::memory_order_relaxed);
+        cache.occ[dev].store(occ, std::memory_order_relaxed);
+    }
     if (ctas_per_sm > 0 && ctas_per_sm < occ) occ = ctas_per_sm;
     const int64_t want = (ntiles + warps_per_cta - 1) / warps_per_cta;
     const int64_t cap = (int64_t)sms * occ;
-    return (int)(want < cap ? want : cap);
+    *grid_out = (int)(want < cap ? want : cap);
+    return cudaSuccess;
 }
 
 TransposeTuning default_tuning(uint32_t elem_bytes) {
@@ -264,10 +287,11 @@ static cudaError_t launch_one(const void *src, void *dst, int64_t rows, int64_t 
     const uint32_t tiles_r = (uint32_t)((rows + 31) / 32), tiles_c = (uint32_t)((cols + 31) / 32);
     const uint32_t ntiles = tiles_r * tiles_c;
     auto k = transpose_kernel<L, EW, VEC, DEPTH, MINB>;
+    static ShapeCache cache;
     const size_t smem = sizeof(uint32_t) * warp_smem_words<L, EW>() * kWarpsT;
-    cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    int grid = 0;
+    const cudaError_t e = grid_for(k, cache, kWarpsT * 32, smem, ntiles, kWarpsT, tu.ctas_per_sm, &grid);
     if (e != cudaSuccess) return e;
-    const int grid = grid_for(k, kWarpsT * 32, smem, ntiles, kWarpsT, tu.ctas_per_sm);
     k<<<grid, kWarpsT * 32, smem, st>>>((const uint32_t *)src, (uint32_t *)dst, rows, cols, ld_src,
                                         ld_dst, seed, tiles_r, tiles_c, ntiles, tu.group);
     return cudaGetLastError();

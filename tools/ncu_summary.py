@@ -1,0 +1,94 @@
+"""Summarise ncu --set full captures (gpurun_out/prof_*.ncu-rep) into profiles/ncu_summary.json.
+
+Run here (no GPU needed):  python tools/ncu_summary.py gpurun_out profiles/ncu_summary.json r01
+Per kernel: duration, DRAM bytes (read + write) per launch, shared-memory wavefronts per request
+for loads and stores, bank conflicts, issue-slot utilisation, occupancy, registers.
+"""
+import csv
+import io
+import json
+import os
+import subprocess
+import sys
+
+CAPTURES = {
+    "transpose_b32_rap": "prof_t32_rap", "transpose_b32_raw": "prof_t32_raw",
+    "transpose_b32_pad": "prof_t32_pad", "transpose_b32_xor": "prof_t32_xor",
+    "transpose_b32_ras": "prof_t32_ras", "transpose_b64_rap": "prof_t64_rap",
+    "sweep_w32": "prof_sweep", "sweep_w32_match": "prof_sweep_match",
+}
+
+WANT = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum",
+        "l1tex__data_pipe_lsu_wavefronts_mem_shared_op_ld.sum",
+        "l1tex__data_pipe_lsu_wavefronts_mem_shared_op_st.sum",
+        "smsp__sass_inst_executed_op_shared_ld.sum", "smsp__sass_inst_executed_op_shared_st.sum",
+        "l1tex__data_bank_conflicts_pipe_lsu_mem_shared_op_ld.sum",
+        "l1tex__data_bank_conflicts_pipe_lsu_mem_shared_op_st.sum",
+        "smsp__issue_active.avg.pct_of_peak_sustained_active",
+        "sm__warps_active.avg.pct_of_peak_sustained_active", "launch__registers_per_thread",
+        "launch__grid_size", "launch__block_size", "dram__throughput.avg.pct_of_peak_sustained_elapsed",
+        "sm__throughput.avg.pct_of_peak_sustained_elapsed", "smsp__inst_executed.sum"]
+
+SCALE = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "ns": 1e-9, "us": 1e-6, "ms": 1e-3,
+         "nsecond": 1e-9, "usecond": 1e-6,
+         "msecond": 1e-3, "second": 1.0}
+
+
+def raw_metrics(rep):
+    out = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    rows = list(csv.reader(io.StringIO(out)))
+    head, units, vals = rows[0], rows[1], rows[2]
+    d = {}
+    for h, u, v in zip(head, units, vals):
+        if h in WANT:
+            try:
+                x = float(v.replace(",", ""))
+            except ValueError:
+                continue
+            d[h] = x * SCALE.get(u, 1.0)
+    d["kernel_name"] = vals[head.index("Kernel Name")] if "Kernel Name" in head else None
+    return d
+
+
+def main(src_dir, dst, tag):
+    kernels = {}
+    for key, stem in CAPTURES.items():
+        rep = os.path.join(src_dir, stem + ".ncu-rep")
+        if not os.path.exists(rep):
+            continue
+        m = raw_metrics(rep)
+        ld_w = m.get("l1tex__data_pipe_lsu_wavefronts_mem_shared_op_ld.sum")
+        st_w = m.get("l1tex__data_pipe_lsu_wavefronts_mem_shared_op_st.sum")
+        ld_i = m.get("smsp__sass_inst_executed_op_shared_ld.sum")
+        st_i = m.get("smsp__sass_inst_executed_op_shared_st.sum")
+        dram = (m.get("dram__bytes_read.sum") or 0) + (m.get("dram__bytes_write.sum") or 0)
+        kernels[key] = {
+            "source": f"profiles/{tag}_{stem}.ncu-rep (ncu --set full --clock-control none)",
+            "kernel_name": m.get("kernel_name"),
+            "duration_us_cold": m.get("gpu__time_duration.sum", 0) * 1e6,
+            "dram_bytes_read": m.get("dram__bytes_read.sum"), "dram_bytes_write": m.get("dram__bytes_write.sum"),
+            "dram_bytes_per_launch": dram or None,
+            "dram_throughput_pct": m.get("dram__throughput.avg.pct_of_peak_sustained_elapsed"),
+            "smem_wavefronts_per_request": {"ld": ld_w / ld_i if ld_i else None,
+                                            "st": st_w / st_i if st_i else None},
+            "smem_bank_conflicts": {"ld": m.get("l1tex__data_bank_conflicts_pipe_lsu_mem_shared_op_ld.sum"),
+                                    "st": m.get("l1tex__data_bank_conflicts_pipe_lsu_mem_shared_op_st.sum")},
+            "issue_active_frac": (m.get("smsp__issue_active.avg.pct_of_peak_sustained_active") or 0) / 100,
+            "warps_active_pct": m.get("sm__warps_active.avg.pct_of_peak_sustained_active"),
+            "registers": m.get("launch__registers_per_thread"), "grid": m.get("launch__grid_size"),
+            "block": m.get("launch__block_size"), "instructions": m.get("smsp__inst_executed.sum"),
+        }
+    os.makedirs(os.path.dirname(dst), exist_ok=True)
+    json.dump({"round": tag, "note": "cold-cache, serialised ncu replays: compare shares and ratios, "
+                                     "not absolute times; dram bytes exclude lines still dirty in L2 at exit",
+               "kernels": kernels}, open(dst, "w"), indent=1)
+    for k, v in kernels.items():
+        print(f"{k:20s} {v['duration_us_cold']:8.1f} us  dram {v['dram_bytes_per_launch'] or 0:.3e} B  "
+              f"smem wf/req ld {v['smem_wavefronts_per_request']['ld']} st {v['smem_wavefronts_per_request']['st']}  "
+              f"issue {v['issue_active_frac']:.3f} regs {v['registers']}")
+
+
+if __name__ == "__main__":
+    main(sys.argv[1] if len(sys.argv) > 1 else "gpurun_out",
+         sys.argv[2] if len(sys.argv) > 2 else "profiles/ncu_summary.json",
+         sys.argv[3] if len(sys.argv) > 3 else "r01")
