@@ -46,7 +46,7 @@ def parse():
     p.add_argument("--impl", default="mine", choices=["mine", "reference"])
     p.add_argument("--workload", default="default",
                    choices=["default", "sweep", "cfg4", "tile", "layouts", "dist"])
-    p.add_argument("--sweep-trials", type=int, default=1 << 24)
+    p.add_argument("--sweep-trials", type=int, default=1 << 16)
     p.add_argument("--sweep-algo", default="default", choices=["default", "match"])
     p.add_argument("--layout", default="rap")
     p.add_argument("--no-e2e", action="store_true")
@@ -192,6 +192,20 @@ def cpu_baseline_sweep():
     el = time.perf_counter() - t0
     return {"value": n * reps / el, "unit": "trials/s", "cores": threads, "kind": "oracle",
             "sample": f"{n * reps} trials of the w=32 sweep (5 patterns x RAW/RAS/RAP) in {el:.1f} s"}
+
+
+def sweep_roofline(tps: float, clocks: dict):
+    """ALU roofline of the sweep: warp instructions per trial (ncu) x trials/s against the issue
+    peak 148 SMs x 4 schedulers x 1 warp-instruction/clk x SM clock."""
+    prof = load_profile("sweep_w32") or {}
+    ipt = prof.get("warp_instructions_per_trial")
+    mhz = (clocks or {}).get("sm_max_mhz") or 1965.0
+    peak = 148 * 4 * mhz * 1e6
+    ach = ipt * tps if ipt else None
+    return {"bound": "alu", "achieved": ach, "peak": peak, "unit": "warp-instructions/s",
+            "frac": ach / peak if ach else None, "traffic": None,
+            "warp_instructions_per_trial": ipt, "profile": prof.get("source"),
+            "issue_active_frac_ncu": prof.get("issue_active_frac")}
 
 
 def reduce_over_ranks(x: float, world: int, dev, op: str) -> float:
@@ -358,18 +372,21 @@ def main():
         line["sweep"] = {"trials_per_s": tps, "trials_per_step": S * world, "w": 32, "algo": args.sweep_algo,
                          "E_ras_stride": E(h[1, 1]), "E_rap_diagonal": E(h[2, 2]), "E_random": E(h[3, 2]),
                          "E_raw_malicious": E(h[4, 0]), "E_rap_stride": E(h[1, 2]),
-                         "kernel_ms_median": statistics.median(r["s_ms"])}
+                         "kernel_ms_median": statistics.median(r["s_ms"]),
+                         "roofline": sweep_roofline(tps / world, r["clocks"])}
         if not do_t:
             line.update(value=tps, unit="trials/s",
                         config={"workload": "cfg2 w=32 congestion sweep, 5 patterns x RAW/RAS/RAP",
                                 "trials_per_step": S * world,
                                 "parallelism": (f"trial ranges x{world} + NCCL all-reduce" if world > 1
                                                 else "single GPU")})
-            prof = load_profile("sweep_w32") or {}
-            line["roofline"] = {"bound": "alu", "achieved": prof.get("issue_active_frac"), "peak": 1.0,
-                                "unit": "fraction of issue slots", "frac": prof.get("issue_active_frac"),
-                                "traffic": None, "profile": prof.get("source"),
-                                "note": "issue-bound integer kernel: achieved = smsp__issue_active from ncu"}
+            line["roofline"] = sweep_roofline(tps / world, r["clocks"])
+    if do_t and do_s:
+        t_share = r["t_sum"] / max(r["t_sum"] + r["s_sum"], 1e-9)
+        line["kernel_time_share"] = {"transpose": t_share, "sweep": 1 - t_share}
+        if t_share < 0.5:                       # the sweep dominates this step: report its roofline
+            line["roofline_transpose"] = line["roofline"]
+            line["roofline"] = line["sweep"]["roofline"]
     line["clocks"] = r["clocks"]
     line["gpu_launches"] = int(reduce_over_ranks(r["launches"], world, dev, "sum"))
 

@@ -18,6 +18,12 @@ CAPTURES = {
     "sweep_w32": "prof_sweep", "sweep_w32_match": "prof_sweep_match",
 }
 
+# work units per captured launch (tools/gpu_profile.sh command lines)
+UNITS = {"sweep_w32": ("trials", 8388608), "sweep_w32_match": ("trials", 4194304),
+         "transpose_b32_rap": ("bytes", 2 * 8192 * 8192 * 4), "transpose_b32_raw": ("bytes", 2 * 8192 * 8192 * 4),
+         "transpose_b32_pad": ("bytes", 2 * 8192 * 8192 * 4), "transpose_b32_xor": ("bytes", 2 * 8192 * 8192 * 4),
+         "transpose_b32_ras": ("bytes", 2 * 8192 * 8192 * 4), "transpose_b64_rap": ("bytes", 2 * 16384 * 16384 * 8)}
+
 WANT = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum",
         "l1tex__data_pipe_lsu_wavefronts_mem_shared_op_ld.sum",
         "l1tex__data_pipe_lsu_wavefronts_mem_shared_op_st.sum",
@@ -78,6 +84,11 @@ def main(src_dir, dst, tag):
             "registers": m.get("launch__registers_per_thread"), "grid": m.get("launch__grid_size"),
             "block": m.get("launch__block_size"), "instructions": m.get("smsp__inst_executed.sum"),
         }
+        if key in UNITS:
+            unit, n = UNITS[key]
+            kernels[key]["units_per_launch"] = {unit: n}
+            if m.get("smsp__inst_executed.sum"):
+                kernels[key][f"warp_instructions_per_{unit[:-1]}"] = m["smsp__inst_executed.sum"] / n
     os.makedirs(os.path.dirname(dst), exist_ok=True)
     json.dump({"round": tag, "note": "cold-cache, serialised ncu replays: compare shares and ratios, "
                                      "not absolute times; dram bytes exclude lines still dirty in L2 at exit",
