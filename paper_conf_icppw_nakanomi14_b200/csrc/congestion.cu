@@ -324,6 +324,192 @@ sweep_kernel(uint32_t w_rt, uint32_t pmask_rt, uint32_t smask_rt, uint64_t seed,
         if (sh_hist[b]) atomicAdd((unsigned long long *)(hist + b), (unsigned long long)sh_hist[b]);
 }
 
+// ------------------------------------------------------------------ C1-C4 sweep, w = 32
+// Same two phases as sweep_kernel, but for w = 32 every bank mask B_b (bit t = bit b of the bank
+// of lane t) is built without per-lane arithmetic where the paper's patterns allow it:
+//   * the broadcast permutation planes ARE the masks of the RAP stride access (bank = P[t]);
+//   * rotations (contiguous access: bank = t + s) are funnel-shift rotations of the constant
+//     lane-index masks;
+//   * the diagonal access (bank = t + P[t] mod 32) is a 5-bit bit-sliced ripple-carry add;
+//   * only data-dependent banks (random cells) take 5 ballots.
+// The congestion is then popc / reduce-max over lane v's mask AND_b (v_b ? B_b : ~B_b) as before.
+__device__ __forceinline__ uint32_t lane_bits(int b) {
+    return b == 0 ? 0xAAAAAAAAu : b == 1 ? 0xCCCCCCCCu : b == 2 ? 0xF0F0F0F0u : b == 3 ? 0xFF00FF00u : 0xFFFF0000u;
+}
+
+struct BankMask { uint32_t b[5]; };
+
+__device__ __forceinline__ BankMask masks_ballot(uint32_t bank) {
+    BankMask B;
+#pragma unroll
+    for (int k = 0; k < 5; ++k) B.b[k] = __ballot_sync(kFull, (bank >> k) & 1u);
+    return B;
+}
+
+__device__ __forceinline__ BankMask masks_lane() {           // bank = t
+    BankMask B;
+#pragma unroll
+    for (int k = 0; k < 5; ++k) B.b[k] = lane_bits(k);
+    return B;
+}
+
+__device__ __forceinline__ BankMask masks_const(uint32_t v) {   // every lane the same bank v
+    BankMask B;
+#pragma unroll
+    for (int k = 0; k < 5; ++k) B.b[k] = ((v >> k) & 1u) ? kFull : 0u;
+    return B;
+}
+
+__device__ __forceinline__ BankMask masks_rot(uint32_t s) {     // bank = (t + s) mod 32
+    BankMask B;
+#pragma unroll
+    for (int k = 0; k < 5; ++k) B.b[k] = __funnelshift_r(lane_bits(k), lane_bits(k), s);
+    return B;
+}
+
+__device__ __forceinline__ BankMask masks_add(const BankMask &X, const BankMask &Y) {   // (x + y) mod 32
+    BankMask S;
+    uint32_t c = 0;
+#pragma unroll
+    for (int k = 0; k < 5; ++k) {
+        S.b[k] = X.b[k] ^ Y.b[k] ^ c;
+        c = (X.b[k] & Y.b[k]) | (c & (X.b[k] ^ Y.b[k]));
+    }
+    return S;
+}
+
+__device__ __forceinline__ uint32_t max_load(const BankMask &B, uint32_t counted, const LaneSel &ls) {
+    uint32_t m = counted;
+#pragma unroll
+    for (int k = 0; k < 5; ++k) m &= B.b[k] ^ ls.nsel[k];
+    return __reduce_max_sync(kFull, __popc(m));
+}
+
+template <uint32_t PM, uint32_t SM>
+__global__ void __launch_bounds__(kSweepWarpsV2 * 32)
+sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint64_t n_trials,
+               uint64_t *__restrict__ hist) {
+    constexpr uint32_t w = 32;
+    constexpr uint32_t npat = __builtin_popcount(PM), nsch = __builtin_popcount(SM);
+    constexpr uint32_t nbins = npat * nsch * (w + 1);
+    constexpr bool any_random = (PM >> RAP_PAT_RANDOM) & 1u;
+    constexpr bool need_r = (SM >> RAP_SCHEME_RAS) & 1u;
+    __shared__ uint32_t sh_hist[nbins];
+    __shared__ uint32_t sh_tr[kSweepWarpsV2][32 * 33];
+    __shared__ uint32_t sh_res[kSweepWarpsV2][32];
+    const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
+    for (uint32_t b = threadIdx.x; b < nbins; b += blockDim.x) sh_hist[b] = 0;
+    __syncthreads();
+    const LaneSel ls(lane);
+    uint32_t *tr = sh_tr[warp];
+    uint32_t *res = sh_res[warp];
+
+    const uint64_t nbatch = (n_trials + 31) / 32;
+    const uint64_t stride = (uint64_t)gridDim.x * kSweepWarpsV2;
+    for (uint64_t bt = (uint64_t)blockIdx.x * kSweepWarpsV2 + warp; bt < nbatch; bt += stride) {
+        const uint64_t n0 = first + bt * 32;
+        const uint32_t nvalid = (uint32_t)min((uint64_t)32, n_trials - bt * 32);
+        // ---- lane mode: trial n0 + lane
+        uint32_t pl[5];
+        lane_perm_planes<32>(seed, n0 + lane, w, pl);
+        const uint32_t p0_lane = plane_value(pl, 0);              // P[0] of this lane's trial
+        uint32_t r0_lane = 0;
+        if (need_r || any_random) {
+#pragma unroll
+            for (int blk = 0; blk < 8; ++blk) {
+                const uint4 cr = need_r ? philox_block(seed, n0 + lane, kDomainRAS, blk) : make_uint4(0, 0, 0, 0);
+                const uint4 cc = any_random ? philox_block(seed, n0 + lane, kDomainRandom, blk) : make_uint4(0, 0, 0, 0);
+                const uint32_t ur[4] = {cr.x, cr.y, cr.z, cr.w};
+                const uint32_t uc[4] = {cc.x, cc.y, cc.z, cc.w};
+#pragma unroll
+                for (int i = 0; i < 4; ++i) {
+                    const uint32_t r = ur[i] >> 27, cell = uc[i] >> 22;   // floor(u*32/2^32), floor(u*1024/2^32)
+                    if (blk == 0 && i == 0) r0_lane = r;
+                    tr[(4 * blk + i) * 33 + lane] = (r << 10) | cell;
+                }
+            }
+        }
+        __syncwarp();
+        // ---- warp mode: lane t is DMM thread t of trial n0 + m
+        for (uint32_t m = 0; m < nvalid; ++m) {
+            BankMask Pm;                                           // bit t = bit b of P[t]
+#pragma unroll
+            for (int b = 0; b < 5; ++b) Pm.b[b] = __shfl_sync(kFull, pl[b], m);
+            const uint32_t P0 = __shfl_sync(kFull, p0_lane, m);
+            const uint32_t r0 = __shfl_sync(kFull, r0_lane, m);
+            const uint32_t packed = tr[lane * 33 + m];
+            const uint32_t rt = packed >> 10;
+            BankMask Rm;
+            if (need_r) Rm = masks_ballot(rt);                      // bit t = bit b of r[t]
+            uint32_t rrow = 0, rcol = 0, Pr = 0, rr = 0, leaders = kFull;
+            if (any_random) {
+                const uint32_t cell = packed & 1023u;
+                rrow = cell >> 5;
+                rcol = cell & 31u;
+                Pr = plane_value(Pm.b, rrow);                      // P[row_t]
+                rr = __shfl_sync(kFull, rt, rrow);                 // r[row_t]
+                const uint32_t same = __match_any_sync(kFull, cell);   // merged requests
+                leaders = __ballot_sync(kFull, (uint32_t)(__ffs(same) - 1) == lane);
+            }
+            uint32_t e = 0;
+            uint32_t c_stride[5] = {0, 0, 0, 0, 0}, c_diag[5] = {0, 0, 0, 0, 0};
+#pragma unroll
+            for (int p = 0; p < 5; ++p) {
+                if (!((PM >> p) & 1u)) continue;
+#pragma unroll
+                for (int s = 0; s < 5; ++s) {
+                    if (!((SM >> s) & 1u)) continue;
+                    uint32_t c;
+                    if (p == RAP_PAT_MALICIOUS && (s == RAP_SCHEME_RAW || s == RAP_SCHEME_RAS) &&
+                        ((PM >> RAP_PAT_STRIDE) & 1u)) {
+                        c = c_stride[s];                            // reading iii: = stride access
+                    } else if (p == RAP_PAT_MALICIOUS && (s == RAP_SCHEME_RAP || s == RAP_SCHEME_XOR) &&
+                               ((PM >> RAP_PAT_DIAGONAL) & 1u)) {
+                        c = c_diag[s];                              // reading iii: = diagonal access
+                    } else {
+                        const int pp = (p == RAP_PAT_MALICIOUS)
+                            ? ((s == RAP_SCHEME_RAW || s == RAP_SCHEME_RAS) ? RAP_PAT_STRIDE
+                               : (s == RAP_SCHEME_PAD) ? -1 : RAP_PAT_DIAGONAL) : p;
+                        BankMask B;
+                        if (s == RAP_SCHEME_RAW) {
+                            B = (pp == RAP_PAT_STRIDE) ? masks_const(0)
+                              : (pp == RAP_PAT_RANDOM) ? masks_ballot(rcol) : masks_lane();
+                        } else if (s == RAP_SCHEME_RAS || s == RAP_SCHEME_RAP) {
+                            const bool isp = (s == RAP_SCHEME_RAP);
+                            if (pp == RAP_PAT_CONTIGUOUS) B = masks_rot(isp ? P0 : r0);
+                            else if (pp == RAP_PAT_STRIDE) B = isp ? Pm : Rm;
+                            else if (pp == RAP_PAT_DIAGONAL) B = masks_add(masks_lane(), isp ? Pm : Rm);
+                            else B = masks_ballot((rcol + (isp ? Pr : rr)) & 31u);
+                        } else {                                    // PAD / XOR: per-lane bank
+                            uint32_t row, col;
+                            switch (pp) {
+                            case RAP_PAT_CONTIGUOUS: row = 0; col = lane; break;
+                            case RAP_PAT_STRIDE: row = lane; col = 0; break;
+                            case RAP_PAT_DIAGONAL: row = lane; col = lane; break;
+                            case RAP_PAT_RANDOM: row = rrow; col = rcol; break;
+                            default: row = lane; col = (32u - lane) & 31u; break;   // PAD anti-diagonal
+                            }
+                            B = masks_ballot(s == RAP_SCHEME_PAD ? ((row + col) & 31u) : (col ^ row));
+                        }
+                        c = max_load(B, pp == RAP_PAT_RANDOM ? leaders : kFull, ls);
+                    }
+                    if (p == RAP_PAT_STRIDE) c_stride[s] = c;
+                    if (p == RAP_PAT_DIAGONAL) c_diag[s] = c;
+                    if (lane == 0) res[e] = c;                      // C4: result slot e
+                    ++e;
+                }
+            }
+            __syncwarp();
+            if (lane < e) atomicAdd(&sh_hist[lane * (w + 1) + res[lane]], 1u);
+            __syncwarp();
+        }
+        __syncwarp();
+    }
+    __syncthreads();
+    for (uint32_t b = threadIdx.x; b < nbins; b += blockDim.x)
+        if (sh_hist[b]) atomicAdd((unsigned long long *)(hist + b), (unsigned long long)sh_hist[b]);
+}
+
 // ------------------------------------------------------------------ C1-C4 sweep (ablation)
 // The north-star sketch, kept as a measured alternative: one warp per trial, Philox blocks
 // spread over lanes, warp Fisher-Yates by __shfl_sync, __match_any_sync histogram.
@@ -505,9 +691,9 @@ cudaError_t launch_sweep(uint32_t w, uint32_t pmask, uint32_t smask, uint64_t se
                          uint64_t n_trials, uint64_t *hist, cudaStream_t st) {
     if (n_trials == 0) return cudaSuccess;
     if (w == 32 && pmask == 31u && smask == 7u)
-        run_sweep<sweep_kernel<32, 31u, 7u>>(kSweepWarpsV2, 32, w, pmask, smask, seed, first, n_trials, hist, st);
+        run_sweep<sweep32_kernel<31u, 7u>>(kSweepWarpsV2, 32, w, pmask, smask, seed, first, n_trials, hist, st);
     else if (w == 32 && pmask == 31u && smask == 31u)
-        run_sweep<sweep_kernel<32, 31u, 31u>>(kSweepWarpsV2, 32, w, pmask, smask, seed, first, n_trials, hist, st);
+        run_sweep<sweep32_kernel<31u, 31u>>(kSweepWarpsV2, 32, w, pmask, smask, seed, first, n_trials, hist, st);
     else if (w == 32)
         run_sweep<sweep_kernel<32, 0u, 0u>>(kSweepWarpsV2, 32, w, pmask, smask, seed, first, n_trials, hist, st);
     else

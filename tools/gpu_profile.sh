@@ -15,7 +15,7 @@ for lay in rap raw pad xor ras; do
 done
 timeout 600 ncu --set full --import-source on --clock-control none -k regex:transpose_kernel -s 3 -c 1 \
     -o "$OUT/prof_t64_rap" -f $B --workload cfg4 --steps 1 --warmup 3 > "$OUT/ncu_t64_rap.log" 2>&1
-timeout 600 ncu --set full --import-source on --clock-control none -k regex:"sweep_kernel" -s 2 -c 1 \
+timeout 600 ncu --set full --import-source on --clock-control none -k regex:"sweep(32)?_kernel" -s 2 -c 1 \
     -o "$OUT/prof_sweep" -f $B --workload sweep --steps 1 --warmup 2 --sweep-trials 8388608 > "$OUT/ncu_sweep.log" 2>&1
 timeout 600 ncu --set full --import-source on --clock-control none -k regex:"sweep_match_kernel" -s 2 -c 1 \
     -o "$OUT/prof_sweep_match" -f $B --workload sweep --sweep-algo match --steps 1 --warmup 2 --sweep-trials 4194304 > "$OUT/ncu_sweep_match.log" 2>&1
