@@ -386,7 +386,7 @@ __device__ __forceinline__ uint32_t max_load(const BankMask &B, uint32_t counted
 }
 
 template <uint32_t PM, uint32_t SM>
-__global__ void __launch_bounds__(kSweepWarpsV2 * 32)
+__global__ void __launch_bounds__(kSweepWarpsV2 * 32, 8)
 sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint64_t n_trials,
                uint64_t *__restrict__ hist) {
     constexpr uint32_t w = 32;
