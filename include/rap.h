@@ -157,6 +157,21 @@ rap_status_t rap_congestion_trace(uint32_t w, uint64_t n_warps, const uint32_t *
 rap_status_t rap_unpack_blocks(const void *d_recv, void *d_out, int64_t G, int64_t M, int64_t ld_out,
                                uint32_t elem_bytes, void *stream);
 
+/* NEXT-1 -- the paper's experiment (Table III, §VI) on this GPU: a 32 x 32 matrix
+ * transposed `reps` times between two shared-memory arrays by one CTA of 1024 threads, with
+ * algorithm CRSW / SRCW / DRDW (§III) under layout RAW / RAS / RAP (both arrays laid
+ * out, reading v).  CTA k uses P = perm(seed, k, 32) or r = shifts(seed, k, 32).
+ * d_out: device uint32_t[n_blocks][1024], logical element (i, j) of the final array (initial
+ * a[i][j] = 32 i + j, so the result is the identity for even reps and the transpose for odd);
+ * d_cycles: device uint64_t[n_blocks], SM clock cycles of the timed loop (reps transposes, each
+ * followed by __syncthreads).  elem_bytes 4 or 8 (the paper used 8-byte doubles in 8-byte bank
+ * mode; B200 banks are 4 bytes).  ncu's shared wavefronts per request over many CTAs is the
+ * hardware's expected congestion of each access. */
+typedef enum { RAP_CRSW = 0, RAP_SRCW = 1, RAP_DRDW = 2 } rap_smem_algorithm_t;
+rap_status_t rap_smem_transpose_bench(uint32_t algorithm, rap_scheme_t scheme, uint32_t elem_bytes,
+                                      uint64_t seed, uint32_t n_blocks, uint32_t reps, uint32_t *d_out,
+                                      uint64_t *d_cycles, void *stream);
+
 #ifdef __cplusplus
 }
 #endif

@@ -62,8 +62,10 @@ def lib():
         L.rap_congestion_sweep_algo.argtypes = [u32, u32, u32, u64, u64, u64, u64p, u32, vp]
         L.rap_congestion_trace.argtypes = [u32, u64, u32p, u32, u64, u64, u64, u64p, vp]
         L.rap_unpack_blocks.argtypes = [vp, vp, i64, i64, i64, u32, vp]
+        L.rap_smem_transpose_bench.argtypes = [u32, i32, u32, u64, u32, u32, u32p, u64p, vp]
         for f in ("rap_perm_gen", "rap_transpose", "rap_congestion", "rap_congestion_sweep",
-                  "rap_congestion_sweep_algo", "rap_congestion_trace", "rap_unpack_blocks"):
+                  "rap_congestion_sweep_algo", "rap_congestion_trace", "rap_unpack_blocks",
+                  "rap_smem_transpose_bench"):
             getattr(L, f).restype = i32
         if L.rap_abi_version() != 1:
             raise ImportError("librap.so ABI version mismatch")
@@ -215,3 +217,19 @@ def unpack_blocks(recv: torch.Tensor, out: torch.Tensor, G: int) -> torch.Tensor
                                        G, M, out.stride(0) if M > 1 else G * M, eb, _stream(recv)),
                "rap_unpack_blocks")
     return out
+
+
+SMEM_ALGORITHMS = {"crsw": 0, "srcw": 1, "drdw": 2}
+
+
+def smem_transpose_bench(algorithm: str, scheme: str, elem_bytes: int = 4, seed: int = 0,
+                         n_blocks: int = 1, reps: int = 1, device="cuda"):
+    """Table III on this GPU: (logical result uint32 [n_blocks, 32, 32], cycles int64 [n_blocks])."""
+    out = torch.empty((n_blocks, 32, 32), dtype=torch.int32, device=device)
+    cyc = torch.empty(n_blocks, dtype=torch.int64, device=device)
+    with torch.cuda.device(out.device):
+        _check(lib().rap_smem_transpose_bench(SMEM_ALGORITHMS[algorithm], SCHEMES[scheme], elem_bytes, seed,
+                                              n_blocks, reps, ctypes.c_void_p(out.data_ptr()),
+                                              ctypes.c_void_p(cyc.data_ptr()), _stream(out)),
+               "rap_smem_transpose_bench")
+    return out, cyc

@@ -151,4 +151,16 @@ rap_status_t rap_unpack_blocks(const void *d_recv, void *d_out, int64_t G, int64
     return from_cuda(rapk::launch_unpack_blocks(d_recv, d_out, G, M, ld_out, elem_bytes, (cudaStream_t)stream));
 }
 
+rap_status_t rap_smem_transpose_bench(uint32_t algorithm, rap_scheme_t scheme, uint32_t elem_bytes,
+                                      uint64_t seed, uint32_t n_blocks, uint32_t reps, uint32_t *d_out,
+                                      uint64_t *d_cycles, void *stream) {
+    if (algorithm > RAP_DRDW) return RAP_ERR_INVALID_ARG;
+    if (scheme != RAP_SCHEME_RAW && scheme != RAP_SCHEME_RAS && scheme != RAP_SCHEME_RAP) return RAP_ERR_INVALID_ARG;
+    if (elem_bytes != 4 && elem_bytes != 8) return RAP_ERR_INVALID_ARG;
+    if (n_blocks == 0) return RAP_OK;
+    if (n_blocks > (1u << 24) || !d_out || !d_cycles) return RAP_ERR_INVALID_ARG;
+    return from_cuda(rapk::launch_smem_bench(algorithm, (int)scheme, elem_bytes, seed, n_blocks, reps, d_out,
+                                             d_cycles, (cudaStream_t)stream));
+}
+
 }  // extern "C"

@@ -51,4 +51,7 @@ cudaError_t launch_trace(uint32_t w, uint64_t n_warps, const uint32_t *cells, ui
 cudaError_t launch_unpack_blocks(const void *recv, void *out, int64_t G, int64_t M, int64_t ld_out,
                                  uint32_t elem_bytes, cudaStream_t st);
 
+cudaError_t launch_smem_bench(uint32_t alg, int scheme, uint32_t elem_bytes, uint64_t seed, uint32_t n_blocks,
+                              uint32_t reps, uint32_t *out, uint64_t *cycles, cudaStream_t st);
+
 }  // namespace rapk

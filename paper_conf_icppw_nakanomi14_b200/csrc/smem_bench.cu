@@ -1,0 +1,77 @@
+// smem_bench.cu -- NEXT-1: the paper's own experiment (Table III, §VI) on B200.
+//
+// One CTA of 1024 threads = 32 warps transposes a 32 x 32 matrix between two shared-memory
+// arrays a and b, `reps` times (a -> b, b -> a, ...), with the three algorithms of §III
+// (P:L787-828): CRSW (contiguous read, stride write), SRCW (stride read, contiguous write) and
+// DRDW (diagonal read, diagonal write), each under the RAW, RAS or RAP layout.  Both arrays carry
+// the layout (reading v: the printed RAP listing P:L1521-1526 would write b column-wise with a
+// 32-way conflict, contradicting Table III's write congestion 1).  Block k uses
+// P = perm(seed, k, 32) / r = shifts(seed, k, 32), so averaging over many blocks measures the
+// EXPECTED congestion; ncu's shared wavefronts per request is the hardware's congestion.
+// Thread (i, j) = (tid / 32, tid % 32) performs, for the source array s and destination d:
+//   CRSW  d[j][i]            <- s[i][j]
+//   SRCW  d[i][j]            <- s[j][i]
+//   DRDW  d[j][(i+j) mod 32] <- s[(i+j) mod 32][j] (reconstructed reading)
+// Element (row, col) of an array lives at row*32 + ((col + sh[row]) mod 32); sh = 0 (RAW),
+// r (RAS) or P (RAP).  Values are logical indices, so the result can be checked exactly.
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "rap_rng.cuh"
+#include "rap_internal.h"
+
+namespace rapk {
+
+template <int SCH>
+__device__ __forceinline__ uint32_t sm_index(uint32_t row, uint32_t col, const uint32_t *sh) {
+    if (SCH == RAP_SCHEME_RAW) return row * 32u + col;
+    return row * 32u + ((col + sh[row]) & 31u);
+}
+
+template <int ALG, int SCH, typename T>
+__global__ void __launch_bounds__(1024, 1)
+smem_transpose_kernel(uint64_t seed, uint32_t reps, uint32_t *__restrict__ out, uint64_t *__restrict__ cycles) {
+    __shared__ T a[1024], b[1024];
+    __shared__ uint32_t sh[32];
+    const uint32_t tid = threadIdx.x, i = tid >> 5, j = tid & 31u;
+    if (i == 0) {
+        uint32_t s = 0;
+        if (SCH == RAP_SCHEME_RAP) s = warp_perm<32>(seed, blockIdx.x, j, 32);
+        if (SCH == RAP_SCHEME_RAS) s = warp_ras_shift(seed, blockIdx.x, j, 32);
+        sh[j] = s;
+    }
+    __syncthreads();
+    a[sm_index<SCH>(i, j, sh)] = (T)(i * 32u + j);              // logical a[i][j] = i*32 + j
+    __syncthreads();
+    // the two addresses are loop-invariant: only the data accesses run inside the timed loop
+    const uint32_t d = (i + j) & 31u;
+    const uint32_t rd = ALG == 0 ? sm_index<SCH>(i, j, sh) : ALG == 1 ? sm_index<SCH>(j, i, sh) : sm_index<SCH>(d, j, sh);
+    const uint32_t wr = ALG == 0 ? sm_index<SCH>(j, i, sh) : ALG == 1 ? sm_index<SCH>(i, j, sh) : sm_index<SCH>(j, d, sh);
+    T *src = a, *dst = b;
+    long long t0 = 0;
+    if (tid == 0) t0 = clock64();
+    for (uint32_t k = 0; k < reps; ++k) {
+        dst[wr] = src[rd];
+        __syncthreads();
+        T *tmp = src; src = dst; dst = tmp;
+    }
+    if (tid == 0) cycles[blockIdx.x] = (uint64_t)(clock64() - t0);
+    out[(size_t)blockIdx.x * 1024 + tid] = (uint32_t)src[sm_index<SCH>(i, j, sh)];   // logical (i, j)
+}
+
+cudaError_t launch_smem_bench(uint32_t alg, int scheme, uint32_t elem_bytes, uint64_t seed, uint32_t n_blocks,
+                              uint32_t reps, uint32_t *out, uint64_t *cycles, cudaStream_t st) {
+#define RAPK_SB(A, S)                                                                              \
+    if (alg == A && scheme == S) {                                                                 \
+        if (elem_bytes == 4) smem_transpose_kernel<A, S, uint32_t><<<n_blocks, 1024, 0, st>>>(seed, reps, out, cycles); \
+        else smem_transpose_kernel<A, S, uint64_t><<<n_blocks, 1024, 0, st>>>(seed, reps, out, cycles);                 \
+        return cudaGetLastError();                                                                 \
+    }
+    RAPK_SB(0, RAP_SCHEME_RAW) RAPK_SB(0, RAP_SCHEME_RAS) RAPK_SB(0, RAP_SCHEME_RAP)
+    RAPK_SB(1, RAP_SCHEME_RAW) RAPK_SB(1, RAP_SCHEME_RAS) RAPK_SB(1, RAP_SCHEME_RAP)
+    RAPK_SB(2, RAP_SCHEME_RAW) RAPK_SB(2, RAP_SCHEME_RAS) RAPK_SB(2, RAP_SCHEME_RAP)
+#undef RAPK_SB
+    return cudaErrorInvalidValue;
+}
+
+}  // namespace rapk

@@ -105,6 +105,23 @@ def test_congestion_trace_perm_validation(L):
     assert L.rap_perm_gen(1, 0, 0, 32, P(0), s) == OK
 
 
+def test_smem_bench_and_unpack_validation(L):
+    d, s = P(0x30000000), P(0)
+    L.rap_smem_transpose_bench.argtypes = [ctypes.c_uint32, ctypes.c_int, ctypes.c_uint32, ctypes.c_uint64,
+                                           ctypes.c_uint32, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_void_p,
+                                           ctypes.c_void_p]
+    assert L.rap_smem_transpose_bench(3, 2, 4, 0, 1, 1, d, d, s) == INVALID      # unknown algorithm
+    assert L.rap_smem_transpose_bench(0, 3, 4, 0, 1, 1, d, d, s) == INVALID      # PAD not in Table III
+    assert L.rap_smem_transpose_bench(0, 2, 2, 0, 1, 1, d, d, s) == INVALID      # elem_bytes
+    assert L.rap_smem_transpose_bench(0, 2, 4, 0, 0, 1, P(0), P(0), s) == OK     # no blocks
+    L.rap_unpack_blocks.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int64, ctypes.c_int64,
+                                    ctypes.c_int64, ctypes.c_uint32, ctypes.c_void_p]
+    assert L.rap_unpack_blocks(d, P(0x40000000), 2, 8, 15, 4, s) == INVALID      # ld_out < G*M
+    assert L.rap_unpack_blocks(d, P(0x30000010), 2, 8, 16, 4, s) == ALIAS
+    assert L.rap_unpack_blocks(d, P(0x40000000), 2, 8, 16, 3, s) == INVALID
+    assert L.rap_unpack_blocks(d, P(0x40000000), 0, 8, 16, 4, s) == OK
+
+
 def test_python_binding_refuses_cpu_tensors(L):
     x = torch.zeros(8, 8)
     with pytest.raises(ValueError):

@@ -313,3 +313,19 @@ def test_dist_world1_nccl(rap, oracle):
         assert np.array_equal(bits(out), oracle.transpose(bits(A)))
     finally:
         dist.destroy_process_group()
+
+
+# ------------------------------------------------------------------ NEXT-1 Table III kernels
+@pytest.mark.parametrize("elem", [4, 8])
+@pytest.mark.parametrize("alg", ["crsw", "srcw", "drdw"])
+@pytest.mark.parametrize("scheme", ["raw", "ras", "rap"])
+def test_smem_transpose_bench_results(rap, oracle, alg, scheme, elem):
+    # each algorithm transposes; odd reps -> A^T, even reps -> A, for every CTA's P/r
+    A = np.arange(1024, dtype=np.int32).reshape(32, 32)
+    AT = oracle.transpose(A)
+    o1, c1 = rap.smem_transpose_bench(alg, scheme, elem, seed=7, n_blocks=40, reps=5)
+    o2, _ = rap.smem_transpose_bench(alg, scheme, elem, seed=7, n_blocks=40, reps=2)
+    o1, o2 = o1.cpu().numpy(), o2.cpu().numpy()
+    assert all(np.array_equal(o1[k], AT) for k in range(40))
+    assert all(np.array_equal(o2[k], A) for k in range(40))
+    assert (c1.cpu().numpy() > 0).all()
