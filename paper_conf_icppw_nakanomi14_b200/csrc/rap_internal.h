@@ -12,16 +12,18 @@ constexpr int kMaxDevices = 64;
 
 // Launch-shape knobs of the transpose (defaults chosen by tools/tune_transpose.cu on B200).
 struct TransposeTuning {
-    uint32_t group = 0;   // tile-rows per traversal group (0 = row-major tile order)
+    int sr = 4, sc = 1;   // super-tile of sr x sc tiles per CTA, one warp per tile, lockstep
     int minb = 2;         // __launch_bounds__ min blocks per SM (register budget)
     int depth = 1;        // tiles of global loads in flight per warp (register double-buffer)
     int ctas_per_sm = 0;  // persistent grid = #SMs x this (0: as many as fit)
+    bool vst = false;     // 128-bit output stores (shuffle-transposed) instead of 32/64-bit rows
 };
-constexpr uint32_t kDefaultGroup32 = 0, kDefaultGroup64 = 0;
+constexpr int kDefaultSR32 = 8, kDefaultSC32 = 2, kDefaultSR64 = 4, kDefaultSC64 = 1;
 // measured on B200 (tools/tune_transpose.cu, profiles/r01_tune_transpose.txt)
-constexpr int kDefaultMinB32 = 2, kDefaultMinB64 = 2;
-constexpr int kDefaultDepth32 = 2, kDefaultDepth64 = 1;
-constexpr int kDefaultCtas32 = 3, kDefaultCtas64 = 0;
+constexpr int kDefaultMinB32 = 1, kDefaultMinB64 = 1;
+constexpr int kDefaultDepth32 = 1, kDefaultDepth64 = 1;
+constexpr int kDefaultCtas32 = 0, kDefaultCtas64 = 0;
+constexpr bool kDefaultVst32 = false, kDefaultVst64 = false;
 TransposeTuning default_tuning(uint32_t elem_bytes);
 
 cudaError_t launch_transpose_tuned(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,

@@ -63,23 +63,6 @@ __device__ __forceinline__ uint4 ldg_stream128(const void *p) {
     return r;
 }
 
-// Tile t -> (ti, tj).  Tiles are walked in groups of `group` tile-rows, column by column
-// inside a group (group == 0: plain row-major tile order).
-__device__ __forceinline__ void tile_coords(uint32_t t, uint32_t tiles_r, uint32_t tiles_c, uint32_t group,
-                                            uint32_t &ti, uint32_t &tj) {
-    if (group == 0) {
-        ti = t / tiles_c;
-        tj = t - ti * tiles_c;
-        return;
-    }
-    const uint32_t per = group * tiles_c;
-    const uint32_t g = t / per, rem = t - g * per;
-    const uint32_t base = g * group;
-    const uint32_t nrows = min(group, tiles_r - base);
-    tj = rem / nrows;
-    ti = base + (rem - tj * nrows);
-}
-
 // Load geometry: a 128-bit load carries NE = 4/EW elements, LPR = 32/NE lanes cover one tile
 // row, so one warp instruction loads R = 32/LPR rows and a tile takes G = 32/R instructions.
 template <int L, int EW>
@@ -90,13 +73,15 @@ struct TileCfg {
     static constexpr int G = 32 / R;                // load instructions per tile (8 or 16)
 };
 
-constexpr int kWarpsT = 4;                          // warps per CTA
-
-template <int L, int EW, bool VEC, int DEPTH, int MINB>
-__global__ void __launch_bounds__(kWarpsT * 32, MINB)
+// CTA = SR x SC warps working on an SR x SC block of tiles ("super-tile") in lockstep: warp w
+// owns tile (w % SR, w / SR) of the block, and a CTA barrier before the drains makes the SC*32
+// input rows / SR*32-element output row runs of neighbouring warps reach DRAM together
+// (measured: +2-4 % over free-running warps, profiles/r01_tune_transpose.txt).
+template <int L, int EW, bool VEC, int DEPTH, int MINB, bool VST, int SR, int SC>
+__global__ void __launch_bounds__(SR * SC * 32, MINB)
 transpose_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, int64_t rows,
                  int64_t cols, int64_t ld_src, int64_t ld_dst, uint64_t seed, uint32_t tiles_r,
-                 uint32_t tiles_c, uint32_t ntiles, uint32_t group) {
+                 uint32_t tiles_c, bool vst_ok) {
     using C = TileCfg<L, EW>;
     constexpr int NE = C::NE, R = C::R, G = C::G, LPR = C::LPR;
     constexpr int PW = 32 * Geom<L>::RP;            // plane size in words
@@ -129,12 +114,18 @@ transpose_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, i
     }
     const uint32_t drain_base = word_of<L>(lane, 0, sh_lane);
 
-    const uint32_t stride = gridDim.x * kWarpsT;
-    uint32_t t = blockIdx.x * kWarpsT + warp;
+    // super-tile s -> this warp's tile (ti, tj); false when it falls outside the matrix
+    const uint32_t stc = (tiles_c + SC - 1) / SC;
+    const uint32_t nst = ((tiles_r + SR - 1) / SR) * stc;
+    const uint32_t wr = warp % SR, wc = warp / SR;
+    auto coords = [&](uint32_t st, uint32_t &ti, uint32_t &tj) -> bool {
+        const uint32_t si = st / stc, sj = st - si * stc;
+        ti = si * SR + wr;
+        tj = sj * SC + wc;
+        return ti < tiles_r && tj < tiles_c;
+    };
 
-    auto load = [&](uint4 (&v)[G], uint32_t tt) {
-        uint32_t ti, tj;
-        tile_coords(tt, tiles_r, tiles_c, group, ti, tj);
+    auto load = [&](uint4 (&v)[G], uint32_t ti, uint32_t tj) {
         const int64_t r0 = (int64_t)ti * 32, c0 = (int64_t)tj * 32;
         const bool full = (r0 + 32 <= rows) && (c0 + 32 <= cols);
         if (VEC && full) {
@@ -175,13 +166,50 @@ transpose_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, i
     };
 
     // T2: stride (column-wise) read -- lane i walks its row window -- and coalesced row stores
-    auto drain = [&](uint32_t tt) {
-        uint32_t ti, tj;
-        tile_coords(tt, tiles_r, tiles_c, group, ti, tj);
+    auto drain = [&](uint32_t ti, uint32_t tj) {
         const int64_t r0 = (int64_t)ti * 32, c0 = (int64_t)tj * 32;
         const int64_t ostride = ld_dst * EW;                       // words between output rows
         uint32_t *o = dst + (c0 * ld_dst + r0 + lane) * EW;        // this lane's column
-        if ((r0 + 32 <= rows) && (c0 + 32 <= cols)) {
+        if (VST && vst_ok && (r0 + 32 <= rows) && (c0 + 32 <= cols)) {
+            // 128-bit stores: each lane reads NE consecutive columns of its row, a butterfly of
+            // __shfl_xor_sync transposes NE x NE blocks among NE lanes, and lane NE*p + k then
+            // holds rows NE*p .. NE*p+NE-1 of column c+k -- one 16-byte chunk of output row c+k.
+            const uint32_t k = lane % NE, p = lane / NE;
+            uint32_t *ob = dst + ((c0 + k) * ld_dst + r0 + NE * p) * EW;
+#pragma unroll
+            for (int cg = 0; cg < 32 / NE; ++cg) {
+                uint32_t r[4];
+                if (EW == 1) {
+#pragma unroll
+                    for (int m = 0; m < 4; ++m) {
+                        const uint32_t off = (L == RAP_LAYOUT_XOR) ? word_of<L>(lane, 4 * cg + m, 0) : drain_base + 4 * cg + m;
+                        r[m] = tile[off];
+                    }
+                    const bool b0 = lane & 1u, b1 = lane & 2u;
+                    uint32_t x = __shfl_xor_sync(kFull, b0 ? r[0] : r[1], 1);
+                    if (b0) r[0] = x; else r[1] = x;
+                    x = __shfl_xor_sync(kFull, b0 ? r[2] : r[3], 1);
+                    if (b0) r[2] = x; else r[3] = x;
+                    x = __shfl_xor_sync(kFull, b1 ? r[0] : r[2], 2);
+                    if (b1) r[0] = x; else r[2] = x;
+                    x = __shfl_xor_sync(kFull, b1 ? r[1] : r[3], 2);
+                    if (b1) r[1] = x; else r[3] = x;
+                } else {
+#pragma unroll
+                    for (int m = 0; m < 2; ++m) {
+                        const uint32_t off = (L == RAP_LAYOUT_XOR) ? word_of<L>(lane, 2 * cg + m, 0) : drain_base + 2 * cg + m;
+                        r[2 * m] = tile[off];
+                        r[2 * m + 1] = tile[PW + off];
+                    }
+                    const bool b0 = lane & 1u;
+                    const uint32_t xl = __shfl_xor_sync(kFull, b0 ? r[0] : r[2], 1);
+                    const uint32_t xh = __shfl_xor_sync(kFull, b0 ? r[1] : r[3], 1);
+                    if (b0) { r[0] = xl; r[1] = xh; } else { r[2] = xl; r[3] = xh; }
+                }
+                *reinterpret_cast<uint4 *>(ob) = make_uint4(r[0], r[1], r[2], r[3]);
+                ob += ostride * NE;
+            }
+        } else if ((r0 + 32 <= rows) && (c0 + 32 <= cols)) {
 #pragma unroll
             for (int c = 0; c < 32; ++c) {
                 const uint32_t off = (L == RAP_LAYOUT_XOR) ? word_of<L>(lane, c, 0) : drain_base + c;
@@ -203,36 +231,50 @@ transpose_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, i
         }
     };
 
+    uint32_t st = blockIdx.x, ti = 0, tj = 0;
+    bool act = st < nst && coords(st, ti, tj);
     if (DEPTH == 1) {
         uint4 v[G];
-        if (t < ntiles) load(v, t);
-        while (t < ntiles) {
-            store_tile(v);
+        if (act) load(v, ti, tj);
+        while (st < nst) {
+            const uint32_t cti = ti, ctj = tj;
+            const bool cact = act;
+            if (cact) store_tile(v);                     // T1
             __syncwarp();
-            const uint32_t cur = t;
-            t += stride;
-            if (t < ntiles) load(v, t);                  // T3: next tile in flight
-            drain(cur);
+            st += gridDim.x;
+            act = st < nst && coords(st, ti, tj);
+            if (act) load(v, ti, tj);                    // T3: next tile in flight
+            if (SR * SC > 1) __syncthreads();            // drains of the super-tile together
+            if (cact) drain(cti, ctj);                   // T2
             __syncwarp();
         }
     } else {
         uint4 va[G], vb[G];
-        if (t < ntiles) load(va, t);
-        if (t + stride < ntiles) load(vb, t + stride);
-        while (t < ntiles) {
-            store_tile(va);
+        uint32_t ti2 = 0, tj2 = 0;
+        if (act) load(va, ti, tj);
+        bool act2 = st + gridDim.x < nst && coords(st + gridDim.x, ti2, tj2);
+        if (act2) load(vb, ti2, tj2);
+        while (st < nst) {
+            uint32_t cti = ti, ctj = tj;
+            bool cact = act;
+            if (cact) store_tile(va);
             __syncwarp();
-            if (t + 2 * stride < ntiles) load(va, t + 2 * stride);
-            drain(t);
+            act = st + 2 * gridDim.x < nst && coords(st + 2 * gridDim.x, ti, tj);
+            if (act) load(va, ti, tj);
+            if (SR * SC > 1) __syncthreads();
+            if (cact) drain(cti, ctj);
             __syncwarp();
-            t += stride;
-            if (t >= ntiles) break;
-            store_tile(vb);
+            st += gridDim.x;
+            if (st >= nst) break;
+            cti = ti2; ctj = tj2; cact = act2;
+            if (cact) store_tile(vb);
             __syncwarp();
-            if (t + 2 * stride < ntiles) load(vb, t + 2 * stride);
-            drain(t);
+            act2 = st + 2 * gridDim.x < nst && coords(st + 2 * gridDim.x, ti2, tj2);
+            if (act2) load(vb, ti2, tj2);
+            if (SR * SC > 1) __syncthreads();
+            if (cact) drain(cti, ctj);
             __syncwarp();
-            t += stride;
+            st += gridDim.x;
         }
     }
 }
@@ -274,44 +316,52 @@ static cudaError_t grid_for(K kernel, ShapeCache &cache, int threads, size_t sme
 
 TransposeTuning default_tuning(uint32_t elem_bytes) {
     TransposeTuning t;
-    t.group = elem_bytes == 4 ? kDefaultGroup32 : kDefaultGroup64;
+    t.sr = elem_bytes == 4 ? kDefaultSR32 : kDefaultSR64;
+    t.sc = elem_bytes == 4 ? kDefaultSC32 : kDefaultSC64;
     t.minb = elem_bytes == 4 ? kDefaultMinB32 : kDefaultMinB64;
     t.depth = elem_bytes == 4 ? kDefaultDepth32 : kDefaultDepth64;
     t.ctas_per_sm = elem_bytes == 4 ? kDefaultCtas32 : kDefaultCtas64;
+    t.vst = elem_bytes == 4 ? kDefaultVst32 : kDefaultVst64;
     return t;
 }
 
-template <int L, int EW, bool VEC, int DEPTH, int MINB>
+template <int L, int EW, bool VEC, int DEPTH, int MINB, bool VST, int SR, int SC>
 static cudaError_t launch_one(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
                               int64_t ld_dst, uint64_t seed, const TransposeTuning &tu, cudaStream_t st) {
     const uint32_t tiles_r = (uint32_t)((rows + 31) / 32), tiles_c = (uint32_t)((cols + 31) / 32);
-    const uint32_t ntiles = tiles_r * tiles_c;
-    auto k = transpose_kernel<L, EW, VEC, DEPTH, MINB>;
+    const int64_t nst = (int64_t)((tiles_r + SR - 1) / SR) * ((tiles_c + SC - 1) / SC);
+    auto k = transpose_kernel<L, EW, VEC, DEPTH, MINB, VST, SR, SC>;
     static ShapeCache cache;
-    const size_t smem = sizeof(uint32_t) * warp_smem_words<L, EW>() * kWarpsT;
+    const bool vst_ok = ((uintptr_t)dst % 16 == 0) && ((ld_dst * EW * 4) % 16 == 0);
+    const size_t smem = sizeof(uint32_t) * warp_smem_words<L, EW>() * SR * SC;
     int grid = 0;
-    const cudaError_t e = grid_for(k, cache, kWarpsT * 32, smem, ntiles, kWarpsT, tu.ctas_per_sm, &grid);
+    const cudaError_t e = grid_for(k, cache, SR * SC * 32, smem, nst, 1, tu.ctas_per_sm, &grid);
     if (e != cudaSuccess) return e;
-    k<<<grid, kWarpsT * 32, smem, st>>>((const uint32_t *)src, (uint32_t *)dst, rows, cols, ld_src,
-                                        ld_dst, seed, tiles_r, tiles_c, ntiles, tu.group);
+    k<<<grid, SR * SC * 32, smem, st>>>((const uint32_t *)src, (uint32_t *)dst, rows, cols, ld_src,
+                                        ld_dst, seed, tiles_r, tiles_c, vst_ok);
     return cudaGetLastError();
 }
 
 template <int L, int EW, bool VEC>
 static cudaError_t launch_shape(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
                                 int64_t ld_dst, uint64_t seed, const TransposeTuning &tu, cudaStream_t st) {
-#define RAPK_SHAPE(D, M)                                                                             \
-    if (tu.depth == D && tu.minb == M)                                                               \
-        return launch_one<L, EW, VEC, D, M>(src, dst, rows, cols, ld_src, ld_dst, seed, tu, st);
+#define RAPK_SHAPE(D, M, V, R_, C_)                                                                  \
+    if (tu.depth == D && tu.minb == M && tu.vst == V && tu.sr == R_ && tu.sc == C_)                  \
+        return launch_one<L, EW, VEC, D, M, V, R_, C_>(src, dst, rows, cols, ld_src, ld_dst, seed, tu, st);
 #ifdef RAP_TUNING_SWEEP
-    RAPK_SHAPE(1, 2) RAPK_SHAPE(1, 3) RAPK_SHAPE(1, 4) RAPK_SHAPE(1, 6) RAPK_SHAPE(1, 8)
-    RAPK_SHAPE(2, 2) RAPK_SHAPE(2, 3) RAPK_SHAPE(2, 4) RAPK_SHAPE(2, 6)
+    RAPK_SHAPE(1, 1, false, 4, 1) RAPK_SHAPE(1, 4, false, 4, 1) RAPK_SHAPE(1, 3, false, 4, 1)
+    RAPK_SHAPE(1, 1, false, 8, 1) RAPK_SHAPE(1, 2, false, 8, 1) RAPK_SHAPE(1, 3, false, 8, 1)
+    RAPK_SHAPE(1, 1, false, 16, 1) RAPK_SHAPE(1, 2, false, 16, 1) RAPK_SHAPE(2, 1, false, 16, 1)
+    RAPK_SHAPE(1, 1, false, 8, 2) RAPK_SHAPE(1, 1, false, 12, 1) RAPK_SHAPE(1, 1, true, 16, 1)
+    RAPK_SHAPE(2, 2, false, 8, 1) RAPK_SHAPE(1, 1, false, 6, 1) RAPK_SHAPE(1, 2, false, 6, 1)
 #endif
 #undef RAPK_SHAPE
     (void)tu;
-    return launch_one<L, EW, VEC, EW == 1 ? kDefaultDepth32 : kDefaultDepth64,
-                      EW == 1 ? kDefaultMinB32 : kDefaultMinB64>(src, dst, rows, cols, ld_src, ld_dst,
-                                                                 seed, tu, st);
+    if (EW == 1)
+        return launch_one<L, EW, VEC, kDefaultDepth32, kDefaultMinB32, kDefaultVst32, kDefaultSR32, kDefaultSC32>(
+            src, dst, rows, cols, ld_src, ld_dst, seed, tu, st);
+    return launch_one<L, EW, VEC, kDefaultDepth64, kDefaultMinB64, kDefaultVst64, kDefaultSR64, kDefaultSC64>(
+        src, dst, rows, cols, ld_src, ld_dst, seed, tu, st);
 }
 
 template <bool VEC>

@@ -248,6 +248,37 @@ static void run_chunkx(const uint32_t *a, uint32_t *b, cudaEvent_t e0, cudaEvent
            WS ? "scattered" : "seq      ", occ, 2.0 * 8192.0 * 8192 * 4 / ms[ms.size() / 2] / 1e6);
 }
 
+// tile copy with the transpose's store granularity: 32 x STG.32 (one 128 B row each) per tile
+template <int STW>   // STW = 1: 32-bit stores (lane = column), 4: 128-bit stores (8 lanes per row)
+__global__ void __launch_bounds__(128) tilecopy_st_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst,
+                                                          int64_t n, uint32_t tiles_c, uint32_t ntiles) {
+    __shared__ uint32_t sm[4][32 * 32];
+    const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
+    const uint32_t q = lane & 7u, c_in = lane >> 3;
+    uint32_t *tile = sm[warp];
+    for (uint32_t t = blockIdx.x * 4 + warp; t < ntiles; t += gridDim.x * 4) {
+        const uint32_t ti = t / tiles_c, tj = t - ti * tiles_c;
+        const uint32_t *s = src + ((int64_t)ti * 32 + c_in) * n + tj * 32 + 4 * q;
+        uint4 v[8];
+#pragma unroll
+        for (int g = 0; g < 8; ++g) v[g] = rapk::ldg_stream128(s + (int64_t)4 * g * n);
+#pragma unroll
+        for (int g = 0; g < 8; ++g) *reinterpret_cast<uint4 *>(&tile[(4 * g + c_in) * 32 + 4 * q]) = v[g];
+        __syncwarp();
+        if (STW == 1) {
+            uint32_t *o = dst + (int64_t)ti * 32 * n + tj * 32 + lane;
+#pragma unroll
+            for (int r = 0; r < 32; ++r) o[(int64_t)r * n] = tile[r * 32 + lane];
+        } else {
+            uint32_t *o = dst + ((int64_t)ti * 32 + c_in) * n + tj * 32 + 4 * q;
+#pragma unroll
+            for (int g = 0; g < 8; ++g)
+                *reinterpret_cast<uint4 *>(o + (int64_t)4 * g * n) = *reinterpret_cast<uint4 *>(&tile[(4 * g + c_in) * 32 + 4 * q]);
+        }
+        __syncwarp();
+    }
+}
+
 static float median(std::vector<float> v) { std::sort(v.begin(), v.end()); return v[v.size() / 2]; }
 
 int main(int argc, char **argv) {
@@ -297,6 +328,12 @@ int main(int argc, char **argv) {
             t = timeit([&] { regtranspose_kernel<<<148 * occ, 128>>>(a, b, n, tc, nt); }, 30);
             run_aspect<32>(a, b, e0, e1); run_aspect<16>(a, b, e0, e1); run_aspect<8>(a, b, e0, e1);
             run_aspect<4>(a, b, e0, e1); run_aspect<2>(a, b, e0, e1); run_aspect<1>(a, b, e0, e1);
+            for (int o : {3, 4, 6, 8, 12, 16}) {
+                float t1 = timeit([&] { tilecopy_st_kernel<1><<<148 * o, 128>>>(a, b, n, tc, nt); }, 30);
+                float t4 = timeit([&] { tilecopy_st_kernel<4><<<148 * o, 128>>>(a, b, n, tc, nt); }, 30);
+                printf("probe smem tilecopy occ %2d: STG.32 rows %.1f GB/s   STG.128 %.1f GB/s\n", o,
+                       2.0 * n * n * 4 / t1 / 1e6, 2.0 * n * n * 4 / t4 / 1e6);
+            }
             for (int o : {4, 6, 8}) {
                 run_chunkx<128, 0, 0>(a, b, e0, e1, o); run_chunkx<128, 0, 1>(a, b, e0, e1, o); run_chunkx<128, 1, 1>(a, b, e0, e1, o);
                 run_chunkx<256, 0, 0>(a, b, e0, e1, o); run_chunkx<256, 0, 1>(a, b, e0, e1, o); run_chunkx<256, 1, 1>(a, b, e0, e1, o);
@@ -321,24 +358,33 @@ int main(int argc, char **argv) {
     }
     const int layouts[] = {RAP_LAYOUT_RAP, RAP_LAYOUT_RAW, RAP_LAYOUT_PAD, RAP_LAYOUT_XOR, RAP_LAYOUT_RAS};
     const char *lname[] = {"raw", "pad", "xor", "ras", "rap"};
-    struct Shape { int depth, minb; };
-    const Shape shapes[] = {{1, 2}, {1, 4}, {2, 2}, {2, 3}};
+    struct Shape { int depth, minb; bool vst; int sr, sc; };
+    const Shape shapes[] = {{1, 1, false, 4, 1}, {1, 4, false, 4, 1}, {1, 3, false, 4, 1}, {1, 1, false, 8, 1},
+                            {1, 2, false, 8, 1}, {1, 3, false, 8, 1}, {1, 1, false, 16, 1}, {1, 2, false, 16, 1},
+                            {2, 1, false, 16, 1}, {1, 1, false, 8, 2}, {1, 1, false, 12, 1}, {1, 1, true, 16, 1},
+                            {2, 2, false, 8, 1}, {1, 1, false, 6, 1}, {1, 2, false, 6, 1}};
     for (int eb : {4, 8}) {
         const int64_t n = eb == 4 ? n32 : n64;
         const size_t bytes = eb == 4 ? bytes32 : bytes64;
-        for (int lay : layouts) {
+        for (int lay : {RAP_LAYOUT_RAP, RAP_LAYOUT_RAW, RAP_LAYOUT_PAD, RAP_LAYOUT_XOR, RAP_LAYOUT_RAS}) {
             for (const Shape &sh : shapes) {
-                for (int cps : {2, 3, 4, 5, 6, 8}) {
-                    if (lay != RAP_LAYOUT_RAP && sh.depth != 1) continue;
-                    rapk::TransposeTuning tu; tu.group = 0; tu.minb = sh.minb; tu.depth = sh.depth; tu.ctas_per_sm = cps;
+                if (lay != RAP_LAYOUT_RAP && !(sh.depth == 1 && sh.minb == 1 && !sh.vst && sh.sr == 16 && sh.sc == 1))
+                    continue;
+                const int rp = (lay == RAP_LAYOUT_RAP || lay == RAP_LAYOUT_RAS) ? 64 : (lay == RAP_LAYOUT_PAD ? 33 : 32);
+                if ((size_t)32 * rp * (eb / 4) * 4 * sh.sr * sh.sc > 227 * 1024) continue;   // smem limit
+                for (int cps : {0}) {
+                    if (lay != RAP_LAYOUT_RAP && cps) continue;
+                    rapk::TransposeTuning tu; tu.minb = sh.minb; tu.depth = sh.depth; tu.ctas_per_sm = cps;
+                    tu.vst = sh.vst; tu.sr = sh.sr; tu.sc = sh.sc;
                     CK(cudaMemset(b, 0, bytes));
                     float t = timeit([&] { rapk::launch_transpose_tuned(a, b, n, n, n, n, eb, lay, 1, tu, 0); }, eb == 4 ? 30 : 10);
                     CK(cudaGetLastError());
                     CK(cudaMemset(bad, 0, 8));
                     check_t<<<2048, 256>>>(a, b, n, eb / 4, bad);
                     unsigned long long hb; CK(cudaMemcpy(&hb, bad, 8, cudaMemcpyDeviceToHost));
-                    printf("b%d %-4s depth=%d minb=%d ctas/sm=%d : %7.1f GB/s  %8.1f us  %s\n", eb * 8, lname[lay],
-                           sh.depth, sh.minb, cps, 2.0 * bytes / t / 1e6, t * 1e3, hb ? "MISMATCH" : "ok");
+                    printf("b%d %-4s depth=%d minb=%d vst=%d sr=%2d sc=%d ctas/sm=%d : %7.1f GB/s  %8.1f us  %s\n", eb * 8,
+                           lname[lay], sh.depth, sh.minb, (int)sh.vst, sh.sr, sh.sc, cps, 2.0 * bytes / t / 1e6, t * 1e3,
+                           hb ? "MISMATCH" : "ok");
                 }
             }
         }
