@@ -387,6 +387,31 @@ def main():
         if t_share < 0.5:                       # the sweep dominates this step: report its roofline
             line["roofline_transpose"] = line["roofline"]
             line["roofline"] = line["sweep"]["roofline"]
+    if wl == "tile":
+        # latency case: the per-call time above includes the Python/ctypes launch path; replaying
+        # 256 launches captured in one CUDA graph gives the device-side time per 32x32 transpose
+        g = torch.cuda.CUDAGraph()
+        cs = torch.cuda.Stream()
+        cs.wait_stream(stream)
+        with torch.cuda.stream(cs):
+            rap.transpose(x, layout=lay, seed=0, out=y)
+            torch.cuda.synchronize()
+            with torch.cuda.graph(g, stream=cs):
+                for _ in range(256):
+                    rap.transpose(x, layout=lay, seed=0, out=y)
+        g.replay()
+        torch.cuda.synchronize()
+        gs, ge = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        gs.record(stream)
+        for _ in range(10):
+            g.replay()
+        ge.record(stream)
+        torch.cuda.synchronize()
+        us = gs.elapsed_time(ge) * 1e3 / (10 * 256)
+        line["tile_latency"] = {"us_per_call_python": statistics.median(r["t_ms"]) * 1e3,
+                                "us_per_transpose_cuda_graph": us,
+                                "note": "2560 graph-replayed launches; includes the in-kernel Philox + "
+                                        "Fisher-Yates of P (T0) and one 8 KiB tile"}
     line["clocks"] = r["clocks"]
     line["gpu_launches"] = int(reduce_over_ranks(r["launches"], world, dev, "sum"))
 

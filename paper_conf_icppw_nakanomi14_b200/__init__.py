@@ -10,6 +10,7 @@ Functions keep the C names without the ``rap_`` prefix:
 """
 from __future__ import annotations
 
+import contextlib
 import ctypes
 import os
 
@@ -77,6 +78,13 @@ def _stream(t: torch.Tensor):
     return ctypes.c_void_p(torch.cuda.current_stream(t.device).cuda_stream)
 
 
+def _on(dev: torch.device):
+    """Make `dev` current for the C call (no-op, and no context-manager cost, when it already is)."""
+    if dev.index is None or dev.index == torch.cuda.current_device():
+        return contextlib.nullcontext()
+    return torch.cuda.device(dev)
+
+
 def _need_cuda(*ts):
     for t in ts:
         if t is not None and not t.is_cuda:
@@ -104,7 +112,7 @@ def perm_gen(seed: int, count: int, w: int = 32, first_index: int = 0,
         out = torch.empty((count, w), dtype=torch.uint8, device=device)
     _need_cuda(out)
     assert out.dtype == torch.uint8 and out.is_contiguous() and out.numel() == count * w
-    with torch.cuda.device(out.device):
+    with _on(out.device):
         _check(lib().rap_perm_gen(seed, first_index, count, w, ctypes.c_void_p(out.data_ptr()),
                                   _stream(out)), "rap_perm_gen")
     return out
@@ -132,7 +140,7 @@ def transpose(x: torch.Tensor, layout: str = "rap", seed: int = 0,
         raise ValueError("out must be a [cols, rows] tensor of x's dtype with unit inner stride")
     ld_src = x.stride(0) if rows > 1 else max(cols, 1)
     ld_dst = out.stride(0) if cols > 1 else max(rows, 1)
-    with torch.cuda.device(x.device):
+    with _on(x.device):
         _check(lib().rap_transpose(ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(out.data_ptr()),
                                    rows, cols, ld_src, ld_dst, eb, LAYOUTS[layout], seed,
                                    _stream(x)), "rap_transpose")
@@ -153,7 +161,7 @@ def congestion(rows: torch.Tensor, cols: torch.Tensor, scheme: str = "rap",
         assert shift.shape == rows.shape
     if out is None:
         out = torch.empty(n, dtype=torch.uint32, device=rows.device)
-    with torch.cuda.device(rows.device):
+    with _on(rows.device):
         _check(lib().rap_congestion(w, n, ctypes.c_void_p(rows.data_ptr()),
                                     ctypes.c_void_p(cols.data_ptr()), SCHEMES[scheme],
                                     ctypes.c_void_p(shift.data_ptr() if shift is not None else 0),
@@ -177,7 +185,7 @@ def congestion_sweep(n_trials: int, seed: int, w: int = 32, patterns=("contiguou
         out = torch.zeros(shape, dtype=torch.int64, device=device)
     _need_cuda(out)
     assert tuple(out.shape) == shape and out.dtype == torch.int64 and out.is_contiguous()
-    with torch.cuda.device(out.device):
+    with _on(out.device):
         _check(lib().rap_congestion_sweep_algo(w, pm, sm, seed, first_trial, n_trials,
                                                ctypes.c_void_p(out.data_ptr()), SWEEP_ALGOS[algo],
                                                _stream(out)), "rap_congestion_sweep")
@@ -195,7 +203,7 @@ def congestion_trace(cells: torch.Tensor, n_trials: int, seed: int, schemes=("ra
     if out is None:
         out = torch.zeros(shape, dtype=torch.int64, device=cells.device)
     assert tuple(out.shape) == shape and out.dtype == torch.int64 and out.is_contiguous()
-    with torch.cuda.device(cells.device):
+    with _on(cells.device):
         _check(lib().rap_congestion_trace(w, n, ctypes.c_void_p(cells.data_ptr()), sm, seed,
                                           first_trial, n_trials, ctypes.c_void_p(out.data_ptr()),
                                           _stream(cells)), "rap_congestion_trace")
@@ -212,7 +220,7 @@ def unpack_blocks(recv: torch.Tensor, out: torch.Tensor, G: int) -> torch.Tensor
     assert GM == G * M and recv.is_contiguous() and out.dtype == recv.dtype
     assert out.shape[0] == M and out.shape[1] >= G * M and out.stride(1) == 1
     eb = recv.element_size()
-    with torch.cuda.device(recv.device):
+    with _on(recv.device):
         _check(lib().rap_unpack_blocks(ctypes.c_void_p(recv.data_ptr()), ctypes.c_void_p(out.data_ptr()),
                                        G, M, out.stride(0) if M > 1 else G * M, eb, _stream(recv)),
                "rap_unpack_blocks")
@@ -227,7 +235,7 @@ def smem_transpose_bench(algorithm: str, scheme: str, elem_bytes: int = 4, seed:
     """Table III on this GPU: (logical result uint32 [n_blocks, 32, 32], cycles int64 [n_blocks])."""
     out = torch.empty((n_blocks, 32, 32), dtype=torch.int32, device=device)
     cyc = torch.empty(n_blocks, dtype=torch.int64, device=device)
-    with torch.cuda.device(out.device):
+    with _on(out.device):
         _check(lib().rap_smem_transpose_bench(SMEM_ALGORITHMS[algorithm], SCHEMES[scheme], elem_bytes, seed,
                                               n_blocks, reps, ctypes.c_void_p(out.data_ptr()),
                                               ctypes.c_void_p(cyc.data_ptr()), _stream(out)),

@@ -56,6 +56,37 @@ def raw_metrics(rep):
     return d
 
 
+def source_smem(rep):
+    """Per-instruction shared-memory wavefronts from the source page: (ld_wf, ld_inst, st_wf, st_inst, excessive)."""
+    out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "sass"],
+                         capture_output=True, text=True).stdout
+    rows = list(csv.reader(io.StringIO(out)))
+    if len(rows) < 3:
+        return None
+    head = rows[1]
+    acc = [0.0] * 5
+    for r in rows[2:]:
+        if len(r) != len(head):
+            continue
+        d = dict(zip(head, r))
+        src = d.get("Source", "")
+        op = src.split()[0] if src.split() else ""
+        if op.startswith("@"):
+            op = src.split()[1]
+        try:
+            wf = float(d.get("L1 Wavefronts Shared") or 0)
+            n = float(d.get("Instructions Executed") or 0)
+            ex = float(d.get("L1 Wavefronts Shared Excessive") or 0)
+        except ValueError:
+            continue
+        if op.startswith("LDS"):
+            acc[0] += wf; acc[1] += n
+        elif op.startswith("STS"):
+            acc[2] += wf; acc[3] += n
+        acc[4] += ex
+    return acc
+
+
 def main(src_dir, dst, tag):
     kernels = {}
     for key, stem in CAPTURES.items():
@@ -84,6 +115,14 @@ def main(src_dir, dst, tag):
             "registers": m.get("launch__registers_per_thread"), "grid": m.get("launch__grid_size"),
             "block": m.get("launch__block_size"), "instructions": m.get("smsp__inst_executed.sum"),
         }
+        sm = source_smem(rep)
+        if sm:
+            kernels[key]["smem_wavefronts_per_request"] = {"ld": sm[0] / sm[1] if sm[1] else None,
+                                                           "st": sm[2] / sm[3] if sm[3] else None}
+            kernels[key]["smem_wavefronts_excessive"] = sm[4]
+            kernels[key]["smem_wavefronts_note"] = ("per-instruction L1 Wavefronts Shared / executed LDS|STS "
+                                                    "(source page); l1tex__data_bank_conflicts also counts "
+                                                    "inter-instruction arbitration")
         if key in UNITS:
             unit, n = UNITS[key]
             kernels[key]["units_per_launch"] = {unit: n}
