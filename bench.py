@@ -45,7 +45,7 @@ def parse():
     p.add_argument("--warmup", type=int, default=5)
     p.add_argument("--impl", default="mine", choices=["mine", "reference"])
     p.add_argument("--workload", default="default",
-                   choices=["default", "sweep", "cfg4", "tile", "layouts", "dist"])
+                   choices=["default", "sweep", "cfg4", "tile", "layouts", "dist", "dist_fused"])
     p.add_argument("--sweep-trials", type=int, default=1 << 16)
     p.add_argument("--sweep-algo", default="default", choices=["default", "match"])
     p.add_argument("--layout", default="rap")
@@ -236,7 +236,11 @@ def main():
     world, rank, local = dist_env()
     dev = torch.device("cuda", local)
     torch.cuda.set_device(dev)
-    if world > 1:
+    if world > 1 or args.workload == "dist_fused":
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        os.environ.setdefault("MASTER_PORT", "29571")
+        os.environ.setdefault("RANK", "0")
+        os.environ.setdefault("WORLD_SIZE", "1")
         dist.init_process_group("nccl", device_id=dev)
     stream = torch.cuda.current_stream()
     peak, peak_src = load_peaks()
@@ -251,7 +255,7 @@ def main():
     elif wl == "tile":
         rows = cols = 32
         dt = torch.float32
-    elif wl == "dist":
+    elif wl in ("dist", "dist_fused"):
         rows, cols = 32768 // world, 32768
         dt = torch.float32
     else:
@@ -264,13 +268,20 @@ def main():
     nbytes = 2 * rows * cols * eb                     # per rank per step
     x = workloads.random_bits(rows, cols, dt, seed=rank, device=dev) if do_t else None
     y = None
+    dist_wl = wl in ("dist", "dist_fused")
     if do_t:
-        y = torch.empty((rows, cols) if wl == "dist" else (cols, rows), dtype=dt, device=dev)
+        y = torch.empty((rows, cols) if dist_wl else (cols, rows), dtype=dt, device=dev)
     work = {}
+    fused = rdist.FusedTranspose((rows, cols), dt, layout=args.layout) if wl == "dist_fused" else None
+    if fused is not None:
+        y = fused.out
     S = args.sweep_trials
     hist = torch.zeros((5, 3, 33), dtype=torch.int64, device=dev)
 
     def step_transpose(lay):
+        if wl == "dist_fused":
+            fused(x)
+            return 1                               # one fused transpose+exchange kernel (+ 2 barriers)
         if wl == "dist":
             rdist.transpose_sharded(x, layout=lay, seed=0, out=y, work=work)
             return 1 if world == 1 else 2          # local transpose (+ unpack)
@@ -324,7 +335,7 @@ def main():
     r = results[lay]
     line = {"metric": METRIC, "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": r["total_ms"] / args.steps, "higher_is_better": True,
-            "scaling": "strong" if wl == "dist" else "weak", "vs_baseline": None,
+            "scaling": "strong" if dist_wl else "weak", "vs_baseline": None,
             "dtype": "u64" if eb == 8 else "u32", "data": "synthetic (seeded random bit patterns)"}
     if do_t:
         gbs = nbytes * world * args.steps / (r["t_sum"] * 1e-3) / 1e9
@@ -334,10 +345,13 @@ def main():
                 "cfg4": "cfg4 16384x16384 float64 RAP transpose (two 32-bit RAP planes)",
                 "tile": "cfg1 32x32 float32 RAP tile (latency case)",
                 "layouts": "cfg3 8192x8192 float32 transpose under 5 smem layouts",
-                "dist": f"cfg5 32768x32768 float32 row-block-sharded transpose over {world} GPU(s)"}[wl]
-        line["config"] = {"workload": desc, "rows": rows * (world if wl == "dist" else 1), "cols": cols,
+                "dist": f"cfg5 32768x32768 float32 row-block-sharded transpose over {world} GPU(s), NCCL all-to-all",
+                "dist_fused": f"cfg5 32768x32768 float32 row-block-sharded transpose over {world} GPU(s), "
+                              "fused: tiles stored straight into peer shards (symmetric memory)"}[wl]
+        line["config"] = {"workload": desc, "rows": rows * (world if dist_wl else 1), "cols": cols,
                           "elem_bytes": eb, "layout": lay,
                           "parallelism": (f"row blocks + NCCL all-to-all, {world} ranks" if wl == "dist"
+                                          else f"row blocks + NVLink peer stores, {world} ranks" if wl == "dist_fused"
                                           else f"replicas x{world}" if world > 1 else "single GPU"),
                           "l2": ("inputs larger than L2 (no flush)" if nbytes // 2 > 126e6
                                  else "input fits in L2 (no flush; latency case)"),
@@ -346,7 +360,7 @@ def main():
             line["config"]["sweep_trials_per_step"] = S * world
         kkey = f"transpose_b{eb * 8}_{lay}"
         prof = load_profile(kkey) or {}
-        if wl == "dist" and world > 1:
+        if dist_wl and world > 1:
             nv = (world - 1) / world * (rows * cols * eb) / (kern_ms * 1e-3) / 1e9
             line["roofline"] = {"bound": "nvlink", "achieved": nv, "peak": NVLINK_GBS, "unit": "GB/s",
                                 "frac": nv / NVLINK_GBS, "traffic": None,
@@ -424,7 +438,9 @@ def main():
 
         def e2e_step():
             dx.copy_(hx, non_blocking=True)
-            if wl == "dist":
+            if wl == "dist_fused":
+                fused(dx)
+            elif wl == "dist":
                 rdist.transpose_sharded(dx, layout=lay, seed=0, out=y, work=work)
             else:
                 rap.transpose(dx, layout=lay, seed=0, out=y)
@@ -468,7 +484,7 @@ def main():
             line["sweep"]["cpu_baseline"] = cpu_baseline_sweep()
     if rank == 0:
         print(json.dumps(line), flush=True)
-    if world > 1:
+    if dist.is_initialized():
         dist.destroy_process_group()
 
 

@@ -102,6 +102,20 @@ rap_status_t rap_transpose(const void *src, void *dst, int64_t rows, int64_t col
                            int64_t ld_src, int64_t ld_dst, uint32_t elem_bytes,
                            rap_layout_t layout, uint64_t seed, void *stream);
 
+/* T4, fused (NEXT-2) -- the row-block-sharded N x N transpose without the all-to-all: rank
+ * `rank` of G holds rows rank*M .. rank*M+M-1 of A (src: M x N, ld_src >= N, N = G*M, M a
+ * multiple of 32) and writes every 32 x 32 output tile straight into the output shard of the
+ * rank that owns it:
+ *     peer_dst[h][(c - h*M) * ld_dst + rank*M + r] = src[r * ld_src + c],   h = c / M,
+ * so out_h = rows h*M .. h*M+M-1 of A^T.  peer_dst: HOST array of G device pointers valid in
+ * this process (peer shards mapped over NVLink -- CUDA IPC / symmetric memory -- or local
+ * buffers for a one-GPU emulation); ld_dst >= N; G <= 16.  One HBM read and one NVLink write
+ * per element; no send/receive buffers, no unpack.  Enqueue only: the caller must make every
+ * rank's kernel complete (a cross-rank barrier) before reading its output shard. */
+rap_status_t rap_transpose_to_peers(const void *src, int64_t M, int64_t N, int64_t ld_src,
+                                    void *const *peer_dst, uint32_t G, uint32_t rank, int64_t ld_dst,
+                                    uint32_t elem_bytes, rap_layout_t layout, uint64_t seed, void *stream);
+
 /* C3 -- the DMM congestion evaluator itself (§II), batched: warp k issues the w
  * requests to logical cells (d_rows[k*w + t], d_cols[k*w + t]) of a w x w matrix laid out
  * by `scheme` with per-warp shift vector d_shift[k*w .. k*w+w-1] (P for RAP, r for RAS;

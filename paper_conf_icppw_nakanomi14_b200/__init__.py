@@ -18,7 +18,8 @@ import torch
 
 from . import build as _build
 
-__all__ = ["perm_gen", "transpose", "congestion", "congestion_sweep", "congestion_trace", "unpack_blocks",
+__all__ = ["perm_gen", "transpose", "transpose_to_peers", "congestion", "congestion_sweep", "congestion_trace",
+           "unpack_blocks", "smem_transpose_bench",
            "LAYOUTS", "SCHEMES", "PATTERNS", "RapError", "lib", "library_path"]
 
 LAYOUTS = {"raw": 0, "pad": 1, "xor": 2, "ras": 3, "rap": 4}
@@ -64,9 +65,11 @@ def lib():
         L.rap_congestion_trace.argtypes = [u32, u64, u32p, u32, u64, u64, u64, u64p, vp]
         L.rap_unpack_blocks.argtypes = [vp, vp, i64, i64, i64, u32, vp]
         L.rap_smem_transpose_bench.argtypes = [u32, i32, u32, u64, u32, u32, u32p, u64p, vp]
+        L.rap_transpose_to_peers.argtypes = [vp, i64, i64, i64, ctypes.POINTER(ctypes.c_void_p), u32, u32, i64,
+                                             u32, i32, u64, vp]
         for f in ("rap_perm_gen", "rap_transpose", "rap_congestion", "rap_congestion_sweep",
                   "rap_congestion_sweep_algo", "rap_congestion_trace", "rap_unpack_blocks",
-                  "rap_smem_transpose_bench"):
+                  "rap_smem_transpose_bench", "rap_transpose_to_peers"):
             getattr(L, f).restype = i32
         if L.rap_abi_version() != 1:
             raise ImportError("librap.so ABI version mismatch")
@@ -145,6 +148,23 @@ def transpose(x: torch.Tensor, layout: str = "rap", seed: int = 0,
                                    rows, cols, ld_src, ld_dst, eb, LAYOUTS[layout], seed,
                                    _stream(x)), "rap_transpose")
     return out
+
+
+def transpose_to_peers(shard: torch.Tensor, peer_ptrs, rank: int, ld_dst: int | None = None,
+                       layout: str = "rap", seed: int = 0) -> None:
+    """Fused sharded transpose (NEXT-2): this rank's row block [M, N] straight into every rank's
+    output shard.  peer_ptrs: G device addresses (ints) of the [M, ld_dst] output shards, valid in
+    this process.  Enqueue only -- the caller barriers across ranks before reading its shard."""
+    _need_cuda(shard)
+    M, N = shard.shape
+    G = len(peer_ptrs)
+    if shard.stride(1) != 1:
+        raise ValueError("shard needs unit inner stride")
+    arr = (ctypes.c_void_p * G)(*[ctypes.c_void_p(int(p)) for p in peer_ptrs])
+    with _on(shard.device):
+        _check(lib().rap_transpose_to_peers(ctypes.c_void_p(shard.data_ptr()), M, N, shard.stride(0) if M > 1 else N,
+                                            arr, G, rank, N if ld_dst is None else ld_dst, shard.element_size(),
+                                            LAYOUTS[layout], seed, _stream(shard)), "rap_transpose_to_peers")
 
 
 def congestion(rows: torch.Tensor, cols: torch.Tensor, scheme: str = "rap",

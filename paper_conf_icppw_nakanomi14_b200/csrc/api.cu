@@ -82,6 +82,35 @@ rap_status_t rap_transpose(const void *src, void *dst, int64_t rows, int64_t col
                                             (int)layout, seed, (cudaStream_t)stream));
 }
 
+rap_status_t rap_transpose_to_peers(const void *src, int64_t M, int64_t N, int64_t ld_src,
+                                    void *const *peer_dst, uint32_t G, uint32_t rank, int64_t ld_dst,
+                                    uint32_t elem_bytes, rap_layout_t layout, uint64_t seed, void *stream) {
+    if (elem_bytes != 4 && elem_bytes != 8) return RAP_ERR_INVALID_ARG;
+    if ((int)layout < RAP_LAYOUT_RAW || (int)layout > RAP_LAYOUT_RAP) return RAP_ERR_INVALID_ARG;
+    if (G < 1 || G > (uint32_t)rapk::kMaxPeers || rank >= G || !peer_dst) return RAP_ERR_INVALID_ARG;
+    if (M <= 0 || M % 32 != 0) return RAP_ERR_INVALID_ARG;
+    int64_t gm;
+    if (!mul_ok((int64_t)G, M, &gm) || N != gm) return RAP_ERR_INVALID_ARG;
+    if (!src || ld_src < N || ld_dst < N) return RAP_ERR_INVALID_ARG;
+    if ((uintptr_t)src % elem_bytes) return RAP_ERR_INVALID_ARG;
+    rapk::PeerOut pe;
+    pe.G = (int)G;
+    pe.M = M;
+    pe.col_off = (int64_t)rank * M;
+    uintptr_t s_lo, s_hi;
+    if (!extent((uintptr_t)src, M, N, ld_src, elem_bytes, &s_lo, &s_hi)) return RAP_ERR_INVALID_ARG;
+    for (uint32_t h = 0; h < G; ++h) {
+        if (!peer_dst[h] || (uintptr_t)peer_dst[h] % elem_bytes) return RAP_ERR_INVALID_ARG;
+        uintptr_t d_lo, d_hi;
+        if (!extent((uintptr_t)peer_dst[h], M, N, ld_dst, elem_bytes, &d_lo, &d_hi)) return RAP_ERR_INVALID_ARG;
+        if (s_lo < d_hi && d_lo < s_hi) return RAP_ERR_ALIAS;
+        pe.ptr[h] = (uint64_t)(uintptr_t)peer_dst[h];
+    }
+    if ((M / 32) * ((N + 31) / 32) >= (int64_t(1) << 31)) return RAP_ERR_UNSUPPORTED;
+    return from_cuda(rapk::launch_transpose_peers(src, M, N, ld_src, pe, ld_dst, elem_bytes, (int)layout,
+                                                  seed, (cudaStream_t)stream));
+}
+
 rap_status_t rap_congestion(uint32_t w, uint64_t n_warps, const uint32_t *d_rows,
                             const uint32_t *d_cols, rap_scheme_t scheme, const uint32_t *d_shift,
                             uint32_t *d_congestion_out, void *stream) {

@@ -9,6 +9,16 @@
 namespace rapk {
 
 constexpr int kMaxDevices = 64;
+constexpr int kMaxPeers = 16;
+
+// Fused-exchange output (NEXT-2): the output shard base of each of the G ranks, as pointers
+// valid in this process (mapped peer memory), M = rows per rank, col_off = rank * M.
+struct PeerOut {
+    uint64_t ptr[kMaxPeers] = {};
+    int64_t M = 1;
+    int64_t col_off = 0;
+    int G = 0;
+};
 
 // Launch-shape knobs of the transpose (defaults chosen by tools/tune_transpose.cu on B200).
 struct TransposeTuning {
@@ -33,6 +43,9 @@ cudaError_t launch_transpose_tuned(const void *src, void *dst, int64_t rows, int
 cudaError_t launch_transpose(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
                              int64_t ld_dst, uint32_t elem_bytes, int layout, uint64_t seed,
                              cudaStream_t st);
+
+cudaError_t launch_transpose_peers(const void *src, int64_t M, int64_t N, int64_t ld_src, const PeerOut &pe,
+                                   int64_t ld_dst, uint32_t elem_bytes, int layout, uint64_t seed, cudaStream_t st);
 
 cudaError_t launch_perm_gen(uint64_t seed, uint64_t first, uint64_t count, uint32_t w, uint8_t *out,
                             cudaStream_t st);

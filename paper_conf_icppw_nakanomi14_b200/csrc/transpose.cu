@@ -77,11 +77,11 @@ struct TileCfg {
 // owns tile (w % SR, w / SR) of the block, and a CTA barrier before the drains makes the SC*32
 // input rows / SR*32-element output row runs of neighbouring warps reach DRAM together
 // (measured: +2-4 % over free-running warps, profiles/r01_tune_transpose.txt).
-template <int L, int EW, bool VEC, int DEPTH, int MINB, bool VST, int SR, int SC>
+template <int L, int EW, bool VEC, int DEPTH, int MINB, bool VST, int SR, int SC, bool PEERS>
 __global__ void __launch_bounds__(SR * SC * 32, MINB)
 transpose_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, int64_t rows,
                  int64_t cols, int64_t ld_src, int64_t ld_dst, uint64_t seed, uint32_t tiles_r,
-                 uint32_t tiles_c, bool vst_ok) {
+                 uint32_t tiles_c, bool vst_ok, PeerOut peers) {
     using C = TileCfg<L, EW>;
     constexpr int NE = C::NE, R = C::R, G = C::G, LPR = C::LPR;
     constexpr int PW = 32 * Geom<L>::RP;            // plane size in words
@@ -169,13 +169,23 @@ transpose_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, i
     auto drain = [&](uint32_t ti, uint32_t tj) {
         const int64_t r0 = (int64_t)ti * 32, c0 = (int64_t)tj * 32;
         const int64_t ostride = ld_dst * EW;                       // words between output rows
-        uint32_t *o = dst + (c0 * ld_dst + r0 + lane) * EW;        // this lane's column
+        // output tile origin: (c0, r0) of dst, or -- fused exchange (NEXT-2) -- of the output
+        // shard of rank h = c0 / M, written straight over NVLink through its mapped pointer
+        uint32_t *obase = dst;
+        int64_t orow = c0, ocol = r0;
+        if (PEERS) {
+            const int64_t h = c0 / peers.M;
+            obase = reinterpret_cast<uint32_t *>(peers.ptr[h]);
+            orow = c0 - h * peers.M;
+            ocol = peers.col_off + r0;
+        }
+        uint32_t *o = obase + (orow * ld_dst + ocol + lane) * EW;    // this lane's column
         if (VST && vst_ok && (r0 + 32 <= rows) && (c0 + 32 <= cols)) {
             // 128-bit stores: each lane reads NE consecutive columns of its row, a butterfly of
             // __shfl_xor_sync transposes NE x NE blocks among NE lanes, and lane NE*p + k then
             // holds rows NE*p .. NE*p+NE-1 of column c+k -- one 16-byte chunk of output row c+k.
             const uint32_t k = lane % NE, p = lane / NE;
-            uint32_t *ob = dst + ((c0 + k) * ld_dst + r0 + NE * p) * EW;
+            uint32_t *ob = obase + ((orow + k) * ld_dst + ocol + NE * p) * EW;
 #pragma unroll
             for (int cg = 0; cg < 32 / NE; ++cg) {
                 uint32_t r[4];
@@ -325,20 +335,25 @@ TransposeTuning default_tuning(uint32_t elem_bytes) {
     return t;
 }
 
-template <int L, int EW, bool VEC, int DEPTH, int MINB, bool VST, int SR, int SC>
+template <int L, int EW, bool VEC, int DEPTH, int MINB, bool VST, int SR, int SC, bool PEERS = false>
 static cudaError_t launch_one(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
-                              int64_t ld_dst, uint64_t seed, const TransposeTuning &tu, cudaStream_t st) {
+                              int64_t ld_dst, uint64_t seed, const TransposeTuning &tu, cudaStream_t st,
+                              const PeerOut &peers = PeerOut{}) {
     const uint32_t tiles_r = (uint32_t)((rows + 31) / 32), tiles_c = (uint32_t)((cols + 31) / 32);
     const int64_t nst = (int64_t)((tiles_r + SR - 1) / SR) * ((tiles_c + SC - 1) / SC);
-    auto k = transpose_kernel<L, EW, VEC, DEPTH, MINB, VST, SR, SC>;
+    auto k = transpose_kernel<L, EW, VEC, DEPTH, MINB, VST, SR, SC, PEERS>;
     static ShapeCache cache;
-    const bool vst_ok = ((uintptr_t)dst % 16 == 0) && ((ld_dst * EW * 4) % 16 == 0);
+    bool vst_ok = ((uintptr_t)dst % 16 == 0) && ((ld_dst * EW * 4) % 16 == 0);
+    if (PEERS) {
+        vst_ok = ((ld_dst * EW * 4) % 16 == 0) && ((peers.col_off * EW * 4) % 16 == 0);
+        for (int h = 0; h < peers.G; ++h) vst_ok = vst_ok && (peers.ptr[h] % 16 == 0);
+    }
     const size_t smem = sizeof(uint32_t) * warp_smem_words<L, EW>() * SR * SC;
     int grid = 0;
     const cudaError_t e = grid_for(k, cache, SR * SC * 32, smem, nst, 1, tu.ctas_per_sm, &grid);
     if (e != cudaSuccess) return e;
     k<<<grid, SR * SC * 32, smem, st>>>((const uint32_t *)src, (uint32_t *)dst, rows, cols, ld_src,
-                                        ld_dst, seed, tiles_r, tiles_c, vst_ok);
+                                        ld_dst, seed, tiles_r, tiles_c, vst_ok, peers);
     return cudaGetLastError();
 }
 
@@ -381,6 +396,35 @@ static cudaError_t dispatch(const void *src, void *dst, int64_t rows, int64_t co
     }
 #undef RAPK_CASE
     return cudaErrorInvalidValue;
+}
+
+template <bool VEC>
+static cudaError_t dispatch_peers(const void *src, int64_t rows, int64_t cols, int64_t ld_src, int64_t ld_dst,
+                                  uint32_t eb, int layout, uint64_t seed, const PeerOut &pe, cudaStream_t st) {
+    const TransposeTuning tu = default_tuning(eb);
+#define RAPK_PEER(LAY)                                                                              \
+    case LAY:                                                                                       \
+        return eb == 4                                                                              \
+            ? launch_one<LAY, 1, VEC, kDefaultDepth32, kDefaultMinB32, kDefaultVst32, kDefaultSR32,  \
+                         kDefaultSC32, true>(src, nullptr, rows, cols, ld_src, ld_dst, seed, tu, st, pe) \
+            : launch_one<LAY, 2, VEC, kDefaultDepth64, kDefaultMinB64, kDefaultVst64, kDefaultSR64,  \
+                         kDefaultSC64, true>(src, nullptr, rows, cols, ld_src, ld_dst, seed, tu, st, pe);
+    switch (layout) {
+        RAPK_PEER(RAP_LAYOUT_RAW)
+        RAPK_PEER(RAP_LAYOUT_PAD)
+        RAPK_PEER(RAP_LAYOUT_XOR)
+        RAPK_PEER(RAP_LAYOUT_RAS)
+        RAPK_PEER(RAP_LAYOUT_RAP)
+    }
+#undef RAPK_PEER
+    return cudaErrorInvalidValue;
+}
+
+cudaError_t launch_transpose_peers(const void *src, int64_t M, int64_t N, int64_t ld_src, const PeerOut &pe,
+                                   int64_t ld_dst, uint32_t elem_bytes, int layout, uint64_t seed, cudaStream_t st) {
+    const bool vec = ((uintptr_t)src % 16 == 0) && ((ld_src * elem_bytes) % 16 == 0);
+    return vec ? dispatch_peers<true>(src, M, N, ld_src, ld_dst, elem_bytes, layout, seed, pe, st)
+               : dispatch_peers<false>(src, M, N, ld_src, ld_dst, elem_bytes, layout, seed, pe, st);
 }
 
 cudaError_t launch_transpose_tuned(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,

@@ -19,6 +19,7 @@ import torch.distributed as dist
 
 from . import congestion_sweep as _sweep
 from . import transpose as _transpose
+from . import transpose_to_peers as _to_peers
 from . import unpack_blocks as _unpack
 
 
@@ -70,3 +71,33 @@ def transpose_sharded(shard: torch.Tensor, group=None, layout: str = "rap", seed
     dist.all_to_all_single(recv, send, group=group)   # T4: M x M blocks, NCCL over NVLink
     up(recv, out, world)                              # T4: place the blocks
     return out
+
+
+class FusedTranspose:
+    """NEXT-2: the sharded transpose as ONE kernel per rank writing over NVLink into the peers'
+    output shards (torch symmetric memory maps every rank's output buffer into every process).
+    No send/receive buffers, no all-to-all, no unpack: each element is read once from local HBM
+    and written once, over NVLink when it belongs to another rank.
+
+        ft = FusedTranspose((M, N), torch.float32, group)
+        out = ft(shard)          # [M, N] symmetric tensor, rows rank*M.. of A^T, valid on return
+    """
+
+    def __init__(self, shape, dtype, group=None, layout: str = "rap", seed: int = 0):
+        from torch.distributed import _symmetric_memory as symm
+        self.group = group if group is not None else dist.group.WORLD
+        self.rank, self.world = dist.get_rank(self.group), dist.get_world_size(self.group)
+        M, N = shape
+        if N != self.world * M or M % 32:
+            raise ValueError("fused transpose needs N = world * M and M a multiple of 32")
+        self.out = symm.empty((M, N), dtype=dtype, device=torch.device("cuda", torch.cuda.current_device()))
+        self.handle = symm.rendezvous(self.out, self.group)
+        self.ptrs = [int(p) for p in self.handle.buffer_ptrs]
+        self.layout, self.seed = layout, seed
+
+    def __call__(self, shard: torch.Tensor) -> torch.Tensor:
+        # every rank must be done reading its shard's previous contents before peers overwrite it
+        self.handle.barrier(channel=0)
+        _to_peers(shard, self.ptrs, self.rank, layout=self.layout, seed=self.seed)
+        self.handle.barrier(channel=0)      # all peers' stores into this shard have landed
+        return self.out

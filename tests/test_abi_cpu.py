@@ -122,6 +122,22 @@ def test_smem_bench_and_unpack_validation(L):
     assert L.rap_unpack_blocks(d, P(0x40000000), 0, 8, 16, 4, s) == OK
 
 
+def test_transpose_to_peers_validation(L):
+    f = L.rap_transpose_to_peers
+    f.argtypes = [ctypes.c_void_p, ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, ctypes.POINTER(ctypes.c_void_p),
+                  ctypes.c_uint32, ctypes.c_uint32, ctypes.c_int64, ctypes.c_uint32, ctypes.c_int, ctypes.c_uint64,
+                  ctypes.c_void_p]
+    peers = (ctypes.c_void_p * 2)(0x40000000, 0x50000000)
+    src, s = P(0x10000000), P(0)
+    assert f(src, 64, 128, 128, peers, 2, 2, 128, 4, 4, 0, s) == INVALID     # rank >= G
+    assert f(src, 48, 96, 96, peers, 2, 0, 96, 4, 4, 0, s) == INVALID        # M not a multiple of 32
+    assert f(src, 64, 100, 128, peers, 2, 0, 128, 4, 4, 0, s) == INVALID     # N != G*M
+    assert f(src, 64, 128, 128, peers, 17, 0, 128, 4, 4, 0, s) == INVALID    # too many peers
+    assert f(src, 64, 128, 128, peers, 2, 0, 100, 4, 4, 0, s) == INVALID     # ld_dst < N
+    alias = (ctypes.c_void_p * 2)(0x10000000, 0x50000000)
+    assert f(src, 64, 128, 128, alias, 2, 0, 128, 4, 4, 0, s) == ALIAS
+
+
 def test_python_binding_refuses_cpu_tensors(L):
     x = torch.zeros(8, 8)
     with pytest.raises(ValueError):

@@ -329,3 +329,52 @@ def test_smem_transpose_bench_results(rap, oracle, alg, scheme, elem):
     assert all(np.array_equal(o1[k], AT) for k in range(40))
     assert all(np.array_equal(o2[k], A) for k in range(40))
     assert (c1.cpu().numpy() > 0).all()
+
+
+# ------------------------------------------------------------------ NEXT-2 fused exchange
+@pytest.mark.parametrize("dtype", [torch.float32, torch.float64])
+@pytest.mark.parametrize("G,M", [(1, 64), (2, 96), (4, 64), (8, 32), (3, 160)])
+@pytest.mark.parametrize("layout", ["rap", "raw"])
+def test_transpose_to_peers_emulated(rap, oracle, dtype, G, M, layout):
+    # G virtual ranks on one GPU: "peer" output shards are local buffers; every rank's kernel
+    # writes its tiles into the owners' shards.  The union must be the oracle's A^T.
+    N = G * M
+    A = workloads.random_bits(N, N, dtype, seed=G * 7 + M)
+    Ad = A.cuda()
+    outs = [torch.zeros((M, N), dtype=dtype, device="cuda") for _ in range(G)]
+    ptrs = [o.data_ptr() for o in outs]
+    for g in range(G):
+        rap.transpose_to_peers(Ad[g * M:(g + 1) * M], ptrs, g, layout=layout, seed=5)
+    torch.cuda.synchronize()
+    assert np.array_equal(bits(torch.cat(outs, 0)), oracle.transpose(bits(A)))
+
+
+def test_transpose_to_peers_padded_pitch(rap, oracle):
+    G, M = 2, 64
+    N = G * M
+    A = workloads.random_bits(N, N, torch.float32, seed=3)
+    outs = [torch.zeros((M, N + 8), dtype=torch.float32, device="cuda") for _ in range(G)]
+    for g in range(G):
+        rap.transpose_to_peers(A.cuda()[g * M:(g + 1) * M], [o.data_ptr() for o in outs], g, ld_dst=N + 8)
+    torch.cuda.synchronize()
+    got = torch.cat([o[:, :N] for o in outs], 0)
+    assert np.array_equal(bits(got), oracle.transpose(bits(A)))
+    assert not bits(torch.cat([o[:, N:] for o in outs], 0)).any()
+
+
+def test_fused_transpose_symmetric_memory_world1(rap, oracle):
+    # the host path of NEXT-2 (symmetric-memory rendezvous + barriers) under a real NCCL group
+    import os
+    import torch.distributed as dist
+    from paper_conf_icppw_nakanomi14_b200 import dist as rdist
+    os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+    os.environ.setdefault("MASTER_PORT", "29563")
+    dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
+    try:
+        A = workloads.random_bits(256, 256, torch.float32, seed=11)
+        ft = rdist.FusedTranspose((256, 256), torch.float32)
+        out = ft(A.cuda())
+        torch.cuda.synchronize()
+        assert np.array_equal(bits(out), oracle.transpose(bits(A)))
+    finally:
+        dist.destroy_process_group()
