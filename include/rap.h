@@ -40,7 +40,8 @@ extern "C" {
 #endif
 
 #define RAP_ABI_VERSION 1
-#define RAP_MAX_W 32
+#define RAP_MAX_W 32          /* warp-wide evaluators: one CUDA warp = one DMM warp          */
+#define RAP_MAX_W_SWEEP 256   /* rap_congestion_sweep: w > 32 runs one trial per CUDA thread */
 
 typedef enum {
     RAP_OK = 0,
@@ -133,7 +134,9 @@ rap_status_t rap_congestion(uint32_t w, uint64_t n_warps, const uint32_t *d_rows
  * d_hist: device uint64_t[npat][nsch][w+1] where npat = popcount(pattern_mask) and
  * nsch = popcount(scheme_mask), patterns/schemes in enum order; ACCUMULATED (+=), so the
  * caller zeroes it once and may split a run into any chunks (bit-identical sums).
- * Masks are bit sets of rap_pattern_t / rap_scheme_t (1..31).  XOR needs w = 2^k. */
+ * Masks are bit sets of rap_pattern_t / rap_scheme_t (1..31).  XOR needs w = 2^k.
+ * 2 <= w <= RAP_MAX_W_SWEEP (256, Table II's widths): w <= 32 maps a DMM warp onto a CUDA warp,
+ * 32 < w <= 256 simulates one trial per CUDA thread (NEXT-3; RAP_SWEEP_DEFAULT only). */
 rap_status_t rap_congestion_sweep(uint32_t w, uint32_t pattern_mask, uint32_t scheme_mask,
                                   uint64_t seed, uint64_t first_trial, uint64_t n_trials,
                                   uint64_t *d_hist, void *stream);

@@ -129,14 +129,16 @@ rap_status_t rap_congestion(uint32_t w, uint64_t n_warps, const uint32_t *d_rows
 rap_status_t rap_congestion_sweep_algo(uint32_t w, uint32_t pattern_mask, uint32_t scheme_mask,
                                        uint64_t seed, uint64_t first_trial, uint64_t n_trials,
                                        uint64_t *d_hist, uint32_t algo, void *stream) {
-    if (w < 2 || w > RAP_MAX_W) return RAP_ERR_INVALID_ARG;
+    if (w < 2 || w > RAP_MAX_W_SWEEP) return RAP_ERR_INVALID_ARG;
+    if (w > RAP_MAX_W && algo != RAP_SWEEP_DEFAULT) return RAP_ERR_UNSUPPORTED;
     if (pattern_mask == 0 || pattern_mask > 31u || scheme_mask == 0 || scheme_mask > 31u)
         return RAP_ERR_INVALID_ARG;
     if (((scheme_mask >> RAP_SCHEME_XOR) & 1u) && !is_pow2(w)) return RAP_ERR_INVALID_ARG;
     if (algo > RAP_SWEEP_MATCH) return RAP_ERR_INVALID_ARG;
     if (n_trials == 0) return RAP_OK;
     if (!d_hist) return RAP_ERR_INVALID_ARG;
-    auto launch = algo == RAP_SWEEP_MATCH ? rapk::launch_sweep_match : rapk::launch_sweep;
+    auto launch = w > RAP_MAX_W ? rapk::launch_sweep_wide
+                : algo == RAP_SWEEP_MATCH ? rapk::launch_sweep_match : rapk::launch_sweep;
     return from_cuda(launch(w, pattern_mask, scheme_mask, seed, first_trial, n_trials, d_hist,
                             (cudaStream_t)stream));
 }

@@ -75,7 +75,7 @@ def test_valid_calls_fail_loudly_without_gpu(L):
 def test_sweep_validation(L):
     h, s = P(0x30000000), P(0)
     assert L.rap_congestion_sweep(1, 31, 7, 1, 0, 10, h, s) == INVALID    # w < 2
-    assert L.rap_congestion_sweep(33, 31, 7, 1, 0, 10, h, s) == INVALID   # w > 32
+    assert L.rap_congestion_sweep(257, 31, 7, 1, 0, 10, h, s) == INVALID  # w > 256
     assert L.rap_congestion_sweep(32, 0, 7, 1, 0, 10, h, s) == INVALID    # empty pattern mask
     assert L.rap_congestion_sweep(32, 32, 7, 1, 0, 10, h, s) == INVALID   # unknown pattern
     assert L.rap_congestion_sweep(32, 31, 64, 1, 0, 10, h, s) == INVALID  # unknown scheme
@@ -87,6 +87,7 @@ def test_sweep_validation(L):
                                             ctypes.c_void_p, ctypes.c_uint32, ctypes.c_void_p]
     assert L.rap_congestion_sweep_algo(32, 31, 7, 1, 0, 10, h, 2, s) == INVALID   # unknown algo
     assert L.rap_congestion_sweep_algo(32, 31, 7, 1, 0, 0, h, 1, s) == OK
+    assert L.rap_congestion_sweep_algo(64, 31, 7, 1, 0, 10, h, 1, s) == UNSUPPORTED  # match kernel: w <= 32
 
 
 def test_congestion_trace_perm_validation(L):

@@ -378,3 +378,33 @@ def test_fused_transpose_symmetric_memory_world1(rap, oracle):
         assert np.array_equal(bits(out), oracle.transpose(bits(A)))
     finally:
         dist.destroy_process_group()
+
+
+# ------------------------------------------------------------------ NEXT-3 wide DMM warps
+@pytest.mark.parametrize("w", [33, 48, 64, 100, 128, 256])
+def test_sweep_wide_bit_exact(rap, oracle, w):
+    N = 3001 if w <= 128 else 1201
+    sch = ["raw", "ras", "rap", "pad"] + (["xor"] if w & (w - 1) == 0 else [])
+    g = rap.congestion_sweep(N, seed=21, w=w, patterns=ALL_PAT, schemes=sch, first_trial=2 ** 35 + 3)
+    o = oracle.sweep(w, ALL_PAT, sch, 21, 2 ** 35 + 3, N)
+    assert np.array_equal(g.cpu().numpy().astype(np.uint64), o)
+
+
+@pytest.mark.parametrize("w,N", [(64, 400_000), (128, 200_000), (256, 100_000)])
+def test_table2_wide_columns_on_gpu(rap, w, N):
+    # Table II columns w = 64, 128, 256 from the GPU sweep: every entry within
+    # rounding (0.005) + the 99% Monte-Carlo interval; contiguous / RAP stride exactly 1.
+    col = [16, 32, 64, 128, 256].index(w)
+    import os
+    from conftest import golden
+    rows = [ln.split() for ln in open(golden("table2.txt")) if ln.strip() and not ln.startswith("#")]
+    table = {(r[0], r[1]): float(r[2 + col]) for r in rows}
+    pats, schs = ["contiguous", "stride", "diagonal", "random"], ["raw", "ras", "rap"]
+    h = rap.congestion_sweep(N, seed=4, w=w, patterns=pats, schemes=schs).cpu().numpy().astype(np.float64)
+    c = np.arange(w + 1)
+    for pi, p in enumerate(pats):
+        for si, s in enumerate(schs):
+            mu = (h[pi, si] * c).sum() / N
+            sd = np.sqrt((h[pi, si] * (c - mu) ** 2).sum() / N)
+            assert abs(mu - table[(p, s)]) <= 0.005 + 2.576 * sd / math.sqrt(N) + 1e-12, (p, s, mu)
+    assert h[0, :, 1].tolist() == [N] * 3 and h[1, 2, 1] == N
