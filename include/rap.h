@@ -79,6 +79,26 @@ typedef enum {
                              /* (t,t); PAD -> (t,(w-t) mod w)       (reading iii)*/
 } rap_pattern_t;
 
+/* §VII: schemes and warp patterns of a w x w x w x w array (NEXT-3). */
+typedef enum {
+    RAP_SCHEME4_RAW = 0,  /* f = 0                                                        */
+    RAP_SCHEME4_RAS = 1,  /* f = r[i][j][k], w^3 independent shifts (domain 1, index (i*w+j)*w+k) */
+    RAP_SCHEME4_1P = 2,   /* f = P[k]                                  (One permutation)   */
+    RAP_SCHEME4_R1P = 3,  /* f = P[i] + P[j] + P[k] mod w              (Repeated one perm.)*/
+    RAP_SCHEME4_3P = 4    /* f = P[i] + Q[j] + R[k] mod w; Q, R from domains 3, 4 (3 perms) */
+} rap_scheme4_t;
+
+typedef enum {
+    RAP_PAT4_CONTIGUOUS = 0,  /* a[0][0][0][t]                                            */
+    RAP_PAT4_STRIDE1 = 1,     /* a[0][0][t][0]                                            */
+    RAP_PAT4_STRIDE2 = 2,     /* a[0][t][0][0]                                            */
+    RAP_PAT4_STRIDE3 = 3,     /* a[t][0][0][0]                                            */
+    RAP_PAT4_RANDOM = 4,      /* w cells of w^4 i.i.d. with replacement (domain 2)        */
+    RAP_PAT4_MALICIOUS = 5    /* RAW, RAS: stride1; 1P: stride2; R1P, 3P: floor(w/6) groups of */
+                              /* the 6 permutations of (3g, 3g+1, 3g+2) at l = 0;  */
+                              /* remaining lanes repeat lane 0's request (merged)          */
+} rap_pattern4_t;
+
 int rap_abi_version(void);
 const char *rap_status_str(rap_status_t s);
 
@@ -140,6 +160,13 @@ rap_status_t rap_congestion(uint32_t w, uint64_t n_warps, const uint32_t *d_rows
 rap_status_t rap_congestion_sweep(uint32_t w, uint32_t pattern_mask, uint32_t scheme_mask,
                                   uint64_t seed, uint64_t first_trial, uint64_t n_trials,
                                   uint64_t *d_hist, void *stream);
+
+/* NEXT-3 -- §VII Monte-Carlo sweep over a w^4 array (Table IV): trial n draws
+ * P, Q, R (domains 0, 3, 4), the random cells (domain 2) and the RAS shifts it needs (domain 1)
+ * and counts the congestion of each selected (rap_pattern4_t, rap_scheme4_t).  4 <= w <= 32;
+ * pattern_mask 1..63, scheme_mask 1..31; d_hist: device uint64_t[npat][nsch][w+1], ACCUMULATED. */
+rap_status_t rap_congestion_sweep4(uint32_t w, uint32_t pattern_mask, uint32_t scheme_mask, uint64_t seed,
+                                   uint64_t first_trial, uint64_t n_trials, uint64_t *d_hist, void *stream);
 
 /* Kernel designs of the sweep (identical histograms):
  *   RAP_SWEEP_DEFAULT  lane-mode bit-sliced Fisher-Yates (one trial per lane, no shuffles)

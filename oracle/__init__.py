@@ -73,9 +73,18 @@ def lib():
         L.oracle_dmm_time.argtypes = [p, u32, u32]
         L.oracle_dmm_time.restype = i64
         L.oracle_max_threads.argtypes = []
+        L.oracle_perm_domain.argtypes = [u64, u64, u32, u32, p]
+        L.oracle_shift4.argtypes = [u32, u32, u32, u32, u32, p, p, p, u64, u64]
+        L.oracle_shift4.restype = i64
+        L.oracle_address4.argtypes = [u32, u32, u32, u32, u32, u32, p, p, p, u64, u64]
+        L.oracle_address4.restype = i64
+        L.oracle_congestion4.argtypes = [u32, u32, p, p, p, p, u32, p, p, p, u64, u64, p]
+        L.oracle_pattern4.argtypes = [u32, u32, u32, u64, u64, p, p, p, p]
+        L.oracle_sweep4.argtypes = [u32, u32, u32, u64, u64, u64, p, ctypes.c_int]
         for name in ("oracle_perm", "oracle_ras_shifts", "oracle_random_cells", "oracle_congestion",
                      "oracle_pattern_cells", "oracle_sweep", "oracle_transpose", "oracle_rap_layout",
-                     "oracle_max_threads"):
+                     "oracle_max_threads", "oracle_perm_domain", "oracle_congestion4", "oracle_pattern4",
+                     "oracle_sweep4"):
             getattr(L, name).restype = ctypes.c_int
         _lib = L
     return _lib
@@ -199,3 +208,50 @@ def dmm_time(congestions, latency: int) -> int:
     if t < 0:
         raise ValueError("oracle dmm_time rejected its arguments")
     return t
+
+
+# ---------------------------------------------------------------- O13: w^4 arrays (paper §VII)
+S4 = {"raw": 0, "ras": 1, "1p": 2, "r1p": 3, "3p": 4}
+P4 = {"contiguous": 0, "stride1": 1, "stride2": 2, "stride3": 3, "random": 4, "malicious": 5}
+
+
+def perm_domain(seed: int, n: int, w: int, d: int) -> np.ndarray:
+    a = np.zeros(w, dtype=np.uint32)
+    _check(lib().oracle_perm_domain(seed, n, w, d, _ptr(a)), "perm_domain")
+    return a
+
+
+def _u32(x, w):
+    return np.ascontiguousarray(np.zeros(w, np.uint32) if x is None else x, dtype=np.uint32)
+
+
+def address4(scheme: int, w: int, i, j, k, l, P=None, Q=None, R=None, seed=0, n=0) -> int:
+    P, Q, R = _u32(P, w), _u32(Q, w), _u32(R, w)
+    a = int(lib().oracle_address4(scheme, w, i, j, k, l, _ptr(P), _ptr(Q), _ptr(R), seed, n))
+    if a < 0:
+        raise ValueError("oracle address4 rejected its arguments")
+    return a
+
+
+def congestion4(w: int, cells, scheme: int, P=None, Q=None, R=None, seed=0, n=0) -> int:
+    c = np.ascontiguousarray(cells, dtype=np.uint32).reshape(-1, 4)
+    ci, cj, ck, cl = (np.ascontiguousarray(c[:, m]) for m in range(4))
+    P, Q, R = _u32(P, w), _u32(Q, w), _u32(R, w)
+    out = np.zeros(1, dtype=np.uint32)
+    _check(lib().oracle_congestion4(w, c.shape[0], _ptr(ci), _ptr(cj), _ptr(ck), _ptr(cl), scheme, _ptr(P),
+                                    _ptr(Q), _ptr(R), seed, n, _ptr(out)), "congestion4")
+    return int(out[0])
+
+
+def pattern4(pattern: int, scheme: int, w: int, seed: int = 0, n: int = 0) -> np.ndarray:
+    c = [np.zeros(w, dtype=np.uint32) for _ in range(4)]
+    _check(lib().oracle_pattern4(pattern, scheme, w, seed, n, *[_ptr(x) for x in c]), "pattern4")
+    return np.stack(c, 1)
+
+
+def sweep4(w: int, patterns, schemes, seed: int, first: int, n_trials: int, threads: int | None = None):
+    pm, sm = _mask(patterns, P4), _mask(schemes, S4)
+    hist = np.zeros((bin(pm).count("1"), bin(sm).count("1"), w + 1), dtype=np.uint64)
+    th = max_threads() if threads is None else threads
+    _check(lib().oracle_sweep4(w, pm, sm, seed, first, n_trials, _ptr(hist), th), "sweep4")
+    return hist

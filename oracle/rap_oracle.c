@@ -36,6 +36,18 @@
  *   O11 RAP layout: phys[i][(j+P[i]) mod w] = logical[i][j] (Fig.6).
  *   O12 DMM time of warps with congestions c_1..c_m: sum(c) + l - 1.
  *
+ *   O13 §VII higher-dimensional RAP: a w x w x w x w array, a[i][j][k][l] at
+ *       address i*w^3 + j*w^2 + k*w + l, bank l; a scheme stores a[i][j][k][l] at
+ *       a[i][j][k][(l + f(i,j,k)) mod w] with
+ *         RAW f = 0;  RAS f = r[i][j][k], r = floor(word(1, i*w^2+j*w+k) * w / 2^32);
+ *         1P  f = P[k];  R1P f = P[i] + P[j] + P[k];  3P f = P[i] + Q[j] + R[k]
+ *       (P, Q, R = Durstenfeld permutations from domains 0, 3, 4 -- reading xiii).
+ *       Warp patterns, lane t: contiguous (0,0,0,t); stride1 (0,0,t,0); stride2 (0,t,0,0);
+ *       stride3 (t,0,0,0); random: w cells of w^4 i.i.d. with replacement (domain 2);
+ *       malicious: RAW, RAS -> stride1; 1P -> stride2; R1P, 3P -> the paper's groups of the 6
+ *       permutations of (x, y, z), group g = (3g, 3g+1, 3g+2), l = 0, lanes past
+ *       6*floor(w/6) repeat lane 0's request (merged).
+ *
  * Every function returns 0 on success and a negative value on a bad argument.
  */
 #include <stdint.h>
@@ -86,16 +98,21 @@ uint32_t oracle_word(uint64_t seed, uint64_t n, uint32_t d, uint32_t t)
 static uint32_t mulshift(uint32_t u, uint32_t m) { return (uint32_t)(((uint64_t)u * m) >> 32); }
 
 /* ---------------- O3: permutation P (Durstenfeld / Fisher-Yates) ---------------- */
-int oracle_perm(uint64_t seed, uint64_t n, uint32_t w, uint32_t *a)
+int oracle_perm_domain(uint64_t seed, uint64_t n, uint32_t w, uint32_t d, uint32_t *a)
 {
     if (w < 1 || w > ORACLE_MAX_W || !a) return -1;
     for (uint32_t i = 0; i < w; ++i) a[i] = i;
     for (uint32_t k = w - 1; k >= 1; --k) {
-        uint32_t u = oracle_word(seed, n, D_FY, w - 1 - k);
+        uint32_t u = oracle_word(seed, n, d, w - 1 - k);
         uint32_t j = mulshift(u, k + 1);
         uint32_t tmp = a[k]; a[k] = a[j]; a[j] = tmp;
     }
     return 0;
+}
+
+int oracle_perm(uint64_t seed, uint64_t n, uint32_t w, uint32_t *a)
+{
+    return oracle_perm_domain(seed, n, w, D_FY, a);
 }
 
 /* ---------------- O4: RAS shift vector ---------------- */
@@ -281,6 +298,161 @@ int64_t oracle_dmm_time(const uint32_t *congestion, uint32_t m, uint32_t latency
     int64_t stages = 0;
     for (uint32_t i = 0; i < m; ++i) stages += congestion[i];
     return stages + latency - 1;
+}
+
+/* ---------------- O13: higher-dimensional RAP (w^4 arrays) ---------------- */
+enum { S4_RAW = 0, S4_RAS = 1, S4_1P = 2, S4_R1P = 3, S4_3P = 4, S4_N = 5 };
+enum { P4_CONTIGUOUS = 0, P4_STRIDE1 = 1, P4_STRIDE2 = 2, P4_STRIDE3 = 3, P4_RANDOM = 4,
+       P4_MALICIOUS = 5, P4_N = 6 };
+enum { D_Q = 3, D_R = 4 };
+
+/* shift f(i,j,k) of a scheme; P, Q, R given, RAS shifts drawn from the counter contract */
+int64_t oracle_shift4(uint32_t scheme, uint32_t w, uint32_t i, uint32_t j, uint32_t k,
+                      const uint32_t *P, const uint32_t *Q, const uint32_t *R, uint64_t seed, uint64_t n)
+{
+    if (i >= w || j >= w || k >= w) return -1;
+    switch (scheme) {
+    case S4_RAW: return 0;
+    case S4_RAS: return mulshift(oracle_word(seed, n, D_RAS, (i * w + j) * w + k), w);
+    case S4_1P: return P[k];
+    case S4_R1P: return ((uint64_t)P[i] + P[j] + P[k]) % w;
+    case S4_3P: return ((uint64_t)P[i] + Q[j] + R[k]) % w;
+    default: return -1;
+    }
+}
+
+/* physical address of a[i][j][k][l] */
+int64_t oracle_address4(uint32_t scheme, uint32_t w, uint32_t i, uint32_t j, uint32_t k, uint32_t l,
+                        const uint32_t *P, const uint32_t *Q, const uint32_t *R, uint64_t seed, uint64_t n)
+{
+    if (l >= w) return -1;
+    int64_t f = oracle_shift4(scheme, w, i, j, k, P, Q, R, seed, n);
+    if (f < 0) return -1;
+    int64_t w2 = (int64_t)w * w;
+    return ((int64_t)i * w2 + (int64_t)j * w) * w + (int64_t)k * w + (l + f) % w;
+}
+
+/* congestion of n requests to cells (i,j,k,l): distinct addresses per bank (address mod w) */
+int oracle_congestion4(uint32_t w, uint32_t nreq, const uint32_t *ci, const uint32_t *cj, const uint32_t *ck,
+                       const uint32_t *cl, uint32_t scheme, const uint32_t *P, const uint32_t *Q,
+                       const uint32_t *R, uint64_t seed, uint64_t n, uint32_t *congestion_out)
+{
+    if (w < 1 || w > ORACLE_MAX_W || nreq > ORACLE_MAX_W || !congestion_out) return -1;
+    int64_t addr[ORACLE_MAX_W];
+    for (uint32_t t = 0; t < nreq; ++t) {
+        addr[t] = oracle_address4(scheme, w, ci[t], cj[t], ck[t], cl[t], P, Q, R, seed, n);
+        if (addr[t] < 0) return -1;
+    }
+    uint32_t count[ORACLE_MAX_W];
+    memset(count, 0, sizeof(count));
+    for (uint32_t t = 0; t < nreq; ++t) {
+        int duplicate = 0;
+        for (uint32_t s = 0; s < t; ++s)
+            if (addr[s] == addr[t]) { duplicate = 1; break; }
+        if (!duplicate) count[addr[t] % w] += 1;
+    }
+    uint32_t c = 0;
+    for (uint32_t b = 0; b < w; ++b)
+        if (count[b] > c) c = count[b];
+    *congestion_out = c;
+    return 0;
+}
+
+int oracle_pattern4(uint32_t pattern, uint32_t scheme, uint32_t w, uint64_t seed, uint64_t n,
+                    uint32_t *ci, uint32_t *cj, uint32_t *ck, uint32_t *cl)
+{
+    if (w < 1 || w > 255 || scheme >= S4_N) return -1;
+    if (pattern == P4_MALICIOUS) {
+        if (scheme == S4_RAW || scheme == S4_RAS) pattern = P4_STRIDE1;
+        else if (scheme == S4_1P) pattern = P4_STRIDE2;
+        else {
+            /* the 6 permutations of (x, y, z) = (3g, 3g+1, 3g+2) share f under R1P */
+            uint32_t groups = w / 6;
+            for (uint32_t t = 0; t < w; ++t) {
+                uint32_t g = t / 6, m = t % 6;
+                if (g >= groups || 3 * g + 2 >= w) { g = 0; m = 0; }
+                uint32_t x = 3 * g, y = 3 * g + 1, z = 3 * g + 2;
+                static const int perm6[6][3] = {{0, 1, 2}, {0, 2, 1}, {1, 0, 2}, {1, 2, 0}, {2, 0, 1}, {2, 1, 0}};
+                uint32_t v[3] = {x, y, z};
+                ci[t] = v[perm6[m][0]]; cj[t] = v[perm6[m][1]]; ck[t] = v[perm6[m][2]]; cl[t] = 0;
+            }
+            return 0;
+        }
+    }
+    for (uint32_t t = 0; t < w; ++t) {
+        ci[t] = cj[t] = ck[t] = cl[t] = 0;
+        switch (pattern) {
+        case P4_CONTIGUOUS: cl[t] = t; break;
+        case P4_STRIDE1: ck[t] = t; break;
+        case P4_STRIDE2: cj[t] = t; break;
+        case P4_STRIDE3: ci[t] = t; break;
+        case P4_RANDOM: {
+            uint64_t w4 = (uint64_t)w * w * w * w;
+            uint32_t cell = (uint32_t)(((uint64_t)oracle_word(seed, n, D_RANDOM, t) * w4) >> 32);
+            cl[t] = cell % w; cell /= w;
+            ck[t] = cell % w; cell /= w;
+            cj[t] = cell % w; cell /= w;
+            ci[t] = cell;
+            break;
+        }
+        default: return -1;
+        }
+    }
+    return 0;
+}
+
+static int sweep4_range(uint32_t w, uint32_t pattern_mask, uint32_t scheme_mask, uint64_t seed,
+                        uint64_t first, uint64_t count, uint64_t *hist)
+{
+    const uint32_t ns = __builtin_popcount(scheme_mask);
+    uint32_t P[ORACLE_MAX_W], Q[ORACLE_MAX_W], R[ORACLE_MAX_W];
+    uint32_t ci[ORACLE_MAX_W], cj[ORACLE_MAX_W], ck[ORACLE_MAX_W], cl[ORACLE_MAX_W];
+    for (uint64_t q = 0; q < count; ++q) {
+        uint64_t n = first + q;
+        oracle_perm_domain(seed, n, w, D_FY, P);
+        oracle_perm_domain(seed, n, w, D_Q, Q);
+        oracle_perm_domain(seed, n, w, D_R, R);
+        uint32_t pi = 0;
+        for (uint32_t p = 0; p < P4_N; ++p) {
+            if (!((pattern_mask >> p) & 1u)) continue;
+            uint32_t si = 0;
+            for (uint32_t sc = 0; sc < S4_N; ++sc) {
+                if (!((scheme_mask >> sc) & 1u)) continue;
+                uint32_t c;
+                if (oracle_pattern4(p, sc, w, seed, n, ci, cj, ck, cl)) return -1;
+                if (oracle_congestion4(w, w, ci, cj, ck, cl, sc, P, Q, R, seed, n, &c)) return -1;
+                hist[((uint64_t)pi * ns + si) * (w + 1) + c] += 1;
+                ++si;
+            }
+            ++pi;
+        }
+    }
+    return 0;
+}
+
+/* hist: u64[popcount(pattern_mask)][popcount(scheme_mask)][w+1], ACCUMULATED */
+int oracle_sweep4(uint32_t w, uint32_t pattern_mask, uint32_t scheme_mask, uint64_t seed,
+                  uint64_t first, uint64_t n_trials, uint64_t *hist, int threads)
+{
+    if (w < 2 || w > 64 || !hist) return -1;
+    if (pattern_mask == 0 || pattern_mask > 63 || scheme_mask == 0 || scheme_mask > 31) return -1;
+    const size_t nbins = (size_t)__builtin_popcount(pattern_mask) * __builtin_popcount(scheme_mask) * (w + 1);
+    if (threads < 1) threads = 1;
+    uint64_t *part = (uint64_t *)calloc((size_t)threads * nbins, sizeof(uint64_t));
+    if (!part) return -2;
+    int err = 0;
+#ifdef _OPENMP
+#pragma omp parallel for num_threads(threads) schedule(static) reduction(|:err)
+#endif
+    for (int th = 0; th < threads; ++th) {
+        uint64_t lo = n_trials * (uint64_t)th / (uint64_t)threads;
+        uint64_t hi = n_trials * (uint64_t)(th + 1) / (uint64_t)threads;
+        err |= sweep4_range(w, pattern_mask, scheme_mask, seed, first + lo, hi - lo, part + (size_t)th * nbins);
+    }
+    for (int th = 0; th < threads; ++th)
+        for (size_t b = 0; b < nbins; ++b) hist[b] += part[(size_t)th * nbins + b];
+    free(part);
+    return err ? -1 : 0;
 }
 
 int oracle_max_threads(void)

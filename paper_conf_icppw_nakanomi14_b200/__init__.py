@@ -64,12 +64,13 @@ def lib():
         L.rap_congestion_sweep_algo.argtypes = [u32, u32, u32, u64, u64, u64, u64p, u32, vp]
         L.rap_congestion_trace.argtypes = [u32, u64, u32p, u32, u64, u64, u64, u64p, vp]
         L.rap_unpack_blocks.argtypes = [vp, vp, i64, i64, i64, u32, vp]
+        L.rap_congestion_sweep4.argtypes = [u32, u32, u32, u64, u64, u64, u64p, vp]
         L.rap_smem_transpose_bench.argtypes = [u32, i32, u32, u64, u32, u32, u32p, u64p, vp]
         L.rap_transpose_to_peers.argtypes = [vp, i64, i64, i64, ctypes.POINTER(ctypes.c_void_p), u32, u32, i64,
                                              u32, i32, u64, vp]
         for f in ("rap_perm_gen", "rap_transpose", "rap_congestion", "rap_congestion_sweep",
                   "rap_congestion_sweep_algo", "rap_congestion_trace", "rap_unpack_blocks",
-                  "rap_smem_transpose_bench", "rap_transpose_to_peers"):
+                  "rap_smem_transpose_bench", "rap_transpose_to_peers", "rap_congestion_sweep4"):
             getattr(L, f).restype = i32
         if L.rap_abi_version() != 1:
             raise ImportError("librap.so ABI version mismatch")
@@ -261,3 +262,22 @@ def smem_transpose_bench(algorithm: str, scheme: str, elem_bytes: int = 4, seed:
                                               ctypes.c_void_p(cyc.data_ptr()), _stream(out)),
                "rap_smem_transpose_bench")
     return out, cyc
+
+
+SCHEMES4 = {"raw": 0, "ras": 1, "1p": 2, "r1p": 3, "3p": 4}
+PATTERNS4 = {"contiguous": 0, "stride1": 1, "stride2": 2, "stride3": 3, "random": 4, "malicious": 5}
+
+
+def congestion_sweep4(n_trials: int, seed: int, w: int = 32, patterns=tuple(PATTERNS4), schemes=tuple(SCHEMES4),
+                      first_trial: int = 0, out: torch.Tensor | None = None, device="cuda") -> torch.Tensor:
+    """§VII sweep over a w^4 array (Table IV): int64 [npat, nsch, w+1], ACCUMULATED into `out`."""
+    pm, sm = _mask(patterns, PATTERNS4), _mask(schemes, SCHEMES4)
+    shape = (bin(pm).count("1"), bin(sm).count("1"), w + 1)
+    if out is None:
+        out = torch.zeros(shape, dtype=torch.int64, device=device)
+    _need_cuda(out)
+    assert tuple(out.shape) == shape and out.dtype == torch.int64 and out.is_contiguous()
+    with _on(out.device):
+        _check(lib().rap_congestion_sweep4(w, pm, sm, seed, first_trial, n_trials, ctypes.c_void_p(out.data_ptr()),
+                                           _stream(out)), "rap_congestion_sweep4")
+    return out

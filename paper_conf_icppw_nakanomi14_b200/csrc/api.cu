@@ -150,6 +150,17 @@ rap_status_t rap_congestion_sweep(uint32_t w, uint32_t pattern_mask, uint32_t sc
                                      d_hist, RAP_SWEEP_DEFAULT, stream);
 }
 
+rap_status_t rap_congestion_sweep4(uint32_t w, uint32_t pattern_mask, uint32_t scheme_mask, uint64_t seed,
+                                   uint64_t first_trial, uint64_t n_trials, uint64_t *d_hist, void *stream) {
+    if (w < 4 || w > RAP_MAX_W) return RAP_ERR_INVALID_ARG;
+    if (pattern_mask == 0 || pattern_mask > 63u || scheme_mask == 0 || scheme_mask > 31u)
+        return RAP_ERR_INVALID_ARG;
+    if (n_trials == 0) return RAP_OK;
+    if (!d_hist) return RAP_ERR_INVALID_ARG;
+    return from_cuda(rapk::launch_sweep4(w, pattern_mask, scheme_mask, seed, first_trial, n_trials, d_hist,
+                                         (cudaStream_t)stream));
+}
+
 rap_status_t rap_congestion_trace(uint32_t w, uint64_t n_warps, const uint32_t *d_cells,
                                   uint32_t scheme_mask, uint64_t seed, uint64_t first_trial,
                                   uint64_t n_trials, uint64_t *d_hist, void *stream) {

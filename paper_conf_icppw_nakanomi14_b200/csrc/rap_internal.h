@@ -62,6 +62,9 @@ cudaError_t launch_sweep_match(uint32_t w, uint32_t pattern_mask, uint32_t schem
 cudaError_t launch_sweep_wide(uint32_t w, uint32_t pattern_mask, uint32_t scheme_mask, uint64_t seed,
                               uint64_t first, uint64_t n_trials, uint64_t *hist, cudaStream_t st);
 
+cudaError_t launch_sweep4(uint32_t w, uint32_t pattern_mask, uint32_t scheme_mask, uint64_t seed,
+                          uint64_t first, uint64_t n_trials, uint64_t *hist, cudaStream_t st);
+
 cudaError_t launch_trace(uint32_t w, uint64_t n_warps, const uint32_t *cells, uint32_t scheme_mask,
                          uint64_t seed, uint64_t first, uint64_t n_trials, uint64_t *hist,
                          cudaStream_t st);

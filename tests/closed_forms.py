@@ -74,3 +74,17 @@ def variance(pmf):
 
 # OEIS A006717: transversals in the cyclic Latin square of order 2n+1 (n = 0..5).
 CYCLIC_TRANSVERSALS_ODD = {1: 1, 3: 3, 5: 15, 7: 133, 9: 2025, 11: 37851}
+
+
+def random_access_cdf_cells(w: int, m: int, cells_per_bank: int) -> Fraction:
+    """w requests i.i.d. uniform over w * cells_per_bank cells (w banks of cells_per_bank cells
+    each), equal cells merged: Pr[max distinct per bank <= m]
+    = w!/(w*c)^w [x^w] (sum_{k<=m} C(c,k) (e^x-1)^k)^w."""
+    n = w
+    egf = [Fraction(0)] * (n + 1)
+    for k in range(0, min(m, cells_per_bank) + 1):
+        term = _exp_minus_one_pow(k, n)
+        cc = comb(cells_per_bank, k)
+        for i in range(n + 1):
+            egf[i] += cc * term[i]
+    return _pow(egf, w, n)[n] * factorial(w) / Fraction(w * cells_per_bank) ** w

@@ -139,6 +139,18 @@ def test_transpose_to_peers_validation(L):
     assert f(src, 64, 128, 128, alias, 2, 0, 128, 4, 4, 0, s) == ALIAS
 
 
+def test_sweep4_validation(L):
+    h, s = P(0x30000000), P(0)
+    f = L.rap_congestion_sweep4
+    f.argtypes = [ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_uint64,
+                  ctypes.c_uint64, ctypes.c_void_p, ctypes.c_void_p]
+    assert f(3, 63, 31, 1, 0, 10, h, s) == INVALID
+    assert f(33, 63, 31, 1, 0, 10, h, s) == INVALID
+    assert f(32, 64, 31, 1, 0, 10, h, s) == INVALID
+    assert f(32, 63, 32, 1, 0, 10, h, s) == INVALID
+    assert f(32, 63, 31, 1, 0, 0, P(0), s) == OK
+
+
 def test_python_binding_refuses_cpu_tensors(L):
     x = torch.zeros(8, 8)
     with pytest.raises(ValueError):

@@ -408,3 +408,31 @@ def test_table2_wide_columns_on_gpu(rap, w, N):
             sd = np.sqrt((h[pi, si] * (c - mu) ** 2).sum() / N)
             assert abs(mu - table[(p, s)]) <= 0.005 + 2.576 * sd / math.sqrt(N) + 1e-12, (p, s, mu)
     assert h[0, :, 1].tolist() == [N] * 3 and h[1, 2, 1] == N
+
+
+# ------------------------------------------------------------------ NEXT-3 §VII w^4 arrays
+ALL_P4 = ["contiguous", "stride1", "stride2", "stride3", "random", "malicious"]
+ALL_S4 = ["raw", "ras", "1p", "r1p", "3p"]
+
+
+@pytest.mark.parametrize("w", [4, 6, 7, 16, 32])
+def test_sweep4_bit_exact(rap, oracle, w):
+    N = 20_000
+    g = rap.congestion_sweep4(N, seed=8, w=w, first_trial=777)
+    o = oracle.sweep4(w, ALL_P4, ALL_S4, 8, 777, N)
+    assert np.array_equal(g.cpu().numpy().astype(np.uint64), o)
+
+
+def test_sweep4_table4_entries_w32(rap):
+    N = 1_000_000
+    h = rap.congestion_sweep4(N, seed=3, w=32).cpu().numpy()
+    one = lambda p, s: h[ALL_P4.index(p), ALL_S4.index(s), 1] == N
+    full = lambda p, s: h[ALL_P4.index(p), ALL_S4.index(s), 32] == N
+    for s in ALL_S4:
+        assert one("contiguous", s)
+    for p in ("stride1", "stride2", "stride3"):
+        assert full(p, "raw") and one(p, "r1p") and one(p, "3p")
+    assert one("stride1", "1p") and full("stride2", "1p") and full("stride3", "1p")
+    # R1P malicious: every group of 6 hits one bank, so the congestion is a multiple of 6
+    mal = h[ALL_P4.index("malicious"), ALL_S4.index("r1p")]
+    assert mal.sum() == N and all(mal[c] == 0 for c in range(33) if c % 6)
