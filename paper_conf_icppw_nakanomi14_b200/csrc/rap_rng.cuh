@@ -30,11 +30,6 @@ __device__ __forceinline__ uint4 philox_block(uint64_t seed, uint64_t n, uint32_
                          (uint32_t)seed, (uint32_t)(seed >> 32));
 }
 
-__device__ __forceinline__ uint32_t pick(uint4 v, uint32_t k);
-
-// one word, word(seed, n, d, t), computed on its own (random access into the stream)
-__device__ __forceinline__ uint32_t word_at(uint64_t seed, uint64_t n, uint32_t d, uint32_t t);
-
 __device__ __forceinline__ uint32_t pick(uint4 v, uint32_t k) {
     uint32_t x = v.x;
     x = (k == 1) ? v.y : x;
@@ -43,6 +38,7 @@ __device__ __forceinline__ uint32_t pick(uint4 v, uint32_t k) {
     return x;
 }
 
+// one word, word(seed, n, d, t), computed on its own (random access into the stream)
 __device__ __forceinline__ uint32_t word_at(uint64_t seed, uint64_t n, uint32_t d, uint32_t t) {
     return pick(philox_block(seed, n, d, t >> 2), t & 3u);
 }
