@@ -216,6 +216,18 @@ rap_status_t rap_smem_transpose_bench(uint32_t algorithm, rap_scheme_t scheme, u
                                       uint64_t seed, uint32_t n_blocks, uint32_t reps, uint32_t *d_out,
                                       uint64_t *d_cycles, void *stream);
 
+/* NEXT-4 -- a data-dependent shared-memory access under a given layout (the paper's motivation:
+ * addresses not known beforehand).  One CTA of 1024 threads applies the
+ * tile permutation `reps` times inside shared memory: thread o writes element o (row o/32,
+ * contiguous) from source element d_src_index[o] of the previous array (a gather), for
+ * o = 0..1023.  d_src_index: device uint16_t[1024], values < 1024 (need not be a permutation).
+ * Layouts: RAW, PAD [32][33], XOR [i][j^i], RAS, RAP; CTA k uses P/r of (seed, k).
+ * d_out: device uint32_t[n_blocks][1024] final array (initial value of element o is o), i.e.
+ * out[o] = src^reps(o); d_cycles: device uint64_t[n_blocks] SM cycles of the timed loop. */
+rap_status_t rap_smem_gather_bench(const uint16_t *d_src_index, rap_layout_t layout, uint64_t seed,
+                                   uint32_t n_blocks, uint32_t reps, uint32_t *d_out, uint64_t *d_cycles,
+                                   void *stream);
+
 #ifdef __cplusplus
 }
 #endif

@@ -81,10 +81,11 @@ def lib():
         L.oracle_congestion4.argtypes = [u32, u32, p, p, p, p, u32, p, p, p, u64, u64, p]
         L.oracle_pattern4.argtypes = [u32, u32, u32, u64, u64, p, p, p, p]
         L.oracle_sweep4.argtypes = [u32, u32, u32, u64, u64, u64, p, ctypes.c_int]
+        L.oracle_gather_power.argtypes = [p, u32, u32, p]
         for name in ("oracle_perm", "oracle_ras_shifts", "oracle_random_cells", "oracle_congestion",
                      "oracle_pattern_cells", "oracle_sweep", "oracle_transpose", "oracle_rap_layout",
                      "oracle_max_threads", "oracle_perm_domain", "oracle_congestion4", "oracle_pattern4",
-                     "oracle_sweep4"):
+                     "oracle_sweep4", "oracle_gather_power"):
             getattr(L, name).restype = ctypes.c_int
         _lib = L
     return _lib
@@ -255,3 +256,11 @@ def sweep4(w: int, patterns, schemes, seed: int, first: int, n_trials: int, thre
     th = max_threads() if threads is None else threads
     _check(lib().oracle_sweep4(w, pm, sm, seed, first, n_trials, _ptr(hist), th), "sweep4")
     return hist
+
+
+def gather_power(idx, reps: int) -> np.ndarray:
+    """x_{k+1}[o] = x_k[idx[o]] applied `reps` times to x_0[o] = o (NEXT-4 reference)."""
+    i = np.ascontiguousarray(idx, dtype=np.uint16)
+    out = np.zeros(i.size, dtype=np.uint32)
+    _check(lib().oracle_gather_power(_ptr(i), i.size, reps, _ptr(out)), "gather_power")
+    return out

@@ -47,6 +47,7 @@
  *       malicious: RAW, RAS -> stride1; 1P -> stride2; R1P, 3P -> the paper's groups of the 6
  *       permutations of (x, y, z), group g = (3g, 3g+1, 3g+2), l = 0, lanes past
  *       6*floor(w/6) repeat lane 0's request (merged).
+ *   O14 data-dependent tile gather (NEXT-4): x_{k+1}[o] = x_k[idx[o]], x_0[o] = o.
  *
  * Every function returns 0 on success and a negative value on a bad argument.
  */
@@ -453,6 +454,22 @@ int oracle_sweep4(uint32_t w, uint32_t pattern_mask, uint32_t scheme_mask, uint6
         for (size_t b = 0; b < nbins; ++b) hist[b] += part[(size_t)th * nbins + b];
     free(part);
     return err ? -1 : 0;
+}
+
+/* ---------------- O14: data-dependent tile gather (NEXT-4) ---------------- */
+/* out = in composed `reps` times with the gather idx: x_{k+1}[o] = x_k[idx[o]], x_0[o] = o */
+int oracle_gather_power(const uint16_t *idx, uint32_t n, uint32_t reps, uint32_t *out)
+{
+    if (!idx || !out || n == 0 || n > 65536) return -1;
+    uint32_t *tmp = (uint32_t *)malloc((size_t)n * sizeof(uint32_t));
+    if (!tmp) return -2;
+    for (uint32_t o = 0; o < n; ++o) { if (idx[o] >= n) { free(tmp); return -1; } out[o] = o; }
+    for (uint32_t k = 0; k < reps; ++k) {
+        for (uint32_t o = 0; o < n; ++o) tmp[o] = out[idx[o]];
+        memcpy(out, tmp, (size_t)n * sizeof(uint32_t));
+    }
+    free(tmp);
+    return 0;
 }
 
 int oracle_max_threads(void)

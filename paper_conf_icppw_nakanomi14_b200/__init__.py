@@ -65,12 +65,14 @@ def lib():
         L.rap_congestion_trace.argtypes = [u32, u64, u32p, u32, u64, u64, u64, u64p, vp]
         L.rap_unpack_blocks.argtypes = [vp, vp, i64, i64, i64, u32, vp]
         L.rap_congestion_sweep4.argtypes = [u32, u32, u32, u64, u64, u64, u64p, vp]
+        L.rap_smem_gather_bench.argtypes = [vp, i32, u64, u32, u32, u32p, u64p, vp]
         L.rap_smem_transpose_bench.argtypes = [u32, i32, u32, u64, u32, u32, u32p, u64p, vp]
         L.rap_transpose_to_peers.argtypes = [vp, i64, i64, i64, ctypes.POINTER(ctypes.c_void_p), u32, u32, i64,
                                              u32, i32, u64, vp]
         for f in ("rap_perm_gen", "rap_transpose", "rap_congestion", "rap_congestion_sweep",
                   "rap_congestion_sweep_algo", "rap_congestion_trace", "rap_unpack_blocks",
-                  "rap_smem_transpose_bench", "rap_transpose_to_peers", "rap_congestion_sweep4"):
+                  "rap_smem_transpose_bench", "rap_transpose_to_peers", "rap_congestion_sweep4",
+                  "rap_smem_gather_bench"):
             getattr(L, f).restype = i32
         if L.rap_abi_version() != 1:
             raise ImportError("librap.so ABI version mismatch")
@@ -281,3 +283,17 @@ def congestion_sweep4(n_trials: int, seed: int, w: int = 32, patterns=tuple(PATT
         _check(lib().rap_congestion_sweep4(w, pm, sm, seed, first_trial, n_trials, ctypes.c_void_p(out.data_ptr()),
                                            _stream(out)), "rap_congestion_sweep4")
     return out
+
+
+def smem_gather_bench(src_index: torch.Tensor, layout: str = "rap", seed: int = 0, n_blocks: int = 1, reps: int = 1):
+    """NEXT-4: apply a 32x32-tile gather `reps` times in shared memory under `layout`.
+    src_index: CUDA int16/uint16 [1024].  Returns (final array int32 [n_blocks, 1024], cycles [n_blocks])."""
+    _need_cuda(src_index)
+    assert src_index.numel() == 1024 and src_index.element_size() == 2 and src_index.is_contiguous()
+    out = torch.empty((n_blocks, 1024), dtype=torch.int32, device=src_index.device)
+    cyc = torch.empty(n_blocks, dtype=torch.int64, device=src_index.device)
+    with _on(out.device):
+        _check(lib().rap_smem_gather_bench(ctypes.c_void_p(src_index.data_ptr()), LAYOUTS[layout], seed, n_blocks,
+                                           reps, ctypes.c_void_p(out.data_ptr()), ctypes.c_void_p(cyc.data_ptr()),
+                                           _stream(out)), "rap_smem_gather_bench")
+    return out, cyc

@@ -205,4 +205,14 @@ rap_status_t rap_smem_transpose_bench(uint32_t algorithm, rap_scheme_t scheme, u
                                              d_cycles, (cudaStream_t)stream));
 }
 
+rap_status_t rap_smem_gather_bench(const uint16_t *d_src_index, rap_layout_t layout, uint64_t seed,
+                                   uint32_t n_blocks, uint32_t reps, uint32_t *d_out, uint64_t *d_cycles,
+                                   void *stream) {
+    if ((int)layout < RAP_LAYOUT_RAW || (int)layout > RAP_LAYOUT_RAP) return RAP_ERR_INVALID_ARG;
+    if (n_blocks == 0) return RAP_OK;
+    if (n_blocks > (1u << 24) || !d_src_index || !d_out || !d_cycles) return RAP_ERR_INVALID_ARG;
+    return from_cuda(rapk::launch_smem_gather(d_src_index, (int)layout, seed, n_blocks, reps, d_out, d_cycles,
+                                              (cudaStream_t)stream));
+}
+
 }  // extern "C"

@@ -75,4 +75,7 @@ cudaError_t launch_unpack_blocks(const void *recv, void *out, int64_t G, int64_t
 cudaError_t launch_smem_bench(uint32_t alg, int scheme, uint32_t elem_bytes, uint64_t seed, uint32_t n_blocks,
                               uint32_t reps, uint32_t *out, uint64_t *cycles, cudaStream_t st);
 
+cudaError_t launch_smem_gather(const uint16_t *src_index, int layout, uint64_t seed, uint32_t n_blocks,
+                               uint32_t reps, uint32_t *out, uint64_t *cycles, cudaStream_t st);
+
 }  // namespace rapk

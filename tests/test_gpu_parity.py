@@ -436,3 +436,15 @@ def test_sweep4_table4_entries_w32(rap):
     # R1P malicious: every group of 6 hits one bank, so the congestion is a multiple of 6
     mal = h[ALL_P4.index("malicious"), ALL_S4.index("r1p")]
     assert mal.sum() == N and all(mal[c] == 0 for c in range(33) if c % 6)
+
+
+# ------------------------------------------------------------------ NEXT-4 data-dependent gather
+@pytest.mark.parametrize("layout", LAYOUT_NAMES)
+def test_smem_gather_results(rap, oracle, layout):
+    for name, idx in workloads.tile_gather_patterns(seed=3).items():
+        for reps in (1, 3):
+            out, cyc = rap.smem_gather_bench(torch.from_numpy(idx.view(np.int16)).cuda(), layout, seed=5,
+                                             n_blocks=8, reps=reps)
+            exp = oracle.gather_power(idx, reps)
+            got = out.cpu().numpy().astype(np.uint32)
+            assert all(np.array_equal(got[k], exp) for k in range(8)), (name, layout, reps)

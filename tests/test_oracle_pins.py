@@ -383,3 +383,15 @@ def test_transpose_strided_source(oracle):
 def test_transpose_empty(oracle):
     A = np.zeros((0, 5), dtype=np.uint32)
     assert oracle.transpose(A).shape == (5, 0)
+
+
+def test_gather_power_definition(oracle):
+    # O14: a permutation applied to the identity is itself; its inverse undoes it; order divides
+    rng = np.random.default_rng(1)
+    p = rng.permutation(1024).astype(np.uint16)
+    assert np.array_equal(oracle.gather_power(p, 1), p)
+    inv = np.argsort(p).astype(np.uint16)
+    assert np.array_equal(oracle.gather_power(p, 2), p[p])
+    t = (np.arange(1024) % 32) * 32 + np.arange(1024) // 32       # transpose is an involution
+    assert np.array_equal(oracle.gather_power(t.astype(np.uint16), 2), np.arange(1024))
+    assert np.array_equal(oracle.gather_power(p, 1)[inv], np.arange(1024))

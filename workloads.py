@@ -89,3 +89,26 @@ def trace_cells(n_warps: int, w: int = 32, seed: int = 0, device="cpu") -> torch
             r, c = cells // w, cells % w
         out[k] = r * w + c
     return torch.from_numpy(out.astype(np.int32)).to(device)
+
+
+def tile_gather_patterns(seed: int = 0):
+    """NEXT-4 inputs: 1024-entry source-index tables of a 32 x 32 tile (thread o = 32 s + t of
+    warp s reads element src[o]).  Each table is a permutation of the tile; the adversarial ones
+    put all 32 reads of a warp into one bank of a deterministic layout (finding 9):
+      identity   warp s reads row s                      (contiguous)
+      transpose  warp s reads column s                   (stride; RAW's worst case)
+      diagonal   warp s reads (t, (t + s) mod 32)        (RAP's worst case, ~3.61)
+      antidiag   warp s reads (t, (s - t) mod 32)        (+1 padding: (row + col) constant -> 32-way)
+      xordiag    warp s reads (t, t xor s)               (XOR swizzle: col xor row constant -> 32-way)
+      random     a seeded uniformly random permutation
+    """
+    t = np.arange(32)
+    tabs = {}
+    rows = lambda f: np.concatenate([f(s) for s in range(32)]).astype(np.uint16)
+    tabs["identity"] = np.arange(1024, dtype=np.uint16)
+    tabs["transpose"] = rows(lambda s: t * 32 + s)
+    tabs["diagonal"] = rows(lambda s: t * 32 + (t + s) % 32)
+    tabs["antidiag"] = rows(lambda s: t * 32 + (s - t) % 32)
+    tabs["xordiag"] = rows(lambda s: t * 32 + (t ^ s))
+    tabs["random"] = np.random.default_rng(seed).permutation(1024).astype(np.uint16)
+    return tabs
