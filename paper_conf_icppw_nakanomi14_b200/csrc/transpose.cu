@@ -369,6 +369,8 @@ static cudaError_t launch_shape(const void *src, void *dst, int64_t rows, int64_
     RAPK_SHAPE(1, 1, false, 16, 1) RAPK_SHAPE(1, 2, false, 16, 1) RAPK_SHAPE(2, 1, false, 16, 1)
     RAPK_SHAPE(1, 1, false, 8, 2) RAPK_SHAPE(1, 1, false, 12, 1) RAPK_SHAPE(1, 1, true, 16, 1)
     RAPK_SHAPE(2, 2, false, 8, 1) RAPK_SHAPE(1, 1, false, 6, 1) RAPK_SHAPE(1, 2, false, 6, 1)
+    RAPK_SHAPE(2, 1, false, 8, 2) RAPK_SHAPE(2, 1, false, 4, 2) RAPK_SHAPE(1, 1, false, 4, 4)
+    RAPK_SHAPE(2, 1, false, 4, 4) RAPK_SHAPE(1, 1, true, 8, 2) RAPK_SHAPE(2, 1, false, 12, 1)
 #endif
 #undef RAPK_SHAPE
     (void)tu;

@@ -359,17 +359,15 @@ int main(int argc, char **argv) {
     const int layouts[] = {RAP_LAYOUT_RAP, RAP_LAYOUT_RAW, RAP_LAYOUT_PAD, RAP_LAYOUT_XOR, RAP_LAYOUT_RAS};
     const char *lname[] = {"raw", "pad", "xor", "ras", "rap"};
     struct Shape { int depth, minb; bool vst; int sr, sc; };
-    const Shape shapes[] = {{1, 1, false, 4, 1}, {1, 4, false, 4, 1}, {1, 3, false, 4, 1}, {1, 1, false, 8, 1},
-                            {1, 2, false, 8, 1}, {1, 3, false, 8, 1}, {1, 1, false, 16, 1}, {1, 2, false, 16, 1},
-                            {2, 1, false, 16, 1}, {1, 1, false, 8, 2}, {1, 1, false, 12, 1}, {1, 1, true, 16, 1},
-                            {2, 2, false, 8, 1}, {1, 1, false, 6, 1}, {1, 2, false, 6, 1}};
+    const Shape shapes[] = {{1, 1, false, 8, 2}, {2, 1, false, 8, 2}, {2, 1, false, 4, 2}, {1, 1, false, 4, 4},
+                            {2, 1, false, 4, 4}, {1, 1, true, 8, 2}, {1, 1, false, 4, 1}, {2, 1, false, 12, 1},
+                            {1, 1, false, 12, 1}, {1, 1, false, 8, 2}};
     for (int eb : {4, 8}) {
         const int64_t n = eb == 4 ? n32 : n64;
         const size_t bytes = eb == 4 ? bytes32 : bytes64;
         for (int lay : {RAP_LAYOUT_RAP, RAP_LAYOUT_RAW, RAP_LAYOUT_PAD, RAP_LAYOUT_XOR, RAP_LAYOUT_RAS}) {
             for (const Shape &sh : shapes) {
-                if (lay != RAP_LAYOUT_RAP && !(sh.depth == 1 && sh.minb == 1 && !sh.vst && sh.sr == 16 && sh.sc == 1))
-                    continue;
+                if (lay != RAP_LAYOUT_RAP) continue;
                 const int rp = (lay == RAP_LAYOUT_RAP || lay == RAP_LAYOUT_RAS) ? 64 : (lay == RAP_LAYOUT_PAD ? 33 : 32);
                 if ((size_t)32 * rp * (eb / 4) * 4 * sh.sr * sh.sc > 227 * 1024) continue;   // smem limit
                 for (int cps : {0}) {
