@@ -234,14 +234,20 @@ def main():
     import workloads
 
     world, rank, local = dist_env()
-    dev = torch.device("cuda", local)
+    # one process per GPU; RAP_BENCH_BACKEND=gloo lets several ranks share one GPU to exercise
+    # the multi-rank code paths on a single-GPU box (NCCL refuses duplicate devices)
+    backend = os.environ.get("RAP_BENCH_BACKEND", "nccl")
+    dev = torch.device("cuda", local % torch.cuda.device_count())
     torch.cuda.set_device(dev)
     if world > 1 or args.workload == "dist_fused":
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
         os.environ.setdefault("MASTER_PORT", "29571")
         os.environ.setdefault("RANK", "0")
         os.environ.setdefault("WORLD_SIZE", "1")
-        dist.init_process_group("nccl", device_id=dev)
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(backend)
     stream = torch.cuda.current_stream()
     peak, peak_src = load_peaks()
     wl = args.workload
@@ -308,7 +314,7 @@ def main():
         launches, ev = 0, []
         barrier()
         torch.cuda.synchronize()
-        with Clocks(local) as clk:
+        with Clocks(dev.index) as clk:
             start = torch.cuda.Event(enable_timing=True)
             end = torch.cuda.Event(enable_timing=True)
             start.record(stream)

@@ -28,7 +28,7 @@ struct TransposeTuning {
     int ctas_per_sm = 0;  // persistent grid = #SMs x this (0: as many as fit)
     bool vst = false;     // 128-bit output stores (shuffle-transposed) instead of 32/64-bit rows
 };
-constexpr int kDefaultSR32 = 8, kDefaultSC32 = 2, kDefaultSR64 = 4, kDefaultSC64 = 1;
+constexpr int kDefaultSR32 = 8, kDefaultSC32 = 2, kDefaultSR64 = 12, kDefaultSC64 = 1;
 // measured on B200 (tools/tune_transpose.cu, profiles/r01_tune_transpose.txt)
 constexpr int kDefaultMinB32 = 1, kDefaultMinB64 = 1;
 constexpr int kDefaultDepth32 = 1, kDefaultDepth64 = 1;
