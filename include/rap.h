@@ -123,6 +123,18 @@ rap_status_t rap_transpose(const void *src, void *dst, int64_t rows, int64_t col
                            int64_t ld_src, int64_t ld_dst, uint32_t elem_bytes,
                            rap_layout_t layout, uint64_t seed, void *stream);
 
+/* T1-T3 from and to HOST memory (the end-to-end call): dst = src^T as rap_transpose, but src
+ * and dst are HOST pointers (pinned memory lets the copies overlap).  The matrix moves in row
+ * bands of a multiple of 32 rows: upload of band b+1, transpose of band b and 2-D download of
+ * band b-1 run concurrently on three internal streams (PCIe in both directions at once).
+ * d_workspace: caller-owned DEVICE buffer of workspace_bytes; it holds 4 band buffers, so it must
+ * fit at least 4 * 32 * cols * elem_bytes bytes (larger = fewer, longer bands).  The call is
+ * SYNCHRONOUS: work queued on `stream` before the call completes first, and dst is valid on
+ * return.  Errors as rap_transpose (+ RAP_ERR_INVALID_ARG for a too-small workspace). */
+rap_status_t rap_transpose_host(const void *h_src, void *h_dst, int64_t rows, int64_t cols, int64_t ld_src,
+                                int64_t ld_dst, uint32_t elem_bytes, rap_layout_t layout, uint64_t seed,
+                                void *d_workspace, size_t workspace_bytes, void *stream);
+
 /* T4, fused (NEXT-2) -- the row-block-sharded N x N transpose without the all-to-all: rank
  * `rank` of G holds rows rank*M .. rank*M+M-1 of A (src: M x N, ld_src >= N, N = G*M, M a
  * multiple of 32) and writes every 32 x 32 output tile straight into the output shard of the

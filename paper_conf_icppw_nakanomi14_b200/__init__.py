@@ -18,7 +18,7 @@ import torch
 
 from . import build as _build
 
-__all__ = ["perm_gen", "transpose", "transpose_to_peers", "congestion", "congestion_sweep", "congestion_trace",
+__all__ = ["perm_gen", "transpose", "transpose_host", "transpose_to_peers", "congestion", "congestion_sweep", "congestion_trace",
            "unpack_blocks", "smem_transpose_bench",
            "LAYOUTS", "SCHEMES", "PATTERNS", "RapError", "lib", "library_path"]
 
@@ -65,6 +65,7 @@ def lib():
         L.rap_congestion_trace.argtypes = [u32, u64, u32p, u32, u64, u64, u64, u64p, vp]
         L.rap_unpack_blocks.argtypes = [vp, vp, i64, i64, i64, u32, vp]
         L.rap_congestion_sweep4.argtypes = [u32, u32, u32, u64, u64, u64, u64p, vp]
+        L.rap_transpose_host.argtypes = [vp, vp, i64, i64, i64, i64, u32, i32, u64, vp, ctypes.c_size_t, vp]
         L.rap_smem_gather_bench.argtypes = [vp, i32, u64, u32, u32, u32p, u64p, vp]
         L.rap_smem_transpose_bench.argtypes = [u32, i32, u32, u64, u32, u32, u32p, u64p, vp]
         L.rap_transpose_to_peers.argtypes = [vp, i64, i64, i64, ctypes.POINTER(ctypes.c_void_p), u32, u32, i64,
@@ -72,7 +73,7 @@ def lib():
         for f in ("rap_perm_gen", "rap_transpose", "rap_congestion", "rap_congestion_sweep",
                   "rap_congestion_sweep_algo", "rap_congestion_trace", "rap_unpack_blocks",
                   "rap_smem_transpose_bench", "rap_transpose_to_peers", "rap_congestion_sweep4",
-                  "rap_smem_gather_bench"):
+                  "rap_smem_gather_bench", "rap_transpose_host"):
             getattr(L, f).restype = i32
         if L.rap_abi_version() != 1:
             raise ImportError("librap.so ABI version mismatch")
@@ -150,6 +151,34 @@ def transpose(x: torch.Tensor, layout: str = "rap", seed: int = 0,
         _check(lib().rap_transpose(ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(out.data_ptr()),
                                    rows, cols, ld_src, ld_dst, eb, LAYOUTS[layout], seed,
                                    _stream(x)), "rap_transpose")
+    return out
+
+
+def transpose_host(x: torch.Tensor, out: torch.Tensor | None = None, layout: str = "rap", seed: int = 0,
+                   workspace_bytes: int = 256 << 20, device="cuda") -> torch.Tensor:
+    """End-to-end transpose of a HOST (ideally pinned) 2-D tensor into a host tensor [cols, rows]:
+    row bands stream through the GPU with upload, RAP transpose and download overlapped.
+    Synchronous.  A device workspace of `workspace_bytes` is taken from torch's allocator."""
+    if x.is_cuda:
+        raise ValueError("transpose_host takes host tensors; use transpose() for device tensors")
+    if x.dim() != 2 or x.element_size() not in (4, 8) or x.stride(1) != 1:
+        raise ValueError("transpose_host expects a 2-D host tensor of 4/8-byte elements, unit inner stride")
+    rows, cols = x.shape
+    if out is None:
+        out = torch.empty((cols, rows), dtype=x.dtype, pin_memory=x.is_pinned())
+    if out.is_cuda or out.shape != (cols, rows) or out.dtype != x.dtype or (out.stride(1) != 1 and rows * cols):
+        raise ValueError("out must be a host [cols, rows] tensor of x's dtype with unit inner stride")
+    dev = torch.device(device) if not isinstance(device, torch.device) else device
+    if dev.index is None:
+        dev = torch.device("cuda", torch.cuda.current_device())
+    eb = x.element_size()
+    need = 4 * 32 * cols * eb
+    ws = torch.empty(max(workspace_bytes, need), dtype=torch.uint8, device=dev)
+    with _on(dev):
+        _check(lib().rap_transpose_host(ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(out.data_ptr()), rows, cols,
+                                        x.stride(0) if rows > 1 else cols, out.stride(0) if cols > 1 else rows, eb,
+                                        LAYOUTS[layout], seed, ctypes.c_void_p(ws.data_ptr()), ws.numel(),
+                                        _stream(ws)), "rap_transpose_host")
     return out
 
 

@@ -82,6 +82,25 @@ rap_status_t rap_transpose(const void *src, void *dst, int64_t rows, int64_t col
                                             (int)layout, seed, (cudaStream_t)stream));
 }
 
+rap_status_t rap_transpose_host(const void *h_src, void *h_dst, int64_t rows, int64_t cols, int64_t ld_src,
+                                int64_t ld_dst, uint32_t elem_bytes, rap_layout_t layout, uint64_t seed,
+                                void *d_workspace, size_t workspace_bytes, void *stream) {
+    if (elem_bytes != 4 && elem_bytes != 8) return RAP_ERR_INVALID_ARG;
+    if ((int)layout < RAP_LAYOUT_RAW || (int)layout > RAP_LAYOUT_RAP) return RAP_ERR_INVALID_ARG;
+    if (rows < 0 || cols < 0) return RAP_ERR_INVALID_ARG;
+    if (rows == 0 || cols == 0) return RAP_OK;
+    if (!h_src || !h_dst || !d_workspace) return RAP_ERR_INVALID_ARG;
+    if (ld_src < cols || ld_dst < rows) return RAP_ERR_INVALID_ARG;
+    uintptr_t s_lo, s_hi, d_lo, d_hi;
+    if (!extent((uintptr_t)h_src, rows, cols, ld_src, elem_bytes, &s_lo, &s_hi) ||
+        !extent((uintptr_t)h_dst, cols, rows, ld_dst, elem_bytes, &d_lo, &d_hi))
+        return RAP_ERR_INVALID_ARG;
+    if (s_lo < d_hi && d_lo < s_hi) return RAP_ERR_ALIAS;
+    if (rapk::host_band_rows(rows, cols, elem_bytes, workspace_bytes) == 0) return RAP_ERR_INVALID_ARG;
+    return from_cuda(rapk::transpose_host(h_src, h_dst, rows, cols, ld_src, ld_dst, elem_bytes, (int)layout, seed,
+                                          d_workspace, workspace_bytes, (cudaStream_t)stream));
+}
+
 rap_status_t rap_transpose_to_peers(const void *src, int64_t M, int64_t N, int64_t ld_src,
                                     void *const *peer_dst, uint32_t G, uint32_t rank, int64_t ld_dst,
                                     uint32_t elem_bytes, rap_layout_t layout, uint64_t seed, void *stream) {

@@ -1,0 +1,100 @@
+// host_pipeline.cu -- rap_transpose_host: the transpose of a HOST matrix into a HOST matrix,
+// pipelined over row bands so that PCIe runs both directions at once.
+//
+//   band b (rows b*RB .. b*RB+RB-1 of src):  H2D (stream in)  ->  rap_transpose kernel
+//   (stream compute)  ->  2-D D2H of the cols x RB result into columns b*RB.. of dst (stream out)
+//
+// Two device buffers per direction (double buffering) live in the caller's workspace; events
+// order the three streams, so band b+1 is uploading while band b is transposed and band b-1 is
+// downloading.  The call is synchronous: it returns once dst holds the result.  Host buffers
+// should be pinned (page-locked) for the copies to overlap; pageable memory still works.
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "rap_internal.h"
+
+namespace rapk {
+
+namespace {
+
+struct Streams {
+    cudaStream_t s[3] = {nullptr, nullptr, nullptr};
+    cudaEvent_t ev[3][2] = {};
+    cudaError_t err = cudaSuccess;
+    Streams() {
+        for (auto &x : s)
+            if (err == cudaSuccess) err = cudaStreamCreateWithFlags(&x, cudaStreamNonBlocking);
+        for (auto &row : ev)
+            for (auto &e : row)
+                if (err == cudaSuccess) err = cudaEventCreateWithFlags(&e, cudaEventDisableTiming);
+    }
+    ~Streams() {
+        for (auto &row : ev)
+            for (auto &e : row)
+                if (e) cudaEventDestroy(e);
+        for (auto &x : s)
+            if (x) cudaStreamDestroy(x);
+    }
+};
+
+}  // namespace
+
+size_t host_band_rows(int64_t rows, int64_t cols, uint32_t eb, size_t work_bytes) {
+    // 4 buffers of band_rows x cols elements; bands a multiple of 32 rows (whole tiles)
+    const size_t per_row = (size_t)cols * eb * 4;
+    if (per_row == 0) return 0;
+    size_t rb = work_bytes / per_row;
+    rb = rb / 32 * 32;
+    const size_t cap = (size_t)((rows + 31) / 32 * 32);
+    return rb < cap ? rb : cap;
+}
+
+cudaError_t transpose_host(const void *h_src, void *h_dst, int64_t rows, int64_t cols, int64_t ld_src,
+                           int64_t ld_dst, uint32_t eb, int layout, uint64_t seed, void *d_work,
+                           size_t work_bytes, cudaStream_t user) {
+    const size_t rb = host_band_rows(rows, cols, eb, work_bytes);
+    if (rb == 0) return cudaErrorInvalidValue;
+    Streams st;
+    if (st.err != cudaSuccess) return st.err;
+    cudaStream_t s_in = st.s[0], s_cmp = st.s[1], s_out = st.s[2];
+    // order after whatever the caller queued on its stream
+    cudaEvent_t start;
+    cudaError_t e = cudaEventCreateWithFlags(&start, cudaEventDisableTiming);
+    if (e != cudaSuccess) return e;
+    cudaEventRecord(start, user);
+    for (cudaStream_t x : {s_in, s_cmp, s_out}) cudaStreamWaitEvent(x, start, 0);
+    const size_t band_bytes = rb * (size_t)cols * eb;
+    uint8_t *din[2] = {(uint8_t *)d_work, (uint8_t *)d_work + band_bytes};
+    uint8_t *dout[2] = {(uint8_t *)d_work + 2 * band_bytes, (uint8_t *)d_work + 3 * band_bytes};
+    const int64_t nb = (rows + (int64_t)rb - 1) / (int64_t)rb;
+    for (int64_t b = 0; b < nb && e == cudaSuccess; ++b) {
+        const int k = (int)(b & 1);
+        const int64_t r0 = b * (int64_t)rb;
+        const int64_t nr = (rows - r0 < (int64_t)rb) ? rows - r0 : (int64_t)rb;
+        // H2D: buffer k is free once the transpose of band b-2 has consumed it
+        if (b >= 2) cudaStreamWaitEvent(s_in, st.ev[1][k], 0);
+        e = cudaMemcpy2DAsync(din[k], (size_t)cols * eb, (const uint8_t *)h_src + (size_t)r0 * ld_src * eb,
+                              (size_t)ld_src * eb, (size_t)cols * eb, (size_t)nr, cudaMemcpyHostToDevice, s_in);
+        if (e != cudaSuccess) break;
+        cudaEventRecord(st.ev[0][k], s_in);
+        // transpose: needs the upload, and out buffer k drained by the D2H of band b-2
+        cudaStreamWaitEvent(s_cmp, st.ev[0][k], 0);
+        if (b >= 2) cudaStreamWaitEvent(s_cmp, st.ev[2][k], 0);
+        e = launch_transpose(din[k], dout[k], nr, cols, cols, nr, eb, layout, seed, s_cmp);
+        if (e != cudaSuccess) break;
+        cudaEventRecord(st.ev[1][k], s_cmp);
+        // D2H: cols rows of nr elements into columns r0 .. r0+nr-1 of dst
+        cudaStreamWaitEvent(s_out, st.ev[1][k], 0);
+        e = cudaMemcpy2DAsync((uint8_t *)h_dst + (size_t)r0 * eb, (size_t)ld_dst * eb, dout[k], (size_t)nr * eb,
+                              (size_t)nr * eb, (size_t)cols, cudaMemcpyDeviceToHost, s_out);
+        if (e != cudaSuccess) break;
+        cudaEventRecord(st.ev[2][k], s_out);
+    }
+    cudaError_t e2 = cudaStreamSynchronize(s_out);
+    cudaStreamSynchronize(s_in);
+    cudaStreamSynchronize(s_cmp);
+    cudaEventDestroy(start);
+    return e != cudaSuccess ? e : e2;
+}
+
+}  // namespace rapk

@@ -78,4 +78,9 @@ cudaError_t launch_smem_bench(uint32_t alg, int scheme, uint32_t elem_bytes, uin
 cudaError_t launch_smem_gather(const uint16_t *src_index, int layout, uint64_t seed, uint32_t n_blocks,
                                uint32_t reps, uint32_t *out, uint64_t *cycles, cudaStream_t st);
 
+size_t host_band_rows(int64_t rows, int64_t cols, uint32_t eb, size_t work_bytes);
+cudaError_t transpose_host(const void *h_src, void *h_dst, int64_t rows, int64_t cols, int64_t ld_src,
+                           int64_t ld_dst, uint32_t eb, int layout, uint64_t seed, void *d_work,
+                           size_t work_bytes, cudaStream_t user);
+
 }  // namespace rapk

@@ -448,3 +448,23 @@ def test_smem_gather_results(rap, oracle, layout):
             exp = oracle.gather_power(idx, reps)
             got = out.cpu().numpy().astype(np.uint32)
             assert all(np.array_equal(got[k], exp) for k in range(8)), (name, layout, reps)
+
+
+# ------------------------------------------------------------------ host-to-host pipeline
+@pytest.mark.parametrize("dtype", [torch.float32, torch.float64])
+@pytest.mark.parametrize("shape,ws", [((1000, 300), 4 * 32 * 300 * 8), ((4096, 2048), 8 << 20),
+                                      ((33, 65), 1 << 20), ((2048, 96), 3 * 32 * 96 * 8 * 4 + 1)])
+def test_transpose_host_pipeline(rap, oracle, dtype, shape, ws):
+    r, c = shape
+    x = workloads.random_bits(r, c, dtype, seed=r + c).pin_memory()
+    y = rap.transpose_host(x, layout="rap", seed=2, workspace_bytes=ws)
+    assert np.array_equal(bits(y), oracle.transpose(bits(x)))
+
+
+def test_transpose_host_strided_pageable(rap, oracle):
+    big = workloads.random_bits(300, 260, torch.float32, seed=8)        # pageable, ld 260
+    xs = big[:, :250]
+    out_big = torch.zeros((250, 310), dtype=torch.float32)
+    rap.transpose_host(xs, out=out_big[:, :300], workspace_bytes=1 << 20)
+    assert np.array_equal(bits(out_big[:, :300]), oracle.transpose(bits(xs)))
+    assert not bits(out_big[:, 300:]).any()
