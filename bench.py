@@ -460,7 +460,7 @@ def main():
                        "h2d_bytes_per_step": hx.numel() * eb * world, "d2h_bytes_per_step": hy.numel() * eb * world,
                        "ms_per_step": ms, "steps": K,
                        "note": "rap_transpose_host: pinned host matrix in, pinned host transpose out; "
-                               "upload / RAP transpose / download of 256 MiB workspace bands overlapped"}
+                               "upload / RAP transpose / download of row bands (128 MiB workspace) overlapped"}
     elif not args.no_e2e and do_t:
         hx = x.cpu().pin_memory()
         hy = torch.empty(tuple(y.shape), dtype=dt).pin_memory()

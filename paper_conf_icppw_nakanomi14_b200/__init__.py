@@ -155,7 +155,7 @@ def transpose(x: torch.Tensor, layout: str = "rap", seed: int = 0,
 
 
 def transpose_host(x: torch.Tensor, out: torch.Tensor | None = None, layout: str = "rap", seed: int = 0,
-                   workspace_bytes: int = 256 << 20, device="cuda") -> torch.Tensor:
+                   workspace_bytes: int = 128 << 20, device="cuda") -> torch.Tensor:
     """End-to-end transpose of a HOST (ideally pinned) 2-D tensor into a host tensor [cols, rows]:
     row bands stream through the GPU with upload, RAP transpose and download overlapped.
     Synchronous.  A device workspace of `workspace_bytes` is taken from torch's allocator."""
