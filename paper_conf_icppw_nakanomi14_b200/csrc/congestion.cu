@@ -4,12 +4,13 @@
 //
 // One CUDA warp simulates one DMM warp of w <= 32 threads (§II): lane t issues the
 // request of DMM thread t.  Congestion: requests to the same address are merged
-// (__match_any_sync on the address, one leader per address), then the number of distinct
-// requests per bank is popc(__match_any_sync(bank)) and the congestion is the warp maximum
-// (__reduce_max_sync).  Permutations come from a warp Fisher-Yates shuffle (rap_rng.cuh);
-// P[i] and r[i] stay in lane i's register and are read with __shfl_sync(., row).
-// Histograms: warp-private u32 counters in shared memory (no atomics: evaluation e is
-// counted by lane e), reduced per CTA and added once to the caller's u64 bins.
+// (one leader per address), then lane v counts the distinct requests to bank v from five
+// 32-bit bank-bit masks (rap_warp.cuh) and the congestion is the warp maximum
+// (__reduce_max_sync).  The default sweep (sweep32_kernel / sweep_kernel) draws each trial's
+// permutation in lane mode as 5 bit planes; the ablation kernel (sweep_match_kernel) keeps the
+// north-star sketch: warp Fisher-Yates by __shfl_sync and __match_any_sync histograms.
+// Histograms: shared-memory u32 counters (evaluation e counted by lane e), reduced per CTA and
+// added once to the caller's u64 bins.
 #include <cuda_runtime.h>
 #include <stdint.h>
 
