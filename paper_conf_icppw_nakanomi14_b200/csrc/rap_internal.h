@@ -27,6 +27,7 @@ struct TransposeTuning {
     int depth = 1;        // tiles of global loads in flight per warp (register double-buffer)
     int ctas_per_sm = 0;  // persistent grid = #SMs x this (0: as many as fit)
     bool vst = false;     // 128-bit output stores (shuffle-transposed) instead of 32/64-bit rows
+    bool tma_store = false;  // drain into a dense staging tile, one TMA bulk tensor store per super-tile
 };
 constexpr int kDefaultSR32 = 8, kDefaultSC32 = 2, kDefaultSR64 = 12, kDefaultSC64 = 1;
 // measured on B200 (tools/tune_transpose.cu, profiles/r01_tune_transpose.txt)

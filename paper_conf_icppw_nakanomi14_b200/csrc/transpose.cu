@@ -20,10 +20,12 @@
 // 64-bit elements: 32 banks of 4 bytes (the paper assumed one double per bank word,
 // P:L278-283, L860), so a tile of doubles is split into two 32-bit RAP planes (low / high
 // words) with identical addressing; every smem access stays a 32-lane 4-byte access.
+#include <cuda.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
 
 #include <atomic>
+#include <cstring>
 
 #include "rap_rng.cuh"
 #include "rap_internal.h"
@@ -77,17 +79,32 @@ struct TileCfg {
 // owns tile (w % SR, w / SR) of the block, and a CTA barrier before the drains makes the SC*32
 // input rows / SR*32-element output row runs of neighbouring warps reach DRAM together
 // (measured: +2-4 % over free-running warps, profiles/r01_tune_transpose.txt).
-template <int L, int EW, bool VEC, int DEPTH, int MINB, bool VST, int SR, int SC, bool PEERS>
+// TMA store path (TMAS): the drains of a super-tile write a dense (SC*32) x (SR*32) staging
+// tile in shared memory (row-contiguous, conflict-free) and one thread stores it to HBM with a
+// single cp.async.bulk.tensor (out-of-range rows/columns of edge super-tiles are clipped by TMA).
+__device__ __forceinline__ void tma_store_2d(const CUtensorMap *map, const void *smem, int32_t x, int32_t y) {
+    const uint32_t s = static_cast<uint32_t>(__cvta_generic_to_shared(smem));
+    asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%1, %2}], [%3];"
+                 :: "l"(map), "r"(x), "r"(y), "r"(s) : "memory");
+    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+}
+__device__ __forceinline__ void tma_wait_read() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
+__device__ __forceinline__ void tma_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+
+template <int L, int EW, bool VEC, int DEPTH, int MINB, bool VST, int SR, int SC, bool PEERS, bool TMAS>
 __global__ void __launch_bounds__(SR * SC * 32, MINB)
 transpose_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, int64_t rows,
                  int64_t cols, int64_t ld_src, int64_t ld_dst, uint64_t seed, uint32_t tiles_r,
-                 uint32_t tiles_c, bool vst_ok, PeerOut peers) {
+                 uint32_t tiles_c, bool vst_ok, PeerOut peers, const __grid_constant__ CUtensorMap tmap) {
+    static_assert(!TMAS || (DEPTH == 1 && !PEERS && SR * 32 <= 256), "TMA store: depth 1, box <= 256");
     using C = TileCfg<L, EW>;
     constexpr int NE = C::NE, R = C::R, G = C::G, LPR = C::LPR;
     constexpr int PW = 32 * Geom<L>::RP;            // plane size in words
     extern __shared__ __align__(16) uint32_t smem_dyn[];
     const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
     uint32_t *tile = smem_dyn + warp * warp_smem_words<L, EW>();
+    uint32_t *staging = smem_dyn + SR * SC * warp_smem_words<L, EW>();   // TMAS: (SC*32) x (SR*32) x EW words
 
     // ---- T0: the per-warp shift vector, lane i holds sh[i] (P[i] for RAP, r[i] for RAS)
     uint32_t sh_lane = 0;
@@ -241,9 +258,41 @@ transpose_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, i
         }
     };
 
+    // TMAS drain: tile (wr, wc) of the super-tile -> staging rows wc*32 + c, columns wr*32 + lane
+    auto drain_staging = [&]() {
+        constexpr int SW = SR * 32;                                // staging row length (elements)
+#pragma unroll
+        for (int c = 0; c < 32; ++c) {
+            const uint32_t off = (L == RAP_LAYOUT_XOR) ? word_of<L>(lane, c, 0) : drain_base + c;
+            const uint32_t e = (wc * 32 + c) * SW + wr * 32 + lane;
+            if (EW == 1) staging[e] = tile[off];
+            else *reinterpret_cast<uint2 *>(staging + 2 * e) = make_uint2(tile[off], tile[PW + off]);
+        }
+    };
+
     uint32_t st = blockIdx.x, ti = 0, tj = 0;
     bool act = st < nst && coords(st, ti, tj);
-    if (DEPTH == 1) {
+    if (TMAS) {
+        uint4 v[G];
+        if (act) load(v, ti, tj);
+        while (st < nst) {
+            const uint32_t si = st / stc, sj = st - si * stc;
+            const bool cact = act;
+            if (cact) store_tile(v);                     // T1
+            __syncwarp();
+            st += gridDim.x;
+            act = st < nst && coords(st, ti, tj);
+            if (act) load(v, ti, tj);                    // T3
+            if (threadIdx.x == 0) tma_wait_read();       // the previous TMA store has read staging
+            __syncthreads();
+            if (cact) drain_staging();                   // T2 into the dense staging tile
+            fence_proxy_async();
+            __syncthreads();
+            if (threadIdx.x == 0)                        // T2: one bulk tensor store per super-tile
+                tma_store_2d(&tmap, staging, (int32_t)(si * SR * 32), (int32_t)(sj * SC * 32));
+        }
+        if (threadIdx.x == 0) tma_wait_all();
+    } else if (DEPTH == 1) {
         uint4 v[G];
         if (act) load(v, ti, tj);
         while (st < nst) {
@@ -335,25 +384,63 @@ TransposeTuning default_tuning(uint32_t elem_bytes) {
     return t;
 }
 
-template <int L, int EW, bool VEC, int DEPTH, int MINB, bool VST, int SR, int SC, bool PEERS = false>
+// cuTensorMapEncodeTiled through the runtime's driver entry point (no libcuda link dependency)
+typedef CUresult (*EncodeTiledFn)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *, const cuuint64_t *,
+                                  const cuuint64_t *, const cuuint32_t *, const cuuint32_t *, CUtensorMapInterleave,
+                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+static EncodeTiledFn encode_tiled() {
+    static EncodeTiledFn fn = [] {
+        void *p = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) != cudaSuccess ||
+            q != cudaDriverEntryPointSuccess)
+            p = nullptr;
+        return reinterpret_cast<EncodeTiledFn>(p);
+    }();
+    return fn;
+}
+
+// 2-D map of the output (rows of `cols` ... ): inner dim = output columns (= input rows)
+static bool make_out_map(CUtensorMap *m, void *dst, int64_t rows, int64_t cols, int64_t ld_dst, int EW,
+                         int box_x, int box_y) {
+    EncodeTiledFn fn = encode_tiled();
+    if (!fn || (uintptr_t)dst % 16 || (ld_dst * EW * 4) % 16) return false;
+    const cuuint64_t dims[2] = {(cuuint64_t)rows, (cuuint64_t)cols};
+    const cuuint64_t strides[1] = {(cuuint64_t)ld_dst * EW * 4};
+    const cuuint32_t box[2] = {(cuuint32_t)box_x, (cuuint32_t)box_y};
+    const cuuint32_t estr[2] = {1, 1};
+    return fn(m, EW == 1 ? CU_TENSOR_MAP_DATA_TYPE_UINT32 : CU_TENSOR_MAP_DATA_TYPE_UINT64, 2, dst, dims, strides,
+              box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+              CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+template <int L, int EW, bool VEC, int DEPTH, int MINB, bool VST, int SR, int SC, bool PEERS = false,
+          bool TMAS = false>
 static cudaError_t launch_one(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
                               int64_t ld_dst, uint64_t seed, const TransposeTuning &tu, cudaStream_t st,
                               const PeerOut &peers = PeerOut{}) {
+    CUtensorMap tmap;
+    memset(&tmap, 0, sizeof(tmap));
+    if (TMAS && !make_out_map(&tmap, dst, rows, cols, ld_dst, EW, SR * 32, SC * 32))
+        return launch_one<L, EW, VEC, DEPTH, MINB, VST, SR, SC, PEERS, false>(src, dst, rows, cols, ld_src,
+                                                                             ld_dst, seed, tu, st, peers);
     const uint32_t tiles_r = (uint32_t)((rows + 31) / 32), tiles_c = (uint32_t)((cols + 31) / 32);
     const int64_t nst = (int64_t)((tiles_r + SR - 1) / SR) * ((tiles_c + SC - 1) / SC);
-    auto k = transpose_kernel<L, EW, VEC, DEPTH, MINB, VST, SR, SC, PEERS>;
+    auto k = transpose_kernel<L, EW, VEC, DEPTH, MINB, VST, SR, SC, PEERS, TMAS>;
     static ShapeCache cache;
     bool vst_ok = ((uintptr_t)dst % 16 == 0) && ((ld_dst * EW * 4) % 16 == 0);
     if (PEERS) {
         vst_ok = ((ld_dst * EW * 4) % 16 == 0) && ((peers.col_off * EW * 4) % 16 == 0);
         for (int h = 0; h < peers.G; ++h) vst_ok = vst_ok && (peers.ptr[h] % 16 == 0);
     }
-    const size_t smem = sizeof(uint32_t) * warp_smem_words<L, EW>() * SR * SC;
+    const size_t smem = sizeof(uint32_t) * (warp_smem_words<L, EW>() * SR * SC +
+                                            (TMAS ? (size_t)SR * 32 * SC * 32 * EW : 0));
     int grid = 0;
     const cudaError_t e = grid_for(k, cache, SR * SC * 32, smem, nst, 1, tu.ctas_per_sm, &grid);
     if (e != cudaSuccess) return e;
     k<<<grid, SR * SC * 32, smem, st>>>((const uint32_t *)src, (uint32_t *)dst, rows, cols, ld_src,
-                                        ld_dst, seed, tiles_r, tiles_c, vst_ok, peers);
+                                        ld_dst, seed, tiles_r, tiles_c, vst_ok, peers, tmap);
     return cudaGetLastError();
 }
 
@@ -361,8 +448,12 @@ template <int L, int EW, bool VEC>
 static cudaError_t launch_shape(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
                                 int64_t ld_dst, uint64_t seed, const TransposeTuning &tu, cudaStream_t st) {
 #define RAPK_SHAPE(D, M, V, R_, C_)                                                                  \
-    if (tu.depth == D && tu.minb == M && tu.vst == V && tu.sr == R_ && tu.sc == C_)                  \
+    if (tu.depth == D && tu.minb == M && tu.vst == V && tu.sr == R_ && tu.sc == C_ && !tu.tma_store)  \
         return launch_one<L, EW, VEC, D, M, V, R_, C_>(src, dst, rows, cols, ld_src, ld_dst, seed, tu, st);
+#define RAPK_TSHAPE(M, R_, C_)                                                                       \
+    if (tu.depth == 1 && tu.minb == M && !tu.vst && tu.sr == R_ && tu.sc == C_ && tu.tma_store)      \
+        return launch_one<L, EW, VEC, 1, M, false, R_, C_, false, true>(src, dst, rows, cols, ld_src, ld_dst, \
+                                                                        seed, tu, st);
 #ifdef RAP_TUNING_SWEEP
     RAPK_SHAPE(1, 1, false, 4, 1) RAPK_SHAPE(1, 4, false, 4, 1) RAPK_SHAPE(1, 3, false, 4, 1)
     RAPK_SHAPE(1, 1, false, 8, 1) RAPK_SHAPE(1, 2, false, 8, 1) RAPK_SHAPE(1, 3, false, 8, 1)
@@ -371,8 +462,11 @@ static cudaError_t launch_shape(const void *src, void *dst, int64_t rows, int64_
     RAPK_SHAPE(2, 2, false, 8, 1) RAPK_SHAPE(1, 1, false, 6, 1) RAPK_SHAPE(1, 2, false, 6, 1)
     RAPK_SHAPE(2, 1, false, 8, 2) RAPK_SHAPE(2, 1, false, 4, 2) RAPK_SHAPE(1, 1, false, 4, 4)
     RAPK_SHAPE(2, 1, false, 4, 4) RAPK_SHAPE(1, 1, true, 8, 2) RAPK_SHAPE(2, 1, false, 12, 1)
+    RAPK_TSHAPE(1, 8, 2) RAPK_TSHAPE(1, 8, 1) RAPK_TSHAPE(1, 4, 2) RAPK_TSHAPE(1, 4, 1) RAPK_TSHAPE(1, 4, 4)
+    RAPK_TSHAPE(2, 4, 2) RAPK_TSHAPE(2, 8, 1)
 #endif
 #undef RAPK_SHAPE
+#undef RAPK_TSHAPE
     (void)tu;
     if (EW == 1)
         return launch_one<L, EW, VEC, kDefaultDepth32, kDefaultMinB32, kDefaultVst32, kDefaultSR32, kDefaultSC32>(

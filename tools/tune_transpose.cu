@@ -358,10 +358,11 @@ int main(int argc, char **argv) {
     }
     const int layouts[] = {RAP_LAYOUT_RAP, RAP_LAYOUT_RAW, RAP_LAYOUT_PAD, RAP_LAYOUT_XOR, RAP_LAYOUT_RAS};
     const char *lname[] = {"raw", "pad", "xor", "ras", "rap"};
-    struct Shape { int depth, minb; bool vst; int sr, sc; };
-    const Shape shapes[] = {{1, 1, false, 8, 2}, {2, 1, false, 8, 2}, {2, 1, false, 4, 2}, {1, 1, false, 4, 4},
-                            {2, 1, false, 4, 4}, {1, 1, true, 8, 2}, {1, 1, false, 4, 1}, {2, 1, false, 12, 1},
-                            {1, 1, false, 12, 1}, {1, 1, false, 8, 2}};
+    struct Shape { int depth, minb; bool vst; int sr, sc; bool tma; };
+    const Shape shapes[] = {{1, 1, false, 8, 2, false}, {1, 1, false, 8, 2, true}, {1, 1, false, 8, 1, true},
+                            {1, 1, false, 4, 2, true}, {1, 1, false, 4, 1, true}, {1, 1, false, 4, 4, true},
+                            {1, 2, false, 4, 2, true}, {1, 2, false, 8, 1, true}, {1, 1, false, 12, 1, false},
+                            {1, 1, false, 4, 1, false}};
     for (int eb : {4, 8}) {
         const int64_t n = eb == 4 ? n32 : n64;
         const size_t bytes = eb == 4 ? bytes32 : bytes64;
@@ -369,19 +370,20 @@ int main(int argc, char **argv) {
             for (const Shape &sh : shapes) {
                 if (lay != RAP_LAYOUT_RAP) continue;
                 const int rp = (lay == RAP_LAYOUT_RAP || lay == RAP_LAYOUT_RAS) ? 64 : (lay == RAP_LAYOUT_PAD ? 33 : 32);
-                if ((size_t)32 * rp * (eb / 4) * 4 * sh.sr * sh.sc > 227 * 1024) continue;   // smem limit
+                if ((size_t)32 * rp * (eb / 4) * 4 * sh.sr * sh.sc + (sh.tma ? (size_t)1024 * eb * sh.sr * sh.sc : 0)
+                    > 227 * 1024) continue;   // smem limit
                 for (int cps : {0}) {
                     if (lay != RAP_LAYOUT_RAP && cps) continue;
                     rapk::TransposeTuning tu; tu.minb = sh.minb; tu.depth = sh.depth; tu.ctas_per_sm = cps;
-                    tu.vst = sh.vst; tu.sr = sh.sr; tu.sc = sh.sc;
+                    tu.vst = sh.vst; tu.sr = sh.sr; tu.sc = sh.sc; tu.tma_store = sh.tma;
                     CK(cudaMemset(b, 0, bytes));
                     float t = timeit([&] { rapk::launch_transpose_tuned(a, b, n, n, n, n, eb, lay, 1, tu, 0); }, eb == 4 ? 30 : 10);
                     CK(cudaGetLastError());
                     CK(cudaMemset(bad, 0, 8));
                     check_t<<<2048, 256>>>(a, b, n, eb / 4, bad);
                     unsigned long long hb; CK(cudaMemcpy(&hb, bad, 8, cudaMemcpyDeviceToHost));
-                    printf("b%d %-4s depth=%d minb=%d vst=%d sr=%2d sc=%d ctas/sm=%d : %7.1f GB/s  %8.1f us  %s\n", eb * 8,
-                           lname[lay], sh.depth, sh.minb, (int)sh.vst, sh.sr, sh.sc, cps, 2.0 * bytes / t / 1e6, t * 1e3,
+                    printf("b%d %-4s depth=%d minb=%d vst=%d tma=%d sr=%2d sc=%d ctas/sm=%d : %7.1f GB/s  %8.1f us  %s\n", eb * 8,
+                           lname[lay], sh.depth, sh.minb, (int)sh.vst, (int)sh.tma, sh.sr, sh.sc, cps, 2.0 * bytes / t / 1e6, t * 1e3,
                            hb ? "MISMATCH" : "ok");
                 }
             }
