@@ -60,6 +60,7 @@ __device__ __forceinline__ uint32_t word_of(uint32_t row, uint32_t col, uint32_t
 
 __device__ __forceinline__ uint4 ldg_stream128(const void *p) {
     uint4 r;
+    // (an L2::256B prefetch hint measured no different, profiles/r01_tune_transpose_tma.txt)
     asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
                  : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
     return r;
