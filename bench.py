@@ -90,9 +90,9 @@ class Clocks:
         try:
             self.proc = subprocess.Popen(
                 ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
-                 "--format=csv,noheader,nounits", "-lms", "50"],
+                 "--format=csv,noheader,nounits", "-lms", "20"],
                 stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
-            time.sleep(0.15)
+            time.sleep(0.1)    # nvidia-smi start-up; samples begin during the soak
         except OSError:
             self.proc = None
         return self
@@ -101,7 +101,6 @@ class Clocks:
         if self.proc is None:
             self.result = {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
             return
-        time.sleep(0.1)
         self.proc.terminate()
         out, _ = self.proc.communicate(timeout=10)
         sm, mx, reasons = [], [], set()
@@ -119,7 +118,7 @@ class Clocks:
                     reasons.add(n)
         self.result = {"sm_mhz": statistics.median(sm) if sm else None,
                        "sm_max_mhz": max(mx) if mx else None, "reasons": sorted(reasons),
-                       "samples": len(sm)}
+                       "samples": len(sm), "window": "timed steps + 0.3 s of identical untimed steps each side"}
 
 
 # ---------------------------------------------------------------------------- reference arm
@@ -302,6 +301,20 @@ def main():
             dist.all_reduce(hist)
         return 1
 
+    soak_hist = torch.zeros_like(hist)
+
+    def soak(lay, seconds):
+        """Identical untimed steps (scratch histogram, far trial range) for `seconds`."""
+        t0, k = time.perf_counter(), 0
+        while time.perf_counter() - t0 < seconds:
+            if do_t:
+                step_transpose(lay)
+            if do_s:
+                rap.congestion_sweep(S, seed=1, first_trial=(1 << 40) + k * S, out=soak_hist, algo=args.sweep_algo)
+            k += 1
+            if k % 16 == 0:
+                torch.cuda.synchronize()
+
     results = {}
     for lay in layouts:
         for k in range(args.warmup):
@@ -315,6 +328,11 @@ def main():
         barrier()
         torch.cuda.synchronize()
         with Clocks(dev.index) as clk:
+            # the sampler runs over the timed steps and ~0.3 s of identical untimed steps on
+            # each side, so every clock sample is taken under this workload
+            soak(lay, 0.3)
+            torch.cuda.synchronize()
+            barrier()
             start = torch.cuda.Event(enable_timing=True)
             end = torch.cuda.Event(enable_timing=True)
             start.record(stream)
@@ -332,6 +350,8 @@ def main():
             end.record(stream)
             torch.cuda.synchronize()
             barrier()
+            soak(lay, 0.3)
+            torch.cuda.synchronize()
         t_ms = [e[0].elapsed_time(e[1]) for e in ev]
         s_ms = [e[2].elapsed_time(e[3]) for e in ev]
         results[lay] = dict(total_ms=rmax(start.elapsed_time(end)), t_sum=rmax(sum(t_ms)), t_ms=t_ms,
