@@ -373,6 +373,31 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
     uint32_t *tr = sh_tr[warp];
     uint32_t *res = sh_res[warp];
 
+    // Accesses whose banks do not depend on the trial's draws -- every non-random pattern under
+    // the deterministic maps RAW / PAD / XOR -- have the same congestion in every trial:
+    // evaluate them once here (same evaluator) and count that value per trial below.
+    uint32_t cfix[5][5];
+#pragma unroll
+    for (int p = 0; p < 5; ++p) {
+#pragma unroll
+        for (int s = 0; s < 5; ++s) {
+            cfix[p][s] = 0;
+            if (!((PM >> p) & 1u) || !((SM >> s) & 1u) || p == RAP_PAT_RANDOM) continue;
+            if (s != RAP_SCHEME_RAW && s != RAP_SCHEME_PAD && s != RAP_SCHEME_XOR) continue;
+            const int pp = (p == RAP_PAT_MALICIOUS)
+                ? ((s == RAP_SCHEME_RAW) ? RAP_PAT_STRIDE : (s == RAP_SCHEME_PAD) ? -1 : RAP_PAT_DIAGONAL) : p;
+            uint32_t row, col;
+            switch (pp) {
+            case RAP_PAT_CONTIGUOUS: row = 0; col = lane; break;
+            case RAP_PAT_STRIDE: row = lane; col = 0; break;
+            case RAP_PAT_DIAGONAL: row = lane; col = lane; break;
+            default: row = lane; col = (32u - lane) & 31u; break;       // PAD anti-diagonal
+            }
+            const uint32_t bank = s == RAP_SCHEME_PAD ? ((row + col) & 31u) : s == RAP_SCHEME_XOR ? (col ^ row) : col;
+            cfix[p][s] = max_load(masks_ballot(bank), kFull, ls);
+        }
+    }
+
     const uint64_t nbatch = (n_trials + 31) / 32;
     const uint64_t stride = (uint64_t)gridDim.x * kSweepWarpsV2;
     for (uint64_t bt = (uint64_t)blockIdx.x * kSweepWarpsV2 + warp; bt < nbatch; bt += stride) {
@@ -429,7 +454,10 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
                 for (int s = 0; s < 5; ++s) {
                     if (!((SM >> s) & 1u)) continue;
                     uint32_t c;
-                    if (p == RAP_PAT_MALICIOUS && (s == RAP_SCHEME_RAW || s == RAP_SCHEME_RAS) &&
+                    if (p != RAP_PAT_RANDOM &&
+                        (s == RAP_SCHEME_RAW || s == RAP_SCHEME_PAD || s == RAP_SCHEME_XOR)) {
+                        c = cfix[p][s];                             // trial-invariant access
+                    } else if (p == RAP_PAT_MALICIOUS && (s == RAP_SCHEME_RAW || s == RAP_SCHEME_RAS) &&
                         ((PM >> RAP_PAT_STRIDE) & 1u)) {
                         c = c_stride[s];                            // reading iii: = stride access
                     } else if (p == RAP_PAT_MALICIOUS && (s == RAP_SCHEME_RAP || s == RAP_SCHEME_XOR) &&
