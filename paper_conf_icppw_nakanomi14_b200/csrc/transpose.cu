@@ -6,17 +6,18 @@
 // row-wise (contiguous) write AND the column-wise (stride) read of the tile are both
 // conflict-free for every P (Theorem 2).
 //
-// B200 design: one warp owns one 32 x 32 tile buffer (no CTA barrier,
-// only __syncwarp), persistent warps stride over the tile grid, and the next tile's global
-// loads are in flight while the current tile is drained.
+// B200 design: one warp owns one 32 x 32 tile buffer (only __syncwarp inside a
+// tile); a CTA of SR x SC warps works on an SR x SC block of tiles and drains it in lockstep
+// (one CTA barrier per super-tile); persistent CTAs stride over super-tiles, and the next
+// tile's global loads are in flight while the current tile is drained.
 //   load  : 128-bit LDG.  One warp instruction covers 4 tile rows x 128 B.  Under RAP the 4
 //           rows are chosen as P^-1(4g+0..3), i.e. rows whose P values cover the 4 residues
 //           mod 4, which makes each of the 4 following STS.32 hit 32 distinct banks:
 //           bank(row, 4q+k) = (4q + k + 4g + c) mod 32 is injective in (c, q).
-//   smem  : STS.32 of element (i, j) at column phys(i, j) of row i.
-//   drain : lane i reads column c of the tile at phys(i, c): the DMM stride access, banks
-//           (c + P[i]) mod 32 distinct because P is a permutation; then 128-byte coalesced
-//           STG.32 of output row c.
+//   smem  : STS.32 of element (i, j) at word i*64 + j + P[i] (unwrapped RAP row window, Geom).
+//   drain : lane i reads column c of the tile at word i*64 + P[i] + c: the DMM stride access,
+//           banks (c + P[i]) mod 32 distinct because P is a permutation; then 128-byte
+//           coalesced STG.32 of output row c (or a staging tile + TMA store, TMAS).
 // 64-bit elements: 32 banks of 4 bytes (the paper assumed one double per bank word,
 // P:L278-283, L860), so a tile of doubles is split into two 32-bit RAP planes (low / high
 // words) with identical addressing; every smem access stays a 32-lane 4-byte access.
@@ -402,7 +403,8 @@ static EncodeTiledFn encode_tiled() {
     return fn;
 }
 
-// 2-D map of the output (rows of `cols` ... ): inner dim = output columns (= input rows)
+// 2-D tensor map of the output (cols rows x rows columns, pitch ld_dst): x = output column (= input
+// row), y = output row (= input column); box = one super-tile's output block
 static bool make_out_map(CUtensorMap *m, void *dst, int64_t rows, int64_t cols, int64_t ld_dst, int EW,
                          int box_x, int box_y) {
     EncodeTiledFn fn = encode_tiled();
