@@ -6,7 +6,11 @@ memory), the current CUDA stream and the enums.  There is no CPU fallback: calli
 CPU tensor, or without the built library, raises.
 
 Functions keep the C names without the ``rap_`` prefix:
-  perm_gen, transpose, congestion, congestion_sweep, congestion_trace.
+  hot path      perm_gen, transpose, congestion, congestion_sweep (+ algo), congestion_trace
+  host / multi  transpose_host (host-to-host pipeline), unpack_blocks, transpose_to_peers
+                (the multi-GPU drivers are in ``dist``)
+  paper §VI/VII smem_transpose_bench (Table III), congestion_sweep4 (§VII, Table IV),
+                smem_gather_bench (data-dependent access under a layout)
 """
 from __future__ import annotations
 
@@ -18,14 +22,18 @@ import torch
 
 from . import build as _build
 
-__all__ = ["perm_gen", "transpose", "transpose_host", "transpose_to_peers", "congestion", "congestion_sweep", "congestion_trace",
-           "unpack_blocks", "smem_transpose_bench",
-           "LAYOUTS", "SCHEMES", "PATTERNS", "RapError", "lib", "library_path"]
+__all__ = ["perm_gen", "transpose", "transpose_host", "transpose_to_peers", "congestion", "congestion_sweep",
+           "congestion_trace", "unpack_blocks", "smem_transpose_bench", "congestion_sweep4", "smem_gather_bench",
+           "LAYOUTS", "SCHEMES", "PATTERNS", "SWEEP_ALGOS", "SMEM_ALGORITHMS", "SCHEMES4", "PATTERNS4",
+           "RapError", "lib", "library_path"]
 
 LAYOUTS = {"raw": 0, "pad": 1, "xor": 2, "ras": 3, "rap": 4}
 SCHEMES = {"raw": 0, "ras": 1, "rap": 2, "pad": 3, "xor": 4}
 SWEEP_ALGOS = {"default": 0, "match": 1}
 PATTERNS = {"contiguous": 0, "stride": 1, "diagonal": 2, "random": 3, "malicious": 4}
+SMEM_ALGORITHMS = {"crsw": 0, "srcw": 1, "drdw": 2}
+SCHEMES4 = {"raw": 0, "ras": 1, "1p": 2, "r1p": 3, "3p": 4}
+PATTERNS4 = {"contiguous": 0, "stride1": 1, "stride2": 2, "stride3": 3, "random": 4, "malicious": 5}
 STATUS = {0: "RAP_OK", 1: "RAP_ERR_INVALID_ARG", 2: "RAP_ERR_UNSUPPORTED", 3: "RAP_ERR_ALIAS",
           4: "RAP_ERR_CUDA"}
 
@@ -286,9 +294,6 @@ def unpack_blocks(recv: torch.Tensor, out: torch.Tensor, G: int) -> torch.Tensor
     return out
 
 
-SMEM_ALGORITHMS = {"crsw": 0, "srcw": 1, "drdw": 2}
-
-
 def smem_transpose_bench(algorithm: str, scheme: str, elem_bytes: int = 4, seed: int = 0,
                          n_blocks: int = 1, reps: int = 1, device="cuda"):
     """Table III on this GPU: (logical result uint32 [n_blocks, 32, 32], cycles int64 [n_blocks])."""
@@ -300,10 +305,6 @@ def smem_transpose_bench(algorithm: str, scheme: str, elem_bytes: int = 4, seed:
                                               ctypes.c_void_p(cyc.data_ptr()), _stream(out)),
                "rap_smem_transpose_bench")
     return out, cyc
-
-
-SCHEMES4 = {"raw": 0, "ras": 1, "1p": 2, "r1p": 3, "3p": 4}
-PATTERNS4 = {"contiguous": 0, "stride1": 1, "stride2": 2, "stride3": 3, "random": 4, "malicious": 5}
 
 
 def congestion_sweep4(n_trials: int, seed: int, w: int = 32, patterns=tuple(PATTERNS4), schemes=tuple(SCHEMES4),
