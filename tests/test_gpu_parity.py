@@ -468,3 +468,24 @@ def test_transpose_host_strided_pageable(rap, oracle):
     rap.transpose_host(xs, out=out_big[:, :300], workspace_bytes=1 << 20)
     assert np.array_equal(bits(out_big[:, :300]), oracle.transpose(bits(xs)))
     assert not bits(out_big[:, 300:]).any()
+
+
+# ------------------------------------------------------------------ randomized shapes / pitches
+def test_transpose_randomized_geometry(rap, oracle):
+    # 60 seeded draws of (rows, cols, source pitch, source offset, destination pitch, dtype, layout):
+    # vector and scalar load paths, partial super-tiles, padded output rows -- all bit-exact
+    rng = np.random.default_rng(2024)
+    for k in range(60):
+        dtype = [torch.float32, torch.float64][k % 2]
+        layout = LAYOUT_NAMES[k % 5]
+        rows, cols = int(rng.integers(1, 700)), int(rng.integers(1, 700))
+        pad_s, off = int(rng.integers(0, 9)), int(rng.integers(0, 5))
+        pad_d = int(rng.integers(0, 9))
+        big = workloads.random_bits(rows, cols + pad_s + off, dtype, seed=k).cuda()
+        xs = big[:, off:off + cols]
+        out_big = torch.zeros((cols, rows + pad_d), dtype=dtype, device="cuda")
+        rap.transpose(xs, layout=layout, seed=k, out=out_big[:, :rows])
+        torch.cuda.synchronize()
+        assert np.array_equal(bits(out_big[:, :rows]), oracle.transpose(bits(xs))), (k, rows, cols, layout)
+        if pad_d:
+            assert not bits(out_big[:, rows:]).any()
