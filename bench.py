@@ -45,7 +45,7 @@ def parse():
     p.add_argument("--warmup", type=int, default=5)
     p.add_argument("--impl", default="mine", choices=["mine", "reference"])
     p.add_argument("--workload", default="default",
-                   choices=["default", "sweep", "cfg4", "tile", "layouts", "dist", "dist_fused"])
+                   choices=["default", "sweep", "trace", "cfg4", "tile", "layouts", "dist", "dist_fused"])
     p.add_argument("--sweep-trials", type=int, default=1 << 16)
     p.add_argument("--sweep-algo", default="default", choices=["default", "match"])
     p.add_argument("--layout", default="rap")
@@ -266,8 +266,8 @@ def main():
     else:
         rows = cols = 8192
         dt = torch.float32
-    do_t = wl != "sweep"
-    do_s = wl in ("default", "sweep")
+    do_t = wl not in ("sweep", "trace")
+    do_s = wl in ("default", "sweep", "trace")
     layouts = ["raw", "pad", "xor", "ras", "rap"] if wl == "layouts" else [args.layout]
     eb = torch.empty((), dtype=dt).element_size()
     nbytes = 2 * rows * cols * eb                     # per rank per step
@@ -293,7 +293,17 @@ def main():
         rap.transpose(x, layout=lay, seed=0, out=y)
         return 1
 
+    # access traces (north star: "synthetic matrices and access traces"): 4096 warps of the paper's
+    # pattern families, each evaluated under every step's trials and all five schemes
+    trace_cells = workloads.trace_cells(4096, 32, seed=rank, device=dev) if wl == "trace" else None
+    trace_hist = torch.zeros((5, 33), dtype=torch.int64, device=dev)
+    TT = max(1, S // 4096)                                 # trials per trace step
+
     def step_sweep(k):
+        if wl == "trace":
+            rap.congestion_trace(trace_cells, TT, seed=1, schemes=("raw", "ras", "rap", "pad", "xor"),
+                                 first_trial=(k * world + rank) * TT, out=trace_hist)
+            return 1
         # this rank's batch of the global trial sequence: step k covers trials
         # [k*S*world, (k+1)*S*world), rank r the r-th slice of it
         rap.congestion_sweep(S, seed=1, first_trial=(k * world + rank) * S, out=hist, algo=args.sweep_algo)
@@ -309,7 +319,10 @@ def main():
         while time.perf_counter() - t0 < seconds:
             if do_t:
                 step_transpose(lay)
-            if do_s:
+            if do_s and wl == "trace":
+                rap.congestion_trace(trace_cells, TT, seed=1, first_trial=(1 << 40) + k * TT,
+                                     schemes=("raw", "ras", "rap", "pad", "xor"), out=torch.zeros_like(trace_hist))
+            elif do_s:
                 rap.congestion_sweep(S, seed=1, first_trial=(1 << 40) + k * S, out=soak_hist, algo=args.sweep_algo)
             k += 1
             if k % 16 == 0:
@@ -404,7 +417,20 @@ def main():
         if wl == "layouts":
             line["layouts_gbs"] = {l: nbytes * world * args.steps / (v["t_sum"] * 1e-3) / 1e9
                                    for l, v in results.items()}
-    if do_s:
+    if wl == "trace":
+        evs = 4096 * TT * 5 * world * args.steps / (r["s_sum"] * 1e-3)
+        th = trace_hist.cpu().numpy()
+        c = np.arange(33)
+        line.update(value=evs, unit="warp-evaluations/s",
+                    config={"workload": "congestion of 4096 synthetic warp traces (row / column / diagonal / "
+                                        "anti-diagonal / permutation / random) under RAW, RAS, RAP, PAD, XOR",
+                            "trials_per_step": TT, "warps": 4096, "schemes": 5})
+        line["trace"] = {"E_by_scheme": {n: float((th[i] * c).sum() / th[i].sum())
+                                         for i, n in enumerate(["raw", "ras", "rap", "pad", "xor"])},
+                         "kernel_ms_median": statistics.median(r["s_ms"])}
+        line["roofline"] = {"bound": "alu", "achieved": None, "peak": None, "unit": "warp-evaluations/s",
+                            "frac": None, "traffic": None, "note": "secondary workload; no ncu capture this round"}
+    elif do_s:
         tps = S * world * args.steps / (r["s_sum"] * 1e-3)
         h = hist.cpu().numpy()
         c = np.arange(33)
@@ -512,7 +538,7 @@ def main():
                        "h2d_bytes_per_step": hx.numel() * eb * world, "d2h_bytes_per_step": hy.numel() * eb * world,
                        "ms_per_step": ms, "steps": K,
                        "note": "pinned host shard -> H2D -> sharded transpose (public API) -> D2H of the result"}
-    elif not args.no_e2e and do_s:
+    elif not args.no_e2e and do_s and wl != "trace":
         hh = torch.empty_like(hist, device="cpu").pin_memory()
         st = torch.cuda.Event(enable_timing=True)
         en = torch.cuda.Event(enable_timing=True)
