@@ -408,7 +408,8 @@ def main():
         else:
             ach = nbytes / (kern_ms * 1e-3) / 1e9
             line["roofline"] = {"bound": "hbm", "achieved": ach, "peak": peak, "unit": "GB/s",
-                                "frac": ach / peak, "traffic": prof.get("dram_bytes_per_launch"),
+                                "frac": ach / peak,
+                                "traffic": prof.get("dram_bytes_per_launch_steady", prof.get("dram_bytes_per_launch")),
                                 "peak_source": peak_src, "frac_of_8TBs_nominal": ach / 8000.0,
                                 "kernel": kkey, "kernel_ms_median": kern_ms,
                                 "algorithmic_bytes_per_launch": nbytes,

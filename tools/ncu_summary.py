@@ -128,6 +128,22 @@ def main(src_dir, dst, tag):
             kernels[key]["units_per_launch"] = {unit: n}
             if m.get("smsp__inst_executed.sum"):
                 kernels[key][f"warp_instructions_per_{unit[:-1]}"] = m["smsp__inst_executed.sum"] / n
+    # steady-state DRAM traffic (ncu --cache-control none, consecutive launches): the dirty lines
+    # a launch leaves in L2 are written back during the next one, so per-launch read + write
+    # bytes here are the true cost (the --set full captures flush caches between replays)
+    for key, stem in (("transpose_b32_rap", "steady_t32"), ("transpose_b64_rap", "steady_t64")):
+        path = os.path.join(src_dir, stem + ".csv")
+        if key not in kernels or not os.path.exists(path):
+            continue
+        txt = open(path).read()
+        txt = txt[txt.index('"ID"'):]
+        per = {}
+        for r in csv.DictReader(io.StringIO(txt)):
+            if r["Metric Name"].startswith("dram__bytes"):
+                per[r["ID"]] = per.get(r["ID"], 0.0) + float(r["Metric Value"].replace(",", "")) * SCALE.get(r["Metric Unit"], 1)
+        if per:
+            kernels[key]["dram_bytes_per_launch_steady"] = sum(per.values()) / len(per)
+            kernels[key]["dram_steady_source"] = f"profiles/{tag}_steady_dram_{stem[-3:]}.csv (--cache-control none)"
     os.makedirs(os.path.dirname(dst), exist_ok=True)
     json.dump({"round": tag, "note": "cold-cache, serialised ncu replays: compare shares and ratios, "
                                      "not absolute times; dram bytes exclude lines still dirty in L2 at exit",
