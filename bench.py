@@ -46,7 +46,9 @@ def parse():
     p.add_argument("--impl", default="mine", choices=["mine", "reference"])
     p.add_argument("--workload", default="default",
                    choices=["default", "sweep", "trace", "cfg4", "tile", "layouts", "dist", "dist_fused"])
-    p.add_argument("--sweep-trials", type=int, default=1 << 16)
+    # default: one full wave of the sweep kernel's resident grid on a B200 (148 SMs x 8 CTAs x
+    # 4 warps x 32 trials per warp batch), so every resident warp evaluates one batch per step
+    p.add_argument("--sweep-trials", type=int, default=148 * 8 * 4 * 32)
     p.add_argument("--sweep-algo", default="default", choices=["default", "match"])
     p.add_argument("--layout", default="rap")
     p.add_argument("--no-e2e", action="store_true")
@@ -194,16 +196,24 @@ def cpu_baseline_sweep():
 
 
 def sweep_roofline(tps: float, clocks: dict):
-    """ALU roofline of the sweep: warp instructions per trial (ncu) x trials/s against the issue
-    peak 148 SMs x 4 schedulers x 1 warp-instruction/clk x SM clock."""
+    """ALU roofline of the sweep.  The binding unit is the ALU pipe (LOP3 / SHF / ISETP / IADD3 ...),
+    which accepts one warp-instruction every 2 cycles per SMSP (B300_MICROARCH.md "Pipe rates"):
+    peak = 148 SMs x 4 SMSPs x 0.5 x SM clock.  achieved = ALU-pipe warp-instructions per trial
+    (from the ncu capture: pipe-active fraction x peak x active cycles / trials) x trials/s.
+    The issue-slot view (all instructions against 1 / clk / SMSP) is reported beside it."""
     prof = load_profile("sweep_w32") or {}
     ipt = prof.get("warp_instructions_per_trial")
+    apt = prof.get("alu_warp_instructions_per_trial")
     mhz = (clocks or {}).get("sm_max_mhz") or 1965.0
-    peak = 148 * 4 * mhz * 1e6
-    ach = ipt * tps if ipt else None
-    return {"bound": "alu", "achieved": ach, "peak": peak, "unit": "warp-instructions/s",
+    peak = 148 * 4 * 0.5 * mhz * 1e6
+    ach = apt * tps if apt else None
+    issue_peak = 148 * 4 * mhz * 1e6
+    return {"bound": "alu", "achieved": ach, "peak": peak, "unit": "ALU-pipe warp-instructions/s",
             "frac": ach / peak if ach else None, "traffic": None,
-            "warp_instructions_per_trial": ipt, "profile": prof.get("source"),
+            "alu_warp_instructions_per_trial": apt, "warp_instructions_per_trial": ipt,
+            "issue_frac": ipt * tps / issue_peak if ipt else None,
+            "peak_source": "148 SMs x 4 SMSPs x 0.5 ALU warp-instr/clk (B300_MICROARCH.md pipe rates) x sm_max_mhz",
+            "profile": prof.get("source"), "alu_pipe_active_frac_ncu": prof.get("alu_pipe_active_frac"),
             "issue_active_frac_ncu": prof.get("issue_active_frac")}
 
 
@@ -268,7 +278,9 @@ def main():
         dt = torch.float32
     do_t = wl not in ("sweep", "trace")
     do_s = wl in ("default", "sweep", "trace")
-    layouts = ["raw", "pad", "xor", "ras", "rap"] if wl == "layouts" else [args.layout]
+    layouts = (["raw", "pad", "xor", "ras", "rap"] if wl == "layouts"
+               else ["rap16", "rap"] if wl == "cfg4" and args.layout == "rap"     # T2b (ii) ablation beside (i)
+               else [args.layout])
     eb = torch.empty((), dtype=dt).element_size()
     nbytes = 2 * rows * cols * eb                     # per rank per step
     x = workloads.random_bits(rows, cols, dt, seed=rank, device=dev) if do_t else None
@@ -370,7 +382,7 @@ def main():
         results[lay] = dict(total_ms=rmax(start.elapsed_time(end)), t_sum=rmax(sum(t_ms)), t_ms=t_ms,
                             s_sum=rmax(sum(s_ms)), s_ms=s_ms, clocks=clk.result, launches=launches)
 
-    lay = "rap" if wl == "layouts" else args.layout
+    lay = "rap" if wl in ("layouts", "cfg4") and "rap" in results else args.layout
     r = results[lay]
     line = {"metric": METRIC, "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": r["total_ms"] / args.steps, "higher_is_better": True,
@@ -415,7 +427,7 @@ def main():
                                 "algorithmic_bytes_per_launch": nbytes,
                                 "smem_wavefronts_per_request": prof.get("smem_wavefronts_per_request"),
                                 "profile": prof.get("source")}
-        if wl == "layouts":
+        if wl in ("layouts", "cfg4") and len(results) > 1:
             line["layouts_gbs"] = {l: nbytes * world * args.steps / (v["t_sum"] * 1e-3) / 1e9
                                    for l, v in results.items()}
     if wl == "trace":

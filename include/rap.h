@@ -57,7 +57,14 @@ typedef enum {
     RAP_LAYOUT_PAD = 1,  /* a[i][j] at [i][j] of a [32][33] array   (+1 padding baseline) */
     RAP_LAYOUT_XOR = 2,  /* a[i][j] at [i][j xor i]                 (XOR-swizzle baseline)*/
     RAP_LAYOUT_RAS = 3,  /* a[i][j] at [i][(j + r[i]) mod 32]          */
-    RAP_LAYOUT_RAP = 4   /* a[i][j] at [i][(j + P[i]) mod 32]        */
+    RAP_LAYOUT_RAP = 4,  /* a[i][j] at [i][(j + P[i]) mod 32]        */
+    RAP_LAYOUT_RAP16 = 5 /* 64-bit elements only (else RAP_ERR_UNSUPPORTED): a tile of     */
+                         /* doubles with one element per PAIR of 4-byte banks, i.e. 16   */
+                         /* "double banks"; a[i][j] at [i][16*(j div 16) + ((j + Q[i mod */
+                         /* 16]) mod 16)], Q = perm(seed, 0, 16).  The paper's RAP with  */
+                         /* w = 16 applied to each half row: every half-warp of a 64-bit */
+                         /* row or column access hits 16 distinct bank pairs (P:L860,    */
+                         /* L1005-1023, DESIGN reading xiv)            */
 } rap_layout_t;
 
 /* Address maps of the DMM congestion evaluator (physical address of logical cell (i,j)). */
@@ -118,7 +125,8 @@ rap_status_t rap_perm_gen(uint64_t seed, uint64_t first_index, uint64_t count, u
  * r = shifts(seed, 0, 32); seed is ignored by RAW/PAD/XOR.  rows == 0 or cols == 0 is a
  * no-op.  Overlapping src/dst -> RAP_ERR_ALIAS.  16-byte aligned src with ld_src a
  * multiple of 16/elem_bytes takes 128-bit loads; anything else takes 32/64-bit loads
- * (still on the GPU). */
+ * (still on the GPU).  RAP_LAYOUT_RAP16 (elem_bytes 8 only) is the 64-bit-element
+ * ablation of T2b: 64-bit global and shared accesses on a [32][32] double tile. */
 rap_status_t rap_transpose(const void *src, void *dst, int64_t rows, int64_t cols,
                            int64_t ld_src, int64_t ld_dst, uint32_t elem_bytes,
                            rap_layout_t layout, uint64_t seed, void *stream);
@@ -144,7 +152,8 @@ rap_status_t rap_transpose_host(const void *h_src, void *h_dst, int64_t rows, in
  * this process (peer shards mapped over NVLink -- CUDA IPC / symmetric memory -- or local
  * buffers for a one-GPU emulation); ld_dst >= N; G <= 16.  One HBM read and one NVLink write
  * per element; no send/receive buffers, no unpack.  Enqueue only: the caller must make every
- * rank's kernel complete (a cross-rank barrier) before reading its output shard. */
+ * rank's kernel complete (a cross-rank barrier) before reading its output shard.
+ * layout RAW..RAP (RAP_LAYOUT_RAP16 -> RAP_ERR_UNSUPPORTED). */
 rap_status_t rap_transpose_to_peers(const void *src, int64_t M, int64_t N, int64_t ld_src,
                                     void *const *peer_dst, uint32_t G, uint32_t rank, int64_t ld_dst,
                                     uint32_t elem_bytes, rap_layout_t layout, uint64_t seed, void *stream);

@@ -27,7 +27,7 @@ __all__ = ["perm_gen", "transpose", "transpose_host", "transpose_to_peers", "con
            "LAYOUTS", "SCHEMES", "PATTERNS", "SWEEP_ALGOS", "SMEM_ALGORITHMS", "SCHEMES4", "PATTERNS4",
            "RapError", "lib", "library_path"]
 
-LAYOUTS = {"raw": 0, "pad": 1, "xor": 2, "ras": 3, "rap": 4}
+LAYOUTS = {"raw": 0, "pad": 1, "xor": 2, "ras": 3, "rap": 4, "rap16": 5}   # rap16: 8-byte elements only
 SCHEMES = {"raw": 0, "ras": 1, "rap": 2, "pad": 3, "xor": 4}
 SWEEP_ALGOS = {"default": 0, "match": 1}
 PATTERNS = {"contiguous": 0, "stride": 1, "diagonal": 2, "random": 3, "malicious": 4}

@@ -118,10 +118,12 @@ constexpr int kSweepWarpsV2 = 4;
 
 template <int W>
 __device__ __forceinline__ void swap_planes(uint32_t (&pl)[5], uint32_t k, uint32_t j) {
+    // j <= k: y holds bit_j ^ bit_k at position j; flipping bits j and k by y swaps them
+    const uint32_t d = k - j, mj = 1u << j;
 #pragma unroll
     for (int b = 0; b < 5; ++b) {
-        const uint32_t d = ((pl[b] >> j) ^ (pl[b] >> k)) & 1u;
-        pl[b] ^= (d << j) | (d << k);
+        const uint32_t y = (pl[b] ^ (pl[b] >> d)) & mj;
+        pl[b] ^= y ^ (y << d);
     }
 }
 
@@ -308,10 +310,9 @@ __device__ __forceinline__ uint32_t lane_bits(int b) {
 
 struct BankMask { uint32_t b[5]; };
 
-__device__ __forceinline__ BankMask masks_ballot(uint32_t bank) {
+__device__ __forceinline__ BankMask masks_ballot(uint32_t bank) {   // bank < 32
     BankMask B;
-#pragma unroll
-    for (int k = 0; k < 5; ++k) B.b[k] = __ballot_sync(kFull, (bank >> k) & 1u);
+    ballot_planes5(bank, B.b);
     return B;
 }
 
@@ -370,6 +371,7 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
     for (uint32_t b = threadIdx.x; b < nbins; b += blockDim.x) sh_hist[b] = 0;
     __syncthreads();
     const LaneSel ls(lane);
+    const uint32_t lt_mask = (1u << lane) - 1u;
     uint32_t *tr = sh_tr[warp];
     uint32_t *res = sh_res[warp];
 
@@ -443,7 +445,7 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
                 Pr = plane_value(Pm.b, rrow);                      // P[row_t]
                 rr = __shfl_sync(kFull, rt, rrow);                 // r[row_t]
                 const uint32_t same = __match_any_sync(kFull, cell);   // merged requests
-                leaders = __ballot_sync(kFull, (uint32_t)(__ffs(same) - 1) == lane);
+                leaders = ballot_zero(same, lt_mask);              // first lane of its cell
             }
             uint32_t e = 0;
             uint32_t c_stride[5] = {0, 0, 0, 0, 0}, c_diag[5] = {0, 0, 0, 0, 0};

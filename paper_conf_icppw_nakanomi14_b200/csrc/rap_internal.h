@@ -45,6 +45,9 @@ cudaError_t launch_transpose(const void *src, void *dst, int64_t rows, int64_t c
                              int64_t ld_dst, uint32_t elem_bytes, int layout, uint64_t seed,
                              cudaStream_t st);
 
+cudaError_t launch_transpose_rap16(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
+                                   int64_t ld_dst, uint64_t seed, cudaStream_t st);
+
 cudaError_t launch_transpose_peers(const void *src, int64_t M, int64_t N, int64_t ld_src, const PeerOut &pe,
                                    int64_t ld_dst, uint32_t elem_bytes, int layout, uint64_t seed, cudaStream_t st);
 

@@ -12,6 +12,36 @@ namespace rapk {
 // with B_k = ballot(bit k of bank), the lanes whose bank equals v are AND_k (v_k ? B_k : ~B_k);
 // popc of that (restricted to the counted lanes) is the load of bank v, and the congestion is
 // the warp maximum (__reduce_max_sync).  Five VOTE + five LOP3 + POPC + REDUX per access.
+// __ballot_sync of the bit selected by M.  Written as and + setp + vote so that ptxas turns the
+// bit tests of up to 7 ballots of one value into a single R2P (register -> predicates) instead
+// of SHF + LOP3 + ISETP per bit (the compiler's lowering of __ballot_sync((x >> k) & 1)).
+template <uint32_t M>
+__device__ __forceinline__ uint32_t ballot_bit(uint32_t x) {
+    uint32_t v;
+    asm volatile("{\n\t.reg .pred p;\n\t.reg .b32 t;\n\tand.b32 t, %1, %2;\n\tsetp.ne.u32 p, t, 0;\n\t"
+                 "vote.sync.ballot.b32 %0, p, 0xffffffff;\n\t}"
+                 : "=r"(v) : "r"(x), "n"(M));
+    return v;
+}
+
+// B[k] = ballot(bit k of x), k = 0..4 (x < 32)
+__device__ __forceinline__ void ballot_planes5(uint32_t x, uint32_t (&B)[5]) {
+    B[0] = ballot_bit<1u>(x);
+    B[1] = ballot_bit<2u>(x);
+    B[2] = ballot_bit<4u>(x);
+    B[3] = ballot_bit<8u>(x);
+    B[4] = ballot_bit<16u>(x);
+}
+
+// ballot of ((x & m) == 0): one LOP3 with a predicate output + VOTE
+__device__ __forceinline__ uint32_t ballot_zero(uint32_t x, uint32_t m) {
+    uint32_t v;
+    asm volatile("{\n\t.reg .pred p;\n\t.reg .b32 t;\n\tand.b32 t, %1, %2;\n\tsetp.eq.u32 p, t, 0;\n\t"
+                 "vote.sync.ballot.b32 %0, p, 0xffffffff;\n\t}"
+                 : "=r"(v) : "r"(x), "r"(m));
+    return v;
+}
+
 struct LaneSel {
     uint32_t nsel[5];        // bit k of lane ? 0 : ~0
     __device__ __forceinline__ explicit LaneSel(uint32_t lane) {
@@ -21,23 +51,26 @@ struct LaneSel {
 };
 
 __device__ __forceinline__ uint32_t max_bank_load(uint32_t bank, uint32_t counted, const LaneSel &ls) {
+    uint32_t B[5];
+    ballot_planes5(bank, B);
     uint32_t m = counted;
 #pragma unroll
-    for (int k = 0; k < 5; ++k) m &= __ballot_sync(kFull, (bank >> k) & 1u) ^ ls.nsel[k];
+    for (int k = 0; k < 5; ++k) m &= B[k] ^ ls.nsel[k];
     return __reduce_max_sync(kFull, __popc(m));
 }
 
 // Merged requests: lanes of `active` that carry the first occurrence of their
 // 10-bit key (the logical cell row*32 + col; every address map is injective on cells).
 __device__ __forceinline__ uint32_t first_occurrences(uint32_t key, uint32_t active, uint32_t lane) {
+    uint32_t b[5];
+    ballot_planes5(key & 31u, b);
     uint32_t same = active;
 #pragma unroll
-    for (int k = 0; k < 10; ++k) {
-        const uint32_t b = __ballot_sync(kFull, (key >> k) & 1u);
-        same &= ((key >> k) & 1u) ? b : ~b;
-    }
-    const bool leader = (same & ((1u << lane) - 1u)) == 0u;
-    return __ballot_sync(kFull, leader) & active;
+    for (int k = 0; k < 5; ++k) same &= ((key >> k) & 1u) ? b[k] : ~b[k];
+    ballot_planes5(key >> 5, b);
+#pragma unroll
+    for (int k = 0; k < 5; ++k) same &= ((key >> (k + 5)) & 1u) ? b[k] : ~b[k];
+    return ballot_zero(same, (1u << lane) - 1u) & active;
 }
 
 }  // namespace rapk

@@ -91,7 +91,7 @@ sweep4_kernel(uint32_t w, uint32_t pmask, uint32_t smask, uint64_t seed, uint64_
                 const uint32_t bank = (l + f) % w;
                 const uint32_t key = ((i * w + j) * w + k) * w + l;     // logical cell, < 2^20
                 const uint32_t same = __match_any_sync(kFull, lane < w ? key : (0x80000000u | lane));
-                const uint32_t counted = __ballot_sync(kFull, (uint32_t)(__ffs(same) - 1) == lane) & active;
+                const uint32_t counted = ballot_zero(same, (1u << lane) - 1u) & active;
                 const uint32_t c = max_bank_load(bank, counted, ls);
                 mine = (lane == e) ? c : mine;
                 ++e;

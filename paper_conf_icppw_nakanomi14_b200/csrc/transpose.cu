@@ -537,6 +537,9 @@ cudaError_t launch_transpose_tuned(const void *src, void *dst, int64_t rows, int
 cudaError_t launch_transpose(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
                              int64_t ld_dst, uint32_t elem_bytes, int layout, uint64_t seed,
                              cudaStream_t st) {
+    if (layout == RAP_LAYOUT_RAP16)
+        return elem_bytes == 8 ? launch_transpose_rap16(src, dst, rows, cols, ld_src, ld_dst, seed, st)
+                               : cudaErrorInvalidValue;
     return launch_transpose_tuned(src, dst, rows, cols, ld_src, ld_dst, elem_bytes, layout, seed,
                                   default_tuning(elem_bytes), st);
 }

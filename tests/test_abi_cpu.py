@@ -53,6 +53,8 @@ def test_transpose_validation(L):
     s = P(0)
     assert L.rap_transpose(a, b, 4, 4, 4, 4, 3, 4, 0, s) == INVALID      # elem_bytes
     assert L.rap_transpose(a, b, 4, 4, 4, 4, 4, 9, 0, s) == INVALID      # layout
+    assert L.rap_transpose(a, b, 4, 4, 4, 4, 4, 6, 0, s) == INVALID      # layout
+    assert L.rap_transpose(a, b, 4, 4, 4, 4, 4, 5, 0, s) == UNSUPPORTED  # RAP16 needs 8-byte elements
     assert L.rap_transpose(a, b, -1, 4, 4, 4, 4, 4, 0, s) == INVALID     # rows < 0
     assert L.rap_transpose(a, b, 4, 8, 4, 4, 4, 4, 0, s) == INVALID      # ld_src < cols
     assert L.rap_transpose(a, b, 8, 4, 4, 4, 4, 4, 0, s) == INVALID      # ld_dst < rows
@@ -137,6 +139,7 @@ def test_transpose_to_peers_validation(L):
     assert f(src, 64, 128, 128, peers, 2, 0, 100, 4, 4, 0, s) == INVALID     # ld_dst < N
     alias = (ctypes.c_void_p * 2)(0x10000000, 0x50000000)
     assert f(src, 64, 128, 128, alias, 2, 0, 128, 4, 4, 0, s) == ALIAS
+    assert f(src, 64, 128, 128, peers, 2, 0, 128, 8, 5, 0, s) == UNSUPPORTED  # RAP16: local transpose only
 
 
 def test_sweep4_validation(L):

@@ -129,6 +129,42 @@ def test_transpose_cfg4_16384_f64(rap, oracle):
         assert np.array_equal(bits(y[c0:c0 + 33]), oracle.transpose(bits(xs[:, c0:c0 + 33])))
 
 
+# T2b (ii): the RAP-16 double tile (8-byte elements only)
+def test_transpose_rap16_shapes(rap, oracle):
+    for i, (r, c) in enumerate(SHAPES + [(384, 64), (385, 33), (31, 1025)]):
+        x = workloads.random_bits(r, c, torch.float64, seed=100 + i)
+        y = rap.transpose(x.cuda(), layout="rap16", seed=i)
+        torch.cuda.synchronize()
+        assert np.array_equal(bits(y), oracle.transpose(bits(x))), (r, c)
+
+
+def test_transpose_rap16_strided(rap, oracle):
+    big = workloads.random_bits(300, 260, torch.float64, seed=4)
+    for (r0, c0, r1, c1) in [(0, 0, 300, 256), (3, 1, 291, 250), (2, 3, 35, 40)]:
+        xs = big.cuda()[r0:r1, c0:c1]
+        out_big = torch.zeros((c1 - c0, (r1 - r0) + 9), dtype=torch.float64, device="cuda")
+        out = out_big[:, 3:3 + (r1 - r0)]
+        rap.transpose(xs, layout="rap16", seed=2, out=out)
+        torch.cuda.synchronize()
+        assert np.array_equal(bits(out), oracle.transpose(bits(big[r0:r1, c0:c1])))
+        assert not bits(out_big[:, :3]).any() and not bits(out_big[:, 3 + (r1 - r0):]).any()
+
+
+def test_transpose_rap16_rejects_32bit(rap):
+    with pytest.raises(rap.RapError, match="UNSUPPORTED"):
+        rap.transpose(torch.zeros((64, 64), device="cuda"), layout="rap16")
+
+
+def test_transpose_rap16_cfg4_16384_f64(rap, oracle):
+    # cfg4 at full size through the RAP-16 ablation (the launch bench.py --workload cfg4 times)
+    x = workloads.random_bits(16384, 16384, torch.float64, seed=0, device="cuda")
+    y = rap.transpose(x, layout="rap16", seed=0)
+    torch.cuda.synchronize()
+    _band_check(oracle, x, y, n_bands=4, band=40, seed=3)
+    ref = rap.transpose(x, layout="rap", seed=0)
+    assert torch.equal(y.view(torch.int64), ref.view(torch.int64))
+
+
 def test_transpose_cfg1_tile(rap, oracle):
     for seed in (0, 1, 2):
         x = workloads.random_bits(32, 32, torch.float32, seed=seed)

@@ -15,6 +15,18 @@ for lay in rap raw pad xor ras; do
 done
 timeout 600 ncu --set full --import-source on --clock-control none -k regex:transpose_kernel -s 3 -c 1 \
     -o "$OUT/prof_t64_rap" -f $B --workload cfg4 --steps 1 --warmup 3 > "$OUT/ncu_t64_rap.log" 2>&1
+timeout 600 ncu --set full --import-source on --clock-control none -k regex:transpose_rap16_kernel -s 3 -c 1 \
+    -o "$OUT/prof_t64_rap16" -f $B --workload cfg4 --steps 1 --warmup 3 > "$OUT/ncu_t64_rap16.log" 2>&1
+# steady-state DRAM bytes per launch: consecutive launches, no cache flush between them
+timeout 600 ncu --cache-control none --clock-control none -k regex:transpose_kernel -s 3 -c 4 --csv \
+    --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum \
+    --log-file "$OUT/steady_t32.csv" $B --steps 4 --warmup 3 --sweep-trials 1024 > /dev/null 2>&1
+timeout 600 ncu --cache-control none --clock-control none -k regex:transpose_kernel -s 3 -c 4 --csv \
+    --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum \
+    --log-file "$OUT/steady_t64.csv" $B --workload cfg4 --layout rap --steps 4 --warmup 3 > /dev/null 2>&1
+timeout 600 ncu --cache-control none --clock-control none -k regex:transpose_rap16_kernel -s 3 -c 4 --csv \
+    --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum \
+    --log-file "$OUT/steady_t64_rap16.csv" $B --workload cfg4 --steps 4 --warmup 3 > /dev/null 2>&1
 timeout 600 ncu --set full --import-source on --clock-control none -k regex:"sweep(32)?_kernel" -s 2 -c 1 \
     -o "$OUT/prof_sweep" -f $B --workload sweep --steps 1 --warmup 2 --sweep-trials 8388608 > "$OUT/ncu_sweep.log" 2>&1
 timeout 600 ncu --set full --import-source on --clock-control none -k regex:"sweep_match_kernel" -s 2 -c 1 \

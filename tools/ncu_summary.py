@@ -15,6 +15,7 @@ CAPTURES = {
     "transpose_b32_rap": "prof_t32_rap", "transpose_b32_raw": "prof_t32_raw",
     "transpose_b32_pad": "prof_t32_pad", "transpose_b32_xor": "prof_t32_xor",
     "transpose_b32_ras": "prof_t32_ras", "transpose_b64_rap": "prof_t64_rap",
+    "transpose_b64_rap16": "prof_t64_rap16",
     "sweep_w32": "prof_sweep", "sweep_w32_match": "prof_sweep_match",
 }
 
@@ -22,7 +23,8 @@ CAPTURES = {
 UNITS = {"sweep_w32": ("trials", 8388608), "sweep_w32_match": ("trials", 4194304),
          "transpose_b32_rap": ("bytes", 2 * 8192 * 8192 * 4), "transpose_b32_raw": ("bytes", 2 * 8192 * 8192 * 4),
          "transpose_b32_pad": ("bytes", 2 * 8192 * 8192 * 4), "transpose_b32_xor": ("bytes", 2 * 8192 * 8192 * 4),
-         "transpose_b32_ras": ("bytes", 2 * 8192 * 8192 * 4), "transpose_b64_rap": ("bytes", 2 * 16384 * 16384 * 8)}
+         "transpose_b32_ras": ("bytes", 2 * 8192 * 8192 * 4), "transpose_b64_rap": ("bytes", 2 * 16384 * 16384 * 8),
+         "transpose_b64_rap16": ("bytes", 2 * 16384 * 16384 * 8)}
 
 WANT = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum",
         "l1tex__data_pipe_lsu_wavefronts_mem_shared_op_ld.sum",
@@ -33,7 +35,13 @@ WANT = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
         "smsp__issue_active.avg.pct_of_peak_sustained_active",
         "sm__warps_active.avg.pct_of_peak_sustained_active", "launch__registers_per_thread",
         "launch__grid_size", "launch__block_size", "dram__throughput.avg.pct_of_peak_sustained_elapsed",
-        "sm__throughput.avg.pct_of_peak_sustained_elapsed", "smsp__inst_executed.sum"]
+        "sm__throughput.avg.pct_of_peak_sustained_elapsed", "smsp__inst_executed.sum",
+        "sm__pipe_alu_cycles_active.avg.pct_of_peak_sustained_active", "sm__cycles_active.avg"]
+
+# ALU pipe (LOP3 / SHF / ISETP / IADD3 / PRMT ...): reciprocal throughput 2 cycles per warp
+# instruction per SMSP (B300_MICROARCH.md "Pipe rates"), i.e. 2 warp-instructions / clk / SM
+ALU_WARP_INST_PER_SM_CLK = 2.0
+N_SMS = 148
 
 SCALE = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "ns": 1e-9, "us": 1e-6, "ms": 1e-3,
          "nsecond": 1e-9, "usecond": 1e-6,
@@ -128,10 +136,17 @@ def main(src_dir, dst, tag):
             kernels[key]["units_per_launch"] = {unit: n}
             if m.get("smsp__inst_executed.sum"):
                 kernels[key][f"warp_instructions_per_{unit[:-1]}"] = m["smsp__inst_executed.sum"] / n
+            alu_pct = m.get("sm__pipe_alu_cycles_active.avg.pct_of_peak_sustained_active")
+            cyc = m.get("sm__cycles_active.avg")
+            if alu_pct is not None and cyc:
+                alu = alu_pct / 100 * ALU_WARP_INST_PER_SM_CLK * N_SMS * cyc
+                kernels[key]["alu_pipe_active_frac"] = alu_pct / 100
+                kernels[key][f"alu_warp_instructions_per_{unit[:-1]}"] = alu / n
     # steady-state DRAM traffic (ncu --cache-control none, consecutive launches): the dirty lines
     # a launch leaves in L2 are written back during the next one, so per-launch read + write
     # bytes here are the true cost (the --set full captures flush caches between replays)
-    for key, stem in (("transpose_b32_rap", "steady_t32"), ("transpose_b64_rap", "steady_t64")):
+    for key, stem in (("transpose_b32_rap", "steady_t32"), ("transpose_b64_rap", "steady_t64"),
+                       ("transpose_b64_rap16", "steady_t64_rap16")):
         path = os.path.join(src_dir, stem + ".csv")
         if key not in kernels or not os.path.exists(path):
             continue
@@ -143,7 +158,7 @@ def main(src_dir, dst, tag):
                 per[r["ID"]] = per.get(r["ID"], 0.0) + float(r["Metric Value"].replace(",", "")) * SCALE.get(r["Metric Unit"], 1)
         if per:
             kernels[key]["dram_bytes_per_launch_steady"] = sum(per.values()) / len(per)
-            kernels[key]["dram_steady_source"] = f"profiles/{tag}_steady_dram_{stem[-3:]}.csv (--cache-control none)"
+            kernels[key]["dram_steady_source"] = f"profiles/{tag}_steady_dram_{stem[7:]}.csv (--cache-control none)"
     os.makedirs(os.path.dirname(dst), exist_ok=True)
     json.dump({"round": tag, "note": "cold-cache, serialised ncu replays: compare shares and ratios, "
                                      "not absolute times; dram bytes exclude lines still dirty in L2 at exit",
