@@ -34,7 +34,9 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if not force and not _stale():
         return LIB
     tmp = LIB + f".tmp{os.getpid()}"
-    cmd = [_nvcc(), *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O2",
+    # RAP_EXTRA_NVCC_FLAGS: launch-shape macros for tuning runs only (e.g. -DRAP_SWEEP_WARPS=8)
+    extra = os.environ.get("RAP_EXTRA_NVCC_FLAGS", "").split()
+    cmd = [_nvcc(), *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O2", *extra,
            "-shared", "-o", tmp, *[os.path.join(CSRC, f) for f in SOURCES]]
     if verbose:
         cmd.insert(1, "-Xptxas=-v")

@@ -114,7 +114,20 @@ __device__ __forceinline__ void flush_hist(uint32_t (*sh)[kMaxBins], int nwarps,
 //             (5 shuffles), unpack P[t]; read r[t] and cell t from shared memory; evaluate
 //             every selected (pattern, scheme) with the ballot evaluator (C3); lane e counts
 //             evaluation e in the CTA histogram (C4).
-constexpr int kSweepWarpsV2 = 4;
+// launch shape of the default sweep (measured on B200, profiles/r01_tune_sweep.txt): 4-warp CTAs,
+// 8 per SM, and a grid of 16 x the resident CTAs so that SMs that finish early pick up more
+// work (+11% over one persistent wave).  The macros exist
+// for tuning builds (RAP_EXTRA_NVCC_FLAGS)
+#ifndef RAP_SWEEP_WARPS
+#define RAP_SWEEP_WARPS 4
+#endif
+#ifndef RAP_SWEEP_MINB
+#define RAP_SWEEP_MINB 8
+#endif
+#ifndef RAP_SWEEP_GRID_MULT
+#define RAP_SWEEP_GRID_MULT 16
+#endif
+constexpr int kSweepWarpsV2 = RAP_SWEEP_WARPS;
 
 template <int W>
 __device__ __forceinline__ void swap_planes(uint32_t (&pl)[5], uint32_t k, uint32_t j) {
@@ -356,7 +369,7 @@ __device__ __forceinline__ uint32_t max_load(const BankMask &B, uint32_t counted
 }
 
 template <uint32_t PM, uint32_t SM>
-__global__ void __launch_bounds__(kSweepWarpsV2 * 32, 8)
+__global__ void __launch_bounds__(kSweepWarpsV2 * 32, RAP_SWEEP_MINB)
 sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint64_t n_trials,
                uint64_t *__restrict__ hist) {
     constexpr uint32_t w = 32;
@@ -677,7 +690,7 @@ static void run_sweep(int warps_per_cta, uint64_t trials_per_item, uint32_t w, u
                       cudaStream_t st) {
     const int threads = warps_per_cta * 32;
     const uint64_t items = (n_trials + trials_per_item - 1) / trials_per_item;
-    const int grid = clamp_grid(items, warps_per_cta, resident_ctas<Kernel>(threads));
+    const int grid = clamp_grid(items, warps_per_cta, RAP_SWEEP_GRID_MULT * resident_ctas<Kernel>(threads));
     // u32 shared counters: keep the trials counted by one CTA below 2^31 per launch
     const uint64_t chunk = (uint64_t)grid * (1ull << 31);
     for (uint64_t done = 0; done < n_trials; done += chunk) {

@@ -99,6 +99,8 @@ def main(src_dir, dst, tag):
     kernels = {}
     for key, stem in CAPTURES.items():
         rep = os.path.join(src_dir, stem + ".ncu-rep")
+        if not os.path.exists(rep):                     # committed copies: profiles/<tag>_<stem>
+            rep = os.path.join(src_dir, f"{tag}_{stem}.ncu-rep")
         if not os.path.exists(rep):
             continue
         m = raw_metrics(rep)
@@ -148,6 +150,8 @@ def main(src_dir, dst, tag):
     for key, stem in (("transpose_b32_rap", "steady_t32"), ("transpose_b64_rap", "steady_t64"),
                        ("transpose_b64_rap16", "steady_t64_rap16")):
         path = os.path.join(src_dir, stem + ".csv")
+        if not os.path.exists(path):
+            path = os.path.join(src_dir, f"{tag}_steady_dram_{stem[7:]}.csv")
         if key not in kernels or not os.path.exists(path):
             continue
         txt = open(path).read()
