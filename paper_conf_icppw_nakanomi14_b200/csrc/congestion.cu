@@ -368,6 +368,44 @@ __device__ __forceinline__ uint32_t max_load(const BankMask &B, uint32_t counted
     return __reduce_max_sync(kFull, __popc(m));
 }
 
+// Per-lane constants of the two rewritten evaluators below (lane v):
+//   E    = AND_k (L_k ^ nsel_k)  -- bit t set iff t == v (the incidence mask of the identity map)
+//   M_k  = L_k ^ nsel_k          -- bit t set iff bit k of t equals bit k of v
+struct LaneEq {
+    uint32_t E, M[5];
+    __device__ __forceinline__ explicit LaneEq(const LaneSel &ls) {
+        E = kFull;
+#pragma unroll
+        for (int k = 0; k < 5; ++k) {
+            M[k] = lane_bits(k) ^ ls.nsel[k];
+            E &= M[k];
+        }
+    }
+};
+
+// max_load(masks_rot(s), kFull): bank(t) = (t + s) mod 32.  Rotation commutes with AND and with
+// XOR by an all-zero / all-one word, so AND_k (rotr(L_k, s) ^ nsel_k) = rotr(AND_k (L_k ^ nsel_k), s)
+// = rotr(E, s): lane v's incidence mask {t : (t + s) mod 32 = v} in one funnel shift instead of
+// 5 shifts + 5 LOP3 (bit-identical; tests/test_gpu_parity.py).
+__device__ __forceinline__ uint32_t max_load_rot(uint32_t s, const LaneEq &le) {
+    return __reduce_max_sync(kFull, __popc(__funnelshift_r(le.E, le.E, s)));
+}
+
+// max_load(masks_add(masks_lane(), Y), kFull): bank(t) = (t + y_t) mod 32, y_t given as planes
+// Y_k.  The ripple-carry sum bit S_k = L_k ^ Y_k ^ c is produced already XORed with the lane's
+// selector (S_k ^ nsel_k = Y_k ^ c ^ M_k, one LOP3 as before), so the incidence mask is a plain
+// AND of five words: two LOP3 instead of five.
+__device__ __forceinline__ uint32_t max_load_add_lane(const BankMask &Y, const LaneEq &le) {
+    uint32_t S[5], c = 0;
+#pragma unroll
+    for (int k = 0; k < 5; ++k) {
+        const uint32_t L = lane_bits(k);
+        S[k] = Y.b[k] ^ c ^ le.M[k];
+        c = (L & Y.b[k]) | (c & (L ^ Y.b[k]));
+    }
+    return __reduce_max_sync(kFull, __popc(S[0] & S[1] & S[2] & S[3] & S[4]));
+}
+
 template <uint32_t PM, uint32_t SM>
 __global__ void __launch_bounds__(kSweepWarpsV2 * 32, RAP_SWEEP_MINB)
 sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint64_t n_trials,
@@ -384,6 +422,7 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
     for (uint32_t b = threadIdx.x; b < nbins; b += blockDim.x) sh_hist[b] = 0;
     __syncthreads();
     const LaneSel ls(lane);
+    const LaneEq le(ls);
     const uint32_t lt_mask = (1u << lane) - 1u;
     uint32_t *tr = sh_tr[warp];
     uint32_t *res = sh_res[warp];
@@ -483,14 +522,20 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
                             ? ((s == RAP_SCHEME_RAW || s == RAP_SCHEME_RAS) ? RAP_PAT_STRIDE
                                : (s == RAP_SCHEME_PAD) ? -1 : RAP_PAT_DIAGONAL) : p;
                         BankMask B;
+                        const bool isp = (s == RAP_SCHEME_RAP);
+                        if ((s == RAP_SCHEME_RAS || s == RAP_SCHEME_RAP) && pp == RAP_PAT_CONTIGUOUS) {
+                            c = max_load_rot(isp ? P0 : r0, le);            // bank t + shift[0]
+                            goto counted;
+                        }
+                        if ((s == RAP_SCHEME_RAS || s == RAP_SCHEME_RAP) && pp == RAP_PAT_DIAGONAL) {
+                            c = max_load_add_lane(isp ? Pm : Rm, le);       // bank t + shift[t]
+                            goto counted;
+                        }
                         if (s == RAP_SCHEME_RAW) {
                             B = (pp == RAP_PAT_STRIDE) ? masks_const(0)
                               : (pp == RAP_PAT_RANDOM) ? masks_ballot(rcol) : masks_lane();
                         } else if (s == RAP_SCHEME_RAS || s == RAP_SCHEME_RAP) {
-                            const bool isp = (s == RAP_SCHEME_RAP);
-                            if (pp == RAP_PAT_CONTIGUOUS) B = masks_rot(isp ? P0 : r0);
-                            else if (pp == RAP_PAT_STRIDE) B = isp ? Pm : Rm;
-                            else if (pp == RAP_PAT_DIAGONAL) B = masks_add(masks_lane(), isp ? Pm : Rm);
+                            if (pp == RAP_PAT_STRIDE) B = isp ? Pm : Rm;
                             else B = masks_ballot((rcol + (isp ? Pr : rr)) & 31u);
                         } else {                                    // PAD / XOR: per-lane bank
                             uint32_t row, col;
@@ -505,6 +550,7 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
                         }
                         c = max_load(B, pp == RAP_PAT_RANDOM ? leaders : kFull, ls);
                     }
+                counted:
                     if (p == RAP_PAT_STRIDE) c_stride[s] = c;
                     if (p == RAP_PAT_DIAGONAL) c_diag[s] = c;
                     if (lane == 0) res[e] = c;                      // C4: result slot e
