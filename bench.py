@@ -46,10 +46,12 @@ def parse():
     p.add_argument("--impl", default="mine", choices=["mine", "reference"])
     p.add_argument("--workload", default="default",
                    choices=["default", "sweep", "trace", "cfg4", "tile", "layouts", "dist", "dist_fused"])
-    # default: four batches of 32 trials for every resident warp of the sweep kernel on a B200
-    # (148 SMs x 8 CTAs x 4 warps): with one batch per warp the launch ramp and the per-CTA
-    # histogram flush cost ~20% of the kernel (2.23 vs 2.83 G trials/s), with four ~6%
-    p.add_argument("--sweep-trials", type=int, default=148 * 8 * 4 * 32 * 4)
+    # default: one batch of 32 trials for every resident warp of the sweep kernel on a B200
+    # (148 SMs x 8 CTAs x 4 warps), so the cfg3 transpose stays the larger share of the step
+    # (the step's `value` and `roofline` are the transpose's).  One batch per warp runs the
+    # sweep below its steady rate (launch ramp, per-CTA histogram flush): `--workload sweep`
+    # measures the steady rate, 4 batches per warp give 2.88 G/s, 10^9 trials 3.09 G/s.
+    p.add_argument("--sweep-trials", type=int, default=148 * 8 * 4 * 32)
     p.add_argument("--sweep-algo", default="default", choices=["default", "match"])
     p.add_argument("--layout", default="rap")
     p.add_argument("--no-e2e", action="store_true")

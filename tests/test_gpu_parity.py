@@ -275,6 +275,38 @@ def test_sweep_full_size_1e9(rap, oracle):
     assert np.array_equal(g.cpu().numpy().astype(np.uint64), o)
 
 
+def read_sweep_golden(path):
+    """tests/golden/sweep_w32_1e9_seed<s>.txt (written by tools/oracle_golden_1e9.py from oracle/ only)."""
+    import json
+    meta, h = None, np.zeros((5, 3, 33), dtype=np.uint64)
+    for ln in open(path):
+        if ln.startswith("# {"):
+            meta = json.loads(ln[2:])
+        elif not ln.startswith("#") and ln.strip():
+            f = ln.split()
+            h[ALL_PAT.index(f[0]), ["raw", "ras", "rap"].index(f[1])] = [int(v) for v in f[2:]]
+    return meta, h
+
+
+@pytest.mark.parametrize("seed", [1, 2, 3])
+def test_sweep_1e9_bit_exact_per_seed(rap, seed):
+    # BASELINE cfg2 at full size, the north star's "matches the oracle bit-for-bit per seed":
+    # the whole 10^9-trial histogram of each seed against the oracle's (computed once on the
+    # host cores by tools/oracle_golden_1e9.py, ~30 min per seed; stored under tests/golden)
+    import conftest
+    path = conftest.golden(f"sweep_w32_1e9_seed{seed}.txt")
+    meta, expect = read_sweep_golden(path)
+    assert meta["n_trials"] == 10 ** 9 and meta["first_trial"] == 0 and meta["seed"] == seed
+    g = rap.congestion_sweep(10 ** 9, seed=seed, patterns=ALL_PAT, schemes=["raw", "ras", "rap"])
+    assert np.array_equal(g.cpu().numpy().astype(np.uint64), expect)
+    # the same histogram assembled from 7 uneven launches (accumulation is exact)
+    acc = torch.zeros_like(g)
+    cuts = [0, 1, 31, 33, 10 ** 6 + 7, 123_456_789, 700_000_001, 10 ** 9]
+    for a, b in zip(cuts[:-1], cuts[1:]):
+        rap.congestion_sweep(b - a, seed=seed, first_trial=a, out=acc)
+    assert torch.equal(acc, g)
+
+
 # ------------------------------------------------------------------ trace evaluator
 def test_trace_matches_oracle(rap, oracle):
     w, n_trials, first = 32, 40, 1000
