@@ -6,6 +6,7 @@ per-seed u64 histograms.
 """
 import itertools
 import math
+import os
 
 import numpy as np
 import pytest
@@ -295,6 +296,8 @@ def test_sweep_1e9_bit_exact_per_seed(rap, seed):
     # host cores by tools/oracle_golden_1e9.py, ~30 min per seed; stored under tests/golden)
     import conftest
     path = conftest.golden(f"sweep_w32_1e9_seed{seed}.txt")
+    if not os.path.exists(path):
+        pytest.skip(f"{path} not generated yet (python tools/oracle_golden_1e9.py)")
     meta, expect = read_sweep_golden(path)
     assert meta["n_trials"] == 10 ** 9 and meta["first_trial"] == 0 and meta["seed"] == seed
     g = rap.congestion_sweep(10 ** 9, seed=seed, patterns=ALL_PAT, schemes=["raw", "ras", "rap"])

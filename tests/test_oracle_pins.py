@@ -7,6 +7,7 @@ vectors, numpy routines, or brute force over all inputs of tiny size.
 """
 import itertools
 import math
+import os
 from fractions import Fraction
 
 import numpy as np
@@ -408,6 +409,8 @@ def test_golden_1e9_histograms_pinned(seed):
     # PMFs by chi-square.
     import json
     path = golden(f"sweep_w32_1e9_seed{seed}.txt")
+    if not os.path.exists(path):
+        pytest.skip(f"{path} not generated yet (python tools/oracle_golden_1e9.py)")
     pats, schs = ["contiguous", "stride", "diagonal", "random", "malicious"], ["raw", "ras", "rap"]
     h, meta = np.zeros((5, 3, 33), dtype=np.float64), None
     for ln in open(path):

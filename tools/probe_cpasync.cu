@@ -8,6 +8,7 @@
 #include <vector>
 #include <algorithm>
 #include <string>
+#include <functional>
 #include "transpose.cu"
 
 namespace rapk {  // the RAP-16 kernel lives in another translation unit; not probed here
@@ -297,28 +298,55 @@ int main(int argc, char **argv) {
         char nm[128]; snprintf(nm, sizeof nm, "wrapped sr=%d sc=%d minb=%d occ=%d", SR, SC, MINB, occ);      \
         check(nm, t);                                                                                        \
     }
-#define CRUN(SR, SC, CL)                                                                                     \
-    {                                                                                                        \
-        auto k = clu_kernel<SR, SC, CL>;                                                                     \
-        const size_t smem = (size_t)SR * SC * 8192;                                                          \
-        CK(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));                \
-        if (CL > 1) CK(cudaFuncSetAttribute(k, cudaFuncAttributeNonPortableClusterSizeAllowed, 1));         \
-        cudaLaunchConfig_t cfg = {};                                                                         \
-        cudaLaunchAttribute at[1];                                                                           \
-        at[0].id = cudaLaunchAttributeClusterDimension;                                                      \
-        at[0].val.clusterDim.x = CL; at[0].val.clusterDim.y = 1; at[0].val.clusterDim.z = 1;                 \
-        cfg.blockDim = dim3(SR * SC * 32); cfg.dynamicSmemBytes = smem; cfg.attrs = at; cfg.numAttrs = 1;     \
-        int ncl = 0;                                                                                         \
-        cfg.gridDim = dim3(148 * CL);                                                                        \
-        CK(cudaOccupancyMaxActiveClusters(&ncl, k, &cfg));                                                   \
-        const uint32_t nst = (uint32_t)((n / 32 / (SR * CL)) * (n / 32 / SC));                               \
-        cfg.gridDim = dim3(std::min<uint32_t>(nst, (uint32_t)ncl) * CL);                                     \
-        float t = timeit([&] { cudaLaunchKernelEx(&cfg, k, (const uint32_t *)a, b, n, (uint64_t)1, (uint32_t)(n / 32)); }, 30); \
-        char nm[128]; snprintf(nm, sizeof nm, "cluster sr=%d sc=%d cl=%d clusters=%d", SR, SC, CL, ncl);     \
-        check(nm, t);                                                                                        \
+    // A/B of the cluster-lockstep variants against the library kernel: every variant is timed in
+    // each of R interleaved rounds (so clock / thermal drift hits all alike); median of rounds
+    std::vector<std::pair<std::string, std::function<void()>>> vs;
+    {
+        rapk::TransposeTuning tu = rapk::default_tuning(4);
+        vs.push_back({"library rap 8x2 (LDG->STS, unwrapped)",
+                      [=] { rapk::launch_transpose_tuned(a, b, n, n, n, n, 4, RAP_LAYOUT_RAP, 1, tu, 0); }});
     }
-    CRUN(8, 2, 1) CRUN(8, 2, 2) CRUN(8, 2, 4) CRUN(16, 1, 1) CRUN(16, 1, 2) CRUN(16, 1, 4) CRUN(8, 1, 2)
-    CRUN(8, 1, 4) CRUN(8, 1, 8) CRUN(4, 2, 4) CRUN(4, 2, 8) CRUN(16, 1, 8) CRUN(8, 2, 8)
-    RUN(8, 2, 2, true, 1, 0)
+    auto add_cluster = [&](auto k, int SR, int SC, int CL) {
+        const size_t smem = (size_t)SR * SC * 8192;
+        CK(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        if (CL > 1) CK(cudaFuncSetAttribute(k, cudaFuncAttributeNonPortableClusterSizeAllowed, 1));
+        cudaLaunchConfig_t cfg = {};
+        static cudaLaunchAttribute at[64][1];
+        static int nat = 0;
+        cudaLaunchAttribute *ap = at[nat++];
+        ap[0].id = cudaLaunchAttributeClusterDimension;
+        ap[0].val.clusterDim.x = CL; ap[0].val.clusterDim.y = 1; ap[0].val.clusterDim.z = 1;
+        cfg.blockDim = dim3(SR * SC * 32); cfg.dynamicSmemBytes = smem; cfg.attrs = ap; cfg.numAttrs = 1;
+        int ncl = 0;
+        cfg.gridDim = dim3(148 * CL);
+        CK(cudaOccupancyMaxActiveClusters(&ncl, k, &cfg));
+        const uint32_t nst = (uint32_t)((n / 32 / (SR * CL)) * (n / 32 / SC));
+        cfg.gridDim = dim3(std::min<uint32_t>(nst, (uint32_t)ncl) * CL);
+        char nm[128]; snprintf(nm, sizeof nm, "cluster sr=%d sc=%d cl=%d clusters=%d", SR, SC, CL, ncl);
+        vs.push_back({nm, [=] { cudaLaunchKernelEx(&cfg, k, (const uint32_t *)a, b, n, (uint64_t)1, (uint32_t)(n / 32)); }});
+    };
+    add_cluster(clu_kernel<8, 2, 1>, 8, 2, 1);
+    add_cluster(clu_kernel<8, 2, 2>, 8, 2, 2);
+    add_cluster(clu_kernel<8, 2, 4>, 8, 2, 4);
+    add_cluster(clu_kernel<8, 1, 4>, 8, 1, 4);
+    add_cluster(clu_kernel<8, 1, 8>, 8, 1, 8);
+    add_cluster(clu_kernel<4, 2, 8>, 4, 2, 8);
+    add_cluster(clu_kernel<4, 1, 8>, 4, 1, 8);
+    add_cluster(clu_kernel<4, 2, 4>, 4, 2, 4);
+    add_cluster(clu_kernel<16, 1, 4>, 16, 1, 4);
+    vs.push_back({"memcpy d2d 256 MiB", [=] { cudaMemcpyAsync(b, a, bytes, cudaMemcpyDeviceToDevice); }});
+    const int R = argc > 1 ? atoi(argv[1]) : 7;
+    std::vector<std::vector<float>> res(vs.size());
+    for (int r = 0; r < R; ++r)
+        for (size_t v = 0; v < vs.size(); ++v) res[v].push_back(timeit(vs[v].second, 20));
+    for (size_t v = 0; v < vs.size(); ++v) {
+        const float t = median(res[v]);
+        if (vs[v].first.rfind("memcpy", 0) == 0) {
+            printf("%-44s: %7.1f GB/s %8.1f us (median of %d rounds)\n", vs[v].first.c_str(), 2.0 * bytes / t / 1e6, t * 1e3, R);
+            continue;
+        }
+        vs[v].second();
+        check(vs[v].first.c_str(), t);
+    }
     return 0;
 }
