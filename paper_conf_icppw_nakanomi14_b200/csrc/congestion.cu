@@ -131,12 +131,16 @@ constexpr int kSweepWarpsV2 = RAP_SWEEP_WARPS;
 
 template <int W>
 __device__ __forceinline__ void swap_planes(uint32_t (&pl)[5], uint32_t k, uint32_t j) {
-    // j <= k: y holds bit_j ^ bit_k at position j; flipping bits j and k by y swaps them
+    // j <= k: y holds bit_j ^ bit_k at position j; flipping bits j and k by y swaps them.
+    // y << d runs on the FMA pipe as y * 2^d (the sweep is bound by the ALU pipe); 2^d is made
+    // in PTX so that the compiler does not turn the multiply back into a shift.
     const uint32_t d = k - j, mj = 1u << j;
+    uint32_t sd;
+    asm("shl.b32 %0, %1, %2;" : "=r"(sd) : "r"(1u), "r"(d));
 #pragma unroll
     for (int b = 0; b < 5; ++b) {
         const uint32_t y = (pl[b] ^ (pl[b] >> d)) & mj;
-        pl[b] ^= y ^ (y << d);
+        pl[b] ^= y ^ (y * sd);
     }
 }
 

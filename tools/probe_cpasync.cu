@@ -236,6 +236,84 @@ clu_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, int64_t
     }
 }
 
+// Warp-specialised variant: T = SR*SC producer warps (LDG.128 -> STS.32 into the RAP tile, the
+// next tile's loads in flight while waiting for a free stage) and T consumer warps (lockstep drain
+// of the super-tile: LDS column reads + 128 B STG rows), two super-tile stages in shared memory,
+// handed over with named barriers (FULL[s] = 1 + s, EMPTY[s] = 3 + s) instead of one CTA barrier.
+__device__ __forceinline__ void nb_sync(int id, int n) { asm volatile("bar.sync %0, %1;" :: "r"(id), "r"(n) : "memory"); }
+__device__ __forceinline__ void nb_arrive(int id, int n) { asm volatile("bar.arrive %0, %1;" :: "r"(id), "r"(n) : "memory"); }
+
+template <int SR, int SC>
+__global__ void __launch_bounds__(2 * SR * SC * 32, 1)
+ws_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, int64_t n, uint64_t seed,
+          uint32_t tiles) {
+    constexpr int T = SR * SC, NT = 2 * T * 32;
+    extern __shared__ __align__(16) uint32_t sm[];
+    const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
+    const bool producer = warp < T;
+    const uint32_t w = producer ? warp : warp - T;          // tile slot in the super-tile
+    uint32_t *tile0 = sm + w * 2048, *tile1 = sm + (T + w) * 2048;
+    const uint32_t P = rapk::warp_perm<32>(seed, 0, lane, 32);
+    const uint32_t stc = tiles / SC, nst = (tiles / SR) * stc;
+    const uint32_t wr = w % SR, wc = w / SR;
+    if (producer) {
+        tile0[P] = lane;
+        __syncwarp();
+        const uint32_t pinv = tile0[lane];
+        __syncwarp();
+        const uint32_t q = lane & 7u, c_in = lane >> 3;
+        uint32_t row_g[8], a_g[8];
+#pragma unroll
+        for (int g = 0; g < 8; ++g) {
+            const uint32_t rr = 4 * g + c_in;
+            row_g[g] = __shfl_sync(0xffffffffu, pinv, rr);
+            a_g[g] = row_g[g] * 64 + 4 * q + rr;
+        }
+        auto load = [&](uint4 (&v)[8], uint32_t st) {
+            const uint32_t si = st / stc, sj = st - si * stc;
+            const int64_t r0 = (int64_t)(si * SR + wr) * 32, c0 = (int64_t)(sj * SC + wc) * 32;
+            const uint32_t *base = src + r0 * n + c0 + 4 * q;
+#pragma unroll
+            for (int g = 0; g < 8; ++g) v[g] = rapk::ldg_stream128(base + (int64_t)row_g[g] * n);
+        };
+        uint4 va[8], vb[8];
+        uint32_t st = blockIdx.x, k = 0;
+        if (st < nst) load(va, st);
+        while (st < nst) {
+            const uint32_t nx = st + gridDim.x;
+            if (nx < nst) load(vb, nx);                      // next tile in flight
+            uint32_t *t = (k & 1) ? tile1 : tile0;
+            if (k >= 2) nb_sync(3 + (k & 1), NT);            // wait: stage drained
+#pragma unroll
+            for (int g = 0; g < 8; ++g) {
+                t[a_g[g] + 0] = va[g].x; t[a_g[g] + 1] = va[g].y;
+                t[a_g[g] + 2] = va[g].z; t[a_g[g] + 3] = va[g].w;
+            }
+            nb_arrive(1 + (k & 1), NT);                      // stage full
+#pragma unroll
+            for (int g = 0; g < 8; ++g) va[g] = vb[g];
+            st = nx; ++k;
+        }
+    } else {
+        const uint32_t drain_base = lane * 64 + P;
+        uint32_t st = blockIdx.x, k = 0;
+        while (st < nst) {
+            const uint32_t *t = (k & 1) ? tile1 : tile0;
+            nb_sync(1 + (k & 1), NT);                        // wait: stage full (all T tiles)
+            const uint32_t si = st / stc, sj = st - si * stc;
+            const int64_t r0 = (int64_t)(si * SR + wr) * 32, c0 = (int64_t)(sj * SC + wc) * 32;
+            uint32_t *o = dst + c0 * n + r0 + lane;
+#pragma unroll
+            for (int c = 0; c < 32; ++c) {
+                *o = t[drain_base + c];
+                o += n;
+            }
+            nb_arrive(3 + (k & 1), NT);                      // stage free
+            st += gridDim.x; ++k;
+        }
+    }
+}
+
 static float median(std::vector<float> v) { std::sort(v.begin(), v.end()); return v[v.size() / 2]; }
 
 int main(int argc, char **argv) {
@@ -334,6 +412,19 @@ int main(int argc, char **argv) {
     add_cluster(clu_kernel<4, 1, 8>, 4, 1, 8);
     add_cluster(clu_kernel<4, 2, 4>, 4, 2, 4);
     add_cluster(clu_kernel<16, 1, 4>, 16, 1, 4);
+    auto add_ws = [&](auto k, int SR, int SC) {
+        const size_t smem = (size_t)2 * SR * SC * 8192;
+        CK(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        const uint32_t nst = (uint32_t)((n / 32 / SR) * (n / 32 / SC));
+        int occ = 1;
+        CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, 2 * SR * SC * 32, smem));
+        const uint32_t grid = std::min<uint32_t>(nst, 148u * occ);
+        char nm[128]; snprintf(nm, sizeof nm, "warp-specialised sr=%d sc=%d (2 stages) occ=%d", SR, SC, occ);
+        vs.push_back({nm, [=] { k<<<grid, 2 * SR * SC * 32, smem>>>(a, b, n, (uint64_t)1, (uint32_t)(n / 32)); }});
+    };
+    add_ws(ws_kernel<8, 1>, 8, 1);
+    add_ws(ws_kernel<4, 2>, 4, 2);
+    add_ws(ws_kernel<4, 1>, 4, 1);
     vs.push_back({"memcpy d2d 256 MiB", [=] { cudaMemcpyAsync(b, a, bytes, cudaMemcpyDeviceToDevice); }});
     const int R = argc > 1 ? atoi(argv[1]) : 7;
     std::vector<std::vector<float>> res(vs.size());
