@@ -297,6 +297,7 @@ def main():
         y = fused.out
     S = args.sweep_trials
     hist = torch.zeros((5, 3, 33), dtype=torch.int64, device=dev)
+    hstep = torch.zeros_like(hist)
 
     def step_transpose(lay):
         if wl == "dist_fused":
@@ -321,9 +322,15 @@ def main():
             return 1
         # this rank's batch of the global trial sequence: step k covers trials
         # [k*S*world, (k+1)*S*world), rank r the r-th slice of it
-        rap.congestion_sweep(S, seed=1, first_trial=(k * world + rank) * S, out=hist, algo=args.sweep_algo)
-        if world > 1:
-            dist.all_reduce(hist)
+        if world == 1:
+            rap.congestion_sweep(S, seed=1, first_trial=k * S, out=hist, algo=args.sweep_algo)
+            return 1
+        # N > 1: this step's batch histogram, all-reduced (the sweep's one exchange), then added
+        # to the run total (all-reducing the running total itself would count earlier steps again)
+        hstep.zero_()
+        rap.congestion_sweep(S, seed=1, first_trial=(k * world + rank) * S, out=hstep, algo=args.sweep_algo)
+        dist.all_reduce(hstep)
+        hist.add_(hstep)
         return 1
 
     soak_hist = torch.zeros_like(hist)
@@ -451,7 +458,9 @@ def main():
         h = hist.cpu().numpy()
         c = np.arange(33)
         E = lambda a: float((a * c).sum() / a.sum())
+        assert (h.sum(-1) == S * world * args.steps).all(), "histogram does not hold every timed trial once"
         line["sweep"] = {"trials_per_s": tps, "trials_per_step": S * world, "w": 32, "algo": args.sweep_algo,
+                         "trials_in_histogram": int(h[0, 0].sum()),
                          "E_ras_stride": E(h[1, 1]), "E_rap_diagonal": E(h[2, 2]), "E_random": E(h[3, 2]),
                          "E_raw_malicious": E(h[4, 0]), "E_rap_stride": E(h[1, 2]),
                          "kernel_ms_median": statistics.median(r["s_ms"]),
