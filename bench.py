@@ -52,6 +52,8 @@ def parse():
     # sweep below its steady rate (launch ramp, per-CTA histogram flush): `--workload sweep`
     # measures the steady rate, 4 batches per warp give 2.88 G/s, 10^9 trials 3.09 G/s.
     p.add_argument("--sweep-trials", type=int, default=148 * 8 * 4 * 32)
+    # --workload trace: each of the 4096 trace warps evaluated under this many trials per step
+    p.add_argument("--trace-trials", type=int, default=256)
     p.add_argument("--sweep-algo", default="default", choices=["default", "match"])
     p.add_argument("--layout", default="rap")
     p.add_argument("--no-e2e", action="store_true")
@@ -220,6 +222,23 @@ def sweep_roofline(tps: float, clocks: dict):
             "issue_active_frac_ncu": prof.get("issue_active_frac")}
 
 
+def trace_roofline(eps: float, clocks: dict):
+    """ALU roofline of the trace evaluator (same pipe model as the sweep): achieved = ALU-pipe
+    warp-instructions per warp-evaluation (ncu capture of trace_kernel<32>) x evaluations/s."""
+    prof = load_profile("trace_w32") or {}
+    ape = prof.get("alu_warp_instructions_per_evaluation")
+    ipe = prof.get("warp_instructions_per_evaluation")
+    mhz = (clocks or {}).get("sm_max_mhz") or 1965.0
+    peak = 148 * 4 * 0.5 * mhz * 1e6
+    ach = ape * eps if ape else None
+    return {"bound": "alu", "achieved": ach, "peak": peak, "unit": "ALU-pipe warp-instructions/s",
+            "frac": ach / peak if ach else None, "traffic": prof.get("dram_bytes_per_launch"),
+            "alu_warp_instructions_per_evaluation": ape, "warp_instructions_per_evaluation": ipe,
+            "issue_frac": ipe * eps / (148 * 4 * mhz * 1e6) if ipe else None,
+            "peak_source": "148 SMs x 4 SMSPs x 0.5 ALU warp-instr/clk (B300_MICROARCH.md pipe rates) x sm_max_mhz",
+            "profile": prof.get("source")}
+
+
 def reduce_over_ranks(x: float, world: int, dev, op: str) -> float:
     if world == 1:
         return x
@@ -313,7 +332,7 @@ def main():
     # pattern families, each evaluated under every step's trials and all five schemes
     trace_cells = workloads.trace_cells(4096, 32, seed=rank, device=dev) if wl == "trace" else None
     trace_hist = torch.zeros((5, 33), dtype=torch.int64, device=dev)
-    TT = max(1, S // 4096)                                 # trials per trace step
+    TT = args.trace_trials                                 # trials per trace step
 
     def step_sweep(k):
         if wl == "trace":
@@ -451,8 +470,7 @@ def main():
         line["trace"] = {"E_by_scheme": {n: float((th[i] * c).sum() / th[i].sum())
                                          for i, n in enumerate(["raw", "ras", "rap", "pad", "xor"])},
                          "kernel_ms_median": statistics.median(r["s_ms"])}
-        line["roofline"] = {"bound": "alu", "achieved": None, "peak": None, "unit": "warp-evaluations/s",
-                            "frac": None, "traffic": None, "note": "secondary workload; no ncu capture this round"}
+        line["roofline"] = trace_roofline(evs / world, r["clocks"])
     elif do_s:
         tps = S * world * args.steps / (r["s_sum"] * 1e-3)
         h = hist.cpu().numpy()
@@ -563,6 +581,25 @@ def main():
                        "h2d_bytes_per_step": hx.numel() * eb * world, "d2h_bytes_per_step": hy.numel() * eb * world,
                        "ms_per_step": ms, "steps": K,
                        "note": "pinned host shard -> H2D -> sharded transpose (public API) -> D2H of the result"}
+    elif not args.no_e2e and wl == "trace":
+        # end to end: the step's access traces uploaded from pinned host memory, evaluated, and
+        # the histogram read back
+        hc = trace_cells.cpu().pin_memory()
+        hh = torch.empty_like(trace_hist, device="cpu").pin_memory()
+        st = torch.cuda.Event(enable_timing=True)
+        en = torch.cuda.Event(enable_timing=True)
+        st.record(stream)
+        for k in range(K):
+            trace_cells.copy_(hc, non_blocking=True)
+            step_sweep(k)
+            hh.copy_(trace_hist, non_blocking=True)
+        en.record(stream)
+        torch.cuda.synchronize()
+        ms = rmax(st.elapsed_time(en)) / K
+        line["e2e"] = {"value": 4096 * TT * 5 * world / (ms * 1e-3), "unit": "warp-evaluations/s",
+                       "h2d_bytes_per_step": hc.numel() * 4 * world, "d2h_bytes_per_step": hh.numel() * 8 * world,
+                       "ms_per_step": ms, "steps": K,
+                       "note": "trace cells H2D from pinned memory + rap_congestion_trace + histogram D2H"}
     elif not args.no_e2e and do_s and wl != "trace":
         hh = torch.empty_like(hist, device="cpu").pin_memory()
         st = torch.cuda.Event(enable_timing=True)

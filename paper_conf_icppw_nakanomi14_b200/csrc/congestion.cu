@@ -629,9 +629,15 @@ sweep_match_kernel(uint32_t w_rt, uint32_t pmask, uint32_t smask, uint64_t seed,
 // ------------------------------------------------------------------ trace evaluator
 constexpr int kTraceChunk = 32;
 
+// W: compile-time w (32: the default bank count, cells split by shift / mask), 0: runtime w.
+// The merge of identical addresses (first_occurrences) depends only on the cells, so it is
+// computed once per trace warp and shared by the schemes; each scheme then costs one shuffle
+// (its shift of the request's row), the bank map and the ballot histogram.
+template <int W>
 __global__ void __launch_bounds__(kSweepWarps * 32)
-trace_kernel(uint32_t w, uint64_t n_warps, const uint32_t *__restrict__ cells, uint32_t smask,
+trace_kernel(uint32_t w_rt, uint64_t n_warps, const uint32_t *__restrict__ cells, uint32_t smask,
              uint64_t seed, uint64_t first, uint64_t n_trials, uint64_t *__restrict__ hist) {
+    const uint32_t w = W ? (uint32_t)W : w_rt;
     __shared__ uint32_t sh_hist[kSweepWarps][kMaxBins];
     const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
     const uint32_t nsch = __popc(smask);
@@ -639,6 +645,7 @@ trace_kernel(uint32_t w, uint64_t n_warps, const uint32_t *__restrict__ cells, u
     for (uint32_t b = lane; b < nbins; b += 32) sh_hist[warp][b] = 0;
     __syncwarp();
     const LaneSel ls(lane);
+    const uint32_t active = (w >= 32) ? kFull : ((1u << w) - 1u);
     const bool need_p = (smask >> RAP_SCHEME_RAP) & 1u, need_r = (smask >> RAP_SCHEME_RAS) & 1u;
     const uint64_t nchunks = (n_warps + kTraceChunk - 1) / kTraceChunk;
     const uint64_t nitems = n_trials * nchunks;
@@ -646,19 +653,24 @@ trace_kernel(uint32_t w, uint64_t n_warps, const uint32_t *__restrict__ cells, u
     for (uint64_t it = (uint64_t)blockIdx.x * kSweepWarps + warp; it < nitems; it += stride) {
         const uint64_t trial = it / nchunks, chunk = it - trial * nchunks;
         const uint64_t n = first + trial;
-        const uint32_t P = need_p ? warp_perm<0>(seed, n, lane, w) : lane;
+        const uint32_t P = need_p ? warp_perm<W>(seed, n, lane, w) : lane;
         const uint32_t r = need_r ? warp_ras_shift(seed, n, lane, w) : 0u;
         const uint64_t k_end = min(n_warps, (chunk + 1) * kTraceChunk);
         for (uint64_t k = chunk * kTraceChunk; k < k_end; ++k) {
             const uint32_t raw_cell = (lane < w) ? cells[k * w + lane] : 0u;
             const bool bad = __any_sync(kFull, raw_cell >= w * w);   // counted in bin 0
             const uint32_t cell = bad ? 0u : raw_cell;
-            const uint32_t row = cell / w, col = cell - (cell / w) * w;
+            const uint32_t row = (W == 32) ? (cell >> 5) : cell / w;
+            const uint32_t col = (W == 32) ? (cell & 31u) : cell - row * w;
+            const uint32_t leaders = first_occurrences(row * 32u + col, active, lane);   // merged requests
             uint32_t mine = 0, e = 0;
 #pragma unroll
             for (int s = 0; s < 5; ++s) {
                 if (!((smask >> s) & 1u)) continue;
-                const uint32_t c = warp_congestion(row, col, s, P, r, lane, w, ls);
+                uint32_t sh = 0;
+                if (s == RAP_SCHEME_RAS || s == RAP_SCHEME_RAP)
+                    sh = __shfl_sync(kFull, s == RAP_SCHEME_RAP ? P : r, row & 31u);
+                const uint32_t c = max_bank_load(bank_of(s, row, col, sh, w), leaders, ls);
                 mine = (lane == e) ? (bad ? 0u : c) : mine;
                 ++e;
             }
@@ -777,12 +789,14 @@ cudaError_t launch_trace(uint32_t w, uint64_t n_warps, const uint32_t *cells, ui
     if (n_trials == 0 || n_warps == 0) return cudaSuccess;
     const int threads = kSweepWarps * 32;
     const uint64_t nchunks = (n_warps + kTraceChunk - 1) / kTraceChunk;
-    const int grid = clamp_grid(n_trials * nchunks, kSweepWarps, resident_ctas<trace_kernel>(threads));
+    auto kern = (w == 32) ? trace_kernel<32> : trace_kernel<0>;
+    const int grid = clamp_grid(n_trials * nchunks, kSweepWarps,
+                                w == 32 ? resident_ctas<trace_kernel<32>>(threads) : resident_ctas<trace_kernel<0>>(threads));
     // counts per warp <= items_per_warp * kTraceChunk; chunk the trial range to stay < 2^31
     const uint64_t trials_chunk = ((uint64_t)grid * kSweepWarps * ((1ull << 31) / kTraceChunk)) / nchunks + 1;
     for (uint64_t done = 0; done < n_trials; done += trials_chunk) {
         const uint64_t cnt = (n_trials - done < trials_chunk) ? n_trials - done : trials_chunk;
-        trace_kernel<<<grid, threads, 0, st>>>(w, n_warps, cells, smask, seed, first + done, cnt, hist);
+        kern<<<grid, threads, 0, st>>>(w, n_warps, cells, smask, seed, first + done, cnt, hist);
     }
     return cudaGetLastError();
 }

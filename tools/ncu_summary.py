@@ -16,11 +16,12 @@ CAPTURES = {
     "transpose_b32_pad": "prof_t32_pad", "transpose_b32_xor": "prof_t32_xor",
     "transpose_b32_ras": "prof_t32_ras", "transpose_b64_rap": "prof_t64_rap",
     "transpose_b64_rap16": "prof_t64_rap16",
-    "sweep_w32": "prof_sweep", "sweep_w32_match": "prof_sweep_match",
+    "sweep_w32": "prof_sweep", "sweep_w32_match": "prof_sweep_match", "trace_w32": "prof_trace",
 }
 
 # work units per captured launch (tools/gpu_profile.sh command lines)
 UNITS = {"sweep_w32": ("trials", 8388608), "sweep_w32_match": ("trials", 4194304),
+         "trace_w32": ("evaluations", 4096 * 296 * 5),
          "transpose_b32_rap": ("bytes", 2 * 8192 * 8192 * 4), "transpose_b32_raw": ("bytes", 2 * 8192 * 8192 * 4),
          "transpose_b32_pad": ("bytes", 2 * 8192 * 8192 * 4), "transpose_b32_xor": ("bytes", 2 * 8192 * 8192 * 4),
          "transpose_b32_ras": ("bytes", 2 * 8192 * 8192 * 4), "transpose_b64_rap": ("bytes", 2 * 16384 * 16384 * 8),
