@@ -629,15 +629,21 @@ sweep_match_kernel(uint32_t w_rt, uint32_t pmask, uint32_t smask, uint64_t seed,
 // ------------------------------------------------------------------ trace evaluator
 constexpr int kTraceChunk = 32;
 
+// RAP_TRACE_MINB: CTAs per SM the register budget is cut for (4: 64 registers, 32 warps per SM)
+#ifndef RAP_TRACE_MINB
+#define RAP_TRACE_MINB 4
+#endif
 // W: compile-time w (32: the default bank count, cells split by shift / mask), 0: runtime w.
-// The merge of identical addresses (first_occurrences) depends only on the cells, so it is
-// computed once per trace warp and shared by the schemes; each scheme then costs one shuffle
-// (its shift of the request's row), the bank map and the ballot histogram.
-template <int W>
-__global__ void __launch_bounds__(kSweepWarps * 32)
-trace_kernel(uint32_t w_rt, uint64_t n_warps, const uint32_t *__restrict__ cells, uint32_t smask,
+// SM: compile-time scheme mask (0: runtime).  The merge of identical addresses depends only on
+// the cells, so the leaders (one lane per distinct cell, one __match_any_sync) are found once per
+// trace warp and shared by the schemes; each scheme then costs one shuffle (its shift of the
+// request's row), the bank map and the ballot histogram.
+template <int W, uint32_t SM>
+__global__ void __launch_bounds__(kSweepWarps * 32, RAP_TRACE_MINB)
+trace_kernel(uint32_t w_rt, uint64_t n_warps, const uint32_t *__restrict__ cells, uint32_t smask_rt,
              uint64_t seed, uint64_t first, uint64_t n_trials, uint64_t *__restrict__ hist) {
     const uint32_t w = W ? (uint32_t)W : w_rt;
+    const uint32_t smask = SM ? SM : smask_rt;
     __shared__ uint32_t sh_hist[kSweepWarps][kMaxBins];
     const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
     const uint32_t nsch = __popc(smask);
@@ -646,6 +652,7 @@ trace_kernel(uint32_t w_rt, uint64_t n_warps, const uint32_t *__restrict__ cells
     __syncwarp();
     const LaneSel ls(lane);
     const uint32_t active = (w >= 32) ? kFull : ((1u << w) - 1u);
+    const uint32_t lt_mask = (1u << lane) - 1u;
     const bool need_p = (smask >> RAP_SCHEME_RAP) & 1u, need_r = (smask >> RAP_SCHEME_RAS) & 1u;
     const uint64_t nchunks = (n_warps + kTraceChunk - 1) / kTraceChunk;
     const uint64_t nitems = n_trials * nchunks;
@@ -656,21 +663,28 @@ trace_kernel(uint32_t w_rt, uint64_t n_warps, const uint32_t *__restrict__ cells
         const uint32_t P = need_p ? warp_perm<W>(seed, n, lane, w) : lane;
         const uint32_t r = need_r ? warp_ras_shift(seed, n, lane, w) : 0u;
         const uint64_t k_end = min(n_warps, (chunk + 1) * kTraceChunk);
+        uint32_t next = (lane < w) ? __ldg(cells + chunk * kTraceChunk * w + lane) : 0u;
         for (uint64_t k = chunk * kTraceChunk; k < k_end; ++k) {
-            const uint32_t raw_cell = (lane < w) ? cells[k * w + lane] : 0u;
+            const uint32_t raw_cell = next;                            // the next trace warp's
+            if (k + 1 < k_end) next = (lane < w) ? __ldg(cells + (k + 1) * w + lane) : 0u;   // load in flight
             const bool bad = __any_sync(kFull, raw_cell >= w * w);   // counted in bin 0
             const uint32_t cell = bad ? 0u : raw_cell;
             const uint32_t row = (W == 32) ? (cell >> 5) : cell / w;
             const uint32_t col = (W == 32) ? (cell & 31u) : cell - row * w;
-            const uint32_t leaders = first_occurrences(row * 32u + col, active, lane);   // merged requests
+            // merged requests: the first lane of each distinct cell is counted
+            const uint32_t same = __match_any_sync(kFull, (lane < w) ? cell : (0x40000000u | lane));
+            const uint32_t leaders = ballot_zero(same, lt_mask) & active;
             uint32_t mine = 0, e = 0;
 #pragma unroll
             for (int s = 0; s < 5; ++s) {
                 if (!((smask >> s) & 1u)) continue;
-                uint32_t sh = 0;
+                uint32_t bank;
                 if (s == RAP_SCHEME_RAS || s == RAP_SCHEME_RAP)
-                    sh = __shfl_sync(kFull, s == RAP_SCHEME_RAP ? P : r, row & 31u);
-                const uint32_t c = max_bank_load(bank_of(s, row, col, sh, w), leaders, ls);
+                    bank = mod_w<W>(col + __shfl_sync(kFull, s == RAP_SCHEME_RAP ? P : r, row & 31u), w);
+                else if (s == RAP_SCHEME_PAD) bank = mod_w<W>(row + col, w);
+                else if (s == RAP_SCHEME_XOR) bank = col ^ row;
+                else bank = col;
+                const uint32_t c = max_bank_load(bank, leaders, ls);
                 mine = (lane == e) ? (bad ? 0u : c) : mine;
                 ++e;
             }
@@ -789,9 +803,12 @@ cudaError_t launch_trace(uint32_t w, uint64_t n_warps, const uint32_t *cells, ui
     if (n_trials == 0 || n_warps == 0) return cudaSuccess;
     const int threads = kSweepWarps * 32;
     const uint64_t nchunks = (n_warps + kTraceChunk - 1) / kTraceChunk;
-    auto kern = (w == 32) ? trace_kernel<32> : trace_kernel<0>;
-    const int grid = clamp_grid(n_trials * nchunks, kSweepWarps,
-                                w == 32 ? resident_ctas<trace_kernel<32>>(threads) : resident_ctas<trace_kernel<0>>(threads));
+    auto kern = (w == 32 && smask == 31u) ? trace_kernel<32, 31u>
+              : (w == 32 && smask == 7u) ? trace_kernel<32, 7u> : (w == 32) ? trace_kernel<32, 0u> : trace_kernel<0, 0u>;
+    const int occ = (w == 32 && smask == 31u) ? resident_ctas<trace_kernel<32, 31u>>(threads)
+                  : (w == 32 && smask == 7u) ? resident_ctas<trace_kernel<32, 7u>>(threads)
+                  : (w == 32) ? resident_ctas<trace_kernel<32, 0u>>(threads) : resident_ctas<trace_kernel<0, 0u>>(threads);
+    const int grid = clamp_grid(n_trials * nchunks, kSweepWarps, occ);
     // counts per warp <= items_per_warp * kTraceChunk; chunk the trial range to stay < 2^31
     const uint64_t trials_chunk = ((uint64_t)grid * kSweepWarps * ((1ull << 31) / kTraceChunk)) / nchunks + 1;
     for (uint64_t done = 0; done < n_trials; done += trials_chunk) {
