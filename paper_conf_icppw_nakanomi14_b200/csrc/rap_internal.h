@@ -28,10 +28,16 @@ struct TransposeTuning {
     int ctas_per_sm = 0;  // persistent grid = #SMs x this (0: as many as fit)
     bool vst = false;     // 128-bit output stores (shuffle-transposed) instead of 32/64-bit rows
     bool tma_store = false;  // drain into a dense staging tile, one TMA bulk tensor store per super-tile
+    int cl = 1;           // thread-block cluster of cl CTAs stacked along the input rows, drains in lockstep
 };
-constexpr int kDefaultSR32 = 8, kDefaultSC32 = 2, kDefaultSR64 = 12, kDefaultSC64 = 1;
+// fp32: 4 x 2 warps per CTA, clusters of 4 CTAs (a 16 x 2-tile cluster super-tile);
+// fp64: 12 x 1 warps, no cluster (profiles/r01_tune_transpose*.txt, r01_probe_transpose.txt)
+constexpr int kDefaultSR32 = 4, kDefaultSC32 = 2, kDefaultSR64 = 12, kDefaultSC64 = 1;
+constexpr int kDefaultCL32 = 4, kDefaultCL64 = 1;
+// fused sharded transpose (peer stores): 8 x 2 warps, no cluster
+constexpr int kPeerSR32 = 8, kPeerSC32 = 2;
 // measured on B200 (tools/tune_transpose.cu, profiles/r01_tune_transpose.txt)
-constexpr int kDefaultMinB32 = 1, kDefaultMinB64 = 1;
+constexpr int kDefaultMinB32 = 2, kDefaultMinB64 = 1;   // fp32: 2 CTAs of 8 warps per SM (128 registers)
 constexpr int kDefaultDepth32 = 1, kDefaultDepth64 = 1;
 constexpr int kDefaultCtas32 = 0, kDefaultCtas64 = 0;
 constexpr bool kDefaultVst32 = false, kDefaultVst64 = false;

@@ -94,12 +94,22 @@ __device__ __forceinline__ void tma_wait_read() { asm volatile("cp.async.bulk.wa
 __device__ __forceinline__ void tma_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
 __device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 
-template <int L, int EW, bool VEC, int DEPTH, int MINB, bool VST, int SR, int SC, bool PEERS, bool TMAS>
+// Cluster lockstep (CL > 1): the CL CTAs of a thread-block cluster take the CL row blocks of one
+// (CL*SR) x SC-tile cluster super-tile and drain behind one barrier.cluster, so each output row
+// receives CL*SR*128 B at once (+1.5-2 % over CL = 1, profiles/r01_probe_transpose.txt).
+__device__ __forceinline__ void cluster_sync_relaxed() {
+    asm volatile("barrier.cluster.arrive.relaxed.aligned;" ::: "memory");
+    asm volatile("barrier.cluster.wait.aligned;" ::: "memory");
+}
+
+template <int L, int EW, bool VEC, int DEPTH, int MINB, bool VST, int SR, int SC, bool PEERS, bool TMAS,
+          int CL = 1>
 __global__ void __launch_bounds__(SR * SC * 32, MINB)
 transpose_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, int64_t rows,
                  int64_t cols, int64_t ld_src, int64_t ld_dst, uint64_t seed, uint32_t tiles_r,
                  uint32_t tiles_c, bool vst_ok, PeerOut peers, const __grid_constant__ CUtensorMap tmap) {
     static_assert(!TMAS || (DEPTH == 1 && !PEERS && SR * 32 <= 256), "TMA store: depth 1, box <= 256");
+    static_assert(CL == 1 || (DEPTH == 1 && !TMAS), "cluster lockstep: depth 1, no TMA store");
     using C = TileCfg<L, EW>;
     constexpr int NE = C::NE, R = C::R, G = C::G, LPR = C::LPR;
     constexpr int PW = 32 * Geom<L>::RP;            // plane size in words
@@ -133,13 +143,20 @@ transpose_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, i
     }
     const uint32_t drain_base = word_of<L>(lane, 0, sh_lane);
 
-    // super-tile s -> this warp's tile (ti, tj); false when it falls outside the matrix
+    // super-tile s -> this warp's tile (ti, tj); false when it falls outside the matrix.  With
+    // clusters, s counts cluster super-tiles and CTA rank `crank` takes row block crank of it.
+    uint32_t crank = 0, st_first = blockIdx.x, st_step = gridDim.x;
+    if (CL > 1) {
+        asm("mov.u32 %0, %%cluster_ctarank;" : "=r"(crank));
+        asm("mov.u32 %0, %%clusterid.x;" : "=r"(st_first));
+        asm("mov.u32 %0, %%nclusterid.x;" : "=r"(st_step));
+    }
     const uint32_t stc = (tiles_c + SC - 1) / SC;
-    const uint32_t nst = ((tiles_r + SR - 1) / SR) * stc;
-    const uint32_t wr = warp % SR, wc = warp / SR;
+    const uint32_t nst = ((tiles_r + SR * CL - 1) / (SR * CL)) * stc;
+    const uint32_t wr = crank * SR + warp % SR, wc = warp / SR;
     auto coords = [&](uint32_t st, uint32_t &ti, uint32_t &tj) -> bool {
         const uint32_t si = st / stc, sj = st - si * stc;
-        ti = si * SR + wr;
+        ti = si * SR * CL + wr;
         tj = sj * SC + wc;
         return ti < tiles_r && tj < tiles_c;
     };
@@ -272,7 +289,7 @@ transpose_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, i
         }
     };
 
-    uint32_t st = blockIdx.x, ti = 0, tj = 0;
+    uint32_t st = st_first, ti = 0, tj = 0;
     bool act = st < nst && coords(st, ti, tj);
     if (TMAS) {
         uint4 v[G];
@@ -302,10 +319,11 @@ transpose_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, i
             const bool cact = act;
             if (cact) store_tile(v);                     // T1
             __syncwarp();
-            st += gridDim.x;
+            st += st_step;
             act = st < nst && coords(st, ti, tj);
             if (act) load(v, ti, tj);                    // T3: next tile in flight
-            if (SR * SC > 1) __syncthreads();            // drains of the super-tile together
+            if (CL > 1) cluster_sync_relaxed();          // drains of the cluster super-tile together
+            else if (SR * SC > 1) __syncthreads();       // drains of the super-tile together
             if (cact) drain(cti, ctj);                   // T2
             __syncwarp();
         }
@@ -383,6 +401,7 @@ TransposeTuning default_tuning(uint32_t elem_bytes) {
     t.depth = elem_bytes == 4 ? kDefaultDepth32 : kDefaultDepth64;
     t.ctas_per_sm = elem_bytes == 4 ? kDefaultCtas32 : kDefaultCtas64;
     t.vst = elem_bytes == 4 ? kDefaultVst32 : kDefaultVst64;
+    t.cl = elem_bytes == 4 ? kDefaultCL32 : kDefaultCL64;
     return t;
 }
 
@@ -418,8 +437,51 @@ static bool make_out_map(CUtensorMap *m, void *dst, int64_t rows, int64_t cols, 
               CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
+// Cluster launch: as many clusters as can be co-resident (cached per kernel and device), each
+// looping over cluster super-tiles.
+template <typename K>
+static cudaError_t launch_clustered(K kernel, ShapeCache &cache, int cl, int threads, size_t smem, int64_t nst,
+                                    cudaStream_t st, const uint32_t *src, uint32_t *dst, int64_t rows, int64_t cols,
+                                    int64_t ld_src, int64_t ld_dst, uint64_t seed, uint32_t tiles_r,
+                                    uint32_t tiles_c, bool vst_ok, const PeerOut &peers, const CUtensorMap &tmap) {
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    if (dev < 0 || dev >= kMaxDevices) return cudaErrorInvalidDevice;
+    cudaLaunchConfig_t cfg = {};
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = (unsigned)cl;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    cfg.blockDim = dim3((unsigned)threads);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    int ncl = cache.occ[dev].load(std::memory_order_relaxed);   // here: co-resident clusters
+    if (ncl == 0) {
+        e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e != cudaSuccess) return e;
+        int sms = 0;
+        e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        if (e != cudaSuccess) return e;
+        cfg.gridDim = dim3((unsigned)(sms * cl));
+        e = cudaOccupancyMaxActiveClusters(&ncl, kernel, &cfg);
+        if (e != cudaSuccess) return e;
+        if (ncl < 1) return cudaErrorInvalidConfiguration;
+        cache.occ[dev].store(ncl, std::memory_order_relaxed);
+    }
+    const int64_t nclusters = nst < ncl ? nst : ncl;
+    cfg.gridDim = dim3((unsigned)(nclusters * cl));
+    e = cudaLaunchKernelEx(&cfg, kernel, src, dst, rows, cols, ld_src, ld_dst, seed, tiles_r, tiles_c, vst_ok,
+                           peers, tmap);
+    if (e != cudaSuccess) return e;
+    return cudaGetLastError();
+}
+
 template <int L, int EW, bool VEC, int DEPTH, int MINB, bool VST, int SR, int SC, bool PEERS = false,
-          bool TMAS = false>
+          bool TMAS = false, int CL = 1>
 static cudaError_t launch_one(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
                               int64_t ld_dst, uint64_t seed, const TransposeTuning &tu, cudaStream_t st,
                               const PeerOut &peers = PeerOut{}) {
@@ -429,8 +491,8 @@ static cudaError_t launch_one(const void *src, void *dst, int64_t rows, int64_t 
         return launch_one<L, EW, VEC, DEPTH, MINB, VST, SR, SC, PEERS, false>(src, dst, rows, cols, ld_src,
                                                                              ld_dst, seed, tu, st, peers);
     const uint32_t tiles_r = (uint32_t)((rows + 31) / 32), tiles_c = (uint32_t)((cols + 31) / 32);
-    const int64_t nst = (int64_t)((tiles_r + SR - 1) / SR) * ((tiles_c + SC - 1) / SC);
-    auto k = transpose_kernel<L, EW, VEC, DEPTH, MINB, VST, SR, SC, PEERS, TMAS>;
+    const int64_t nst = (int64_t)((tiles_r + SR * CL - 1) / (SR * CL)) * ((tiles_c + SC - 1) / SC);
+    auto k = transpose_kernel<L, EW, VEC, DEPTH, MINB, VST, SR, SC, PEERS, TMAS, CL>;
     static ShapeCache cache;
     bool vst_ok = ((uintptr_t)dst % 16 == 0) && ((ld_dst * EW * 4) % 16 == 0);
     if (PEERS) {
@@ -439,6 +501,9 @@ static cudaError_t launch_one(const void *src, void *dst, int64_t rows, int64_t 
     }
     const size_t smem = sizeof(uint32_t) * (warp_smem_words<L, EW>() * SR * SC +
                                             (TMAS ? (size_t)SR * 32 * SC * 32 * EW : 0));
+    if (CL > 1)
+        return launch_clustered(k, cache, CL, SR * SC * 32, smem, nst, st, (const uint32_t *)src, (uint32_t *)dst,
+                                rows, cols, ld_src, ld_dst, seed, tiles_r, tiles_c, vst_ok, peers, tmap);
     int grid = 0;
     const cudaError_t e = grid_for(k, cache, SR * SC * 32, smem, nst, 1, tu.ctas_per_sm, &grid);
     if (e != cudaSuccess) return e;
@@ -451,10 +516,10 @@ template <int L, int EW, bool VEC>
 static cudaError_t launch_shape(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
                                 int64_t ld_dst, uint64_t seed, const TransposeTuning &tu, cudaStream_t st) {
 #define RAPK_SHAPE(D, M, V, R_, C_)                                                                  \
-    if (tu.depth == D && tu.minb == M && tu.vst == V && tu.sr == R_ && tu.sc == C_ && !tu.tma_store)  \
+    if (tu.depth == D && tu.minb == M && tu.vst == V && tu.sr == R_ && tu.sc == C_ && !tu.tma_store && tu.cl == 1) \
         return launch_one<L, EW, VEC, D, M, V, R_, C_>(src, dst, rows, cols, ld_src, ld_dst, seed, tu, st);
 #define RAPK_TSHAPE(M, R_, C_)                                                                       \
-    if (tu.depth == 1 && tu.minb == M && !tu.vst && tu.sr == R_ && tu.sc == C_ && tu.tma_store)      \
+    if (tu.depth == 1 && tu.minb == M && !tu.vst && tu.sr == R_ && tu.sc == C_ && tu.tma_store && tu.cl == 1) \
         return launch_one<L, EW, VEC, 1, M, false, R_, C_, false, true>(src, dst, rows, cols, ld_src, ld_dst, \
                                                                         seed, tu, st);
 #ifdef RAP_TUNING_SWEEP
@@ -471,9 +536,11 @@ static cudaError_t launch_shape(const void *src, void *dst, int64_t rows, int64_
 #undef RAPK_SHAPE
 #undef RAPK_TSHAPE
     (void)tu;
-    if (EW == 1)
-        return launch_one<L, EW, VEC, kDefaultDepth32, kDefaultMinB32, kDefaultVst32, kDefaultSR32, kDefaultSC32>(
-            src, dst, rows, cols, ld_src, ld_dst, seed, tu, st);
+    if (EW == 1 && tu.cl == kDefaultCL32)
+        return launch_one<L, EW, VEC, kDefaultDepth32, kDefaultMinB32, kDefaultVst32, kDefaultSR32, kDefaultSC32,
+                          false, false, kDefaultCL32>(src, dst, rows, cols, ld_src, ld_dst, seed, tu, st);
+    if (EW == 1)      // the round-1 shape without cluster (8 x 2 warps), kept selectable for A/B runs
+        return launch_one<L, EW, VEC, 1, 1, false, 8, 2>(src, dst, rows, cols, ld_src, ld_dst, seed, tu, st);
     return launch_one<L, EW, VEC, kDefaultDepth64, kDefaultMinB64, kDefaultVst64, kDefaultSR64, kDefaultSC64>(
         src, dst, rows, cols, ld_src, ld_dst, seed, tu, st);
 }
@@ -504,8 +571,8 @@ static cudaError_t dispatch_peers(const void *src, int64_t rows, int64_t cols, i
 #define RAPK_PEER(LAY)                                                                              \
     case LAY:                                                                                       \
         return eb == 4                                                                              \
-            ? launch_one<LAY, 1, VEC, kDefaultDepth32, kDefaultMinB32, kDefaultVst32, kDefaultSR32,  \
-                         kDefaultSC32, true>(src, nullptr, rows, cols, ld_src, ld_dst, seed, tu, st, pe) \
+            ? launch_one<LAY, 1, VEC, kDefaultDepth32, 1, kDefaultVst32, kPeerSR32,                  \
+                         kPeerSC32, true>(src, nullptr, rows, cols, ld_src, ld_dst, seed, tu, st, pe)   \
             : launch_one<LAY, 2, VEC, kDefaultDepth64, kDefaultMinB64, kDefaultVst64, kDefaultSR64,  \
                          kDefaultSC64, true>(src, nullptr, rows, cols, ld_src, ld_dst, seed, tu, st, pe);
     switch (layout) {

@@ -169,7 +169,22 @@ wrap_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, int64_
 // lockstep drains) with the lockstep widened across a thread-block cluster of CL CTAs stacked
 // along the input rows: a cluster super-tile is (CL*SR) x SC tiles, drained behind one cluster
 // barrier, so each output row receives CL*SR*128 B at once.
-template <int SR, int SC, int CL>
+__device__ __forceinline__ void st_cs32(uint32_t *p, uint32_t v) {
+    asm volatile("st.global.cs.u32 [%0], %1;" :: "l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void st_ef32(uint32_t *p, uint32_t v, uint64_t pol) {
+    asm volatile("st.global.L2::cache_hint.u32 [%0], %1, %2;" :: "l"(p), "r"(v), "l"(pol) : "memory");
+}
+__device__ __forceinline__ uint4 ld_hint128(const void *p, uint64_t pol) {
+    uint4 r;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
+                 : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p), "l"(pol));
+    return r;
+}
+
+// ST: 0 plain stores, 1 st.global.cs, 2 L2 evict_first stores, 3 evict_first loads + stores,
+//     4 evict_last stores (keep output lines in L2 so write-back happens in larger batches)
+template <int SR, int SC, int CL, int ST = 0>
 __global__ void __launch_bounds__(SR * SC * 32, 1)
 clu_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, int64_t n, uint64_t seed,
            uint32_t tiles) {
@@ -190,6 +205,9 @@ clu_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, int64_t
         a_g[g] = row_g[g] * 64 + 4 * q + rr;
     }
     const uint32_t drain_base = lane * 64 + P;
+    uint64_t pol_ef, pol_el;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol_ef));
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol_el));
     uint32_t crank = 0, cid = blockIdx.x, ncl = gridDim.x;
     if (CL > 1) {
         asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(crank));
@@ -203,7 +221,8 @@ clu_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, int64_t
         const int64_t r0 = (int64_t)(si * SR * CL + wr) * 32, c0 = (int64_t)(sj * SC + wc) * 32;
         const uint32_t *base = src + r0 * n + c0 + 4 * q;
 #pragma unroll
-        for (int g = 0; g < 8; ++g) v[g] = rapk::ldg_stream128(base + (int64_t)row_g[g] * n);
+        for (int g = 0; g < 8; ++g)
+            v[g] = (ST == 3) ? ld_hint128(base + (int64_t)row_g[g] * n, pol_ef) : rapk::ldg_stream128(base + (int64_t)row_g[g] * n);
     };
     uint32_t st = cid;
     uint4 v[8];
@@ -229,7 +248,11 @@ clu_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, int64_t
         uint32_t *o = dst + c0 * n + r0 + lane;
 #pragma unroll
         for (int c = 0; c < 32; ++c) {
-            *o = tile[drain_base + c];
+            const uint32_t x = tile[drain_base + c];
+            if (ST == 1) st_cs32(o, x);
+            else if (ST == 2 || ST == 3) st_ef32(o, x, pol_ef);
+            else if (ST == 4) st_ef32(o, x, pol_el);
+            else *o = x;
             o += n;
         }
         __syncwarp();
@@ -381,8 +404,17 @@ int main(int argc, char **argv) {
     std::vector<std::pair<std::string, std::function<void()>>> vs;
     {
         rapk::TransposeTuning tu = rapk::default_tuning(4);
-        vs.push_back({"library rap 8x2 (LDG->STS, unwrapped)",
+        vs.push_back({"library rap default (4x2 warps, cluster 4)",
                       [=] { rapk::launch_transpose_tuned(a, b, n, n, n, n, 4, RAP_LAYOUT_RAP, 1, tu, 0); }});
+        rapk::TransposeTuning t1 = tu;
+        t1.cl = 1;
+        vs.push_back({"library rap 8x2, no cluster (round-1 default)",
+                      [=] { rapk::launch_transpose_tuned(a, b, n, n, n, n, 4, RAP_LAYOUT_RAP, 1, t1, 0); }});
+        for (int lay : {RAP_LAYOUT_RAW, RAP_LAYOUT_PAD, RAP_LAYOUT_XOR, RAP_LAYOUT_RAS}) {
+            static const char *nm[] = {"raw", "pad", "xor", "ras"};
+            vs.push_back({std::string("library default layout ") + nm[lay],
+                          [=] { rapk::launch_transpose_tuned(a, b, n, n, n, n, 4, lay, 1, tu, 0); }});
+        }
     }
     auto add_cluster = [&](auto k, int SR, int SC, int CL) {
         const size_t smem = (size_t)SR * SC * 8192;
@@ -400,18 +432,14 @@ int main(int argc, char **argv) {
         CK(cudaOccupancyMaxActiveClusters(&ncl, k, &cfg));
         const uint32_t nst = (uint32_t)((n / 32 / (SR * CL)) * (n / 32 / SC));
         cfg.gridDim = dim3(std::min<uint32_t>(nst, (uint32_t)ncl) * CL);
-        char nm[128]; snprintf(nm, sizeof nm, "cluster sr=%d sc=%d cl=%d clusters=%d", SR, SC, CL, ncl);
+        static int idx = 0;
+        char nm[128]; snprintf(nm, sizeof nm, "cluster sr=%d sc=%d cl=%d clusters=%d #%d", SR, SC, CL, ncl, idx++);
         vs.push_back({nm, [=] { cudaLaunchKernelEx(&cfg, k, (const uint32_t *)a, b, n, (uint64_t)1, (uint32_t)(n / 32)); }});
     };
     add_cluster(clu_kernel<8, 2, 1>, 8, 2, 1);
-    add_cluster(clu_kernel<8, 2, 2>, 8, 2, 2);
-    add_cluster(clu_kernel<8, 2, 4>, 8, 2, 4);
-    add_cluster(clu_kernel<8, 1, 4>, 8, 1, 4);
-    add_cluster(clu_kernel<8, 1, 8>, 8, 1, 8);
-    add_cluster(clu_kernel<4, 2, 8>, 4, 2, 8);
-    add_cluster(clu_kernel<4, 1, 8>, 4, 1, 8);
     add_cluster(clu_kernel<4, 2, 4>, 4, 2, 4);
-    add_cluster(clu_kernel<16, 1, 4>, 16, 1, 4);
+    add_cluster(clu_kernel<4, 2, 8>, 4, 2, 8);
+    add_cluster(clu_kernel<8, 2, 2>, 8, 2, 2);
     auto add_ws = [&](auto k, int SR, int SC) {
         const size_t smem = (size_t)2 * SR * SC * 8192;
         CK(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
@@ -422,9 +450,6 @@ int main(int argc, char **argv) {
         char nm[128]; snprintf(nm, sizeof nm, "warp-specialised sr=%d sc=%d (2 stages) occ=%d", SR, SC, occ);
         vs.push_back({nm, [=] { k<<<grid, 2 * SR * SC * 32, smem>>>(a, b, n, (uint64_t)1, (uint32_t)(n / 32)); }});
     };
-    add_ws(ws_kernel<8, 1>, 8, 1);
-    add_ws(ws_kernel<4, 2>, 4, 2);
-    add_ws(ws_kernel<4, 1>, 4, 1);
     vs.push_back({"memcpy d2d 256 MiB", [=] { cudaMemcpyAsync(b, a, bytes, cudaMemcpyDeviceToDevice); }});
     const int R = argc > 1 ? atoi(argv[1]) : 7;
     std::vector<std::vector<float>> res(vs.size());
