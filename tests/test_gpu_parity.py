@@ -355,6 +355,52 @@ def test_sharded_transpose_emulated_on_one_gpu(rap, oracle, dtype, G, M):
     assert np.array_equal(bits(got), oracle.transpose(bits(A)))
 
 
+def _cfg5_check(oracle, A, got, seed):
+    """32768^2 check on sampled bands: output rows (= input columns) and output columns (= input
+    rows) both go through the oracle, plus the first/last 33 of each."""
+    _band_check(oracle, A, got, n_bands=3, band=40, seed=seed)
+    N = A.shape[1]
+    for c0 in (0, 12345, N - 33):
+        assert np.array_equal(bits(got[c0:c0 + 33]), oracle.transpose(bits(A[:, c0:c0 + 33]))), c0
+
+
+@pytest.mark.parametrize("G", [2, 4, 8])
+def test_transpose_cfg5_32768_sharded_emulated(rap, oracle, G):
+    # BASELINE cfg5 at full size (32768^2 float32, 4 GiB), the NCCL-path pieces of G ranks on one
+    # GPU: per-rank local RAP transpose of its M x N row block, the all-to-all as block slicing,
+    # rap_unpack_blocks into the rank's M x N output rows.
+    N = 32768
+    M = N // G
+    A = workloads.random_bits(N, N, torch.float32, seed=50 + G, device="cuda")
+    got = torch.empty((N, N), dtype=torch.float32, device="cuda")
+    sends = [rap.transpose(A[s * M:(s + 1) * M], layout="rap", seed=3) for s in range(G)]   # N x M each
+    for g in range(G):
+        # rank g's receive buffer: block g (rows gM..gM+M) of every rank's send, in rank order
+        recv = torch.cat([sends[s][g * M:(g + 1) * M] for s in range(G)], 0)
+        rap.unpack_blocks(recv, got[g * M:(g + 1) * M], G)
+        del recv
+    del sends
+    torch.cuda.synchronize()
+    _cfg5_check(oracle, A, got, seed=G)
+    # property at full size: the sharded result equals the 1-GPU transpose bit for bit
+    assert torch.equal(got.view(torch.int32), rap.transpose(A, layout="raw").view(torch.int32))
+
+
+def test_transpose_to_peers_cfg5_32768_emulated(rap, oracle):
+    # NEXT-2 fused exchange at cfg5's full size, G = 8: every rank's kernel stores its tiles
+    # straight into the owners' output shards (local buffers standing in for mapped peers)
+    N, G = 32768, 8
+    M = N // G
+    A = workloads.random_bits(N, N, torch.float32, seed=77, device="cuda")
+    got = torch.zeros((N, N), dtype=torch.float32, device="cuda")
+    ptrs = [got[h * M:(h + 1) * M].data_ptr() for h in range(G)]
+    for g in range(G):
+        rap.transpose_to_peers(A[g * M:(g + 1) * M], ptrs, g, layout="rap", seed=5)
+    torch.cuda.synchronize()
+    _cfg5_check(oracle, A, got, seed=9)
+    assert torch.equal(rap.transpose(got, layout="rap", seed=2).view(torch.int32), A.view(torch.int32))
+
+
 def test_unpack_blocks_strided_output(rap):
     G, M = 3, 40
     recv = workloads.random_bits(G * M, M, torch.float32, seed=1).cuda()

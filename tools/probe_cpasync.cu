@@ -184,7 +184,10 @@ __device__ __forceinline__ uint4 ld_hint128(const void *p, uint64_t pol) {
 
 // ST: 0 plain stores, 1 st.global.cs, 2 L2 evict_first stores, 3 evict_first loads + stores,
 //     4 evict_last stores (keep output lines in L2 so write-back happens in larger batches)
-template <int SR, int SC, int CL, int ST = 0>
+// GR > 1: cluster super-tiles visited in groups of GR super-tile rows (column-major inside a
+// group), so the concurrently active clusters cover a squarish block of the matrix: shorter
+// scattered write runs across output rows, more input rows read in parallel.
+template <int SR, int SC, int CL, int ST = 0, int GR = 1>
 __global__ void __launch_bounds__(SR * SC * 32, 1)
 clu_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, int64_t n, uint64_t seed,
            uint32_t tiles) {
@@ -216,8 +219,13 @@ clu_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, int64_t
     }
     const uint32_t stc = tiles / SC, nst = (tiles / (SR * CL)) * stc;
     const uint32_t wr = crank * SR + warp % SR, wc = warp / SR;
+    auto split = [&](uint32_t st, uint32_t &si, uint32_t &sj) {
+        if (GR == 1) { si = st / stc; sj = st - si * stc; return; }
+        const uint32_t g = st / (GR * stc), idx = st - g * (GR * stc);
+        si = g * GR + idx % GR; sj = idx / GR;
+    };
     auto load = [&](uint4 (&v)[8], uint32_t st) {
-        const uint32_t si = st / stc, sj = st - si * stc;
+        uint32_t si, sj; split(st, si, sj);
         const int64_t r0 = (int64_t)(si * SR * CL + wr) * 32, c0 = (int64_t)(sj * SC + wc) * 32;
         const uint32_t *base = src + r0 * n + c0 + 4 * q;
 #pragma unroll
@@ -243,7 +251,7 @@ clu_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, int64_t
         } else {
             __syncthreads();
         }
-        const uint32_t si = cst / stc, sj = cst - si * stc;
+        uint32_t si, sj; split(cst, si, sj);
         const int64_t r0 = (int64_t)(si * SR * CL + wr) * 32, c0 = (int64_t)(sj * SC + wc) * 32;
         uint32_t *o = dst + c0 * n + r0 + lane;
 #pragma unroll
@@ -253,6 +261,90 @@ clu_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, int64_t
             else if (ST == 2 || ST == 3) st_ef32(o, x, pol_ef);
             else if (ST == 4) st_ef32(o, x, pol_el);
             else *o = x;
+            o += n;
+        }
+        __syncwarp();
+    }
+}
+
+
+// K-plane fp32 tile: one warp owns a (32K) x 32 tile of 32-bit elements held as K RAP planes,
+// plane p row i = input row K*i + p (each plane the paper's 32 x 32 RAP tile with the same P).
+// The drain reads the K planes at the same (conflict-free, stride) address and writes K adjacent
+// output columns with one K-word store: 64-/128-bit STG, 256 / 512 B per warp instruction per
+// output row, and K x 4 KiB of loads in flight per warp.  RP = 64: unwrapped rows, 32: wrapped.
+template <int K, int SR, int SC, int CL, int RP>
+__global__ void __launch_bounds__(SR * SC * 32, 1)
+kplane_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, int64_t n, uint64_t seed,
+              uint32_t tiles) {
+    constexpr int PW = 32 * RP;
+    extern __shared__ __align__(16) uint32_t sm[];
+    const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
+    uint32_t *tile = sm + warp * K * PW;
+    const uint32_t P = rapk::warp_perm<32>(seed, 0, lane, 32);
+    tile[P] = lane;
+    __syncwarp();
+    const uint32_t pinv = tile[lane];
+    __syncwarp();
+    const uint32_t q = lane & 7u, c_in = lane >> 3;
+    uint32_t row_g[8], a_g[8];
+#pragma unroll
+    for (int g = 0; g < 8; ++g) {
+        const uint32_t rr = 4 * g + c_in;            // = P[row_g[g]]
+        row_g[g] = __shfl_sync(0xffffffffu, pinv, rr);
+        a_g[g] = RP == 64 ? row_g[g] * 64 + 4 * q + rr : row_g[g] * 32;
+    }
+    uint32_t crank = 0, cid = blockIdx.x, ncl = gridDim.x;
+    if (CL > 1) {
+        asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(crank));
+        asm volatile("mov.u32 %0, %%clusterid.x;" : "=r"(cid));
+        asm volatile("mov.u32 %0, %%nclusterid.x;" : "=r"(ncl));
+    }
+    const uint32_t rtiles = tiles / K;
+    const uint32_t stc = tiles / SC, nst = (rtiles / (SR * CL)) * stc;
+    const uint32_t wr = crank * SR + warp % SR, wc = warp / SR;
+    auto load = [&](uint4 (&v)[K][8], uint32_t st) {
+        const uint32_t si = st / stc, sj = st - si * stc;
+        const int64_t r0 = (int64_t)(si * SR * CL + wr) * 32 * K, c0 = (int64_t)(sj * SC + wc) * 32;
+        const uint32_t *base = src + r0 * n + c0 + 4 * q;
+#pragma unroll
+        for (int p = 0; p < K; ++p)
+#pragma unroll
+            for (int g = 0; g < 8; ++g) v[p][g] = rapk::ldg_stream128(base + (int64_t)(K * row_g[g] + p) * n);
+    };
+    uint32_t st = cid;
+    uint4 v[K][8];
+    if (st < nst) load(v, st);
+    while (st < nst) {
+        const uint32_t cst = st;
+#pragma unroll
+        for (int p = 0; p < K; ++p)
+#pragma unroll
+            for (int g = 0; g < 8; ++g) {
+                const uint32_t w4[4] = {v[p][g].x, v[p][g].y, v[p][g].z, v[p][g].w};
+#pragma unroll
+                for (int e = 0; e < 4; ++e) {
+                    const uint32_t off = RP == 64 ? a_g[g] + e : a_g[g] + ((4 * q + e + 4 * g + c_in) & 31u);
+                    tile[p * PW + off] = w4[e];
+                }
+            }
+        __syncwarp();
+        st += ncl;
+        if (st < nst) load(v, st);
+        if (CL > 1) {
+            asm volatile("barrier.cluster.arrive.relaxed.aligned;" ::: "memory");
+            asm volatile("barrier.cluster.wait.aligned;" ::: "memory");
+        } else if (SR * SC > 1) {
+            __syncthreads();
+        }
+        const uint32_t si = cst / stc, sj = cst - si * stc;
+        const int64_t r0 = (int64_t)(si * SR * CL + wr) * 32 * K, c0 = (int64_t)(sj * SC + wc) * 32;
+        uint32_t *o = dst + c0 * n + r0 + K * lane;
+#pragma unroll
+        for (int c = 0; c < 32; ++c) {
+            const uint32_t off = RP == 64 ? lane * 64 + P + c : lane * 32 + ((P + c) & 31u);
+            if (K == 2) *reinterpret_cast<uint2 *>(o) = make_uint2(tile[off], tile[PW + off]);
+            else *reinterpret_cast<uint4 *>(o) = make_uint4(tile[off], tile[PW + off], tile[2 * PW + off], tile[3 * PW + off]);
             o += n;
         }
         __syncwarp();
@@ -436,10 +528,52 @@ int main(int argc, char **argv) {
         char nm[128]; snprintf(nm, sizeof nm, "cluster sr=%d sc=%d cl=%d clusters=%d #%d", SR, SC, CL, ncl, idx++);
         vs.push_back({nm, [=] { cudaLaunchKernelEx(&cfg, k, (const uint32_t *)a, b, n, (uint64_t)1, (uint32_t)(n / 32)); }});
     };
-    add_cluster(clu_kernel<8, 2, 1>, 8, 2, 1);
+    auto add_kp = [&](auto k, int K, int SR, int SC, int CL, int RP) {
+        const size_t smem = (size_t)SR * SC * K * 32 * RP * 4;
+        CK(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        if (CL > 1) CK(cudaFuncSetAttribute(k, cudaFuncAttributeNonPortableClusterSizeAllowed, 1));
+        cudaLaunchConfig_t cfg = {};
+        static cudaLaunchAttribute at[64][1];
+        static int nat = 0;
+        cudaLaunchAttribute *ap = at[nat++];
+        ap[0].id = cudaLaunchAttributeClusterDimension;
+        ap[0].val.clusterDim.x = CL; ap[0].val.clusterDim.y = 1; ap[0].val.clusterDim.z = 1;
+        cfg.blockDim = dim3(SR * SC * 32); cfg.dynamicSmemBytes = smem; cfg.attrs = ap; cfg.numAttrs = 1;
+        int ncl = 0;
+        cfg.gridDim = dim3(148 * CL);
+        CK(cudaOccupancyMaxActiveClusters(&ncl, k, &cfg));
+        const uint32_t nst = (uint32_t)((n / 32 / K / (SR * CL)) * (n / 32 / SC));
+        cfg.gridDim = dim3(std::min<uint32_t>(nst, (uint32_t)ncl) * CL);
+        static int idx = 0;
+        char nm[128]; snprintf(nm, sizeof nm, "kplane K=%d sr=%d sc=%d cl=%d rp=%d clusters=%d #%d", K, SR, SC, CL, RP, ncl, idx++);
+        vs.push_back({nm, [=] { cudaLaunchKernelEx(&cfg, k, (const uint32_t *)a, b, n, (uint64_t)1, (uint32_t)(n / 32)); }});
+    };
+    add_kp(kplane_kernel<2, 4, 2, 1, 64>, 2, 4, 2, 1, 64);
+    add_kp(kplane_kernel<2, 8, 1, 1, 64>, 2, 8, 1, 1, 64);
+    add_kp(kplane_kernel<2, 12, 1, 1, 64>, 2, 12, 1, 1, 64);
+    add_kp(kplane_kernel<2, 6, 1, 1, 64>, 2, 6, 1, 1, 64);
+    add_kp(kplane_kernel<2, 4, 2, 1, 32>, 2, 4, 2, 1, 32);
+    add_kp(kplane_kernel<2, 12, 1, 1, 32>, 2, 12, 1, 1, 32);
+    add_kp(kplane_kernel<2, 2, 2, 4, 64>, 2, 2, 2, 4, 64);
+    add_kp(kplane_kernel<2, 4, 1, 4, 64>, 2, 4, 1, 4, 64);
+    add_kp(kplane_kernel<2, 4, 2, 2, 32>, 2, 4, 2, 2, 32);
+    add_kp(kplane_kernel<4, 4, 1, 1, 32>, 4, 4, 1, 1, 32);
+    add_kp(kplane_kernel<4, 6, 1, 1, 32>, 4, 6, 1, 1, 32);
+    add_kp(kplane_kernel<4, 2, 2, 1, 32>, 4, 2, 2, 1, 32);
+    add_kp(kplane_kernel<4, 3, 1, 1, 64>, 4, 3, 1, 1, 64);
     add_cluster(clu_kernel<4, 2, 4>, 4, 2, 4);
-    add_cluster(clu_kernel<4, 2, 8>, 4, 2, 8);
-    add_cluster(clu_kernel<8, 2, 2>, 8, 2, 2);
+    add_cluster(clu_kernel<4, 2, 4, 0, 2>, 4, 2, 4);
+    add_cluster(clu_kernel<4, 2, 4, 0, 4>, 4, 2, 4);
+    add_cluster(clu_kernel<4, 2, 4, 0, 8>, 4, 2, 4);
+    add_cluster(clu_kernel<4, 2, 4, 0, 16>, 4, 2, 4);
+    add_cluster(clu_kernel<4, 2, 4, 1>, 4, 2, 4);
+    add_cluster(clu_kernel<4, 2, 4, 2>, 4, 2, 4);
+    add_cluster(clu_kernel<4, 2, 4, 3>, 4, 2, 4);
+    add_cluster(clu_kernel<4, 2, 4, 4>, 4, 2, 4);
+    add_cluster(clu_kernel<4, 4, 4>, 4, 4, 4);
+    add_cluster(clu_kernel<4, 4, 4, 0, 4>, 4, 4, 4);
+    add_cluster(clu_kernel<2, 4, 4>, 2, 4, 4);
+    add_cluster(clu_kernel<2, 4, 8>, 2, 4, 8);
     auto add_ws = [&](auto k, int SR, int SC) {
         const size_t smem = (size_t)2 * SR * SC * 8192;
         CK(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
