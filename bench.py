@@ -38,6 +38,27 @@ SCH = ["raw", "ras", "rap"]
 NVLINK_GBS = 770.0   # measured peer copy per direction (B200_PROFILING.md); 900 nominal
 
 
+# The JSON line goes to the process's original stdout; everything else that native code prints
+# on fd 1 (NCCL's "NCCL version" banner, NCCL_DEBUG=INFO lines) is sent to stderr, so rank 0's
+# stdout carries exactly one line.
+_JSON_OUT = None
+
+
+def emit(line: dict):
+    global _JSON_OUT
+    out = _JSON_OUT if _JSON_OUT is not None else sys.stdout
+    out.write(json.dumps(line) + "\n")
+    out.flush()
+
+
+def route_native_stdout_to_stderr():
+    global _JSON_OUT
+    if _JSON_OUT is None:
+        sys.stdout.flush()
+        _JSON_OUT = os.fdopen(os.dup(1), "w")
+        os.dup2(2, 1)
+
+
 def parse():
     p = argparse.ArgumentParser()
     p.add_argument("--gpus", type=int, default=1)
@@ -128,6 +149,44 @@ class Clocks:
                        "samples": len(sm), "window": "timed steps + 0.3 s of identical untimed steps each side"}
 
 
+# ---------------------------------------------------------------------------- workload config
+DESC = {"default": "cfg3 8192x8192 float32 RAP transpose + cfg2 w=32 sweep batch",
+        "cfg4": "cfg4 16384x16384 float64 RAP transpose (two 32-bit RAP planes)",
+        "tile": "cfg1 32x32 float32 RAP tile (latency case)",
+        "layouts": "cfg3 8192x8192 float32 transpose under 5 smem layouts",
+        "dist": "cfg5 32768x32768 float32 row-block-sharded transpose over {world} GPU(s), NCCL all-to-all",
+        "dist_fused": "cfg5 32768x32768 float32 row-block-sharded transpose over {world} GPU(s), "
+                      "fused: tiles stored straight into peer shards (symmetric memory)",
+        "sweep": "cfg2 w=32 congestion sweep, 5 patterns x RAW/RAS/RAP",
+        "trace": "congestion of 4096 synthetic warp traces (row / column / diagonal / "
+                 "anti-diagonal / permutation / random) under RAW, RAS, RAP, PAD, XOR"}
+
+
+def arm_config(args, world: int) -> dict:
+    """The `config` object of the JSON line for args.workload -- one definition for both arms."""
+    wl = args.workload
+    if wl == "sweep":
+        return {"workload": DESC[wl], "trials_per_step": args.sweep_trials * world,
+                "parallelism": f"trial ranges x{world} + NCCL all-reduce" if world > 1 else "single GPU"}
+    if wl == "trace":
+        return {"workload": DESC[wl], "trials_per_step": args.trace_trials, "warps": 4096, "schemes": 5}
+    n = {"cfg4": 16384, "tile": 32, "dist": 32768, "dist_fused": 32768}.get(wl, 8192)
+    eb = 8 if wl == "cfg4" else 4
+    lay = "rap" if wl in ("layouts", "cfg4") else args.layout
+    rows_rank = n // world if wl in ("dist", "dist_fused") else n
+    nbytes = 2 * rows_rank * n * eb
+    cfg = {"workload": DESC[wl].format(world=world), "rows": n, "cols": n, "elem_bytes": eb, "layout": lay,
+           "parallelism": (f"row blocks + NCCL all-to-all, {world} ranks" if wl == "dist"
+                           else f"row blocks + NVLink peer stores, {world} ranks" if wl == "dist_fused"
+                           else f"replicas x{world}" if world > 1 else "single GPU"),
+           "l2": ("inputs larger than L2 (no flush)" if nbytes // 2 > 126e6
+                  else "input fits in L2 (no flush; latency case)"),
+           "algorithmic_bytes_per_step_per_rank": nbytes}
+    if wl == "default":
+        cfg["sweep_trials_per_step"] = args.sweep_trials * world
+    return cfg
+
+
 # ---------------------------------------------------------------------------- reference arm
 def run_reference(args):
     """The CPU oracle, as it stands, on the host cores, on a bounded sample of the workload."""
@@ -139,35 +198,67 @@ def run_reference(args):
     import oracle
     import workloads
     threads = oracle.max_threads()
-    if args.workload == "sweep":
-        n = 20000
-        unit, what = "trials/s", f"{n} trials of the w=32 sweep (5 patterns x RAW/RAS/RAP) per step"
-        fn = lambda k: oracle.sweep(32, ALL_PAT, SCH, 1, k * n, n, threads=threads)
-        work, cfg = n, {"workload": "cfg2 w=32 congestion sweep (oracle sample)"}
+    wl = args.workload
+    cfg = arm_config(args, world)          # the same workload / config as our arm's line
+    n_sw = 20000                           # oracle sweep sample: trials per step
+
+    def sweep_sample(k):
+        oracle.sweep(32, ALL_PAT, SCH, 1, k * n_sw, n_sw, threads=threads)
+
+    sweep_s = 0.0
+    if wl == "sweep":
+        unit, what = "trials/s", f"{n_sw} trials of the w=32 sweep (5 patterns x RAW/RAS/RAP) per step"
+        fn, work = sweep_sample, n_sw
+    elif wl == "trace":
+        # the oracle's direct DMM congestion (O8) per (trace warp, trial, scheme), as the parity
+        # test computes it: 64 of the 4096 trace warps x 4 trials x 5 schemes per step
+        cells = workloads.trace_cells(4096, 32, seed=0).numpy()[:64]
+        SCH5 = ["raw", "ras", "rap", "pad", "xor"]
+
+        def fn(k):
+            for n in range(4 * k, 4 * k + 4):
+                P, r = oracle.perm(1, n, 32), oracle.ras_shifts(1, n, 32)
+                for cw in cells:
+                    for s in SCH5:
+                        oracle.congestion(32, cw // 32, cw % 32, oracle.SCHEMES[s], {"ras": r, "rap": P}.get(s))
+        unit, work = "warp-evaluations/s", 64 * 4 * 5
+        what = "64 of the 4096 trace warps x 4 trials x 5 schemes per step, oracle congestion (O8) one by one"
     else:
         rows, cols, dt = {"cfg4": (16384, 16384, torch.float64), "dist": (32768, 32768, torch.float32),
-                          "tile": (32, 32, torch.float32)}.get(args.workload, (8192, 8192, torch.float32))
+                          "dist_fused": (32768, 32768, torch.float32),
+                          "tile": (32, 32, torch.float32)}.get(wl, (8192, 8192, torch.float32))
         band = min(rows, 512)
         x = workloads.as_bits_numpy(workloads.random_bits(band, cols, dt, seed=0))
         unit = "GB/s"
         what = f"{band} x {cols} row band of the {rows}x{cols} {str(dt)[6:]} matrix per step, naive oracle transpose"
-        fn = lambda k: oracle.transpose(x, threads=threads)
+        if wl == "default":
+            what += f"; plus {n_sw} oracle sweep trials per step, timed apart (`sweep`)"
         work = 2 * x.nbytes / 1e9
-        cfg = {"workload": f"{rows}x{cols} {str(dt)[6:]} transpose (oracle sample)", "rows": rows, "cols": cols}
+
+        def fn(k):
+            nonlocal sweep_s
+            oracle.transpose(x, threads=threads)
+            if wl == "default":                  # the step's second half, timed apart like our arm's
+                t = time.perf_counter()
+                sweep_sample(k)
+                sweep_s += time.perf_counter() - t
     for k in range(args.warmup):
         fn(k)
+    sweep_s = 0.0
     t0 = time.perf_counter()
     for k in range(args.steps):
         fn(args.warmup + k)
     el = time.perf_counter() - t0
-    value = work * args.steps / el
+    value = work * args.steps / (el - sweep_s)
     line = {"impl": "reference", "metric": METRIC, "value": value, "unit": unit, "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": el / args.steps * 1e3,
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
-            "dtype": "u64" if args.workload == "cfg4" else "u32", "data": "synthetic", "config": cfg,
+            "higher_is_better": True, "scaling": "strong" if wl in ("dist", "dist_fused") else "weak",
+            "vs_baseline": None, "dtype": "u64" if wl == "cfg4" else "u32", "data": "synthetic", "config": cfg,
             "cpu_baseline": {"value": value, "unit": unit, "cores": threads, "kind": "oracle", "sample": what},
             "e2e": {"value": value, "unit": unit, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
-    print(json.dumps(line), flush=True)
+    if wl == "default":
+        line["sweep"] = {"trials_per_s": n_sw * args.steps / sweep_s, "trials_per_step": n_sw}
+    emit(line)
 
 
 # ---------------------------------------------------------------------------- helpers
@@ -252,6 +343,7 @@ def reduce_over_ranks(x: float, world: int, dev, op: str) -> float:
 # ---------------------------------------------------------------------------- our arm
 def main():
     args = parse()
+    route_native_stdout_to_stderr()
     if args.impl == "reference":
         return run_reference(args)
     import numpy as np
@@ -421,23 +513,8 @@ def main():
         gbs = nbytes * world * args.steps / (r["t_sum"] * 1e-3) / 1e9
         kern_ms = statistics.median(r["t_ms"])
         line.update(value=gbs, unit="GB/s")
-        desc = {"default": "cfg3 8192x8192 float32 RAP transpose + cfg2 w=32 sweep batch",
-                "cfg4": "cfg4 16384x16384 float64 RAP transpose (two 32-bit RAP planes)",
-                "tile": "cfg1 32x32 float32 RAP tile (latency case)",
-                "layouts": "cfg3 8192x8192 float32 transpose under 5 smem layouts",
-                "dist": f"cfg5 32768x32768 float32 row-block-sharded transpose over {world} GPU(s), NCCL all-to-all",
-                "dist_fused": f"cfg5 32768x32768 float32 row-block-sharded transpose over {world} GPU(s), "
-                              "fused: tiles stored straight into peer shards (symmetric memory)"}[wl]
-        line["config"] = {"workload": desc, "rows": rows * (world if dist_wl else 1), "cols": cols,
-                          "elem_bytes": eb, "layout": lay,
-                          "parallelism": (f"row blocks + NCCL all-to-all, {world} ranks" if wl == "dist"
-                                          else f"row blocks + NVLink peer stores, {world} ranks" if wl == "dist_fused"
-                                          else f"replicas x{world}" if world > 1 else "single GPU"),
-                          "l2": ("inputs larger than L2 (no flush)" if nbytes // 2 > 126e6
-                                 else "input fits in L2 (no flush; latency case)"),
-                          "algorithmic_bytes_per_step_per_rank": nbytes}
-        if do_s:
-            line["config"]["sweep_trials_per_step"] = S * world
+        line["config"] = arm_config(args, world)
+        assert line["config"]["layout"] == lay and line["config"]["algorithmic_bytes_per_step_per_rank"] == nbytes
         kkey = f"transpose_b{eb * 8}_{lay}"
         prof = load_profile(kkey) or {}
         if dist_wl and world > 1:
@@ -464,9 +541,7 @@ def main():
         th = trace_hist.cpu().numpy()
         c = np.arange(33)
         line.update(value=evs, unit="warp-evaluations/s",
-                    config={"workload": "congestion of 4096 synthetic warp traces (row / column / diagonal / "
-                                        "anti-diagonal / permutation / random) under RAW, RAS, RAP, PAD, XOR",
-                            "trials_per_step": TT, "warps": 4096, "schemes": 5})
+                    config=arm_config(args, world))
         line["trace"] = {"E_by_scheme": {n: float((th[i] * c).sum() / th[i].sum())
                                          for i, n in enumerate(["raw", "ras", "rap", "pad", "xor"])},
                          "kernel_ms_median": statistics.median(r["s_ms"])}
@@ -485,10 +560,7 @@ def main():
                          "roofline": sweep_roofline(tps / world, r["clocks"])}
         if not do_t:
             line.update(value=tps, unit="trials/s",
-                        config={"workload": "cfg2 w=32 congestion sweep, 5 patterns x RAW/RAS/RAP",
-                                "trials_per_step": S * world,
-                                "parallelism": (f"trial ranges x{world} + NCCL all-reduce" if world > 1
-                                                else "single GPU")})
+                        config=arm_config(args, world))
             line["roofline"] = sweep_roofline(tps / world, r["clocks"])
     if do_t and do_s:
         t_share = r["t_sum"] / max(r["t_sum"] + r["s_sum"], 1e-9)
@@ -619,7 +691,7 @@ def main():
         if do_s and do_t:
             line["sweep"]["cpu_baseline"] = cpu_baseline_sweep()
     if rank == 0:
-        print(json.dumps(line), flush=True)
+        emit(line)
     if dist.is_initialized():
         dist.destroy_process_group()
 
