@@ -15,7 +15,9 @@
  * Conventions (all entry points):
  *   - Ownership: the caller owns every buffer.  Pointers named d_* (and src/dst of
  *     rap_transpose) are DEVICE pointers on the current CUDA device.  The library keeps no
- *     allocation and no mutable global state; calls are thread-safe.
+ *     memory allocation and no shared mutable state; calls are thread-safe.  (Cached per
+ *     kernel: the launch shape; per calling thread and device: rap_transpose_host's three
+ *     streams and their events, created on first use and destroyed at thread exit.)
  *   - Asynchrony: device work is enqueued on `stream` (a cudaStream_t passed as void*;
  *     NULL = the legacy default stream) and returns immediately; results are valid once
  *     the stream is synchronised.
@@ -134,7 +136,8 @@ rap_status_t rap_transpose(const void *src, void *dst, int64_t rows, int64_t col
 /* T1-T3 from and to HOST memory (the end-to-end call): dst = src^T as rap_transpose, but src
  * and dst are HOST pointers (pinned memory lets the copies overlap).  The matrix moves in row
  * bands of a multiple of 32 rows: upload of band b+1, transpose of band b and 2-D download of
- * band b-1 run concurrently on three internal streams (PCIe in both directions at once).
+ * band b-1 run concurrently on three internal streams (PCIe in both directions at once); band
+ * heights ramp up at the start and down at the end so the pipeline fills and drains quickly.
  * d_workspace: caller-owned DEVICE buffer of workspace_bytes; it holds 4 band buffers, so it must
  * fit at least 4 * 32 * cols * elem_bytes bytes (larger = fewer, longer bands).  The call is
  * SYNCHRONOUS: work queued on `stream` before the call completes first, and dst is valid on
