@@ -57,12 +57,16 @@ size_t host_band_rows(int64_t rows, int64_t cols, uint32_t eb, size_t work_bytes
     return rb < cap ? rb : cap;
 }
 
-// Band heights for `rows` rows with full bands of rb rows: a doubling ramp from rb/16 (at least
+// Band heights for `rows` rows with full bands of rb rows: a doubling ramp from rb/4 (at least
 // 32 rows) up to rb at the head, full bands in the middle, the mirrored ramp at the tail.
+#ifndef RAP_HOST_RAMP_DIV
+#define RAP_HOST_RAMP_DIV 4    // smallest ramp band = rb / RAP_HOST_RAMP_DIV (0: no ramp); narrower bands
+                               // make the strided download slow (256 B of each 32 KiB row: 32 GB/s)
+#endif
 static std::vector<int64_t> band_plan(int64_t rows, int64_t rb) {
     std::vector<int64_t> head;
     int64_t ramp = 0;
-    const int64_t s0 = rb / 16 / 32 * 32;
+    const int64_t s0 = RAP_HOST_RAMP_DIV ? rb / RAP_HOST_RAMP_DIV / 32 * 32 : rb;
     for (int64_t s = s0 < 32 ? 32 : s0; s < rb; s *= 2) {
         head.push_back(s);
         ramp += s;

@@ -43,6 +43,15 @@ for width in (256, 512, 1024, 2048, 4096, 8192, 32768):
     a, b = t_of(d2h), t_of(h2d)
     print(f"width {width:6d} B x {h:7d} rows: D2H 2-D {N / a / 1e9:5.1f} GB/s, H2D 2-D {N / b / 1e9:5.1f} GB/s", flush=True)
 
+# the band download's real shape: 4 KiB of each 32 KiB output row (cfg3, 1024-row bands)
+for width, pitch in ((4096, 32768), (2048, 32768), (256, 32768), (8192, 65536)):
+    h = N // pitch
+
+    def d2h():
+        assert rt.cudaMemcpy2DAsync(host_big.data_ptr(), pitch, dev.data_ptr(), width, width, h, 2, None) == 0
+    a = t_of(d2h)
+    print(f"D2H 2-D width {width} B, host pitch {pitch} B: {width * h / a / 1e9:5.1f} GB/s", flush=True)
+
 x = torch.zeros((64, 64), dtype=torch.float32).pin_memory()
 y = torch.empty((64, 64), dtype=torch.float32).pin_memory()
 t = t_of(lambda: rap.transpose_host(x, out=y), reps=50)
