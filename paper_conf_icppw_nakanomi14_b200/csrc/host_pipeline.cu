@@ -6,7 +6,7 @@
 //
 // Two device buffers per direction (double buffering) live in the caller's workspace; events
 // order the three streams, so band b+1 is uploading while band b is transposed and band b-1 is
-// downloading.  Band heights ramp geometrically (RB/16, RB/8, .. RB) at the start and back down
+// downloading.  Band heights ramp (RB/4, RB/2, then RB) at the start and back down
 // at the end, so the pipeline fills (first upload) and drains (last download) on small bands
 // while the middle runs in full-size bands.  The call is synchronous: it returns once dst holds the result.  Host buffers
 // should be pinned (page-locked) for the copies to overlap; pageable memory still works.

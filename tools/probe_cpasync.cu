@@ -351,6 +351,110 @@ kplane_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, int6
     }
 }
 
+
+// Memory-level-parallelism variants of the cluster kernel: MINB CTAs per SM (register budget),
+// DEPTH tiles of loads in flight per warp (1 or 2 register buffers), RP = 64 unwrapped / 32
+// wrapped RAP rows (half the shared memory per warp).
+template <int SR, int SC, int CL, int MINB, int DEPTH, int RP>
+__global__ void __launch_bounds__(SR * SC * 32, MINB)
+mlp_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, int64_t n, uint64_t seed,
+           uint32_t tiles) {
+    extern __shared__ __align__(16) uint32_t sm[];
+    const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
+    uint32_t *tile = sm + warp * 32 * RP;
+    const uint32_t P = rapk::warp_perm<32>(seed, 0, lane, 32);
+    tile[P] = lane;
+    __syncwarp();
+    const uint32_t pinv = tile[lane];
+    __syncwarp();
+    const uint32_t q = lane & 7u, c_in = lane >> 3;
+    uint32_t row_g[8], a_g[8];
+#pragma unroll
+    for (int g = 0; g < 8; ++g) {
+        const uint32_t rr = 4 * g + c_in;
+        row_g[g] = __shfl_sync(0xffffffffu, pinv, rr);
+        a_g[g] = RP == 64 ? row_g[g] * 64 + 4 * q + rr : row_g[g] * 32;
+    }
+    uint32_t crank = 0, cid = blockIdx.x, ncl = gridDim.x;
+    if (CL > 1) {
+        asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(crank));
+        asm volatile("mov.u32 %0, %%clusterid.x;" : "=r"(cid));
+        asm volatile("mov.u32 %0, %%nclusterid.x;" : "=r"(ncl));
+    }
+    const uint32_t stc = tiles / SC, nst = (tiles / (SR * CL)) * stc;
+    const uint32_t wr = crank * SR + warp % SR, wc = warp / SR;
+    auto load = [&](uint4 (&v)[8], uint32_t st) {
+        const uint32_t si = st / stc, sj = st - si * stc;
+        const int64_t r0 = (int64_t)(si * SR * CL + wr) * 32, c0 = (int64_t)(sj * SC + wc) * 32;
+        const uint32_t *base = src + r0 * n + c0 + 4 * q;
+#pragma unroll
+        for (int g = 0; g < 8; ++g) v[g] = rapk::ldg_stream128(base + (int64_t)row_g[g] * n);
+    };
+    auto store = [&](const uint4 (&v)[8]) {
+#pragma unroll
+        for (int g = 0; g < 8; ++g) {
+            const uint32_t w4[4] = {v[g].x, v[g].y, v[g].z, v[g].w};
+#pragma unroll
+            for (int e = 0; e < 4; ++e)
+                tile[RP == 64 ? a_g[g] + e : a_g[g] + ((4 * q + e + 4 * g + c_in) & 31u)] = w4[e];
+        }
+    };
+    auto sync = [&]() {
+        if (CL > 1) {
+            asm volatile("barrier.cluster.arrive.relaxed.aligned;" ::: "memory");
+            asm volatile("barrier.cluster.wait.aligned;" ::: "memory");
+        } else if (SR * SC > 1) {
+            __syncthreads();
+        }
+    };
+    auto drain = [&](uint32_t cst) {
+        const uint32_t si = cst / stc, sj = cst - si * stc;
+        const int64_t r0 = (int64_t)(si * SR * CL + wr) * 32, c0 = (int64_t)(sj * SC + wc) * 32;
+        uint32_t *o = dst + c0 * n + r0 + lane;
+#pragma unroll
+        for (int c = 0; c < 32; ++c) {
+            *o = tile[RP == 64 ? lane * 64 + P + c : lane * 32 + ((P + c) & 31u)];
+            o += n;
+        }
+    };
+    uint32_t st = cid;
+    if (DEPTH == 1) {
+        uint4 v[8];
+        if (st < nst) load(v, st);
+        while (st < nst) {
+            const uint32_t cst = st;
+            store(v);
+            __syncwarp();
+            st += ncl;
+            if (st < nst) load(v, st);
+            sync();
+            drain(cst);
+            __syncwarp();
+        }
+    } else {
+        uint4 va[8], vb[8];
+        if (st < nst) load(va, st);
+        if (st + ncl < nst) load(vb, st + ncl);
+        while (st < nst) {
+            store(va);
+            __syncwarp();
+            if (st + 2 * ncl < nst) load(va, st + 2 * ncl);
+            sync();
+            drain(st);
+            __syncwarp();
+            st += ncl;
+            if (st >= nst) break;
+            store(vb);
+            __syncwarp();
+            if (st + 2 * ncl < nst) load(vb, st + 2 * ncl);
+            sync();
+            drain(st);
+            __syncwarp();
+            st += ncl;
+        }
+    }
+}
+
 // Warp-specialised variant: T = SR*SC producer warps (LDG.128 -> STS.32 into the RAP tile, the
 // next tile's loads in flight while waiting for a free stage) and T consumer warps (lockstep drain
 // of the super-tile: LDS column reads + 128 B STG rows), two super-tile stages in shared memory,
@@ -548,32 +652,35 @@ int main(int argc, char **argv) {
         char nm[128]; snprintf(nm, sizeof nm, "kplane K=%d sr=%d sc=%d cl=%d rp=%d clusters=%d #%d", K, SR, SC, CL, RP, ncl, idx++);
         vs.push_back({nm, [=] { cudaLaunchKernelEx(&cfg, k, (const uint32_t *)a, b, n, (uint64_t)1, (uint32_t)(n / 32)); }});
     };
-    add_kp(kplane_kernel<2, 4, 2, 1, 64>, 2, 4, 2, 1, 64);
-    add_kp(kplane_kernel<2, 8, 1, 1, 64>, 2, 8, 1, 1, 64);
-    add_kp(kplane_kernel<2, 12, 1, 1, 64>, 2, 12, 1, 1, 64);
-    add_kp(kplane_kernel<2, 6, 1, 1, 64>, 2, 6, 1, 1, 64);
-    add_kp(kplane_kernel<2, 4, 2, 1, 32>, 2, 4, 2, 1, 32);
-    add_kp(kplane_kernel<2, 12, 1, 1, 32>, 2, 12, 1, 1, 32);
-    add_kp(kplane_kernel<2, 2, 2, 4, 64>, 2, 2, 2, 4, 64);
-    add_kp(kplane_kernel<2, 4, 1, 4, 64>, 2, 4, 1, 4, 64);
-    add_kp(kplane_kernel<2, 4, 2, 2, 32>, 2, 4, 2, 2, 32);
-    add_kp(kplane_kernel<4, 4, 1, 1, 32>, 4, 4, 1, 1, 32);
-    add_kp(kplane_kernel<4, 6, 1, 1, 32>, 4, 6, 1, 1, 32);
-    add_kp(kplane_kernel<4, 2, 2, 1, 32>, 4, 2, 2, 1, 32);
-    add_kp(kplane_kernel<4, 3, 1, 1, 64>, 4, 3, 1, 1, 64);
-    add_cluster(clu_kernel<4, 2, 4>, 4, 2, 4);
-    add_cluster(clu_kernel<4, 2, 4, 0, 2>, 4, 2, 4);
-    add_cluster(clu_kernel<4, 2, 4, 0, 4>, 4, 2, 4);
-    add_cluster(clu_kernel<4, 2, 4, 0, 8>, 4, 2, 4);
-    add_cluster(clu_kernel<4, 2, 4, 0, 16>, 4, 2, 4);
-    add_cluster(clu_kernel<4, 2, 4, 1>, 4, 2, 4);
-    add_cluster(clu_kernel<4, 2, 4, 2>, 4, 2, 4);
-    add_cluster(clu_kernel<4, 2, 4, 3>, 4, 2, 4);
-    add_cluster(clu_kernel<4, 2, 4, 4>, 4, 2, 4);
-    add_cluster(clu_kernel<4, 4, 4>, 4, 4, 4);
-    add_cluster(clu_kernel<4, 4, 4, 0, 4>, 4, 4, 4);
-    add_cluster(clu_kernel<2, 4, 4>, 2, 4, 4);
-    add_cluster(clu_kernel<2, 4, 8>, 2, 4, 8);
+    auto add_mlp = [&](auto k, int SR, int SC, int CL, int MINB, int DEPTH, int RP) {
+        const size_t smem = (size_t)SR * SC * 32 * RP * 4;
+        CK(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        if (CL > 1) CK(cudaFuncSetAttribute(k, cudaFuncAttributeNonPortableClusterSizeAllowed, 1));
+        cudaLaunchConfig_t cfg = {};
+        static cudaLaunchAttribute at[64][1];
+        static int nat = 0;
+        cudaLaunchAttribute *ap = at[nat++];
+        ap[0].id = cudaLaunchAttributeClusterDimension;
+        ap[0].val.clusterDim.x = CL; ap[0].val.clusterDim.y = 1; ap[0].val.clusterDim.z = 1;
+        cfg.blockDim = dim3(SR * SC * 32); cfg.dynamicSmemBytes = smem; cfg.attrs = ap; cfg.numAttrs = 1;
+        int ncl = 0;
+        cfg.gridDim = dim3(148 * CL);
+        CK(cudaOccupancyMaxActiveClusters(&ncl, k, &cfg));
+        const uint32_t nst = (uint32_t)((n / 32 / (SR * CL)) * (n / 32 / SC));
+        cfg.gridDim = dim3(std::min<uint32_t>(nst, (uint32_t)ncl) * CL);
+        cudaFuncAttributes fa; cudaFuncGetAttributes(&fa, k);
+        char nm[160]; snprintf(nm, sizeof nm, "mlp sr=%d sc=%d cl=%d minb=%d depth=%d rp=%d regs=%d clusters=%d", SR, SC, CL, MINB, DEPTH, RP, fa.numRegs, ncl);
+        vs.push_back({nm, [=] { cudaLaunchKernelEx(&cfg, k, (const uint32_t *)a, b, n, (uint64_t)1, (uint32_t)(n / 32)); }});
+    };
+    add_mlp(mlp_kernel<4, 2, 4, 2, 1, 64>, 4, 2, 4, 2, 1, 64);
+    add_mlp(mlp_kernel<4, 2, 4, 3, 1, 64>, 4, 2, 4, 3, 1, 64);
+    add_mlp(mlp_kernel<4, 2, 4, 2, 2, 64>, 4, 2, 4, 2, 2, 64);
+    add_mlp(mlp_kernel<4, 2, 2, 3, 1, 64>, 4, 2, 2, 3, 1, 64);
+    add_mlp(mlp_kernel<2, 2, 8, 6, 1, 64>, 2, 2, 8, 6, 1, 64);
+    add_mlp(mlp_kernel<2, 4, 4, 3, 1, 64>, 2, 4, 4, 3, 1, 64);
+    add_mlp(mlp_kernel<2, 2, 4, 4, 2, 64>, 2, 2, 4, 4, 2, 64);
+    add_mlp(mlp_kernel<8, 2, 1, 1, 2, 64>, 8, 2, 1, 1, 2, 64);
+    add_mlp(mlp_kernel<4, 4, 4, 1, 2, 64>, 4, 4, 4, 1, 2, 64);
     auto add_ws = [&](auto k, int SR, int SC) {
         const size_t smem = (size_t)2 * SR * SC * 8192;
         CK(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
