@@ -59,7 +59,7 @@ def route_native_stdout_to_stderr():
         os.dup2(2, 1)
 
 
-def parse():
+def parse(argv=None):
     p = argparse.ArgumentParser()
     p.add_argument("--gpus", type=int, default=1)
     p.add_argument("--steps", type=int, default=50)
@@ -74,12 +74,13 @@ def parse():
     # measures the steady rate, 4 batches per warp give 2.88 G/s, 10^9 trials 3.09 G/s.
     p.add_argument("--sweep-trials", type=int, default=148 * 8 * 4 * 32)
     # --workload trace: each of the 4096 trace warps evaluated under this many trials per step
-    p.add_argument("--trace-trials", type=int, default=256)
+    # (2048: a 0.6 ms launch, past the launch ramp; 256 trials run at ~80 % of that rate)
+    p.add_argument("--trace-trials", type=int, default=2048)
     p.add_argument("--sweep-algo", default="default", choices=["default", "match"])
     p.add_argument("--layout", default="rap")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu", action="store_true")
-    return p.parse_args()
+    return p.parse_args(argv)
 
 
 def dist_env():
@@ -210,19 +211,8 @@ def run_reference(args):
         unit, what = "trials/s", f"{n_sw} trials of the w=32 sweep (5 patterns x RAW/RAS/RAP) per step"
         fn, work = sweep_sample, n_sw
     elif wl == "trace":
-        # the oracle's direct DMM congestion (O8) per (trace warp, trial, scheme), as the parity
-        # test computes it: 64 of the 4096 trace warps x 4 trials x 5 schemes per step
-        cells = workloads.trace_cells(4096, 32, seed=0).numpy()[:64]
-        SCH5 = ["raw", "ras", "rap", "pad", "xor"]
-
-        def fn(k):
-            for n in range(4 * k, 4 * k + 4):
-                P, r = oracle.perm(1, n, 32), oracle.ras_shifts(1, n, 32)
-                for cw in cells:
-                    for s in SCH5:
-                        oracle.congestion(32, cw // 32, cw % 32, oracle.SCHEMES[s], {"ras": r, "rap": P}.get(s))
-        unit, work = "warp-evaluations/s", 64 * 4 * 5
-        what = "64 of the 4096 trace warps x 4 trials x 5 schemes per step, oracle congestion (O8) one by one"
+        fn, work, what = oracle_trace_sample()
+        unit = "warp-evaluations/s"
     else:
         rows, cols, dt = {"cfg4": (16384, 16384, torch.float64), "dist": (32768, 32768, torch.float32),
                           "dist_fused": (32768, 32768, torch.float32),
@@ -254,7 +244,8 @@ def run_reference(args):
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": el / args.steps * 1e3,
             "higher_is_better": True, "scaling": "strong" if wl in ("dist", "dist_fused") else "weak",
             "vs_baseline": None, "dtype": "u64" if wl == "cfg4" else "u32", "data": "synthetic", "config": cfg,
-            "cpu_baseline": {"value": value, "unit": unit, "cores": threads, "kind": "oracle", "sample": what},
+            "cpu_baseline": {"value": value, "unit": unit, "cores": 1 if wl == "trace" else threads, "kind": "oracle",
+                             "sample": what},
             "e2e": {"value": value, "unit": unit, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     if wl == "default":
         line["sweep"] = {"trials_per_s": n_sw * args.steps / sweep_s, "trials_per_step": n_sw}
@@ -277,6 +268,36 @@ def cpu_baseline_transpose(rows, cols, dt):
     return {"value": 2 * x.nbytes * reps / el / 1e9, "unit": "GB/s", "cores": threads, "kind": "oracle",
             "sample": f"{band} x {cols} row band of the {rows}x{cols} matrix, naive oracle transpose, "
                       f"{reps} reps in {el:.1f} s"}
+
+
+def oracle_trace_sample():
+    """(fn(k), evaluations per call, description): the oracle's direct DMM congestion (O8) per
+    (trace warp, trial, scheme), as the parity test computes it -- 64 of the 4096 trace warps x
+    4 trials x 5 schemes per call."""
+    import oracle
+    import workloads
+    cells = workloads.trace_cells(4096, 32, seed=0).numpy()[:64]
+    sch5 = ["raw", "ras", "rap", "pad", "xor"]
+
+    def fn(k):
+        for n in range(4 * k, 4 * k + 4):
+            P, r = oracle.perm(1, n, 32), oracle.ras_shifts(1, n, 32)
+            for cw in cells:
+                for s in sch5:
+                    oracle.congestion(32, cw // 32, cw % 32, oracle.SCHEMES[s], {"ras": r, "rap": P}.get(s))
+    return fn, 64 * 4 * 5, "64 of the 4096 trace warps x 4 trials x 5 schemes per call, oracle congestion (O8) one by one"
+
+
+def cpu_baseline_trace():
+    fn, work, what = oracle_trace_sample()
+    fn(0)
+    reps, t0 = 0, time.perf_counter()
+    while time.perf_counter() - t0 < 3.0:
+        fn(reps)
+        reps += 1
+    el = time.perf_counter() - t0
+    return {"value": work * reps / el, "unit": "warp-evaluations/s", "cores": 1, "kind": "oracle",
+            "sample": f"{what}; {reps} calls in {el:.1f} s (single thread: one ctypes call per evaluation)"}
 
 
 def cpu_baseline_sweep():
@@ -544,7 +565,11 @@ def main():
                     config=arm_config(args, world))
         line["trace"] = {"E_by_scheme": {n: float((th[i] * c).sum() / th[i].sum())
                                          for i, n in enumerate(["raw", "ras", "rap", "pad", "xor"])},
-                         "kernel_ms_median": statistics.median(r["s_ms"])}
+                         "kernel_ms_median": statistics.median(r["s_ms"]),
+                         # RAW / PAD / XOR use no random numbers: the kernel evaluates them once per
+                         # (trace warp, block of 32 trials) and counts the result for every trial;
+                         # the per-trial Monte-Carlo work is the RAS and RAP evaluations
+                         "ras_rap_evaluations_per_s": evs * 2 / 5}
         line["roofline"] = trace_roofline(evs / world, r["clocks"])
     elif do_s:
         tps = S * world * args.steps / (r["s_sum"] * 1e-3)
@@ -687,7 +712,8 @@ def main():
                        "d2h_bytes_per_step": hh.numel() * 8, "ms_per_step": ms, "steps": K,
                        "note": "sweep batch through the public API + D2H of the histogram (inputs are counters)"}
     if rank == 0 and not args.no_cpu and world == 1:
-        line["cpu_baseline"] = cpu_baseline_transpose(rows, cols, dt) if do_t else cpu_baseline_sweep()
+        line["cpu_baseline"] = (cpu_baseline_transpose(rows, cols, dt) if do_t
+                                else cpu_baseline_trace() if wl == "trace" else cpu_baseline_sweep())
         if do_s and do_t:
             line["sweep"]["cpu_baseline"] = cpu_baseline_sweep()
     if rank == 0:

@@ -694,6 +694,99 @@ trace_kernel(uint32_t w_rt, uint64_t n_warps, const uint32_t *__restrict__ cells
     flush_hist(sh_hist, kSweepWarps, nbins, hist);
 }
 
+
+// w = 32 trace evaluator.  Work unit = (block of kTraceTB trials, range of kTraceTK trace warps).
+// The CTA first draws P and r of its kTraceTB trials into shared memory (one warp Fisher-Yates
+// per trial), then each warp takes trace warps of the range and, per trace warp:
+//   * decodes the 32 cells and finds the merged-request leaders ONCE (one __match_any_sync);
+//   * evaluates the trial-invariant schemes RAW / PAD / XOR once and counts the result for every
+//     trial of the block (their bank maps use no random numbers);
+//   * for each trial of the block evaluates RAS / RAP: the shift of the lane's row is one LDS.U8
+//     (P_t[row] -- lanes of equal rows share a word, so one wavefront), bank = col + shift (the
+//     ballots read bits 0..4 only, which is the "mod 32"), 5 ballots, popc, reduce-max.
+// Histograms live in registers: lane L of the warp counts congestion L+1 for each scheme, flushed
+// with one u64 atomic per non-zero counter at the end.
+#ifndef RAP_TRACE_TB
+#define RAP_TRACE_TB 32
+#endif
+#ifndef RAP_TRACE_TK
+#define RAP_TRACE_TK 64
+#endif
+#ifndef RAP_TRACE_WARPS
+#define RAP_TRACE_WARPS 8
+#endif
+constexpr int kTraceTB = RAP_TRACE_TB;     // trials per unit (P, r of the block in shared memory)
+constexpr int kTraceTK = RAP_TRACE_TK;     // trace warps per unit
+constexpr int kTraceWarps = RAP_TRACE_WARPS;
+
+#ifndef RAP_TRACE32_MINB
+#define RAP_TRACE32_MINB 4
+#endif
+
+template <uint32_t SM>
+__global__ void __launch_bounds__(kTraceWarps * 32, RAP_TRACE32_MINB)
+trace32_kernel(uint64_t n_warps, const uint32_t *__restrict__ cells, uint64_t seed, uint64_t first,
+               uint64_t n_trials, uint64_t *__restrict__ hist) {
+    constexpr uint32_t nsch = __builtin_popcount(SM);
+    constexpr bool need_p = (SM >> RAP_SCHEME_RAP) & 1u, need_r = (SM >> RAP_SCHEME_RAS) & 1u;
+    __shared__ uint8_t shP[kTraceTB][32], shR[kTraceTB][32];
+    const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
+    const LaneSel ls(lane);
+    const uint32_t lt_mask = (1u << lane) - 1u;
+    uint32_t hc[nsch];                                      // lane L: count of congestion L + 1
+#pragma unroll
+    for (uint32_t e = 0; e < nsch; ++e) hc[e] = 0;
+    uint32_t hbad = 0;                                      // evaluations of warps with a bad cell
+    const uint64_t nkc = (n_warps + kTraceTK - 1) / kTraceTK;
+    const uint64_t ntb = (n_trials + kTraceTB - 1) / kTraceTB;
+    for (uint64_t unit = blockIdx.x; unit < ntb * nkc; unit += gridDim.x) {
+        const uint64_t tb = unit / nkc, kc = unit - tb * nkc;
+        const uint64_t t0 = tb * kTraceTB;
+        const uint32_t tcnt = (uint32_t)min((uint64_t)kTraceTB, n_trials - t0);
+        __syncthreads();                                    // the previous unit is done with shP / shR
+        for (uint32_t t = warp; t < tcnt; t += kTraceWarps) {
+            if (need_p) shP[t][lane] = (uint8_t)warp_perm<32>(seed, first + t0 + t, lane, 32);
+            if (need_r) shR[t][lane] = (uint8_t)warp_ras_shift(seed, first + t0 + t, lane, 32);
+        }
+        __syncthreads();
+        const uint64_t k_end = min(n_warps, (kc + 1) * kTraceTK);
+        for (uint64_t k = kc * kTraceTK + warp; k < k_end; k += kTraceWarps) {
+            const uint32_t raw_cell = __ldg(cells + k * 32 + lane);
+            if (__any_sync(kFull, raw_cell >= 1024u)) {     // invalid trace warp: bin 0
+                hbad += tcnt;
+                continue;
+            }
+            const uint32_t row = raw_cell >> 5, col = raw_cell & 31u;
+            // merged requests: the first lane of each distinct cell is counted
+            const uint32_t same = __match_any_sync(kFull, raw_cell);
+            const uint32_t leaders = ballot_zero(same, lt_mask);
+            uint32_t e = 0;
+#pragma unroll
+            for (int s = 0; s < 5; ++s) {
+                if (!((SM >> s) & 1u)) continue;
+                if (s == RAP_SCHEME_RAW || s == RAP_SCHEME_PAD || s == RAP_SCHEME_XOR) {
+                    const uint32_t bank = s == RAP_SCHEME_RAW ? col : s == RAP_SCHEME_PAD ? row + col : (col ^ row);
+                    const uint32_t c = max_bank_load(bank, leaders, ls);
+                    hc[e] += (c == lane + 1u) ? tcnt : 0u;
+                } else {
+                    const uint8_t *sh = s == RAP_SCHEME_RAP ? &shP[0][0] : &shR[0][0];
+#pragma unroll 4
+                    for (uint32_t t = 0; t < tcnt; ++t) {
+                        const uint32_t c = max_bank_load(col + sh[t * 32 + row], leaders, ls);
+                        hc[e] += (c == lane + 1u) ? 1u : 0u;
+                    }
+                }
+                ++e;
+            }
+        }
+    }
+#pragma unroll
+    for (uint32_t e = 0; e < nsch; ++e) {
+        if (hc[e]) atomicAdd((unsigned long long *)(hist + e * 33 + lane + 1), (unsigned long long)hc[e]);
+        if (lane == 0 && hbad) atomicAdd((unsigned long long *)(hist + e * 33), (unsigned long long)hbad);
+    }
+}
+
 // ------------------------------------------------------------------ batched evaluator
 __global__ void __launch_bounds__(256)
 congestion_kernel(uint32_t w, uint64_t n_warps, const uint32_t *__restrict__ rows,
@@ -797,17 +890,49 @@ cudaError_t launch_sweep_match(uint32_t w, uint32_t pmask, uint32_t smask, uint6
     return cudaGetLastError();
 }
 
+template <uint32_t SM>
+static void run_trace32(uint64_t n_warps, const uint32_t *cells, uint64_t seed, uint64_t first, uint64_t n_trials,
+                        uint64_t *hist, cudaStream_t st) {
+    const int threads = kTraceWarps * 32;
+    const uint64_t nkc = (n_warps + kTraceTK - 1) / kTraceTK;
+    const int cap = resident_ctas<trace32_kernel<SM>>(threads);
+    // per-lane u32 counters: a warp evaluates at most ceil(units / grid) units of
+    // (kTraceTK / kTraceWarps) trace warps x kTraceTB trials per launch -- keep that below 2^31
+    const uint64_t per_unit = (uint64_t)(kTraceTK / kTraceWarps) * kTraceTB;
+    const uint64_t max_units = (1ull << 31) / per_unit;     // per CTA per launch
+    const uint64_t tb_chunk = max_units * (uint64_t)cap / nkc + 1;  // trial blocks per launch
+    const uint64_t trials_chunk = tb_chunk * kTraceTB;
+    for (uint64_t done = 0; done < n_trials; done += trials_chunk) {
+        const uint64_t cnt = (n_trials - done < trials_chunk) ? n_trials - done : trials_chunk;
+        const uint64_t units = ((cnt + kTraceTB - 1) / kTraceTB) * nkc;
+        const int grid = (int)(units < (uint64_t)cap ? units : (uint64_t)cap);
+        trace32_kernel<SM><<<grid, threads, 0, st>>>(n_warps, cells, seed, first + done, cnt, hist);
+    }
+}
+
 cudaError_t launch_trace(uint32_t w, uint64_t n_warps, const uint32_t *cells, uint32_t smask,
                          uint64_t seed, uint64_t first, uint64_t n_trials, uint64_t *hist,
                          cudaStream_t st) {
     if (n_trials == 0 || n_warps == 0) return cudaSuccess;
+    if (w == 32) {
+#define RAPK_TRACE32(M) case M: run_trace32<M>(n_warps, cells, seed, first, n_trials, hist, st); break;
+        switch (smask) {
+            RAPK_TRACE32(1) RAPK_TRACE32(2) RAPK_TRACE32(3) RAPK_TRACE32(4) RAPK_TRACE32(5) RAPK_TRACE32(6)
+            RAPK_TRACE32(7) RAPK_TRACE32(8) RAPK_TRACE32(9) RAPK_TRACE32(10) RAPK_TRACE32(11) RAPK_TRACE32(12)
+            RAPK_TRACE32(13) RAPK_TRACE32(14) RAPK_TRACE32(15) RAPK_TRACE32(16) RAPK_TRACE32(17) RAPK_TRACE32(18)
+            RAPK_TRACE32(19) RAPK_TRACE32(20) RAPK_TRACE32(21) RAPK_TRACE32(22) RAPK_TRACE32(23) RAPK_TRACE32(24)
+            RAPK_TRACE32(25) RAPK_TRACE32(26) RAPK_TRACE32(27) RAPK_TRACE32(28) RAPK_TRACE32(29) RAPK_TRACE32(30)
+            RAPK_TRACE32(31)
+            default: return cudaErrorInvalidValue;
+        }
+#undef RAPK_TRACE32
+        return cudaGetLastError();
+    }
+    // 2 <= w < 32: the generic evaluator, one warp per (trial, chunk of 32 trace warps)
     const int threads = kSweepWarps * 32;
     const uint64_t nchunks = (n_warps + kTraceChunk - 1) / kTraceChunk;
-    auto kern = (w == 32 && smask == 31u) ? trace_kernel<32, 31u>
-              : (w == 32 && smask == 7u) ? trace_kernel<32, 7u> : (w == 32) ? trace_kernel<32, 0u> : trace_kernel<0, 0u>;
-    const int occ = (w == 32 && smask == 31u) ? resident_ctas<trace_kernel<32, 31u>>(threads)
-                  : (w == 32 && smask == 7u) ? resident_ctas<trace_kernel<32, 7u>>(threads)
-                  : (w == 32) ? resident_ctas<trace_kernel<32, 0u>>(threads) : resident_ctas<trace_kernel<0, 0u>>(threads);
+    auto kern = trace_kernel<0, 0u>;
+    const int occ = resident_ctas<trace_kernel<0, 0u>>(threads);
     const int grid = clamp_grid(n_trials * nchunks, kSweepWarps, occ);
     // counts per warp <= items_per_warp * kTraceChunk; chunk the trial range to stay < 2^31
     const uint64_t trials_chunk = ((uint64_t)grid * kSweepWarps * ((1ull << 31) / kTraceChunk)) / nchunks + 1;

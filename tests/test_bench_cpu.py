@@ -3,7 +3,6 @@
 The driver runs `bench.py --impl reference` beside our arm and divides the two `value`s, so the
 reference line must carry the same metric, unit and config as our arm's line for that workload.
 """
-import argparse
 import json
 import os
 import subprocess
@@ -26,7 +25,7 @@ def _run(*argv, env=None):
 
 
 def _args(workload):
-    return argparse.Namespace(workload=workload, sweep_trials=148 * 8 * 4 * 32, trace_trials=256, layout="rap")
+    return bench.parse(["--workload", workload])
 
 
 @pytest.mark.parametrize("workload,unit", [("default", "GB/s"), ("sweep", "trials/s"),

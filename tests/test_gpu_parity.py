@@ -327,6 +327,50 @@ def test_trace_matches_oracle(rap, oracle):
     assert np.array_equal(g.cpu().numpy().astype(np.uint64), expect)
 
 
+def _trace_oracle(oracle, cl, seed, first, n_trials, schemes, w=32):
+    """Histogram of the oracle's direct DMM congestion (O8) per (trial, trace warp, scheme); a
+    trace warp with a cell >= w*w counts in bin 0."""
+    expect = np.zeros((len(schemes), w + 1), dtype=np.uint64)
+    for n in range(first, first + n_trials):
+        P, r = oracle.perm(seed, n, w), oracle.ras_shifts(seed, n, w)
+        for k in range(cl.shape[0]):
+            if (cl[k] >= w * w).any():
+                expect[:, 0] += 1
+                continue
+            rows, cols = cl[k] // w, cl[k] % w
+            for si, s in enumerate(schemes):
+                expect[si, oracle.congestion(w, rows, cols, oracle.SCHEMES[s], {"ras": r, "rap": P}.get(s))] += 1
+    return expect
+
+
+@pytest.mark.parametrize("schemes", [["ras"], ["rap", "xor"], ["pad"], ["raw", "ras", "rap"], ALL_SCH])
+def test_trace_w32_masks_ragged_invalid(rap, oracle, schemes):
+    # ragged against the kernel's units (64 trace warps x 32 trials), a bad cell, every mask shape
+    w, n_trials, first = 32, 70, 12345
+    cells = workloads.trace_cells(131, w, seed=8)
+    cells[77, 5] = w * w + 3
+    g = rap.congestion_trace(cells.cuda(), n_trials, seed=9, schemes=schemes, first_trial=first)
+    expect = _trace_oracle(oracle, cells.numpy(), 9, first, n_trials, schemes)
+    assert np.array_equal(g.cpu().numpy().astype(np.uint64), expect)
+    assert (g[:, 0] == n_trials).all()
+
+
+def test_trace_bench_size_sampled_and_additive(rap, oracle):
+    # the bench workload (4096 trace warps x 256 trials, five schemes): a 48-warp sample of it
+    # against the oracle one by one, and additivity over trial ranges at full size
+    cells = workloads.trace_cells(4096, 32, seed=0)
+    rng = np.random.default_rng(5)
+    pick = np.sort(rng.choice(4096, 48, replace=False))
+    sub = cells[pick].contiguous()
+    g = rap.congestion_trace(sub.cuda(), 256, seed=1, schemes=ALL_SCH)
+    assert np.array_equal(g.cpu().numpy().astype(np.uint64), _trace_oracle(oracle, sub.numpy(), 1, 0, 256, ALL_SCH))
+    cd = cells.cuda()
+    full = rap.congestion_trace(cd, 256, seed=1, schemes=ALL_SCH)
+    parts = rap.congestion_trace(cd, 100, seed=1, schemes=ALL_SCH)
+    rap.congestion_trace(cd, 156, seed=1, schemes=ALL_SCH, first_trial=100, out=parts)
+    assert torch.equal(full, parts) and (full.sum(-1) == 4096 * 256).all()
+
+
 def test_trace_small_w_and_invalid(rap, oracle):
     w = 8
     cells = workloads.trace_cells(13, w, seed=1)

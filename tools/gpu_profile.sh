@@ -31,7 +31,7 @@ timeout 600 ncu --set full --import-source on --clock-control none -k regex:"swe
     -o "$OUT/prof_sweep" -f $B --workload sweep --steps 1 --warmup 2 --sweep-trials 8388608 > "$OUT/ncu_sweep.log" 2>&1
 timeout 600 ncu --set full --import-source on --clock-control none -k regex:"sweep_match_kernel" -s 2 -c 1 \
     -o "$OUT/prof_sweep_match" -f $B --workload sweep --sweep-algo match --steps 1 --warmup 2 --sweep-trials 4194304 > "$OUT/ncu_sweep_match.log" 2>&1
-# trace evaluator: 4096 warps x 296 trials x 5 schemes per launch
-timeout 600 ncu --set full --import-source on --clock-control none -k regex:"trace_kernel" -s 2 -c 1 \
-    -o "$OUT/prof_trace" -f $B --workload trace --steps 1 --warmup 2 --trace-trials 296 > "$OUT/ncu_trace.log" 2>&1
+# trace evaluator: 4096 warps x 2048 trials x 5 schemes per launch
+timeout 600 ncu --set full --import-source on --clock-control none -k regex:"trace(32)?_kernel" -s 2 -c 1 \
+    -o "$OUT/prof_trace" -f $B --workload trace --steps 1 --warmup 2 --trace-trials 2048 > "$OUT/ncu_trace.log" 2>&1
 ls -la "$OUT"

@@ -21,7 +21,7 @@ CAPTURES = {
 
 # work units per captured launch (tools/gpu_profile.sh command lines)
 UNITS = {"sweep_w32": ("trials", 8388608), "sweep_w32_match": ("trials", 4194304),
-         "trace_w32": ("evaluations", 4096 * 296 * 5),
+         "trace_w32": ("evaluations", 4096 * 2048 * 5),
          "transpose_b32_rap": ("bytes", 2 * 8192 * 8192 * 4), "transpose_b32_raw": ("bytes", 2 * 8192 * 8192 * 4),
          "transpose_b32_pad": ("bytes", 2 * 8192 * 8192 * 4), "transpose_b32_xor": ("bytes", 2 * 8192 * 8192 * 4),
          "transpose_b32_ras": ("bytes", 2 * 8192 * 8192 * 4), "transpose_b64_rap": ("bytes", 2 * 16384 * 16384 * 8),
