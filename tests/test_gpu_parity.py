@@ -118,6 +118,29 @@ def test_transpose_cfg3_8192_f32(rap, oracle, layout):
     assert torch.equal(z.view(torch.int32), x.view(torch.int32))
 
 
+def test_transpose_beyond_2pow32_elements(rap, oracle):
+    # 65600 x 65600 fp32 = 4.3e9 elements (17.2 GB each way): every element offset needs 64 bits;
+    # ragged in both dimensions (65600 = 2050 tiles, not a multiple of the 16 x 2 cluster super-tile)
+    n = 65600
+    x = workloads.random_bits(n, n, torch.float32, seed=21, device="cuda")
+    y = rap.transpose(x, layout="rap", seed=4)
+    torch.cuda.synchronize()
+    _band_check(oracle, x, y, n_bands=2, band=33, seed=3)
+    for c0 in (0, 40000, n - 17):
+        assert np.array_equal(bits(y[c0:c0 + 17]), oracle.transpose(bits(x[:, c0:c0 + 17]))), c0
+    z = rap.transpose(y, layout="rap", seed=5)
+    assert torch.equal(z.view(torch.int32), x.view(torch.int32))
+
+
+@pytest.mark.parametrize("shape", [((1 << 27) + 5, 3), (3, (1 << 27) + 5), ((1 << 22) + 1, 33)])
+def test_transpose_extreme_aspect(rap, oracle, shape):
+    # tall / wide extremes: one partial tile column or row over millions of tiles
+    x = workloads.random_bits(*shape, torch.float64, seed=22, device="cuda")
+    y = rap.transpose(x, layout="rap", seed=6)
+    torch.cuda.synchronize()
+    assert np.array_equal(bits(y), oracle.transpose(bits(x), threads=oracle.max_threads()))
+
+
 def test_transpose_cfg4_16384_f64(rap, oracle):
     x = workloads.random_bits(16384, 16384, torch.float64, seed=0, device="cuda")
     y = rap.transpose(x, layout="rap", seed=0)
