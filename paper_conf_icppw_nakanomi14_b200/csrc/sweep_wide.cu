@@ -136,15 +136,182 @@ sweep_wide_kernel(uint32_t w, uint32_t pmask, uint32_t smask, uint64_t seed, uin
         if (sh_hist[b]) atomicAdd((unsigned long long *)(hist + b), (unsigned long long)sh_hist[b]);
 }
 
+// ---------------------------------------------------------------- one CUDA warp per trial
+// The default for 32 < w <= 256.  A warp simulates one DMM warp of w threads: lane L plays DMM
+// threads t = L + 32 i (i < NI = ceil(w / 32)).  Per trial, in the warp's shared-memory slice:
+//   * Philox words are drawn in parallel (lane L: blocks L, L + 32 of each domain); the FY draws
+//     become j_t = floor(u_t (w - t) / 2^32) in jv[], the RAS shifts r[], the random cells stay in
+//     registers;
+//   * Durstenfeld on a[] is one sequential chain (lane 0; k = w-1 .. 1: swap a[k], a[jv[w-1-k]]);
+//   * merged requests: slice by slice, a request leads if it is the lowest lane of
+//     its cell in the slice (__match_any_sync) and the cell's bit in a w*w-bit bitmap is not yet
+//     set by an earlier slice; the bits are cleared again afterwards (O(w) per trial);
+//   * each (pattern, scheme): every lane adds its requests to the per-bank counters cnt[] with
+//     shared atomics -- congestion = max over requests of the returned count + 1 (= max over
+//     banks), reduce-max over the warp -- then zeroes the counters it touched.
+constexpr int kWideWarps = 8;
+#ifndef RAP_WIDE_MINB
+#define RAP_WIDE_MINB 4
+#endif
+
+struct WideSlice {           // per-warp shared-memory slice, in 32-bit words
+    uint32_t *a, *r, *jv, *cnt, *bm;
+};
+
+__host__ __device__ inline uint32_t wide_warp_words(uint32_t w) {
+    return 4 * w + (w * w + 31) / 32;
+}
+
+template <int NI>
+__global__ void __launch_bounds__(kWideWarps * 32, RAP_WIDE_MINB)
+sweep_wide_warp_kernel(uint32_t w, uint32_t pmask, uint32_t smask, uint64_t seed, uint64_t first,
+                       uint64_t n_trials, uint64_t *__restrict__ hist) {
+    extern __shared__ __align__(16) uint32_t dyn[];
+    const uint32_t npat = __popc(pmask), nsch = __popc(smask);
+    const uint32_t nbins = npat * nsch * (w + 1);
+    const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
+    uint32_t *sh_hist = dyn;
+    uint32_t *mine = dyn + ((nbins + 3) & ~3u) + warp * wide_warp_words(w);
+    WideSlice S{mine, mine + w, mine + 2 * w, mine + 3 * w, mine + 4 * w};
+    for (uint32_t b = threadIdx.x; b < nbins; b += blockDim.x) sh_hist[b] = 0;
+    for (uint32_t b = lane; b < 4 * w + (w * w + 31) / 32; b += 32) mine[b] = 0;
+    __syncthreads();
+    const bool any_random = (pmask >> RAP_PAT_RANDOM) & 1u;
+    const bool need_r = (smask >> RAP_SCHEME_RAS) & 1u;
+    const uint32_t nblk = (w + 3) / 4;                      // Philox blocks per domain
+
+    const uint64_t stride = (uint64_t)gridDim.x * kWideWarps;
+    for (uint64_t i = (uint64_t)blockIdx.x * kWideWarps + warp; i < n_trials; i += stride) {
+        const uint64_t n = first + i;
+        // ---- C1: draws, lanes in parallel
+        uint32_t cellv[NI];
+#pragma unroll
+        for (int q = 0; q < NI; ++q) cellv[q] = 0;
+        for (uint32_t blk = lane; blk < nblk; blk += 32) {
+            const uint4 f = philox_block(seed, n, kDomainFY, blk);
+            const uint32_t fw[4] = {f.x, f.y, f.z, f.w};
+#pragma unroll
+            for (int c = 0; c < 4; ++c) {
+                const uint32_t t = 4 * blk + c;               // FY word t -> k = w - 1 - t
+                if (t + 1 < w) S.jv[t] = mulshift(fw[c], w - t);
+            }
+            if (need_r) {
+                const uint4 g = philox_block(seed, n, kDomainRAS, blk);
+                const uint32_t gw[4] = {g.x, g.y, g.z, g.w};
+#pragma unroll
+                for (int c = 0; c < 4; ++c)
+                    if (4 * blk + c < w) S.r[4 * blk + c] = mulshift(gw[c], w);
+            }
+        }
+        if (any_random) {
+#pragma unroll
+            for (int q = 0; q < NI; ++q) {
+                const uint32_t t = lane + 32u * q;
+                if (t < w) cellv[q] = mulshift(pick(philox_block(seed, n, kDomainRandom, t >> 2), t & 3u), w * w);
+            }
+        }
+#pragma unroll
+        for (int q = 0; q < NI; ++q) {
+            const uint32_t t = lane + 32u * q;
+            if (t < w) S.a[t] = t;
+        }
+        __syncwarp();
+        // ---- C2: Durstenfeld, one sequential chain
+        if (lane == 0) {
+            for (uint32_t k = w - 1; k >= 1; --k) {
+                const uint32_t j = S.jv[w - 1 - k];
+                const uint32_t x = S.a[k];
+                S.a[k] = S.a[j];
+                S.a[j] = x;
+            }
+        }
+        // ---- merged requests of the random pattern
+        uint32_t lead = 0;                                    // bit q: request lane + 32q counts
+        if (any_random) {
+#pragma unroll
+            for (int q = 0; q < NI; ++q) {
+                const uint32_t t = lane + 32u * q;
+                const bool valid = t < w;
+                const uint32_t c = cellv[q];
+                const uint32_t same = __match_any_sync(kFull, valid ? c : (0x80000000u | lane));
+                const bool first_in_slice = (__ffs(same) - 1) == (int)lane;
+                const bool seen = valid && ((S.bm[c >> 5] >> (c & 31u)) & 1u);
+                if (valid && first_in_slice && !seen) lead |= 1u << q;
+                __syncwarp();
+                if (valid) atomicOr(&S.bm[c >> 5], 1u << (c & 31u));
+                __syncwarp();
+            }
+#pragma unroll
+            for (int q = 0; q < NI; ++q)
+                if (lane + 32u * q < w) S.bm[cellv[q] >> 5] = 0u;
+        }
+        __syncwarp();
+        // ---- C3 + C4: every selected (pattern, scheme)
+        uint32_t e = 0;
+        for (int p = 0; p < 5; ++p) {
+            if (!((pmask >> p) & 1u)) continue;
+            for (int s = 0; s < 5; ++s) {
+                if (!((smask >> s) & 1u)) continue;
+                int pp = p;                                   // reading iii: malicious
+                if (p == RAP_PAT_MALICIOUS)
+                    pp = (s == RAP_SCHEME_RAW || s == RAP_SCHEME_RAS) ? RAP_PAT_STRIDE
+                       : (s == RAP_SCHEME_PAD) ? -1 : RAP_PAT_DIAGONAL;
+                uint32_t bankv[NI];
+                uint32_t mx = 0;
+#pragma unroll
+                for (int q = 0; q < NI; ++q) {
+                    const uint32_t t = lane + 32u * q;
+                    bankv[q] = 0xffffffffu;
+                    if (t >= w) continue;
+                    if (pp == RAP_PAT_RANDOM && !((lead >> q) & 1u)) continue;      // merged
+                    uint32_t row, col;
+                    switch (pp) {
+                    case RAP_PAT_CONTIGUOUS: row = 0; col = t; break;
+                    case RAP_PAT_STRIDE: row = t; col = 0; break;
+                    case RAP_PAT_DIAGONAL: row = t; col = t; break;
+                    case RAP_PAT_RANDOM: row = cellv[q] / w; col = cellv[q] - row * w; break;
+                    default: row = t; col = t == 0 ? 0u : w - t; break;               // PAD anti-diagonal
+                    }
+                    uint32_t bank;
+                    if (s == RAP_SCHEME_RAS || s == RAP_SCHEME_RAP) {
+                        bank = col + (s == RAP_SCHEME_RAP ? S.a[row] : S.r[row]);
+                        bank = bank >= w ? bank - w : bank;
+                    } else if (s == RAP_SCHEME_PAD) {
+                        bank = row + col;
+                        bank = bank >= w ? bank - w : bank;
+                    } else if (s == RAP_SCHEME_XOR) {
+                        bank = col ^ row;
+                    } else {
+                        bank = col;
+                    }
+                    bankv[q] = bank;
+                    const uint32_t v = atomicAdd(&S.cnt[bank], 1u) + 1u;
+                    mx = v > mx ? v : mx;
+                }
+                mx = __reduce_max_sync(kFull, mx);
+                __syncwarp();
+#pragma unroll
+                for (int q = 0; q < NI; ++q)
+                    if (bankv[q] != 0xffffffffu) S.cnt[bankv[q]] = 0u;
+                if (lane == 0) atomicAdd(&sh_hist[e * (w + 1) + mx], 1u);
+                __syncwarp();
+                ++e;
+            }
+        }
+    }
+    __syncthreads();
+    for (uint32_t b = threadIdx.x; b < nbins; b += blockDim.x)
+        if (sh_hist[b]) atomicAdd((unsigned long long *)(hist + b), (unsigned long long)sh_hist[b]);
+}
+
 size_t wide_smem_bytes(uint32_t w, uint32_t pmask, uint32_t smask) {
     const uint32_t nbins = __builtin_popcount(pmask) * __builtin_popcount(smask) * (w + 1);
     return 4 * (size_t)((nbins + 3) & ~3u) + 2 * (size_t)4 * w * kWideThreads +
            4 * (size_t)((w + 31) / 32) * kWideThreads;
 }
 
-cudaError_t launch_sweep_wide(uint32_t w, uint32_t pmask, uint32_t smask, uint64_t seed, uint64_t first,
-                              uint64_t n_trials, uint64_t *hist, cudaStream_t st) {
-    if (n_trials == 0) return cudaSuccess;
+static cudaError_t launch_sweep_wide_thread(uint32_t w, uint32_t pmask, uint32_t smask, uint64_t seed,
+                                            uint64_t first, uint64_t n_trials, uint64_t *hist, cudaStream_t st) {
     const size_t smem = wide_smem_bytes(w, pmask, smask);
     cudaError_t e = cudaFuncSetAttribute(sweep_wide_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
@@ -163,6 +330,50 @@ cudaError_t launch_sweep_wide(uint32_t w, uint32_t pmask, uint32_t smask, uint64
         sweep_wide_kernel<<<grid, kWideThreads, smem, st>>>(w, pmask, smask, seed, first + done, cnt, hist);
     }
     return cudaGetLastError();
+}
+
+template <int NI>
+static cudaError_t launch_wide_warp(uint32_t w, uint32_t pmask, uint32_t smask, uint64_t seed, uint64_t first,
+                                    uint64_t n_trials, uint64_t *hist, cudaStream_t st) {
+    const uint32_t nbins = __builtin_popcount(pmask) * __builtin_popcount(smask) * (w + 1);
+    const size_t smem = 4 * ((size_t)((nbins + 3) & ~3u) + (size_t)kWideWarps * wide_warp_words(w));
+    auto k = sweep_wide_warp_kernel<NI>;
+    cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    int dev = 0, sms = 148, occ = 1;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, kWideWarps * 32, smem);
+    if (occ < 1) occ = 1;
+    const uint64_t want = (n_trials + kWideWarps - 1) / kWideWarps;
+    const uint64_t cap = (uint64_t)sms * occ;
+    const int grid = (int)(want < cap ? want : cap);
+    const uint64_t chunk = (uint64_t)grid * (1ull << 31);    // u32 CTA counters stay below 2^31
+    for (uint64_t done = 0; done < n_trials; done += chunk) {
+        const uint64_t cnt = (n_trials - done < chunk) ? n_trials - done : chunk;
+        k<<<grid, kWideWarps * 32, smem, st>>>(w, pmask, smask, seed, first + done, cnt, hist);
+    }
+    return cudaGetLastError();
+}
+
+// RAP_SWEEP_WIDE_THREAD: the one-trial-per-thread kernel above (the round-1 design, an ablation)
+cudaError_t launch_sweep_wide(uint32_t w, uint32_t pmask, uint32_t smask, uint64_t seed, uint64_t first,
+                              uint64_t n_trials, uint64_t *hist, cudaStream_t st) {
+    if (n_trials == 0) return cudaSuccess;
+#ifdef RAP_SWEEP_WIDE_THREAD
+    return launch_sweep_wide_thread(w, pmask, smask, seed, first, n_trials, hist, st);
+#else
+    switch ((w + 31) / 32) {
+    case 2: return launch_wide_warp<2>(w, pmask, smask, seed, first, n_trials, hist, st);
+    case 3: return launch_wide_warp<3>(w, pmask, smask, seed, first, n_trials, hist, st);
+    case 4: return launch_wide_warp<4>(w, pmask, smask, seed, first, n_trials, hist, st);
+    case 5: return launch_wide_warp<5>(w, pmask, smask, seed, first, n_trials, hist, st);
+    case 6: return launch_wide_warp<6>(w, pmask, smask, seed, first, n_trials, hist, st);
+    case 7: return launch_wide_warp<7>(w, pmask, smask, seed, first, n_trials, hist, st);
+    case 8: return launch_wide_warp<8>(w, pmask, smask, seed, first, n_trials, hist, st);
+    default: return launch_sweep_wide_thread(w, pmask, smask, seed, first, n_trials, hist, st);
+    }
+#endif
 }
 
 }  // namespace rapk
