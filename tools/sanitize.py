@@ -33,10 +33,15 @@ rap.congestion_sweep(5000, seed=1)
 rap.congestion_sweep(5000, seed=1, schemes=("raw", "ras", "rap", "pad", "xor"))
 rap.congestion_sweep(3000, seed=1, w=7, schemes=("raw", "ras", "rap", "pad"))
 rap.congestion_sweep(300, seed=1, w=64)
+rap.congestion_sweep(200, seed=1, w=100, schemes=("raw", "ras", "rap", "pad"))
+rap.congestion_sweep(100, seed=1, w=256, schemes=("raw", "ras", "rap", "pad", "xor"))
 rap.congestion_sweep(2000, seed=1, algo="match")
 rap.congestion_sweep4(2000, seed=1, w=16)
 cells = workloads.trace_cells(20, 32, seed=1).to(dev)
 rap.congestion_trace(cells, 10, seed=1, schemes=("raw", "ras", "rap", "pad", "xor"))
+cells2 = workloads.trace_cells(131, 32, seed=2)
+cells2[7, 3] = 5000                                   # invalid trace warp -> bin 0
+rap.congestion_trace(cells2.to(dev), 70, seed=1, schemes=("ras", "xor"), first_trial=33)
 t = lambda a: torch.from_numpy(np.asarray(a, dtype=np.int32)).to(dev)
 rr = np.random.default_rng(0).integers(0, 32, (50, 32))
 rap.congestion(t(rr), t(rr[::-1].copy()), "rap", shift=t(np.stack([np.random.default_rng(k).permutation(32) for k in range(50)])))
