@@ -490,39 +490,53 @@ def main():
             if do_s:
                 step_sweep(k)
         torch.cuda.synchronize()
-        hist.zero_()
-        launches, ev = 0, []
-        barrier()
-        torch.cuda.synchronize()
-        with Clocks(dev.index) as clk:
-            # the sampler runs over the timed steps and ~0.3 s of identical untimed steps on
-            # each side, so every clock sample is taken under this workload
-            soak(lay, 0.3)
-            torch.cuda.synchronize()
+        first_clocks = None
+        for attempt in range(2):
+            hist.zero_()
+            launches, ev = 0, []
             barrier()
-            start = torch.cuda.Event(enable_timing=True)
-            end = torch.cuda.Event(enable_timing=True)
-            start.record(stream)
-            for k in range(args.steps):
-                e = [torch.cuda.Event(enable_timing=True) for _ in range(4)]
-                e[0].record(stream)
-                if do_t:
-                    launches += step_transpose(lay)
-                e[1].record(stream)
-                e[2].record(stream)
-                if do_s:
-                    launches += step_sweep(k)
-                e[3].record(stream)
-                ev.append(e)
-            end.record(stream)
             torch.cuda.synchronize()
-            barrier()
-            soak(lay, 0.3)
-            torch.cuda.synchronize()
-        t_ms = [e[0].elapsed_time(e[1]) for e in ev]
-        s_ms = [e[2].elapsed_time(e[3]) for e in ev]
-        results[lay] = dict(total_ms=rmax(start.elapsed_time(end)), t_sum=rmax(sum(t_ms)), t_ms=t_ms,
-                            s_sum=rmax(sum(s_ms)), s_ms=s_ms, clocks=clk.result, launches=launches)
+            with Clocks(dev.index) as clk:
+                # the sampler runs over the timed steps and ~0.3 s of identical untimed steps on
+                # each side, so every clock sample is taken under this workload
+                soak(lay, 0.3)
+                torch.cuda.synchronize()
+                barrier()
+                start = torch.cuda.Event(enable_timing=True)
+                end = torch.cuda.Event(enable_timing=True)
+                start.record(stream)
+                for k in range(args.steps):
+                    e = [torch.cuda.Event(enable_timing=True) for _ in range(4)]
+                    e[0].record(stream)
+                    if do_t:
+                        launches += step_transpose(lay)
+                    e[1].record(stream)
+                    e[2].record(stream)
+                    if do_s:
+                        launches += step_sweep(k)
+                    e[3].record(stream)
+                    ev.append(e)
+                end.record(stream)
+                torch.cuda.synchronize()
+                barrier()
+                soak(lay, 0.3)
+                torch.cuda.synchronize()
+            t_ms = [e[0].elapsed_time(e[1]) for e in ev]
+            s_ms = [e[2].elapsed_time(e[3]) for e in ev]
+            results[lay] = dict(total_ms=rmax(start.elapsed_time(end)), t_sum=rmax(sum(t_ms)), t_ms=t_ms,
+                                s_sum=rmax(sum(s_ms)), s_ms=s_ms, clocks=clk.result, launches=launches)
+            # a timed region that saw thermal / hardware slowdown, or SM clocks well below max with
+            # no reason given, is measured once more (every rank agrees through the max)
+            c = clk.result
+            bad = bool(set(c.get("reasons") or []) & {"hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown"})
+            bad = bad or bool(c.get("sm_mhz") and c.get("sm_max_mhz") and not c.get("reasons")
+                              and c["sm_mhz"] < 0.85 * c["sm_max_mhz"])
+            if attempt == 0 and rmax(1.0 if bad else 0.0) > 0:
+                first_clocks = c
+                continue
+            if first_clocks is not None:
+                results[lay]["clocks"] = dict(c, remeasured=True, first_attempt=first_clocks)
+            break
 
     lay = "rap" if wl in ("layouts", "cfg4") and "rap" in results else args.layout
     r = results[lay]
