@@ -162,10 +162,11 @@ __host__ __device__ inline uint32_t wide_warp_words(uint32_t w) {
     return 4 * w + (w * w + 31) / 32;
 }
 
-template <int NI>
+template <int NI, uint32_t PM, uint32_t SM>
 __global__ void __launch_bounds__(kWideWarps * 32, RAP_WIDE_MINB)
-sweep_wide_warp_kernel(uint32_t w, uint32_t pmask, uint32_t smask, uint64_t seed, uint64_t first,
+sweep_wide_warp_kernel(uint32_t w, uint32_t pmask_rt, uint32_t smask_rt, uint64_t seed, uint64_t first,
                        uint64_t n_trials, uint64_t *__restrict__ hist) {
+    const uint32_t pmask = PM ? PM : pmask_rt, smask = SM ? SM : smask_rt;
     extern __shared__ __align__(16) uint32_t dyn[];
     const uint32_t npat = __popc(pmask), nsch = __popc(smask);
     const uint32_t nbins = npat * nsch * (w + 1);
@@ -218,15 +219,24 @@ sweep_wide_warp_kernel(uint32_t w, uint32_t pmask, uint32_t smask, uint64_t seed
         __syncwarp();
         // ---- C2: Durstenfeld, one sequential chain
         if (lane == 0) {
-            for (uint32_t k = w - 1; k >= 1; --k) {
-                const uint32_t j = S.jv[w - 1 - k];
-                const uint32_t x = S.a[k];
-                S.a[k] = S.a[j];
+            const uint32_t *jp = S.jv;
+            uint32_t *ak = S.a + (w - 1);
+#pragma unroll 4
+            for (uint32_t k = w - 1; k >= 1; --k, ++jp, --ak) {
+                const uint32_t j = *jp;
+                const uint32_t x = *ak;
+                *ak = S.a[j];
                 S.a[j] = x;
             }
         }
-        // ---- merged requests of the random pattern
+        // ---- merged requests of the random pattern; row / col of each random cell
         uint32_t lead = 0;                                    // bit q: request lane + 32q counts
+        uint32_t rrow[NI], rcol[NI];
+#pragma unroll
+        for (int q = 0; q < NI; ++q) {
+            rrow[q] = cellv[q] / w;
+            rcol[q] = cellv[q] - rrow[q] * w;
+        }
         if (any_random) {
 #pragma unroll
             for (int q = 0; q < NI; ++q) {
@@ -248,8 +258,10 @@ sweep_wide_warp_kernel(uint32_t w, uint32_t pmask, uint32_t smask, uint64_t seed
         __syncwarp();
         // ---- C3 + C4: every selected (pattern, scheme)
         uint32_t e = 0;
+#pragma unroll
         for (int p = 0; p < 5; ++p) {
             if (!((pmask >> p) & 1u)) continue;
+#pragma unroll
             for (int s = 0; s < 5; ++s) {
                 if (!((smask >> s) & 1u)) continue;
                 int pp = p;                                   // reading iii: malicious
@@ -269,7 +281,7 @@ sweep_wide_warp_kernel(uint32_t w, uint32_t pmask, uint32_t smask, uint64_t seed
                     case RAP_PAT_CONTIGUOUS: row = 0; col = t; break;
                     case RAP_PAT_STRIDE: row = t; col = 0; break;
                     case RAP_PAT_DIAGONAL: row = t; col = t; break;
-                    case RAP_PAT_RANDOM: row = cellv[q] / w; col = cellv[q] - row * w; break;
+                    case RAP_PAT_RANDOM: row = rrow[q]; col = rcol[q]; break;
                     default: row = t; col = t == 0 ? 0u : w - t; break;               // PAD anti-diagonal
                     }
                     uint32_t bank;
@@ -337,7 +349,10 @@ static cudaError_t launch_wide_warp(uint32_t w, uint32_t pmask, uint32_t smask, 
                                     uint64_t n_trials, uint64_t *hist, cudaStream_t st) {
     const uint32_t nbins = __builtin_popcount(pmask) * __builtin_popcount(smask) * (w + 1);
     const size_t smem = 4 * ((size_t)((nbins + 3) & ~3u) + (size_t)kWideWarps * wide_warp_words(w));
-    auto k = sweep_wide_warp_kernel<NI>;
+    // compile-time masks for the Table II sweeps (5 patterns x RAW/RAS/RAP, and all 5 schemes)
+    auto k = (pmask == 31u && smask == 7u) ? sweep_wide_warp_kernel<NI, 31u, 7u>
+           : (pmask == 31u && smask == 31u) ? sweep_wide_warp_kernel<NI, 31u, 31u>
+           : sweep_wide_warp_kernel<NI, 0u, 0u>;
     cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     int dev = 0, sms = 148, occ = 1;
