@@ -67,12 +67,13 @@ def parse(argv=None):
     p.add_argument("--impl", default="mine", choices=["mine", "reference"])
     p.add_argument("--workload", default="default",
                    choices=["default", "sweep", "trace", "cfg4", "tile", "layouts", "dist", "dist_fused"])
-    # default: one batch of 32 trials for every resident warp of the sweep kernel on a B200
-    # (148 SMs x 8 CTAs x 4 warps), so the cfg3 transpose stays the larger share of the step
-    # (the step's `value` and `roofline` are the transpose's).  One batch per warp runs the
-    # sweep below its steady rate (launch ramp, per-CTA histogram flush): `--workload sweep`
-    # measures the steady rate, 4 batches per warp give 2.88 G/s, 10^9 trials 3.09 G/s.
-    p.add_argument("--sweep-trials", type=int, default=148 * 8 * 4 * 32)
+    # default workload: one batch of 32 trials for every resident warp of the sweep kernel on a
+    # B200 (148 SMs x 8 CTAs x 4 warps), so the cfg3 transpose stays the larger share of the step
+    # (the step's `value` and `roofline` are the transpose's).  One batch per warp runs the sweep
+    # below its steady rate (launch ramp and tail of a single wave).  `--workload sweep` (cfg2)
+    # defaults to 64 batches per warp (9.7 M trials, ~3 ms per step): the steady rate, as the
+    # 10^9-trial cfg2 run sees it.
+    p.add_argument("--sweep-trials", type=int, default=None)
     # --workload trace: each of the 4096 trace warps evaluated under this many trials per step
     # (2048: a 0.6 ms launch, past the launch ramp; 256 trials run at ~80 % of that rate)
     p.add_argument("--trace-trials", type=int, default=2048)
@@ -80,7 +81,10 @@ def parse(argv=None):
     p.add_argument("--layout", default="rap")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu", action="store_true")
-    return p.parse_args(argv)
+    a = p.parse_args(argv)
+    if a.sweep_trials is None:
+        a.sweep_trials = 148 * 8 * 4 * 32 * (64 if a.workload == "sweep" else 1)
+    return a
 
 
 def dist_env():
