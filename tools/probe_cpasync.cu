@@ -672,15 +672,31 @@ int main(int argc, char **argv) {
         char nm[160]; snprintf(nm, sizeof nm, "mlp sr=%d sc=%d cl=%d minb=%d depth=%d rp=%d regs=%d clusters=%d", SR, SC, CL, MINB, DEPTH, RP, fa.numRegs, ncl);
         vs.push_back({nm, [=] { cudaLaunchKernelEx(&cfg, k, (const uint32_t *)a, b, n, (uint64_t)1, (uint32_t)(n / 32)); }});
     };
-    add_mlp(mlp_kernel<4, 2, 4, 2, 1, 64>, 4, 2, 4, 2, 1, 64);
-    add_mlp(mlp_kernel<4, 2, 4, 3, 1, 64>, 4, 2, 4, 3, 1, 64);
-    add_mlp(mlp_kernel<4, 2, 4, 2, 2, 64>, 4, 2, 4, 2, 2, 64);
-    add_mlp(mlp_kernel<4, 2, 2, 3, 1, 64>, 4, 2, 2, 3, 1, 64);
-    add_mlp(mlp_kernel<2, 2, 8, 6, 1, 64>, 2, 2, 8, 6, 1, 64);
-    add_mlp(mlp_kernel<2, 4, 4, 3, 1, 64>, 2, 4, 4, 3, 1, 64);
-    add_mlp(mlp_kernel<2, 2, 4, 4, 2, 64>, 2, 2, 4, 4, 2, 64);
-    add_mlp(mlp_kernel<8, 2, 1, 1, 2, 64>, 8, 2, 1, 1, 2, 64);
-    add_mlp(mlp_kernel<4, 4, 4, 1, 2, 64>, 4, 4, 4, 1, 2, 64);
+    // grid size: cluster counts that divide the 2048 cluster super-tiles evenly vs all co-resident
+    auto add_grid = [&](int want) {
+        auto k = mlp_kernel<4, 2, 4, 2, 1, 64>;
+        const size_t smem = (size_t)8 * 32 * 64 * 4;
+        CK(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        cudaLaunchConfig_t cfg = {};
+        static cudaLaunchAttribute at[16][1];
+        static int nat = 0;
+        cudaLaunchAttribute *ap = at[nat++];
+        ap[0].id = cudaLaunchAttributeClusterDimension;
+        ap[0].val.clusterDim.x = 4; ap[0].val.clusterDim.y = 1; ap[0].val.clusterDim.z = 1;
+        cfg.blockDim = dim3(256); cfg.dynamicSmemBytes = smem; cfg.attrs = ap; cfg.numAttrs = 1;
+        int ncl = 0;
+        cfg.gridDim = dim3(148 * 4);
+        CK(cudaOccupancyMaxActiveClusters(&ncl, k, &cfg));
+        const int use = want > 0 ? std::min(want, ncl) : ncl;
+        cfg.gridDim = dim3(use * 4);
+        char nm[128]; snprintf(nm, sizeof nm, "cluster 4x2x4 grid %d of %d clusters", use, ncl);
+        vs.push_back({nm, [=] { cudaLaunchKernelEx(&cfg, k, (const uint32_t *)a, b, n, (uint64_t)1, (uint32_t)(n / 32)); }});
+    };
+    add_grid(0);
+    add_grid(64);
+    add_grid(68);
+    add_grid(57);
+    add_grid(32);
     auto add_ws = [&](auto k, int SR, int SC) {
         const size_t smem = (size_t)2 * SR * SC * 8192;
         CK(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
