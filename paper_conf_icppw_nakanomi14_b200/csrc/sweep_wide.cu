@@ -150,6 +150,9 @@ sweep_wide_kernel(uint32_t w, uint32_t pmask, uint32_t smask, uint64_t seed, uin
 //     shared atomics -- congestion = max over requests of the returned count + 1 (= max over
 //     banks), reduce-max over the warp -- then zeroes the counters it touched.
 constexpr int kWideWarps = 8;
+#ifndef RAP_WIDE_LANE_FY
+#define RAP_WIDE_LANE_FY 1
+#endif
 #ifndef RAP_WIDE_MINB
 #define RAP_WIDE_MINB 4
 #endif
@@ -316,6 +319,168 @@ sweep_wide_warp_kernel(uint32_t w, uint32_t pmask_rt, uint32_t smask_rt, uint64_
         if (sh_hist[b]) atomicAdd((unsigned long long *)(hist + b), (unsigned long long)sh_hist[b]);
 }
 
+
+// Lane-mode Durstenfeld variant (RAP_WIDE_LANE_FY, default): a warp takes a batch of 32 trials;
+// in lane mode lane L runs the whole Durstenfeld chain of trial n0 + L on its own column of a
+// [k][32] byte table (w <= 256 fits u8), so 32 chains advance together instead of one; then in
+// warp mode the trials are evaluated one after the other as in sweep_wide_warp_kernel, the RAP
+// shift of row r of trial m being byte r*32 + (m ^ sw(r)).  The XOR swizzle
+// sw(k) = ((k >> 2) & 7) << 2 keeps both access shapes conflict-free: a lane-mode row k is 32
+// consecutive bytes, and a warp-mode column read of 32 distinct rows lands in 32 distinct banks
+// (bank = 8 (r & 3) + ((m >> 2) ^ ((r >> 2) & 7))).
+__host__ __device__ inline uint32_t wide_lane_words(uint32_t w) {
+    return 8 * w + 3 * w + (w * w + 31) / 32;      // perm table, r, cells, cnt, merge bitmap
+}
+
+__device__ __forceinline__ uint32_t pt_off(uint32_t k, uint32_t col) { return k * 32u + (col ^ (((k >> 2) & 7u) << 2)); }
+
+template <int NI, uint32_t PM, uint32_t SM>
+__global__ void __launch_bounds__(kWideWarps * 32, RAP_WIDE_MINB)
+sweep_wide_lane_kernel(uint32_t w, uint32_t pmask_rt, uint32_t smask_rt, uint64_t seed, uint64_t first,
+                       uint64_t n_trials, uint64_t *__restrict__ hist) {
+    const uint32_t pmask = PM ? PM : pmask_rt, smask = SM ? SM : smask_rt;
+    extern __shared__ __align__(16) uint32_t dyn[];
+    const uint32_t npat = __popc(pmask), nsch = __popc(smask);
+    const uint32_t nbins = npat * nsch * (w + 1);
+    const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
+    uint32_t *sh_hist = dyn;
+    uint32_t *mine = dyn + ((nbins + 3) & ~3u) + warp * wide_lane_words(w);
+    uint8_t *pt = reinterpret_cast<uint8_t *>(mine);          // [w][32] bytes, swizzled
+    uint32_t *rsh = mine + 8 * w, *cw = mine + 9 * w, *cnt = mine + 10 * w, *bm = mine + 11 * w;
+    for (uint32_t b = threadIdx.x; b < nbins; b += blockDim.x) sh_hist[b] = 0;
+    for (uint32_t b = lane; b < wide_lane_words(w); b += 32) mine[b] = 0;
+    __syncthreads();
+    const bool any_random = (pmask >> RAP_PAT_RANDOM) & 1u;
+    const bool need_r = (smask >> RAP_SCHEME_RAS) & 1u;
+    const uint32_t nblk = (w + 3) / 4;
+
+    const uint64_t nbatch = (n_trials + 31) / 32;
+    const uint64_t stride = (uint64_t)gridDim.x * kWideWarps;
+    for (uint64_t bt = (uint64_t)blockIdx.x * kWideWarps + warp; bt < nbatch; bt += stride) {
+        const uint64_t n0 = first + bt * 32;
+        const uint32_t nvalid = (uint32_t)min((uint64_t)32, n_trials - bt * 32);
+        // ---- C1 + C2 in lane mode: P of trial n0 + lane (include/rap.h counter contract)
+        for (uint32_t k = 0; k < w; ++k) pt[pt_off(k, lane)] = (uint8_t)k;
+        {
+            WordStream fy{seed, n0 + lane, kDomainFY};
+            for (uint32_t k = w - 1; k >= 1; --k) {
+                const uint32_t j = mulshift(fy(w - 1 - k), k + 1);
+                const uint32_t ok = pt_off(k, lane), oj = pt_off(j, lane);
+                const uint8_t x = pt[ok];
+                pt[ok] = pt[oj];
+                pt[oj] = x;
+            }
+        }
+        __syncwarp();
+        // ---- warp mode: trial n0 + m
+        for (uint32_t m = 0; m < nvalid; ++m) {
+            const uint64_t n = n0 + m;
+            for (uint32_t blk = lane; blk < nblk; blk += 32) {
+                if (need_r) {
+                    const uint4 g = philox_block(seed, n, kDomainRAS, blk);
+                    const uint32_t gw[4] = {g.x, g.y, g.z, g.w};
+#pragma unroll
+                    for (int c = 0; c < 4; ++c)
+                        if (4 * blk + c < w) rsh[4 * blk + c] = mulshift(gw[c], w);
+                }
+                if (any_random) {
+                    const uint4 g = philox_block(seed, n, kDomainRandom, blk);
+                    const uint32_t gw[4] = {g.x, g.y, g.z, g.w};
+#pragma unroll
+                    for (int c = 0; c < 4; ++c)
+                        if (4 * blk + c < w) cw[4 * blk + c] = mulshift(gw[c], w * w);
+                }
+            }
+            __syncwarp();
+            uint32_t cellv[NI], rrow[NI], rcol[NI];
+            uint32_t lead = 0;
+            if (any_random) {
+#pragma unroll
+                for (int q = 0; q < NI; ++q) {
+                    const uint32_t t = lane + 32u * q;
+                    cellv[q] = t < w ? cw[t] : 0u;
+                    rrow[q] = cellv[q] / w;
+                    rcol[q] = cellv[q] - rrow[q] * w;
+                }
+#pragma unroll
+                for (int q = 0; q < NI; ++q) {          // merged requests, slice by slice
+                    const uint32_t t = lane + 32u * q;
+                    const bool valid = t < w;
+                    const uint32_t c = cellv[q];
+                    const uint32_t same = __match_any_sync(kFull, valid ? c : (0x80000000u | lane));
+                    const bool first_in_slice = (__ffs(same) - 1) == (int)lane;
+                    const bool seen = valid && ((bm[c >> 5] >> (c & 31u)) & 1u);
+                    if (valid && first_in_slice && !seen) lead |= 1u << q;
+                    __syncwarp();
+                    if (valid) atomicOr(&bm[c >> 5], 1u << (c & 31u));
+                    __syncwarp();
+                }
+#pragma unroll
+                for (int q = 0; q < NI; ++q)
+                    if (lane + 32u * q < w) bm[cellv[q] >> 5] = 0u;
+            }
+            __syncwarp();
+            uint32_t e = 0;
+#pragma unroll
+            for (int p = 0; p < 5; ++p) {
+                if (!((pmask >> p) & 1u)) continue;
+#pragma unroll
+                for (int s = 0; s < 5; ++s) {
+                    if (!((smask >> s) & 1u)) continue;
+                    int pp = p;                                   // reading iii: malicious
+                    if (p == RAP_PAT_MALICIOUS)
+                        pp = (s == RAP_SCHEME_RAW || s == RAP_SCHEME_RAS) ? RAP_PAT_STRIDE
+                           : (s == RAP_SCHEME_PAD) ? -1 : RAP_PAT_DIAGONAL;
+                    uint32_t bankv[NI];
+                    uint32_t mx = 0;
+#pragma unroll
+                    for (int q = 0; q < NI; ++q) {
+                        const uint32_t t = lane + 32u * q;
+                        bankv[q] = 0xffffffffu;
+                        if (t >= w) continue;
+                        if (pp == RAP_PAT_RANDOM && !((lead >> q) & 1u)) continue;      // merged
+                        uint32_t row, col;
+                        switch (pp) {
+                        case RAP_PAT_CONTIGUOUS: row = 0; col = t; break;
+                        case RAP_PAT_STRIDE: row = t; col = 0; break;
+                        case RAP_PAT_DIAGONAL: row = t; col = t; break;
+                        case RAP_PAT_RANDOM: row = rrow[q]; col = rcol[q]; break;
+                        default: row = t; col = t == 0 ? 0u : w - t; break;           // PAD anti-diagonal
+                        }
+                        uint32_t bank;
+                        if (s == RAP_SCHEME_RAS || s == RAP_SCHEME_RAP) {
+                            bank = col + (s == RAP_SCHEME_RAP ? (uint32_t)pt[pt_off(row, m)] : rsh[row]);
+                            bank = bank >= w ? bank - w : bank;
+                        } else if (s == RAP_SCHEME_PAD) {
+                            bank = row + col;
+                            bank = bank >= w ? bank - w : bank;
+                        } else if (s == RAP_SCHEME_XOR) {
+                            bank = col ^ row;
+                        } else {
+                            bank = col;
+                        }
+                        bankv[q] = bank;
+                        const uint32_t v = atomicAdd(&cnt[bank], 1u) + 1u;
+                        mx = v > mx ? v : mx;
+                    }
+                    mx = __reduce_max_sync(kFull, mx);
+                    __syncwarp();
+#pragma unroll
+                    for (int q = 0; q < NI; ++q)
+                        if (bankv[q] != 0xffffffffu) cnt[bankv[q]] = 0u;
+                    if (lane == 0) atomicAdd(&sh_hist[e * (w + 1) + mx], 1u);
+                    __syncwarp();
+                    ++e;
+                }
+            }
+        }
+        __syncwarp();
+    }
+    __syncthreads();
+    for (uint32_t b = threadIdx.x; b < nbins; b += blockDim.x)
+        if (sh_hist[b]) atomicAdd((unsigned long long *)(hist + b), (unsigned long long)sh_hist[b]);
+}
+
 size_t wide_smem_bytes(uint32_t w, uint32_t pmask, uint32_t smask) {
     const uint32_t nbins = __builtin_popcount(pmask) * __builtin_popcount(smask) * (w + 1);
     return 4 * (size_t)((nbins + 3) & ~3u) + 2 * (size_t)4 * w * kWideThreads +
@@ -350,6 +515,30 @@ static cudaError_t launch_wide_warp(uint32_t w, uint32_t pmask, uint32_t smask, 
     const uint32_t nbins = __builtin_popcount(pmask) * __builtin_popcount(smask) * (w + 1);
     const size_t smem = 4 * ((size_t)((nbins + 3) & ~3u) + (size_t)kWideWarps * wide_warp_words(w));
     // compile-time masks for the Table II sweeps (5 patterns x RAW/RAS/RAP, and all 5 schemes)
+#if RAP_WIDE_LANE_FY
+    const size_t smem_l = 4 * ((size_t)((nbins + 3) & ~3u) + (size_t)kWideWarps * wide_lane_words(w));
+    if (smem_l <= 227 * 1024) {
+        auto kl = (pmask == 31u && smask == 7u) ? sweep_wide_lane_kernel<NI, 31u, 7u>
+                : (pmask == 31u && smask == 31u) ? sweep_wide_lane_kernel<NI, 31u, 31u>
+                : sweep_wide_lane_kernel<NI, 0u, 0u>;
+        cudaError_t e = cudaFuncSetAttribute(kl, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_l);
+        if (e != cudaSuccess) return e;
+        int dev = 0, sms = 148, occ = 1;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kl, kWideWarps * 32, smem_l);
+        if (occ < 1) occ = 1;
+        const uint64_t want = (n_trials + 32 * kWideWarps - 1) / (32 * kWideWarps);
+        const uint64_t cap = (uint64_t)sms * occ;
+        const int grid = (int)(want < cap ? want : cap);
+        const uint64_t chunk = (uint64_t)grid * (1ull << 31);  // u32 CTA counters stay below 2^31
+        for (uint64_t done = 0; done < n_trials; done += chunk) {
+            const uint64_t cnt = (n_trials - done < chunk) ? n_trials - done : chunk;
+            kl<<<grid, kWideWarps * 32, smem_l, st>>>(w, pmask, smask, seed, first + done, cnt, hist);
+        }
+        return cudaGetLastError();
+    }
+#endif
     auto k = (pmask == 31u && smask == 7u) ? sweep_wide_warp_kernel<NI, 31u, 7u>
            : (pmask == 31u && smask == 31u) ? sweep_wide_warp_kernel<NI, 31u, 31u>
            : sweep_wide_warp_kernel<NI, 0u, 0u>;
