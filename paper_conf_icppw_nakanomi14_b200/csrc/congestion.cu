@@ -877,6 +877,8 @@ cudaError_t launch_sweep(uint32_t w, uint32_t pmask, uint32_t smask, uint64_t se
         run_sweep<sweep32_kernel<31u, 31u>>(kSweepWarpsV2, 32, w, pmask, smask, seed, first, n_trials, hist, st);
     else if (w == 32)
         run_sweep<sweep_kernel<32, 0u, 0u>>(kSweepWarpsV2, 32, w, pmask, smask, seed, first, n_trials, hist, st);
+    else if (pmask == 31u && smask == 7u)      // w < 32 with the Table II masks fixed at compile time
+        run_sweep<sweep_kernel<0, 31u, 7u>>(kSweepWarpsV2, 32, w, pmask, smask, seed, first, n_trials, hist, st);
     else
         run_sweep<sweep_kernel<0, 0u, 0u>>(kSweepWarpsV2, 32, w, pmask, smask, seed, first, n_trials, hist, st);
     return cudaGetLastError();
