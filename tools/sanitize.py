@@ -32,6 +32,7 @@ rap.perm_gen(seed=1, count=10, w=7)
 rap.congestion_sweep(5000, seed=1)
 rap.congestion_sweep(5000, seed=1, schemes=("raw", "ras", "rap", "pad", "xor"))
 rap.congestion_sweep(3000, seed=1, w=7, schemes=("raw", "ras", "rap", "pad"))
+rap.congestion_sweep(3000, seed=1, w=16)
 rap.congestion_sweep(300, seed=1, w=64)
 rap.congestion_sweep(200, seed=1, w=100, schemes=("raw", "ras", "rap", "pad"))
 rap.congestion_sweep(100, seed=1, w=256, schemes=("raw", "ras", "rap", "pad", "xor"))
