@@ -574,6 +574,16 @@ def test_sweep_wide_bit_exact(rap, oracle, w):
     assert np.array_equal(g.cpu().numpy().astype(np.uint64), o)
 
 
+@pytest.mark.parametrize("w", [16, 24, 64, 96, 256])
+def test_sweep_default_masks_other_w(rap, oracle, w):
+    # the compile-time-mask kernels (5 patterns x RAW/RAS/RAP) off w = 32: the w < 32 warp kernel
+    # and the lane-mode wide kernel; trial count ragged against the 32-trial batches
+    N = 2777 if w <= 96 else 997
+    g = rap.congestion_sweep(N, seed=5, w=w, first_trial=12345)
+    o = oracle.sweep(w, ALL_PAT, ["raw", "ras", "rap"], 5, 12345, N)
+    assert np.array_equal(g.cpu().numpy().astype(np.uint64), o)
+
+
 @pytest.mark.parametrize("w,N", [(64, 400_000), (128, 200_000), (256, 100_000)])
 def test_table2_wide_columns_on_gpu(rap, w, N):
     # Table II columns w = 64, 128, 256 from the GPU sweep: every entry within
