@@ -36,6 +36,8 @@ constexpr int kDefaultSR32 = 4, kDefaultSC32 = 2, kDefaultSR64 = 12, kDefaultSC6
 constexpr int kDefaultCL32 = 4, kDefaultCL64 = 1;
 // fused sharded transpose (peer stores): 8 x 2 warps, no cluster
 constexpr int kPeerSR32 = 8, kPeerSC32 = 2;
+// up to this many 32 x 32 tiles: one single-warp CTA per tile
+constexpr int64_t kSmallTiles = 8;
 // measured on B200 (tools/tune_transpose.cu, profiles/r01_tune_transpose.txt)
 constexpr int kDefaultMinB32 = 2, kDefaultMinB64 = 1;   // fp32: 2 CTAs of 8 warps per SM (128 registers)
 constexpr int kDefaultDepth32 = 1, kDefaultDepth64 = 1;

@@ -536,6 +536,10 @@ static cudaError_t launch_shape(const void *src, void *dst, int64_t rows, int64_
 #undef RAPK_SHAPE
 #undef RAPK_TSHAPE
     (void)tu;
+    // a handful of tiles (cfg1's single 32 x 32 tile): one warp per CTA, one CTA per tile -- no
+    // cluster, no idle warps of a super-tile computing P, the cheapest launch
+    if (((rows + 31) / 32) * ((cols + 31) / 32) <= kSmallTiles)
+        return launch_one<L, EW, VEC, 1, 1, false, 1, 1>(src, dst, rows, cols, ld_src, ld_dst, seed, tu, st);
     if (EW == 1 && tu.cl == kDefaultCL32)
         return launch_one<L, EW, VEC, kDefaultDepth32, kDefaultMinB32, kDefaultVst32, kDefaultSR32, kDefaultSC32,
                           false, false, kDefaultCL32>(src, dst, rows, cols, ld_src, ld_dst, seed, tu, st);
