@@ -601,6 +601,10 @@ def main():
                          "E_raw_malicious": E(h[4, 0]), "E_rap_stride": E(h[1, 2]),
                          "kernel_ms_median": statistics.median(r["s_ms"]),
                          "roofline": sweep_roofline(tps / world, r["clocks"])}
+        if do_t and S <= 148 * 8 * 4 * 32:
+            line["sweep"]["note"] = ("one batch of 32 trials per resident warp per step: a single wave, below the "
+                                     "kernel's steady rate (launch ramp and tail); `--workload sweep` times 64 "
+                                     "batches per warp per launch (profiles/r01_bench_sweep.json)")
         if not do_t:
             line.update(value=tps, unit="trials/s",
                         config=arm_config(args, world))
