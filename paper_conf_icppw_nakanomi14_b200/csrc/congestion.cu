@@ -706,6 +706,9 @@ trace_kernel(uint32_t w_rt, uint64_t n_warps, const uint32_t *__restrict__ cells
 //     ballots read bits 0..4 only, which is the "mod 32"), 5 ballots, popc, reduce-max.
 // Histograms live in registers: lane L of the warp counts congestion L+1 for each scheme, flushed
 // with one u64 atomic per non-zero counter at the end.
+#ifndef RAP_TRACE_GENERIC
+#define RAP_TRACE_GENERIC 0
+#endif
 #ifndef RAP_TRACE_TB
 #define RAP_TRACE_TB 32
 #endif
@@ -723,10 +726,22 @@ constexpr int kTraceWarps = RAP_TRACE_WARPS;
 #define RAP_TRACE32_MINB 4
 #endif
 
-template <uint32_t SM>
+// trace32_kernel helpers: lanes that play DMM threads, and (x mod w) for x < 2w -- for W = 32 the
+// ballots read bits 0..4 only, which is already the reduction mod 32
+template <int W>
+__device__ __forceinline__ bool lane_active(uint32_t w) { return W == 32 || (threadIdx.x & 31u) < w; }
+template <int W>
+__device__ __forceinline__ uint32_t wrap_w(uint32_t x, uint32_t w) { return W == 32 ? x : (x >= w ? x - w : x); }
+
+// W = 32: compile-time w (cells split by shift / mask, the ballots' bits 0..4 are the "mod 32");
+// W = 0: runtime w < 32 (lanes >= w idle, explicit mod w, w + 1 bins per scheme).
+template <int W, uint32_t SM>
 __global__ void __launch_bounds__(kTraceWarps * 32, RAP_TRACE32_MINB)
-trace32_kernel(uint64_t n_warps, const uint32_t *__restrict__ cells, uint64_t seed, uint64_t first,
+trace32_kernel(uint32_t w_rt, uint64_t n_warps, const uint32_t *__restrict__ cells, uint64_t seed, uint64_t first,
                uint64_t n_trials, uint64_t *__restrict__ hist) {
+    const uint32_t w = W ? (uint32_t)W : w_rt;
+    const bool active = lane_active<W>(w);
+    const uint32_t amask = (w >= 32) ? kFull : ((1u << w) - 1u);
     constexpr uint32_t nsch = __builtin_popcount(SM);
     constexpr bool need_p = (SM >> RAP_SCHEME_RAP) & 1u, need_r = (SM >> RAP_SCHEME_RAS) & 1u;
     __shared__ uint8_t shP[kTraceTB][32], shR[kTraceTB][32];
@@ -745,34 +760,35 @@ trace32_kernel(uint64_t n_warps, const uint32_t *__restrict__ cells, uint64_t se
         const uint32_t tcnt = (uint32_t)min((uint64_t)kTraceTB, n_trials - t0);
         __syncthreads();                                    // the previous unit is done with shP / shR
         for (uint32_t t = warp; t < tcnt; t += kTraceWarps) {
-            if (need_p) shP[t][lane] = (uint8_t)warp_perm<32>(seed, first + t0 + t, lane, 32);
-            if (need_r) shR[t][lane] = (uint8_t)warp_ras_shift(seed, first + t0 + t, lane, 32);
+            if (need_p) shP[t][lane] = (uint8_t)warp_perm<W>(seed, first + t0 + t, lane, w);
+            if (need_r) shR[t][lane] = (uint8_t)warp_ras_shift(seed, first + t0 + t, lane, w);
         }
         __syncthreads();
         const uint64_t k_end = min(n_warps, (kc + 1) * kTraceTK);
         for (uint64_t k = kc * kTraceTK + warp; k < k_end; k += kTraceWarps) {
-            const uint32_t raw_cell = __ldg(cells + k * 32 + lane);
-            if (__any_sync(kFull, raw_cell >= 1024u)) {     // invalid trace warp: bin 0
+            const uint32_t raw_cell = active ? __ldg(cells + k * w + lane) : 0u;
+            if (__any_sync(kFull, active && raw_cell >= w * w)) {     // invalid trace warp: bin 0
                 hbad += tcnt;
                 continue;
             }
-            const uint32_t row = raw_cell >> 5, col = raw_cell & 31u;
+            const uint32_t row = W == 32 ? raw_cell >> 5 : raw_cell / w;
+            const uint32_t col = W == 32 ? raw_cell & 31u : raw_cell - row * w;
             // merged requests: the first lane of each distinct cell is counted
-            const uint32_t same = __match_any_sync(kFull, raw_cell);
-            const uint32_t leaders = ballot_zero(same, lt_mask);
+            const uint32_t same = __match_any_sync(kFull, active ? raw_cell : (0x80000000u | lane));
+            const uint32_t leaders = ballot_zero(same, lt_mask) & amask;
             uint32_t e = 0;
 #pragma unroll
             for (int s = 0; s < 5; ++s) {
                 if (!((SM >> s) & 1u)) continue;
                 if (s == RAP_SCHEME_RAW || s == RAP_SCHEME_PAD || s == RAP_SCHEME_XOR) {
-                    const uint32_t bank = s == RAP_SCHEME_RAW ? col : s == RAP_SCHEME_PAD ? row + col : (col ^ row);
+                    const uint32_t bank = s == RAP_SCHEME_RAW ? col : s == RAP_SCHEME_PAD ? wrap_w<W>(row + col, w) : (col ^ row);
                     const uint32_t c = max_bank_load(bank, leaders, ls);
                     hc[e] += (c == lane + 1u) ? tcnt : 0u;
                 } else {
                     const uint8_t *sh = s == RAP_SCHEME_RAP ? &shP[0][0] : &shR[0][0];
 #pragma unroll 4
                     for (uint32_t t = 0; t < tcnt; ++t) {
-                        const uint32_t c = max_bank_load(col + sh[t * 32 + row], leaders, ls);
+                        const uint32_t c = max_bank_load(wrap_w<W>(col + sh[t * 32 + row], w), leaders, ls);
                         hc[e] += (c == lane + 1u) ? 1u : 0u;
                     }
                 }
@@ -782,8 +798,8 @@ trace32_kernel(uint64_t n_warps, const uint32_t *__restrict__ cells, uint64_t se
     }
 #pragma unroll
     for (uint32_t e = 0; e < nsch; ++e) {
-        if (hc[e]) atomicAdd((unsigned long long *)(hist + e * 33 + lane + 1), (unsigned long long)hc[e]);
-        if (lane == 0 && hbad) atomicAdd((unsigned long long *)(hist + e * 33), (unsigned long long)hbad);
+        if (hc[e]) atomicAdd((unsigned long long *)(hist + e * (w + 1) + lane + 1), (unsigned long long)hc[e]);
+        if (lane == 0 && hbad) atomicAdd((unsigned long long *)(hist + e * (w + 1)), (unsigned long long)hbad);
     }
 }
 
@@ -892,12 +908,12 @@ cudaError_t launch_sweep_match(uint32_t w, uint32_t pmask, uint32_t smask, uint6
     return cudaGetLastError();
 }
 
-template <uint32_t SM>
-static void run_trace32(uint64_t n_warps, const uint32_t *cells, uint64_t seed, uint64_t first, uint64_t n_trials,
-                        uint64_t *hist, cudaStream_t st) {
+template <int W, uint32_t SM>
+static void run_trace32(uint32_t w, uint64_t n_warps, const uint32_t *cells, uint64_t seed, uint64_t first,
+                        uint64_t n_trials, uint64_t *hist, cudaStream_t st) {
     const int threads = kTraceWarps * 32;
     const uint64_t nkc = (n_warps + kTraceTK - 1) / kTraceTK;
-    const int cap = resident_ctas<trace32_kernel<SM>>(threads);
+    const int cap = resident_ctas<trace32_kernel<W, SM>>(threads);
     // per-lane u32 counters: a warp evaluates at most ceil(units / grid) units of
     // (kTraceTK / kTraceWarps) trace warps x kTraceTB trials per launch -- keep that below 2^31
     const uint64_t per_unit = (uint64_t)(kTraceTK / kTraceWarps) * kTraceTB;
@@ -908,7 +924,7 @@ static void run_trace32(uint64_t n_warps, const uint32_t *cells, uint64_t seed, 
         const uint64_t cnt = (n_trials - done < trials_chunk) ? n_trials - done : trials_chunk;
         const uint64_t units = ((cnt + kTraceTB - 1) / kTraceTB) * nkc;
         const int grid = (int)(units < (uint64_t)cap ? units : (uint64_t)cap);
-        trace32_kernel<SM><<<grid, threads, 0, st>>>(n_warps, cells, seed, first + done, cnt, hist);
+        trace32_kernel<W, SM><<<grid, threads, 0, st>>>(w, n_warps, cells, seed, first + done, cnt, hist);
     }
 }
 
@@ -916,8 +932,10 @@ cudaError_t launch_trace(uint32_t w, uint64_t n_warps, const uint32_t *cells, ui
                          uint64_t seed, uint64_t first, uint64_t n_trials, uint64_t *hist,
                          cudaStream_t st) {
     if (n_trials == 0 || n_warps == 0) return cudaSuccess;
-    if (w == 32) {
-#define RAPK_TRACE32(M) case M: run_trace32<M>(n_warps, cells, seed, first, n_trials, hist, st); break;
+#if !RAP_TRACE_GENERIC
+    {
+#define RAPK_TRACE32(M) case M: if (w == 32) run_trace32<32, M>(w, n_warps, cells, seed, first, n_trials, hist, st); \
+                                else run_trace32<0, M>(w, n_warps, cells, seed, first, n_trials, hist, st); break;
         switch (smask) {
             RAPK_TRACE32(1) RAPK_TRACE32(2) RAPK_TRACE32(3) RAPK_TRACE32(4) RAPK_TRACE32(5) RAPK_TRACE32(6)
             RAPK_TRACE32(7) RAPK_TRACE32(8) RAPK_TRACE32(9) RAPK_TRACE32(10) RAPK_TRACE32(11) RAPK_TRACE32(12)
@@ -930,7 +948,9 @@ cudaError_t launch_trace(uint32_t w, uint64_t n_warps, const uint32_t *cells, ui
 #undef RAPK_TRACE32
         return cudaGetLastError();
     }
-    // 2 <= w < 32: the generic evaluator, one warp per (trial, chunk of 32 trace warps)
+#endif
+    // RAP_TRACE_GENERIC (ablation): the first evaluator, one warp per (trial, chunk of 32 trace
+    // warps), leaders and trial-invariant schemes recomputed for every trial
     const int threads = kSweepWarps * 32;
     const uint64_t nchunks = (n_warps + kTraceChunk - 1) / kTraceChunk;
     auto kern = trace_kernel<0, 0u>;

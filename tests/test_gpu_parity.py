@@ -394,6 +394,17 @@ def test_trace_bench_size_sampled_and_additive(rap, oracle):
     assert torch.equal(full, parts) and (full.sum(-1) == 4096 * 256).all()
 
 
+@pytest.mark.parametrize("w", [2, 5, 8, 16, 31])
+def test_trace_small_w_matches_oracle(rap, oracle, w):
+    # w < 32: lanes >= w idle, banks reduced mod w, w + 1 bins per scheme; ragged units, bad cell
+    schemes = ["raw", "ras", "rap", "pad"] + (["xor"] if w & (w - 1) == 0 else [])
+    cells = workloads.trace_cells(70, w, seed=w)
+    cells[3, 0] = w * w                                  # invalid -> bin 0
+    g = rap.congestion_trace(cells.cuda(), 45, seed=11, schemes=schemes, first_trial=77)
+    expect = _trace_oracle(oracle, cells.numpy(), 11, 77, 45, schemes, w=w)
+    assert np.array_equal(g.cpu().numpy().astype(np.uint64), expect)
+
+
 def test_trace_small_w_and_invalid(rap, oracle):
     w = 8
     cells = workloads.trace_cells(13, w, seed=1)
