@@ -43,6 +43,9 @@ rap.congestion_trace(cells, 10, seed=1, schemes=("raw", "ras", "rap", "pad", "xo
 cells2 = workloads.trace_cells(131, 32, seed=2)
 cells2[7, 3] = 5000                                   # invalid trace warp -> bin 0
 rap.congestion_trace(cells2.to(dev), 70, seed=1, schemes=("ras", "xor"), first_trial=33)
+cells3 = workloads.trace_cells(40, 8, seed=3)
+cells3[2, 1] = 64                                     # w = 8: invalid trace warp
+rap.congestion_trace(cells3.to(dev), 37, seed=1, schemes=("raw", "ras", "rap", "pad", "xor"))
 t = lambda a: torch.from_numpy(np.asarray(a, dtype=np.int32)).to(dev)
 rr = np.random.default_rng(0).integers(0, 32, (50, 32))
 rap.congestion(t(rr), t(rr[::-1].copy()), "rap", shift=t(np.stack([np.random.default_rng(k).permutation(32) for k in range(50)])))
