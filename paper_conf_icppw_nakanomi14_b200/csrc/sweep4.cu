@@ -22,9 +22,19 @@ constexpr int kSweep4Warps = 8;
 constexpr int kMaxBins4 = 6 * 5 * (RAP_MAX_W + 1);
 constexpr uint32_t kDomainQ = 3, kDomainR = 4;
 
+// x mod w / x div w: masks and shifts when w is a compile-time power of two (W = 16, 32)
+template <int W>
+__device__ __forceinline__ uint32_t md(uint32_t x, uint32_t w) { return (W && !(W & (W - 1))) ? (x & (W - 1)) : x % w; }
+template <int W>
+__device__ __forceinline__ uint32_t dv(uint32_t x, uint32_t w) {
+    return (W && !(W & (W - 1))) ? (x >> __builtin_ctz(W ? W : 1)) : x / w;
+}
+
+template <int W>
 __global__ void __launch_bounds__(kSweep4Warps * 32)
-sweep4_kernel(uint32_t w, uint32_t pmask, uint32_t smask, uint64_t seed, uint64_t first, uint64_t n_trials,
+sweep4_kernel(uint32_t w_rt, uint32_t pmask, uint32_t smask, uint64_t seed, uint64_t first, uint64_t n_trials,
               uint64_t *__restrict__ hist) {
+    const uint32_t w = W ? (uint32_t)W : w_rt;
     __shared__ uint32_t sh_hist[kMaxBins4];
     const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
     const uint32_t nbins = __popc(pmask) * __popc(smask) * (w + 1);
@@ -37,9 +47,9 @@ sweep4_kernel(uint32_t w, uint32_t pmask, uint32_t smask, uint64_t seed, uint64_
     const uint64_t stride = (uint64_t)gridDim.x * kSweep4Warps;
     for (uint64_t it = (uint64_t)blockIdx.x * kSweep4Warps + warp; it < n_trials; it += stride) {
         const uint64_t n = first + it;
-        const uint32_t P = need_p ? warp_perm<0>(seed, n, lane, w) : lane;
-        const uint32_t Q = need_qr ? warp_fisher_yates<0>(lane_word(seed, n, kDomainQ, lane), lane, w) : lane;
-        const uint32_t R = need_qr ? warp_fisher_yates<0>(lane_word(seed, n, kDomainR, lane), lane, w) : lane;
+        const uint32_t P = need_p ? warp_perm<W == 32 ? 32 : 0>(seed, n, lane, w) : lane;
+        const uint32_t Q = need_qr ? warp_fisher_yates<W == 32 ? 32 : 0>(lane_word(seed, n, kDomainQ, lane), lane, w) : lane;
+        const uint32_t R = need_qr ? warp_fisher_yates<W == 32 ? 32 : 0>(lane_word(seed, n, kDomainR, lane), lane, w) : lane;
         uint32_t cell_rnd = 0;
         if ((pmask >> RAP_PAT4_RANDOM) & 1u) {
             const uint64_t w4 = (uint64_t)w * w * w * w;
@@ -62,9 +72,9 @@ sweep4_kernel(uint32_t w, uint32_t pmask, uint32_t smask, uint64_t seed, uint64_
                 case RAP_PAT4_STRIDE3: i = lane; break;
                 case RAP_PAT4_RANDOM: {
                     uint32_t c = cell_rnd;
-                    l = c % w; c /= w;
-                    k = c % w; c /= w;
-                    j = c % w; i = c / w;
+                    l = md<W>(c, w); c = dv<W>(c, w);
+                    k = md<W>(c, w); c = dv<W>(c, w);
+                    j = md<W>(c, w); i = dv<W>(c, w);
                     break;
                 }
                 default: {                                          // 6-permutation groups
@@ -79,19 +89,28 @@ sweep4_kernel(uint32_t w, uint32_t pmask, uint32_t smask, uint64_t seed, uint64_
                     break;
                 }
                 }
+                // only the shuffles this scheme needs (s is warp-uniform)
                 uint32_t f = 0;
-                const uint32_t Pi = __shfl_sync(kFull, P, i & 31u), Pj = __shfl_sync(kFull, P, j & 31u);
-                const uint32_t Pk = __shfl_sync(kFull, P, k & 31u);
-                const uint32_t Qj = __shfl_sync(kFull, Q, j & 31u), Rk = __shfl_sync(kFull, R, k & 31u);
-                if (s == RAP_SCHEME4_RAS)
+                if (s == RAP_SCHEME4_RAS) {
                     f = mulshift(word_at(seed, n, kDomainRAS, (i * w + j) * w + k), w);
-                else if (s == RAP_SCHEME4_1P) f = Pk;
-                else if (s == RAP_SCHEME4_R1P) f = (Pi + Pj + Pk) % w;
-                else if (s == RAP_SCHEME4_3P) f = (Pi + Qj + Rk) % w;
-                const uint32_t bank = (l + f) % w;
-                const uint32_t key = ((i * w + j) * w + k) * w + l;     // logical cell, < 2^20
-                const uint32_t same = __match_any_sync(kFull, lane < w ? key : (0x80000000u | lane));
-                const uint32_t counted = ballot_zero(same, (1u << lane) - 1u) & active;
+                } else if (s == RAP_SCHEME4_1P) {
+                    f = __shfl_sync(kFull, P, k & 31u);
+                } else if (s == RAP_SCHEME4_R1P) {
+                    f = md<W>(__shfl_sync(kFull, P, i & 31u) + __shfl_sync(kFull, P, j & 31u) +
+                              __shfl_sync(kFull, P, k & 31u), w);
+                } else if (s == RAP_SCHEME4_3P) {
+                    f = md<W>(__shfl_sync(kFull, P, i & 31u) + __shfl_sync(kFull, Q, j & 31u) +
+                              __shfl_sync(kFull, R, k & 31u), w);
+                }
+                const uint32_t bank = md<W>(l + f, w);
+                // merged requests: only the random cells and the clamped 6-permutation groups can
+                // repeat a cell; every other pattern's w cells are distinct
+                uint32_t counted = active;
+                if (pp == RAP_PAT4_RANDOM || pp == -1) {
+                    const uint32_t key = ((i * w + j) * w + k) * w + l;  // logical cell, < 2^20
+                    const uint32_t same = __match_any_sync(kFull, lane < w ? key : (0x80000000u | lane));
+                    counted = ballot_zero(same, (1u << lane) - 1u) & active;
+                }
                 const uint32_t c = max_bank_load(bank, counted, ls);
                 mine = (lane == e) ? c : mine;
                 ++e;
@@ -110,7 +129,8 @@ cudaError_t launch_sweep4(uint32_t w, uint32_t pmask, uint32_t smask, uint64_t s
     int dev = 0, sms = 148, occ = 1;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, sweep4_kernel, kSweep4Warps * 32, 0);
+    auto k = w == 32 ? sweep4_kernel<32> : w == 16 ? sweep4_kernel<16> : sweep4_kernel<0>;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, kSweep4Warps * 32, 0);
     if (occ < 1) occ = 1;
     const uint64_t want = (n_trials + kSweep4Warps - 1) / kSweep4Warps;
     const uint64_t cap = (uint64_t)sms * occ;
@@ -118,7 +138,7 @@ cudaError_t launch_sweep4(uint32_t w, uint32_t pmask, uint32_t smask, uint64_t s
     const uint64_t chunk = (uint64_t)grid * (1ull << 31) / 32;    // u32 CTA counters
     for (uint64_t done = 0; done < n_trials; done += chunk) {
         const uint64_t cnt = (n_trials - done < chunk) ? n_trials - done : chunk;
-        sweep4_kernel<<<grid, kSweep4Warps * 32, 0, st>>>(w, pmask, smask, seed, first + done, cnt, hist);
+        k<<<grid, kSweep4Warps * 32, 0, st>>>(w, pmask, smask, seed, first + done, cnt, hist);
     }
     return cudaGetLastError();
 }
