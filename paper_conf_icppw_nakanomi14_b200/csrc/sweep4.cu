@@ -56,6 +56,7 @@ sweep4_kernel(uint32_t w_rt, uint32_t pmask, uint32_t smask, uint64_t seed, uint
             cell_rnd = (uint32_t)(((uint64_t)lane_word(seed, n, kDomainRandom, lane) * w4) >> 32);
         }
         uint32_t mine = 0, e = 0;
+        uint32_t c_s1[5] = {0, 0, 0, 0, 0}, c_s2[5] = {0, 0, 0, 0, 0};   // stride1 / stride2 results
         for (int p = 0; p < 6; ++p) {
             if (!((pmask >> p) & 1u)) continue;
             for (int s = 0; s < 5; ++s) {
@@ -64,6 +65,14 @@ sweep4_kernel(uint32_t w_rt, uint32_t pmask, uint32_t smask, uint64_t seed, uint
                 if (p == RAP_PAT4_MALICIOUS)
                     pp = (s == RAP_SCHEME4_RAW || s == RAP_SCHEME4_RAS) ? RAP_PAT4_STRIDE1
                        : (s == RAP_SCHEME4_1P) ? RAP_PAT4_STRIDE2 : -1;
+                // malicious = an access already evaluated this trial (reading xiii): reuse it
+                if (p == RAP_PAT4_MALICIOUS && ((pp == RAP_PAT4_STRIDE1 && ((pmask >> RAP_PAT4_STRIDE1) & 1u)) ||
+                                                (pp == RAP_PAT4_STRIDE2 && ((pmask >> RAP_PAT4_STRIDE2) & 1u)))) {
+                    const uint32_t c = pp == RAP_PAT4_STRIDE1 ? c_s1[s] : c_s2[s];
+                    mine = (lane == e) ? c : mine;
+                    ++e;
+                    continue;
+                }
                 uint32_t i = 0, j = 0, k = 0, l = 0;
                 switch (pp) {
                 case RAP_PAT4_CONTIGUOUS: l = lane; break;
@@ -112,6 +121,8 @@ sweep4_kernel(uint32_t w_rt, uint32_t pmask, uint32_t smask, uint64_t seed, uint
                     counted = ballot_zero(same, (1u << lane) - 1u) & active;
                 }
                 const uint32_t c = max_bank_load(bank, counted, ls);
+                if (p == RAP_PAT4_STRIDE1) c_s1[s] = c;
+                if (p == RAP_PAT4_STRIDE2) c_s2[s] = c;
                 mine = (lane == e) ? c : mine;
                 ++e;
             }
