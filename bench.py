@@ -418,7 +418,7 @@ def main():
     do_t = wl not in ("sweep", "trace")
     do_s = wl in ("default", "sweep", "trace")
     layouts = (["raw", "pad", "xor", "ras", "rap"] if wl == "layouts"
-               else ["rap16", "rap"] if wl == "cfg4" and args.layout == "rap"     # T2b (ii) ablation beside (i)
+               else ["rap16", "rap2p", "rap"] if wl == "cfg4" and args.layout == "rap"     # T2b ablations beside the 8-byte-slot RAP
                else [args.layout])
     eb = torch.empty((), dtype=dt).element_size()
     nbytes = 2 * rows * cols * eb                     # per rank per step

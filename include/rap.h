@@ -41,9 +41,10 @@
 extern "C" {
 #endif
 
-#define RAP_ABI_VERSION 1
+#define RAP_ABI_VERSION 2
 #define RAP_MAX_W 32          /* warp-wide evaluators: one CUDA warp = one DMM warp          */
-#define RAP_MAX_W_SWEEP 256   /* rap_congestion_sweep: w > 32 runs one trial per CUDA thread */
+#define RAP_MAX_W_SWEEP 256   /* rap_congestion_sweep: 32 < w <= 256 spans one CUDA warp over  */
+                              /* w/32 request slices (sweep_wide.cu)                          */
 
 typedef enum {
     RAP_OK = 0,
@@ -60,14 +61,22 @@ typedef enum {
     RAP_LAYOUT_XOR = 2,  /* a[i][j] at [i][j xor i]                 (XOR-swizzle baseline)*/
     RAP_LAYOUT_RAS = 3,  /* a[i][j] at [i][(j + r[i]) mod 32]          */
     RAP_LAYOUT_RAP = 4,  /* a[i][j] at [i][(j + P[i]) mod 32]        */
-    RAP_LAYOUT_RAP16 = 5 /* 64-bit elements only (else RAP_ERR_UNSUPPORTED): a tile of     */
+    RAP_LAYOUT_RAP16 = 5,/* 64-bit elements only (else RAP_ERR_UNSUPPORTED): a tile of     */
                          /* doubles with one element per PAIR of 4-byte banks, i.e. 16   */
                          /* "double banks"; a[i][j] at [i][16*(j div 16) + ((j + Q[i mod */
                          /* 16]) mod 16)], Q = perm(seed, 0, 16).  The paper's RAP with  */
                          /* w = 16 applied to each half row: every half-warp of a 64-bit */
                          /* row or column access hits 16 distinct bank pairs (P:L860,    */
                          /* L1005-1023, DESIGN reading xiv)            */
+    RAP_LAYOUT_RAP2P = 6 /* 64-bit elements only: the w = 32 RAP map on two 32-bit planes */
+                         /* (low words, high words), every smem access 4 bytes wide      */
+                         /* (the round-1 default, kept as an ablation)   */
 } rap_layout_t;
+/* With elem_bytes == 8, RAW..RAP keep ONE 8-byte element per tile slot: RAP is the paper's map
+ * a[i][(j + P[i]) mod 32] on doubles, P = perm(seed, 0, 32) (where a
+ * bank held one double).  B200 banks are 4 bytes, so a 64-bit access is served per half-warp
+ * (16 doubles = 128 B per wavefront); the kernel assigns rows to lanes so that every half-warp
+ * of the row write and of the column read hits 16 distinct bank pairs (DESIGN reading xv). */
 
 /* Address maps of the DMM congestion evaluator (physical address of logical cell (i,j)). */
 typedef enum {
@@ -111,11 +120,19 @@ typedef enum {
 int rap_abi_version(void);
 const char *rap_status_str(rap_status_t s);
 
-/* T0 -- permutations P_n = perm(seed, n, w) for n = first_index .. first_index+count-1
- * (§IV).  d_perm_out: device uint8_t[count][w]; row k holds P_{first_index+k}.
- * 2 <= w <= 32.  count == 0 is a no-op. */
-rap_status_t rap_perm_gen(uint64_t seed, uint64_t first_index, uint64_t count, uint32_t w,
-                          uint8_t *d_perm_out, void *stream);
+/* T0 -- one permutation P = perm(seed, index, w) of {0..w-1}, on the HOST (P:L316-320, L959-962
+ * §IV: "P is selected uniformly at random from all w! permutations"; the counter contract above
+ * fixes which one).  perm_out: host uint32_t[w], caller-owned; 2 <= w <= 256 (Table II's widths).
+ * Deterministic and synchronous; no GPU involved.  This is how every transpose launch obtains
+ * its P (index 0): computed once per call on the host and passed to the kernel by value
+ * (the paper: the random numbers are "computed beforehand"). */
+rap_status_t rap_perm_gen(uint64_t seed, uint64_t index, uint32_t w, uint32_t *perm_out);
+
+/* T0, batched on the device -- P_n = perm(seed, n, w) for n = first_index .. first_index+count-1.
+ * d_perm_out: device uint8_t[count][w]; row k holds P_{first_index+k}.  2 <= w <= 32; one warp
+ * per permutation (warp Fisher-Yates, one shuffle per swap).  count == 0 is a no-op. */
+rap_status_t rap_perm_gen_batch(uint64_t seed, uint64_t first_index, uint64_t count, uint32_t w,
+                                uint8_t *d_perm_out, void *stream);
 
 /* T1-T3 -- out-of-place transpose staged through 32 x 32 shared-memory tiles in `layout`
  * (§III; RAP layout P:L1005-1023 §IV, RAP CRSW listing P:L1515-1546 §VI):
@@ -124,11 +141,12 @@ rap_status_t rap_perm_gen(uint64_t seed, uint64_t first_index, uint64_t count, u
  * ld_dst >= rows (elements).  elem_bytes in {4, 8}: a raw bit copy (float32/float64 NaN
  * payloads, -0, subnormals are preserved).  The tile layout changes only where an element
  * sits in shared memory, never the result.  RAP uses P = perm(seed, 0, 32), RAS uses
- * r = shifts(seed, 0, 32); seed is ignored by RAW/PAD/XOR.  rows == 0 or cols == 0 is a
+ * r = shifts(seed, 0, 32), both computed on the host at launch (rap_perm_gen); seed is ignored
+ * by RAW/PAD/XOR.  rows == 0 or cols == 0 is a
  * no-op.  Overlapping src/dst -> RAP_ERR_ALIAS.  16-byte aligned src with ld_src a
  * multiple of 16/elem_bytes takes 128-bit loads; anything else takes 32/64-bit loads
- * (still on the GPU).  RAP_LAYOUT_RAP16 (elem_bytes 8 only) is the 64-bit-element
- * ablation of T2b: 64-bit global and shared accesses on a [32][32] double tile. */
+ * (still on the GPU).  RAP_LAYOUT_RAP16 and RAP_LAYOUT_RAP2P (elem_bytes 8 only) are the
+ * 64-bit-element ablations of T2b. */
 rap_status_t rap_transpose(const void *src, void *dst, int64_t rows, int64_t cols,
                            int64_t ld_src, int64_t ld_dst, uint32_t elem_bytes,
                            rap_layout_t layout, uint64_t seed, void *stream);
@@ -156,7 +174,8 @@ rap_status_t rap_transpose_host(const void *h_src, void *h_dst, int64_t rows, in
  * buffers for a one-GPU emulation); ld_dst >= N; G <= 16.  One HBM read and one NVLink write
  * per element; no send/receive buffers, no unpack.  Enqueue only: the caller must make every
  * rank's kernel complete (a cross-rank barrier) before reading its output shard.
- * layout RAW..RAP (RAP_LAYOUT_RAP16 -> RAP_ERR_UNSUPPORTED). */
+ * layout RAW..RAP (RAP16 / RAP2P -> RAP_ERR_UNSUPPORTED); 64-bit elements are staged as two
+ * 32-bit planes here. */
 rap_status_t rap_transpose_to_peers(const void *src, int64_t M, int64_t N, int64_t ld_src,
                                     void *const *peer_dst, uint32_t G, uint32_t rank, int64_t ld_dst,
                                     uint32_t elem_bytes, rap_layout_t layout, uint64_t seed, void *stream);
@@ -179,8 +198,10 @@ rap_status_t rap_congestion(uint32_t w, uint64_t n_warps, const uint32_t *d_rows
  * nsch = popcount(scheme_mask), patterns/schemes in enum order; ACCUMULATED (+=), so the
  * caller zeroes it once and may split a run into any chunks (bit-identical sums).
  * Masks are bit sets of rap_pattern_t / rap_scheme_t (1..31).  XOR needs w = 2^k.
- * 2 <= w <= RAP_MAX_W_SWEEP (256, Table II's widths): w <= 32 maps a DMM warp onto a CUDA warp,
- * 32 < w <= 256 simulates one trial per CUDA thread (NEXT-3; RAP_SWEEP_DEFAULT only). */
+ * 2 <= w <= RAP_MAX_W_SWEEP (256, Table II's widths): w <= 32 maps a DMM warp onto a CUDA warp;
+ * 32 < w <= 256 (NEXT-3; RAP_SWEEP_DEFAULT only) gives a CUDA warp a batch of 32 trials: each
+ * lane runs one trial's Durstenfeld chain, then lane L plays DMM threads L + 32i of one trial at
+ * a time (merged requests by __match_any_sync + a w*w-bit bitmap, bank counts by shared atomics). */
 rap_status_t rap_congestion_sweep(uint32_t w, uint32_t pattern_mask, uint32_t scheme_mask,
                                   uint64_t seed, uint64_t first_trial, uint64_t n_trials,
                                   uint64_t *d_hist, void *stream);
@@ -244,7 +265,8 @@ rap_status_t rap_smem_transpose_bench(uint32_t algorithm, rap_scheme_t scheme, u
  * addresses not known beforehand).  One CTA of 1024 threads applies the
  * tile permutation `reps` times inside shared memory: thread o writes element o (row o/32,
  * contiguous) from source element d_src_index[o] of the previous array (a gather), for
- * o = 0..1023.  d_src_index: device uint16_t[1024], values < 1024 (need not be a permutation).
+ * o = 0..1023.  d_src_index: device uint16_t[1024], values < 1024 (need not be a permutation;
+ * the host cannot validate device data, so the kernel uses each index mod 1024).
  * Layouts: RAW, PAD [32][33], XOR [i][j^i], RAS, RAP; CTA k uses P/r of (seed, k).
  * d_out: device uint32_t[n_blocks][1024] final array (initial value of element o is o), i.e.
  * out[o] = src^reps(o); d_cycles: device uint64_t[n_blocks] SM cycles of the timed loop. */

@@ -6,7 +6,7 @@ memory), the current CUDA stream and the enums.  There is no CPU fallback: calli
 CPU tensor, or without the built library, raises.
 
 Functions keep the C names without the ``rap_`` prefix:
-  hot path      perm_gen, transpose, congestion, congestion_sweep (+ algo), congestion_trace
+  hot path      perm_gen (host), perm_gen_batch, transpose, congestion, congestion_sweep (+ algo), congestion_trace
   host / multi  transpose_host (host-to-host pipeline), unpack_blocks, transpose_to_peers
                 (the multi-GPU drivers are in ``dist``)
   paper §VI/VII smem_transpose_bench (Table III), congestion_sweep4 (§VII, Table IV),
@@ -22,12 +22,12 @@ import torch
 
 from . import build as _build
 
-__all__ = ["perm_gen", "transpose", "transpose_host", "transpose_to_peers", "congestion", "congestion_sweep",
+__all__ = ["perm_gen", "perm_gen_batch", "transpose", "transpose_host", "transpose_to_peers", "congestion", "congestion_sweep",
            "congestion_trace", "unpack_blocks", "smem_transpose_bench", "congestion_sweep4", "smem_gather_bench",
            "LAYOUTS", "SCHEMES", "PATTERNS", "SWEEP_ALGOS", "SMEM_ALGORITHMS", "SCHEMES4", "PATTERNS4",
            "RapError", "lib", "library_path"]
 
-LAYOUTS = {"raw": 0, "pad": 1, "xor": 2, "ras": 3, "rap": 4, "rap16": 5}   # rap16: 8-byte elements only
+LAYOUTS = {"raw": 0, "pad": 1, "xor": 2, "ras": 3, "rap": 4, "rap16": 5, "rap2p": 6}   # rap16/rap2p: 8-byte only
 SCHEMES = {"raw": 0, "ras": 1, "rap": 2, "pad": 3, "xor": 4}
 SWEEP_ALGOS = {"default": 0, "match": 1}
 PATTERNS = {"contiguous": 0, "stride": 1, "diagonal": 2, "random": 3, "malicious": 4}
@@ -65,7 +65,8 @@ def lib():
         L.rap_abi_version.restype = i32
         L.rap_status_str.argtypes = [i32]
         L.rap_status_str.restype = ctypes.c_char_p
-        L.rap_perm_gen.argtypes = [u64, u64, u64, u32, u8p, vp]
+        L.rap_perm_gen.argtypes = [u64, u64, u32, ctypes.POINTER(u32)]
+        L.rap_perm_gen_batch.argtypes = [u64, u64, u64, u32, u8p, vp]
         L.rap_transpose.argtypes = [vp, vp, i64, i64, i64, i64, u32, i32, u64, vp]
         L.rap_congestion.argtypes = [u32, u64, u32p, u32p, i32, u32p, u32p, vp]
         L.rap_congestion_sweep.argtypes = [u32, u32, u32, u64, u64, u64, u64p, vp]
@@ -78,12 +79,12 @@ def lib():
         L.rap_smem_transpose_bench.argtypes = [u32, i32, u32, u64, u32, u32, u32p, u64p, vp]
         L.rap_transpose_to_peers.argtypes = [vp, i64, i64, i64, ctypes.POINTER(ctypes.c_void_p), u32, u32, i64,
                                              u32, i32, u64, vp]
-        for f in ("rap_perm_gen", "rap_transpose", "rap_congestion", "rap_congestion_sweep",
+        for f in ("rap_perm_gen", "rap_perm_gen_batch", "rap_transpose", "rap_congestion", "rap_congestion_sweep",
                   "rap_congestion_sweep_algo", "rap_congestion_trace", "rap_unpack_blocks",
                   "rap_smem_transpose_bench", "rap_transpose_to_peers", "rap_congestion_sweep4",
                   "rap_smem_gather_bench", "rap_transpose_host"):
             getattr(L, f).restype = i32
-        if L.rap_abi_version() != 1:
+        if L.rap_abi_version() != 2:
             raise ImportError("librap.so ABI version mismatch")
         _lib = L
     return _lib
@@ -127,16 +128,24 @@ def _mask(sel, table) -> int:
     return m
 
 
-def perm_gen(seed: int, count: int, w: int = 32, first_index: int = 0,
-             device="cuda", out: torch.Tensor | None = None) -> torch.Tensor:
-    """Permutations P_n = perm(seed, n, w), n = first_index .. +count-1 -> uint8 [count, w]."""
+def perm_gen(seed: int, index: int = 0, w: int = 32) -> list[int]:
+    """P = perm(seed, index, w) computed by the library on the host (rap_perm_gen): the P every
+    transpose launch uses (index 0)."""
+    buf = (ctypes.c_uint32 * w)()
+    _check(lib().rap_perm_gen(seed, index, w, buf), "rap_perm_gen")
+    return list(buf)
+
+
+def perm_gen_batch(seed: int, count: int, w: int = 32, first_index: int = 0,
+                   device="cuda", out: torch.Tensor | None = None) -> torch.Tensor:
+    """Permutations P_n = perm(seed, n, w), n = first_index .. +count-1 -> uint8 [count, w], on the GPU."""
     if out is None:
         out = torch.empty((count, w), dtype=torch.uint8, device=device)
     _need_cuda(out)
     assert out.dtype == torch.uint8 and out.is_contiguous() and out.numel() == count * w
     with _on(out.device):
-        _check(lib().rap_perm_gen(seed, first_index, count, w, ctypes.c_void_p(out.data_ptr()),
-                                  _stream(out)), "rap_perm_gen")
+        _check(lib().rap_perm_gen_batch(seed, first_index, count, w, ctypes.c_void_p(out.data_ptr()),
+                                        _stream(out)), "rap_perm_gen_batch")
     return out
 
 

@@ -6,6 +6,7 @@
 
 #include "../../include/rap.h"
 #include "rap_internal.h"
+#include "rap_rng.cuh"
 
 namespace {
 
@@ -52,8 +53,14 @@ const char *rap_status_str(rap_status_t s) {
     return "RAP_ERR_UNKNOWN";
 }
 
-rap_status_t rap_perm_gen(uint64_t seed, uint64_t first_index, uint64_t count, uint32_t w,
-                          uint8_t *d_perm_out, void *stream) {
+rap_status_t rap_perm_gen(uint64_t seed, uint64_t index, uint32_t w, uint32_t *perm_out) {
+    if (w < 2 || w > RAP_MAX_W_SWEEP || !perm_out) return RAP_ERR_INVALID_ARG;
+    rapk::perm_serial(seed, index, w, perm_out);
+    return RAP_OK;
+}
+
+rap_status_t rap_perm_gen_batch(uint64_t seed, uint64_t first_index, uint64_t count, uint32_t w,
+                                uint8_t *d_perm_out, void *stream) {
     if (w < 2 || w > RAP_MAX_W) return RAP_ERR_INVALID_ARG;
     if (count == 0) return RAP_OK;
     if (!d_perm_out || count > (UINT64_MAX / w)) return RAP_ERR_INVALID_ARG;
@@ -65,8 +72,8 @@ rap_status_t rap_transpose(const void *src, void *dst, int64_t rows, int64_t col
                            int64_t ld_dst, uint32_t elem_bytes, rap_layout_t layout, uint64_t seed,
                            void *stream) {
     if (elem_bytes != 4 && elem_bytes != 8) return RAP_ERR_INVALID_ARG;
-    if ((int)layout < RAP_LAYOUT_RAW || (int)layout > RAP_LAYOUT_RAP16) return RAP_ERR_INVALID_ARG;
-    if (layout == RAP_LAYOUT_RAP16 && elem_bytes != 8) return RAP_ERR_UNSUPPORTED;
+    if ((int)layout < RAP_LAYOUT_RAW || (int)layout > RAP_LAYOUT_RAP2P) return RAP_ERR_INVALID_ARG;
+    if ((layout == RAP_LAYOUT_RAP16 || layout == RAP_LAYOUT_RAP2P) && elem_bytes != 8) return RAP_ERR_UNSUPPORTED;
     if (rows < 0 || cols < 0) return RAP_ERR_INVALID_ARG;
     if (rows == 0 || cols == 0) return RAP_OK;
     if (!src || !dst) return RAP_ERR_INVALID_ARG;
@@ -87,8 +94,8 @@ rap_status_t rap_transpose_host(const void *h_src, void *h_dst, int64_t rows, in
                                 int64_t ld_dst, uint32_t elem_bytes, rap_layout_t layout, uint64_t seed,
                                 void *d_workspace, size_t workspace_bytes, void *stream) {
     if (elem_bytes != 4 && elem_bytes != 8) return RAP_ERR_INVALID_ARG;
-    if ((int)layout < RAP_LAYOUT_RAW || (int)layout > RAP_LAYOUT_RAP16) return RAP_ERR_INVALID_ARG;
-    if (layout == RAP_LAYOUT_RAP16 && elem_bytes != 8) return RAP_ERR_UNSUPPORTED;
+    if ((int)layout < RAP_LAYOUT_RAW || (int)layout > RAP_LAYOUT_RAP2P) return RAP_ERR_INVALID_ARG;
+    if ((layout == RAP_LAYOUT_RAP16 || layout == RAP_LAYOUT_RAP2P) && elem_bytes != 8) return RAP_ERR_UNSUPPORTED;
     if (rows < 0 || cols < 0) return RAP_ERR_INVALID_ARG;
     if (rows == 0 || cols == 0) return RAP_OK;
     if (!h_src || !h_dst || !d_workspace) return RAP_ERR_INVALID_ARG;
@@ -107,8 +114,8 @@ rap_status_t rap_transpose_to_peers(const void *src, int64_t M, int64_t N, int64
                                     void *const *peer_dst, uint32_t G, uint32_t rank, int64_t ld_dst,
                                     uint32_t elem_bytes, rap_layout_t layout, uint64_t seed, void *stream) {
     if (elem_bytes != 4 && elem_bytes != 8) return RAP_ERR_INVALID_ARG;
-    if ((int)layout < RAP_LAYOUT_RAW || (int)layout > RAP_LAYOUT_RAP16) return RAP_ERR_INVALID_ARG;
-    if (layout == RAP_LAYOUT_RAP16) return RAP_ERR_UNSUPPORTED;
+    if ((int)layout < RAP_LAYOUT_RAW || (int)layout > RAP_LAYOUT_RAP2P) return RAP_ERR_INVALID_ARG;
+    if (layout == RAP_LAYOUT_RAP16 || layout == RAP_LAYOUT_RAP2P) return RAP_ERR_UNSUPPORTED;
     if (G < 1 || G > (uint32_t)rapk::kMaxPeers || rank >= G || !peer_dst) return RAP_ERR_INVALID_ARG;
     if (M <= 0 || M % 32 != 0) return RAP_ERR_INVALID_ARG;
     int64_t gm;
@@ -152,11 +159,11 @@ rap_status_t rap_congestion_sweep_algo(uint32_t w, uint32_t pattern_mask, uint32
                                        uint64_t seed, uint64_t first_trial, uint64_t n_trials,
                                        uint64_t *d_hist, uint32_t algo, void *stream) {
     if (w < 2 || w > RAP_MAX_W_SWEEP) return RAP_ERR_INVALID_ARG;
+    if (algo > RAP_SWEEP_MATCH) return RAP_ERR_INVALID_ARG;
     if (w > RAP_MAX_W && algo != RAP_SWEEP_DEFAULT) return RAP_ERR_UNSUPPORTED;
     if (pattern_mask == 0 || pattern_mask > 31u || scheme_mask == 0 || scheme_mask > 31u)
         return RAP_ERR_INVALID_ARG;
     if (((scheme_mask >> RAP_SCHEME_XOR) & 1u) && !is_pow2(w)) return RAP_ERR_INVALID_ARG;
-    if (algo > RAP_SWEEP_MATCH) return RAP_ERR_INVALID_ARG;
     if (n_trials == 0) return RAP_OK;
     if (!d_hist) return RAP_ERR_INVALID_ARG;
     auto launch = w > RAP_MAX_W ? rapk::launch_sweep_wide

@@ -4,12 +4,41 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <atomic>
+
 #include "../../include/rap.h"
 
 namespace rapk {
 
 constexpr int kMaxDevices = 64;
 constexpr int kMaxPeers = 16;
+
+// T0 at launch time: the shift vector of the tile layout, computed once per call on the host
+// (perm_serial / ras_serial of rap_rng.cuh, index 0) and passed to the kernel by value, so no
+// warp spends its prologue on Philox + Fisher-Yates.  RAP: sh = P, inv = P^-1; RAP-16: sh = Q
+// (w = 16) and inv = Q^-1; RAS: sh = r.  Unused for RAW / PAD / XOR.
+struct TileShifts {
+    uint32_t sh[8];    // byte i of the 32-byte vector = sh[i / 4] >> (8 * (i % 4))
+    uint32_t inv[8];
+};
+
+// byte i (< 32) of a packed TileShifts vector: uniform constant-bank words + a per-lane select
+// (a dynamic index into a kernel parameter would copy the struct to local memory)
+__device__ __forceinline__ uint32_t shift_byte(const uint32_t (&w)[8], uint32_t i) {
+    uint32_t x = w[0];
+#pragma unroll
+    for (int k = 1; k < 8; ++k) x = ((i >> 2) == (uint32_t)k) ? w[k] : x;
+    return (x >> (8u * (i & 3u))) & 0xffu;
+}
+TileShifts tile_shifts(int layout, uint64_t seed);
+
+// Launch shape cached per kernel instantiation and device: the dynamic-smem attribute and the
+// occupancy query run once.  `occ` (0 = unknown) is published with release after `sms`, and
+// read with acquire, so a reader that sees occ != 0 also sees sms.
+struct ShapeCache {
+    std::atomic<int> occ[kMaxDevices];
+    std::atomic<int> sms[kMaxDevices];
+};
 
 // Fused-exchange output (NEXT-2): the output shard base of each of the G ranks, as pointers
 // valid in this process (mapped peer memory), M = rows per rank, col_off = rank * M.
@@ -29,6 +58,7 @@ struct TransposeTuning {
     bool vst = false;     // 128-bit output stores (shuffle-transposed) instead of 32/64-bit rows
     bool tma_store = false;  // drain into a dense staging tile, one TMA bulk tensor store per super-tile
     int cl = 1;           // thread-block cluster of cl CTAs stacked along the input rows, drains in lockstep
+    bool force_planes = false;  // 64-bit elements through the two-plane kernel for every layout (tuning A/B)
 };
 // fp32: 4 x 2 warps per CTA, clusters of 4 CTAs (a 16 x 2-tile cluster super-tile);
 // fp64: 12 x 1 warps, no cluster (profiles/r01_tune_transpose*.txt, r01_probe_transpose.txt)
@@ -56,11 +86,42 @@ cudaError_t launch_transpose(const void *src, void *dst, int64_t rows, int64_t c
 cudaError_t launch_transpose_rap16(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
                                    int64_t ld_dst, uint64_t seed, cudaStream_t st);
 
+// 64-bit elements, one element per 8 bytes of the tile (transpose64.cu): layouts RAW..RAP
+cudaError_t launch_transpose64(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
+                               int64_t ld_dst, int layout, uint64_t seed, cudaStream_t st);
+
 cudaError_t launch_transpose_peers(const void *src, int64_t M, int64_t N, int64_t ld_src, const PeerOut &pe,
                                    int64_t ld_dst, uint32_t elem_bytes, int layout, uint64_t seed, cudaStream_t st);
 
 cudaError_t launch_perm_gen(uint64_t seed, uint64_t first, uint64_t count, uint32_t w, uint8_t *out,
                             cudaStream_t st);
+
+// occupancy-capped persistent grid for `want` work units (ShapeCache above)
+template <typename K>
+cudaError_t cached_grid(K kernel, ShapeCache &cache, int threads, size_t smem, int64_t want, int ctas_per_sm,
+                        int *grid_out) {
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    if (dev < 0 || dev >= kMaxDevices) return cudaErrorInvalidDevice;
+    int occ = cache.occ[dev].load(std::memory_order_acquire);
+    int sms = cache.sms[dev].load(std::memory_order_relaxed);
+    if (occ == 0) {
+        e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e != cudaSuccess) return e;
+        e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        if (e != cudaSuccess) return e;
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kernel, threads, smem);
+        if (e != cudaSuccess) return e;
+        if (occ < 1) occ = 1;
+        cache.sms[dev].store(sms, std::memory_order_relaxed);
+        cache.occ[dev].store(occ, std::memory_order_release);
+    }
+    if (ctas_per_sm > 0 && ctas_per_sm < occ) occ = ctas_per_sm;
+    const int64_t cap = (int64_t)sms * occ;
+    *grid_out = (int)(want < cap ? want : cap);
+    return cudaSuccess;
+}
 
 cudaError_t launch_congestion(uint32_t w, uint64_t n_warps, const uint32_t *rows, const uint32_t *cols,
                               int scheme, const uint32_t *shift, uint32_t *out, cudaStream_t st);

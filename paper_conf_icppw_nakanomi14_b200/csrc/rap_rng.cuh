@@ -13,24 +13,34 @@ namespace rapk {
 constexpr unsigned kFull = 0xffffffffu;
 constexpr uint32_t kDomainFY = 0, kDomainRAS = 1, kDomainRandom = 2;
 
-__device__ __forceinline__ uint4 philox4x32_10(uint4 c, uint32_t k0, uint32_t k1) {
+// high word of the 64-bit product (UMULHI on the device); the host build serves rap_perm_gen
+// and the launch-time shift vectors of the transposes (the same functions, not a second copy)
+__host__ __device__ __forceinline__ uint32_t umulhi32(uint32_t a, uint32_t b) {
+#ifdef __CUDA_ARCH__
+    return __umulhi(a, b);
+#else
+    return (uint32_t)(((uint64_t)a * b) >> 32);
+#endif
+}
+
+__host__ __device__ __forceinline__ uint4 philox4x32_10(uint4 c, uint32_t k0, uint32_t k1) {
 #pragma unroll
     for (int round = 0; round < 10; ++round) {
         if (round) { k0 += 0x9E3779B9u; k1 += 0xBB67AE85u; }
-        const uint32_t lo0 = 0xD2511F53u * c.x, hi0 = __umulhi(0xD2511F53u, c.x);
-        const uint32_t lo1 = 0xCD9E8D57u * c.z, hi1 = __umulhi(0xCD9E8D57u, c.z);
+        const uint32_t lo0 = 0xD2511F53u * c.x, hi0 = umulhi32(0xD2511F53u, c.x);
+        const uint32_t lo1 = 0xCD9E8D57u * c.z, hi1 = umulhi32(0xCD9E8D57u, c.z);
         c = make_uint4(hi1 ^ c.y ^ k0, lo1, hi0 ^ c.w ^ k1, lo0);
     }
     return c;
 }
 
 // The 4 words t = 4*blk .. 4*blk+3 of domain d for index n.
-__device__ __forceinline__ uint4 philox_block(uint64_t seed, uint64_t n, uint32_t d, uint32_t blk) {
+__host__ __device__ __forceinline__ uint4 philox_block(uint64_t seed, uint64_t n, uint32_t d, uint32_t blk) {
     return philox4x32_10(make_uint4((uint32_t)n, (uint32_t)(n >> 32), blk, d),
                          (uint32_t)seed, (uint32_t)(seed >> 32));
 }
 
-__device__ __forceinline__ uint32_t pick(uint4 v, uint32_t k) {
+__host__ __device__ __forceinline__ uint32_t pick(uint4 v, uint32_t k) {
     uint32_t x = v.x;
     x = (k == 1) ? v.y : x;
     x = (k == 2) ? v.z : x;
@@ -44,7 +54,31 @@ __device__ __forceinline__ uint32_t word_at(uint64_t seed, uint64_t n, uint32_t 
 }
 
 // floor(u * m / 2^32)
-__device__ __forceinline__ uint32_t mulshift(uint32_t u, uint32_t m) { return __umulhi(u, m); }
+__host__ __device__ __forceinline__ uint32_t mulshift(uint32_t u, uint32_t m) { return umulhi32(u, m); }
+
+// Serial form of T0 (one thread / the host): a = perm(seed, n, w), 2 <= w <= 256, Durstenfeld
+// for k = w-1 .. 1 with j = floor(word(0, w-1-k) * (k+1) / 2^32), swap a[k], a[j].
+__host__ __device__ inline void perm_serial(uint64_t seed, uint64_t n, uint32_t w, uint32_t *a) {
+    for (uint32_t k = 0; k < w; ++k) a[k] = k;
+    uint4 blk = make_uint4(0u, 0u, 0u, 0u);
+    for (uint32_t t = 0; t + 1 < w; ++t) {
+        if ((t & 3u) == 0) blk = philox_block(seed, n, kDomainFY, t >> 2);
+        const uint32_t k = w - 1 - t;
+        const uint32_t j = mulshift(pick(blk, t & 3u), k + 1);
+        const uint32_t x = a[k];
+        a[k] = a[j];
+        a[j] = x;
+    }
+}
+
+// Serial RAS shifts r[i] = floor(word(1, i) * w / 2^32), i < w.
+__host__ __device__ inline void ras_serial(uint64_t seed, uint64_t n, uint32_t w, uint32_t *r) {
+    uint4 blk = make_uint4(0u, 0u, 0u, 0u);
+    for (uint32_t i = 0; i < w; ++i) {
+        if ((i & 3u) == 0) blk = philox_block(seed, n, kDomainRAS, i >> 2);
+        r[i] = mulshift(pick(blk, i & 3u), w);
+    }
+}
 
 // word(seed, n, d, t) for t = lane: each of the first ceil(w/4) lanes computes one Philox
 // block, every lane then picks its word with 4 shuffles.

@@ -90,7 +90,9 @@ smem_gather_kernel(const uint16_t *__restrict__ src_index, uint64_t seed, uint32
     }
     __syncthreads();
     a[lay_index<L>(i, j, sh)] = i * 32u + j;
-    const uint32_t g = src_index[tid];
+    // indices >= 1024 are reduced mod 1024 on the device (the host cannot see device data; an
+    // out-of-range index must not address past the tile, include/rap.h)
+    const uint32_t g = src_index[tid] & 1023u;
     const uint32_t rd = lay_index<L>(g >> 5, g & 31u, sh);
     const uint32_t wr = lay_index<L>(i, j, sh);
     __syncthreads();

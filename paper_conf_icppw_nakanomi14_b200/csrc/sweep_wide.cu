@@ -2,14 +2,18 @@
 // (Table II's w = 64, 128, 256 columns, §V; "the value of w may be increased in
 // future GPUs").
 //
-// A DMM warp of w > 32 threads does not fit one CUDA warp, so here ONE CUDA THREAD SIMULATES ONE
-// TRIAL: it draws its permutation (Durstenfeld on a private array), its RAS shifts and its random
-// cells from the same counter contract as every other kernel (rap_rng.cuh / include/rap.h), then
-// walks the w requests of each (pattern, scheme), counting distinct requests per bank in a private
-// array.  Private arrays live in shared memory laid out [index][thread] (element k of thread t at
-// k*T + t), so at any step the T threads of a CTA touch T consecutive 16-bit slots: no bank
-// conflicts whatever index each thread uses.  Merged requests (random cells) are found once per
-// trial: a request is a leader if no earlier request of the trial has the same cell.
+// Default design (sweep_wide_lane_kernel): a CUDA warp takes a batch of 32 trials.
+// In LANE mode each lane runs the Durstenfeld chain of its own trial on a swizzled [k][32] byte
+// table (conflict-free both for a lane-mode row and a warp-mode column read); in WARP mode lane L
+// plays DMM threads L + 32i of one trial at a time -- Philox words drawn by all lanes, merged
+// requests by __match_any_sync per 32-request slice plus a w^2-bit bitmap across slices, bank
+// counts by shared atomics (the congestion is the largest returned count).
+//
+// The first design, ONE CUDA THREAD PER TRIAL (sweep_wide_kernel below, built with
+// -DRAP_SWEEP_WIDE_THREAD): the thread draws its permutation (Durstenfeld on a private array),
+// its RAS shifts and its random cells from the same counter contract as every other kernel
+// (rap_rng.cuh / include/rap.h), then walks the w requests of each (pattern, scheme), counting
+// distinct requests per bank in a private array laid out [index][thread] in shared memory.
 #include <cuda_runtime.h>
 #include <stdint.h>
 

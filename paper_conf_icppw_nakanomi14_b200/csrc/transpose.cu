@@ -106,7 +106,7 @@ template <int L, int EW, bool VEC, int DEPTH, int MINB, bool VST, int SR, int SC
           int CL = 1>
 __global__ void __launch_bounds__(SR * SC * 32, MINB)
 transpose_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, int64_t rows,
-                 int64_t cols, int64_t ld_src, int64_t ld_dst, uint64_t seed, uint32_t tiles_r,
+                 int64_t cols, int64_t ld_src, int64_t ld_dst, const TileShifts ts, uint32_t tiles_r,
                  uint32_t tiles_c, bool vst_ok, PeerOut peers, const __grid_constant__ CUtensorMap tmap) {
     static_assert(!TMAS || (DEPTH == 1 && !PEERS && SR * 32 <= 256), "TMA store: depth 1, box <= 256");
     static_assert(CL == 1 || (DEPTH == 1 && !TMAS), "cluster lockstep: depth 1, no TMA store");
@@ -118,22 +118,16 @@ transpose_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, i
     uint32_t *tile = smem_dyn + warp * warp_smem_words<L, EW>();
     uint32_t *staging = smem_dyn + SR * SC * warp_smem_words<L, EW>();   // TMAS: (SC*32) x (SR*32) x EW words
 
-    // ---- T0: the per-warp shift vector, lane i holds sh[i] (P[i] for RAP, r[i] for RAS)
+    // ---- T0: the shift vector of the launch (computed once on the host, tile_shifts), lane i
+    // holds sh[i] (P[i] for RAP, r[i] for RAS)
     uint32_t sh_lane = 0;
-    if (L == RAP_LAYOUT_RAP) sh_lane = warp_perm<32>(seed, 0, lane, 32);
-    if (L == RAP_LAYOUT_RAS) sh_lane = warp_ras_shift(seed, 0, lane, 32);
+    if (L == RAP_LAYOUT_RAP || L == RAP_LAYOUT_RAS) sh_lane = shift_byte(ts.sh, lane);
     // load group g: this lane loads tile row row_g[g], chunk q (elements NE*q .. NE*q+NE-1).
     // RAP: the R rows of group g are P^-1(R*g + 0..R-1) -- one row per residue of P mod R --
     // so each STS of the group hits 32 distinct banks.
     const uint32_t q = lane % LPR, c_in = lane / LPR;
     uint32_t row_g[G], a_g[G];
-    uint32_t pinv = lane;
-    if (L == RAP_LAYOUT_RAP) {
-        tile[sh_lane] = lane;
-        __syncwarp();
-        pinv = tile[lane];
-        __syncwarp();
-    }
+    const uint32_t pinv = (L == RAP_LAYOUT_RAP) ? shift_byte(ts.inv, lane) : lane;
 #pragma unroll
     for (int g = 0; g < G; ++g) {
         const uint32_t rr = (uint32_t)(R * g) + c_in;
@@ -359,38 +353,24 @@ transpose_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, i
 }
 
 // ------------------------------------------------------------------ launchers
-// Host-side launch shape, cached per kernel instantiation and device: the dynamic-smem
-// attribute and the occupancy query run once, so a launch costs one cudaGetDevice + one launch.
-struct ShapeCache {
-    std::atomic<int> occ[kMaxDevices];      // 0 = not yet known
-    std::atomic<int> sms[kMaxDevices];
-};
-
-template <typename K>
-static cudaError_t grid_for(K kernel, ShapeCache &cache, int threads, size_t smem, int64_t ntiles,
-                            int warps_per_cta, int ctas_per_sm, int *grid_out) {
-    int dev = 0;
-    cudaError_t e = cudaGetDevice(&dev);
-    if (e != cudaSuccess) return e;
-    if (dev < 0 || dev >= kMaxDevices) return cudaErrorInvalidDevice;
-    int occ = cache.occ[dev].load(std::memory_order_relaxed);
-    int sms = cache.sms[dev].load(std::memory_order_relaxed);
-    if (occ == 0) {
-        e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        if (e != cudaSuccess) return e;
-        e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        if (e != cudaSuccess) return e;
-        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kernel, threads, smem);
-        if (e != cudaSuccess) return e;
-        if (occ < 1) occ = 1;
-        cache.sms[dev].store(sms, std::memory_order_relaxed);
-        cache.occ[dev].store(occ, std::memory_order_relaxed);
+// T0 at launch time: RAP's P (and P^-1) / RAS's r for index 0 of `seed`, on the host (the
+// rap_rng.cuh functions compiled for the host: the same code as every kernel's draws)
+TileShifts tile_shifts(int layout, uint64_t seed) {
+    TileShifts t;
+    uint32_t a[32];
+    memset(&t, 0, sizeof(t));
+    const uint32_t w = layout == RAP_LAYOUT_RAP16 ? 16u : 32u;
+    if (layout == RAP_LAYOUT_RAP || layout == RAP_LAYOUT_RAP2P || layout == RAP_LAYOUT_RAP16) {
+        perm_serial(seed, 0, w, a);
+        for (uint32_t i = 0; i < w; ++i) {
+            t.sh[i / 4] |= a[i] << (8 * (i % 4));
+            t.inv[a[i] / 4] |= i << (8 * (a[i] % 4));
+        }
+    } else if (layout == RAP_LAYOUT_RAS) {
+        ras_serial(seed, 0, w, a);
+        for (uint32_t i = 0; i < w; ++i) t.sh[i / 4] |= a[i] << (8 * (i % 4));
     }
-    if (ctas_per_sm > 0 && ctas_per_sm < occ) occ = ctas_per_sm;
-    const int64_t want = (ntiles + warps_per_cta - 1) / warps_per_cta;
-    const int64_t cap = (int64_t)sms * occ;
-    *grid_out = (int)(want < cap ? want : cap);
-    return cudaSuccess;
+    return t;
 }
 
 TransposeTuning default_tuning(uint32_t elem_bytes) {
@@ -442,7 +422,7 @@ static bool make_out_map(CUtensorMap *m, void *dst, int64_t rows, int64_t cols, 
 template <typename K>
 static cudaError_t launch_clustered(K kernel, ShapeCache &cache, int cl, int threads, size_t smem, int64_t nst,
                                     cudaStream_t st, const uint32_t *src, uint32_t *dst, int64_t rows, int64_t cols,
-                                    int64_t ld_src, int64_t ld_dst, uint64_t seed, uint32_t tiles_r,
+                                    int64_t ld_src, int64_t ld_dst, const TileShifts &ts, uint32_t tiles_r,
                                     uint32_t tiles_c, bool vst_ok, const PeerOut &peers, const CUtensorMap &tmap) {
     int dev = 0;
     cudaError_t e = cudaGetDevice(&dev);
@@ -459,7 +439,7 @@ static cudaError_t launch_clustered(K kernel, ShapeCache &cache, int cl, int thr
     cfg.stream = st;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
-    int ncl = cache.occ[dev].load(std::memory_order_relaxed);   // here: co-resident clusters
+    int ncl = cache.occ[dev].load(std::memory_order_acquire);   // here: co-resident clusters
     if (ncl == 0) {
         e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return e;
@@ -470,11 +450,11 @@ static cudaError_t launch_clustered(K kernel, ShapeCache &cache, int cl, int thr
         e = cudaOccupancyMaxActiveClusters(&ncl, kernel, &cfg);
         if (e != cudaSuccess) return e;
         if (ncl < 1) return cudaErrorInvalidConfiguration;
-        cache.occ[dev].store(ncl, std::memory_order_relaxed);
+        cache.occ[dev].store(ncl, std::memory_order_release);
     }
     const int64_t nclusters = nst < ncl ? nst : ncl;
     cfg.gridDim = dim3((unsigned)(nclusters * cl));
-    e = cudaLaunchKernelEx(&cfg, kernel, src, dst, rows, cols, ld_src, ld_dst, seed, tiles_r, tiles_c, vst_ok,
+    e = cudaLaunchKernelEx(&cfg, kernel, src, dst, rows, cols, ld_src, ld_dst, ts, tiles_r, tiles_c, vst_ok,
                            peers, tmap);
     if (e != cudaSuccess) return e;
     return cudaGetLastError();
@@ -501,14 +481,15 @@ static cudaError_t launch_one(const void *src, void *dst, int64_t rows, int64_t 
     }
     const size_t smem = sizeof(uint32_t) * (warp_smem_words<L, EW>() * SR * SC +
                                             (TMAS ? (size_t)SR * 32 * SC * 32 * EW : 0));
+    const TileShifts ts = tile_shifts(L, seed);
     if (CL > 1)
         return launch_clustered(k, cache, CL, SR * SC * 32, smem, nst, st, (const uint32_t *)src, (uint32_t *)dst,
-                                rows, cols, ld_src, ld_dst, seed, tiles_r, tiles_c, vst_ok, peers, tmap);
+                                rows, cols, ld_src, ld_dst, ts, tiles_r, tiles_c, vst_ok, peers, tmap);
     int grid = 0;
-    const cudaError_t e = grid_for(k, cache, SR * SC * 32, smem, nst, 1, tu.ctas_per_sm, &grid);
+    const cudaError_t e = cached_grid(k, cache, SR * SC * 32, smem, nst, tu.ctas_per_sm, &grid);
     if (e != cudaSuccess) return e;
     k<<<grid, SR * SC * 32, smem, st>>>((const uint32_t *)src, (uint32_t *)dst, rows, cols, ld_src,
-                                        ld_dst, seed, tiles_r, tiles_c, vst_ok, peers, tmap);
+                                        ld_dst, ts, tiles_r, tiles_c, vst_ok, peers, tmap);
     return cudaGetLastError();
 }
 
@@ -553,6 +534,12 @@ template <bool VEC>
 static cudaError_t dispatch(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
                             int64_t ld_dst, uint32_t eb, int layout, uint64_t seed,
                             const TransposeTuning &tu, cudaStream_t st) {
+    // 64-bit elements: one element per 8 bytes of the tile (transpose64.cu) for RAW..RAP; the
+    // round-1 design, two 32-bit planes under the w = 32 RAP map, is layout RAP2P
+    if (eb == 8 && layout == RAP_LAYOUT_RAP2P)
+        return launch_shape<RAP_LAYOUT_RAP, 2, VEC>(src, dst, rows, cols, ld_src, ld_dst, seed, tu, st);
+    if (eb == 8 && !tu.force_planes)
+        return launch_transpose64(src, dst, rows, cols, ld_src, ld_dst, layout, seed, st);
 #define RAPK_CASE(LAY)                                                                             \
     case LAY:                                                                                      \
         return eb == 4 ? launch_shape<LAY, 1, VEC>(src, dst, rows, cols, ld_src, ld_dst, seed, tu, st) \

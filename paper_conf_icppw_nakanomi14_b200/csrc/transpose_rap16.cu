@@ -32,13 +32,13 @@ constexpr int kR16SR = 12;                  // warps (tiles) per CTA, stacked al
 template <int SR>
 __global__ void __launch_bounds__(SR * 32, 1)
 transpose_rap16_kernel(const uint2 *__restrict__ src, uint2 *__restrict__ dst, int64_t rows, int64_t cols,
-                       int64_t ld_src, int64_t ld_dst, uint64_t seed, uint32_t tiles_r, uint32_t tiles_c) {
+                       int64_t ld_src, int64_t ld_dst, const TileShifts ts, uint32_t tiles_r, uint32_t tiles_c) {
     extern __shared__ __align__(16) uint2 smem_r16[];
     const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
     uint2 *tile = smem_r16 + warp * (32 * kR16Pitch);
 
-    // T0: lanes 0..15 hold Q[lane] (Durstenfeld at w = 16, domain 0, index 0)
-    const uint32_t qv = warp_perm<16>(seed, 0, lane, 16);
+    // T0: lanes 0..15 hold Q[lane] (Durstenfeld at w = 16, domain 0, index 0; host, tile_shifts)
+    const uint32_t qv = shift_byte(ts.sh, lane & 15u);
     // T1 offsets: lane j writes row i at i*64 + st_off[i mod 16]
     uint32_t st_off[16];
 #pragma unroll
@@ -113,27 +113,14 @@ cudaError_t launch_transpose_rap16(const void *src, void *dst, int64_t rows, int
     constexpr int SR = kR16SR;
     auto k = transpose_rap16_kernel<SR>;
     const size_t smem = sizeof(uint2) * 32 * kR16Pitch * SR;
-    static int occ_cache[kMaxDevices] = {}, sms_cache[kMaxDevices] = {};
-    int dev = 0;
-    cudaError_t e = cudaGetDevice(&dev);
-    if (e != cudaSuccess) return e;
-    if (dev < 0 || dev >= kMaxDevices) return cudaErrorInvalidDevice;
-    if (occ_cache[dev] == 0) {
-        e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        if (e != cudaSuccess) return e;
-        int sms = 0, occ = 0;
-        e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        if (e != cudaSuccess) return e;
-        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, SR * 32, smem);
-        if (e != cudaSuccess) return e;
-        sms_cache[dev] = sms;
-        occ_cache[dev] = occ < 1 ? 1 : occ;
-    }
+    static ShapeCache cache;
     const uint32_t tiles_r = (uint32_t)((rows + 31) / 32), tiles_c = (uint32_t)((cols + 31) / 32);
     const int64_t nst = (int64_t)((tiles_r + SR - 1) / SR) * tiles_c;
-    const int64_t cap = (int64_t)sms_cache[dev] * occ_cache[dev];
-    const int grid = (int)(nst < cap ? nst : cap);
-    k<<<grid, SR * 32, smem, st>>>((const uint2 *)src, (uint2 *)dst, rows, cols, ld_src, ld_dst, seed, tiles_r,
+    int grid = 0;
+    const cudaError_t e = cached_grid(k, cache, SR * 32, smem, nst, 0, &grid);
+    if (e != cudaSuccess) return e;
+    const TileShifts ts = tile_shifts(RAP_LAYOUT_RAP16, seed);
+    k<<<grid, SR * 32, smem, st>>>((const uint2 *)src, (uint2 *)dst, rows, cols, ld_src, ld_dst, ts, tiles_r,
                                    tiles_c);
     return cudaGetLastError();
 }

@@ -29,15 +29,23 @@ def trial_slice(n_trials: int, rank: int, world: int, first_trial: int = 0):
     return lo, hi - lo
 
 
-def congestion_sweep(n_trials: int, seed: int, group=None, first_trial: int = 0, local=None, **kw):
-    """All-reduced histogram of [first_trial, first_trial + n_trials) swept across the group."""
+def congestion_sweep(n_trials: int, seed: int, group=None, first_trial: int = 0, local=None,
+                     out: torch.Tensor | None = None, **kw):
+    """All-reduced histogram of [first_trial, first_trial + n_trials) swept across the group.
+
+    The ranks sweep into a FRESH zeroed histogram, which is all-reduced and then added to `out`
+    (if given): all-reducing a buffer that already holds counts would multiply them by the world
+    size."""
     on = dist.is_initialized()
     rank, world = (dist.get_rank(group), dist.get_world_size(group)) if on else (0, 1)
     first, count = trial_slice(n_trials, rank, world, first_trial)
     fn = local if local is not None else _sweep
-    h = fn(count, seed, first_trial=first, **kw)
+    h = fn(count, seed, first_trial=first, **kw)          # zero-initialised by the callee
     if world > 1:
         dist.all_reduce(h, op=dist.ReduceOp.SUM, group=group)
+    if out is not None:
+        out.add_(h)
+        return out
     return h
 
 

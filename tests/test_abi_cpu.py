@@ -37,7 +37,7 @@ def test_exports_every_declared_symbol(L):
             "rap_congestion_trace", "rap_status_str", "rap_abi_version"} <= set(names)
     for n in names:
         assert hasattr(L, n), n
-    assert L.rap_abi_version() == 1
+    assert L.rap_abi_version() == 2
 
 
 def test_status_strings(L):
@@ -53,7 +53,8 @@ def test_transpose_validation(L):
     s = P(0)
     assert L.rap_transpose(a, b, 4, 4, 4, 4, 3, 4, 0, s) == INVALID      # elem_bytes
     assert L.rap_transpose(a, b, 4, 4, 4, 4, 4, 9, 0, s) == INVALID      # layout
-    assert L.rap_transpose(a, b, 4, 4, 4, 4, 4, 6, 0, s) == INVALID      # layout
+    assert L.rap_transpose(a, b, 4, 4, 4, 4, 4, 7, 0, s) == INVALID      # layout
+    assert L.rap_transpose(a, b, 4, 4, 4, 4, 4, 6, 0, s) == UNSUPPORTED  # RAP2P needs 8-byte elements
     assert L.rap_transpose(a, b, 4, 4, 4, 4, 4, 5, 0, s) == UNSUPPORTED  # RAP16 needs 8-byte elements
     assert L.rap_transpose(a, b, -1, 4, 4, 4, 4, 4, 0, s) == INVALID     # rows < 0
     assert L.rap_transpose(a, b, 4, 8, 4, 4, 4, 4, 0, s) == INVALID      # ld_src < cols
@@ -71,7 +72,7 @@ def test_valid_calls_fail_loudly_without_gpu(L):
     a, b = P(0x10000000), P(0x20000000)
     assert L.rap_transpose(a, b, 64, 64, 64, 64, 4, 4, 0, P(0)) == CUDA
     assert L.rap_congestion_sweep(32, 31, 7, 1, 0, 1000, P(0x30000000), P(0)) == CUDA
-    assert L.rap_perm_gen(1, 0, 10, 32, P(0x30000000), P(0)) == CUDA
+    assert L.rap_perm_gen_batch(1, 0, 10, 32, P(0x30000000), P(0)) == CUDA
 
 
 def test_sweep_validation(L):
@@ -102,10 +103,25 @@ def test_congestion_trace_perm_validation(L):
     assert L.rap_congestion_trace(32, 4, d, 0, 1, 0, 5, d, s) == INVALID
     assert L.rap_congestion_trace(32, 4, P(0), 7, 1, 0, 5, d, s) == INVALID
     assert L.rap_congestion_trace(32, 0, d, 7, 1, 0, 5, d, s) == OK
-    assert L.rap_perm_gen(1, 0, 4, 33, d, s) == INVALID
-    assert L.rap_perm_gen(1, 0, 4, 1, d, s) == INVALID
-    assert L.rap_perm_gen(1, 0, 4, 32, P(0), s) == INVALID
-    assert L.rap_perm_gen(1, 0, 0, 32, P(0), s) == OK
+    assert L.rap_perm_gen_batch(1, 0, 4, 33, d, s) == INVALID
+    assert L.rap_perm_gen_batch(1, 0, 4, 1, d, s) == INVALID
+    assert L.rap_perm_gen_batch(1, 0, 4, 32, P(0), s) == INVALID
+    assert L.rap_perm_gen_batch(1, 0, 0, 32, P(0), s) == OK
+    buf = (ctypes.c_uint32 * 300)()
+    assert L.rap_perm_gen(1, 0, 1, buf) == INVALID                       # w < 2
+    assert L.rap_perm_gen(1, 0, 257, buf) == INVALID                     # w > 256
+    assert L.rap_perm_gen(1, 0, 32, None) == INVALID
+
+
+@pytest.mark.parametrize("w", [2, 3, 5, 16, 31, 32, 33, 64, 100, 256])
+def test_host_perm_gen_matches_oracle(L, oracle, w):
+    """§8(b) rap_perm_gen (host, the P every transpose launch passes to its kernel) equals the
+    oracle's O3 Durstenfeld permutation for many (seed, index): a pure host call, no GPU."""
+    import numpy as np
+    for seed in (0, 1, 77, (1 << 64) - 1):
+        for index in (0, 1, 2, 12345, (1 << 32) + 7, (1 << 64) - 1):
+            assert np.array_equal(np.array(rap.perm_gen(seed, index, w)), oracle.perm(seed, index, w)), \
+                (seed, index, w)
 
 
 def test_smem_bench_and_unpack_validation(L):

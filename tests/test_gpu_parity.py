@@ -39,10 +39,21 @@ def bits(t):
 @pytest.mark.parametrize("w", [2, 3, 5, 16, 31, 32])
 def test_perm_gen_matches_oracle(rap, oracle, w):
     first, count = 12345678901, 3000
-    P = rap.perm_gen(seed=77, count=count, w=w, first_index=first).cpu().numpy()
-    for k in range(0, count, 7):
+    P = rap.perm_gen_batch(seed=77, count=count, w=w, first_index=first).cpu().numpy()
+    for k in range(count):
         assert np.array_equal(P[k], oracle.perm(77, first + k, w).astype(np.uint8)), k
     assert all(sorted(row) == list(range(w)) for row in P.tolist())
+
+
+def test_perm_gen_batch_1e6_indices(rap, oracle):
+    """10^6 consecutive indices (straddling 2^32, so the counter's high word changes) at w = 32,
+    every permutation compared with the oracle's O3, and the host call (rap_perm_gen) agrees."""
+    first, count = (1 << 32) - 500_000, 1_000_000
+    P = rap.perm_gen_batch(seed=3, count=count, w=32, first_index=first).cpu().numpy()
+    for k in range(count):
+        assert np.array_equal(P[k], oracle.perm(3, first + k, 32)), k
+    for k in range(0, count, 9973):
+        assert rap.perm_gen(3, first + k, 32) == P[k].tolist()
 
 
 # ------------------------------------------------------------------ T1-T3 transpose
@@ -92,6 +103,11 @@ def test_transpose_result_independent_of_seed(rap):
         assert torch.equal(rap.transpose(x, layout="rap", seed=s).view(torch.int32), ref.view(torch.int32))
 
 
+def _full_check(oracle, x_dev, y_dev):
+    """Every element: the oracle transposes the whole matrix (multi-threaded plain loops)."""
+    assert np.array_equal(bits(y_dev), oracle.transpose(bits(x_dev), threads=oracle.max_threads()))
+
+
 def _band_check(oracle, x_dev, y_dev, n_bands=6, band=48, seed=0):
     """Full-size check on sampled row bands: the oracle transposes each band of x."""
     rows, cols = x_dev.shape
@@ -109,10 +125,7 @@ def test_transpose_cfg3_8192_f32(rap, oracle, layout):
     x = workloads.random_bits(8192, 8192, torch.float32, seed=0, device="cuda")
     y = rap.transpose(x, layout=layout, seed=0)
     torch.cuda.synchronize()
-    if layout == "rap":
-        assert np.array_equal(bits(y), oracle.transpose(bits(x), threads=oracle.max_threads()))
-    else:
-        _band_check(oracle, x, y, seed=1)
+    _full_check(oracle, x, y)
     # property at any size: transposing twice is the identity (bit-exact)
     z = rap.transpose(y, layout=layout, seed=1)
     assert torch.equal(z.view(torch.int32), x.view(torch.int32))
@@ -141,16 +154,48 @@ def test_transpose_extreme_aspect(rap, oracle, shape):
     assert np.array_equal(bits(y), oracle.transpose(bits(x), threads=oracle.max_threads()))
 
 
-def test_transpose_cfg4_16384_f64(rap, oracle):
+@pytest.mark.parametrize("layout", ["rap", "rap2p", "rap16"])
+def test_transpose_cfg4_16384_f64(rap, oracle, layout):
+    # BASELINE cfg4 at full size, in the launch configuration bench.py times: all 2^28 doubles
+    # compared with the oracle (rap: the paper's w = 32 map on 8-byte slots, the headline;
+    # rap2p: two 32-bit planes; rap16: RAP over 16 double banks)
     x = workloads.random_bits(16384, 16384, torch.float64, seed=0, device="cuda")
-    y = rap.transpose(x, layout="rap", seed=0)
+    y = rap.transpose(x, layout=layout, seed=0)
     torch.cuda.synchronize()
-    _band_check(oracle, x, y, n_bands=4, band=40, seed=2)
-    del x
-    # column bands too (output rows)
-    xs = workloads.random_bits(16384, 16384, torch.float64, seed=0, device="cuda")
-    for c0 in (0, 7777, 16384 - 33):
-        assert np.array_equal(bits(y[c0:c0 + 33]), oracle.transpose(bits(xs[:, c0:c0 + 33])))
+    _full_check(oracle, x, y)
+    z = rap.transpose(y, layout=layout, seed=9)
+    assert torch.equal(z.view(torch.int64), x.view(torch.int64))
+
+
+@pytest.mark.parametrize("layout", ["raw", "pad", "xor", "ras"])
+def test_transpose_cfg4_16384_f64_baselines(rap, layout):
+    # the baseline layouts on 8-byte slots at cfg4 size: equal to the RAP result (itself
+    # checked in full against the oracle above) and an involution
+    x = workloads.random_bits(16384, 16384, torch.float64, seed=0, device="cuda")
+    ref = rap.transpose(x, layout="rap", seed=0)
+    y = rap.transpose(x, layout=layout, seed=3)
+    assert torch.equal(y.view(torch.int64), ref.view(torch.int64))
+
+
+def test_transpose64_seeds_and_ragged(rap, oracle):
+    # the 8-byte-slot kernel under many P (the P^-1 row grouping and drain lanes depend on P)
+    # on ragged shapes spanning several 12-warp super-tiles
+    for i, (r, c) in enumerate([(385, 33), (31, 1025), (800, 417), (1024, 96)]):
+        x = workloads.random_bits(r, c, torch.float64, seed=200 + i)
+        for seed in (0, 1, 2, 3, 12345, 2 ** 64 - 1):
+            y = rap.transpose(x.cuda(), layout="rap", seed=seed)
+            torch.cuda.synchronize()
+            assert np.array_equal(bits(y), oracle.transpose(bits(x))), (r, c, seed)
+
+
+def test_transpose_rap2p_shapes(rap, oracle):
+    for i, (r, c) in enumerate(SHAPES + [(384, 64), (385, 33)]):
+        x = workloads.random_bits(r, c, torch.float64, seed=300 + i)
+        y = rap.transpose(x.cuda(), layout="rap2p", seed=i)
+        torch.cuda.synchronize()
+        assert np.array_equal(bits(y), oracle.transpose(bits(x))), (r, c)
+    with pytest.raises(rap.RapError, match="UNSUPPORTED"):
+        rap.transpose(torch.zeros((64, 64), device="cuda"), layout="rap2p")
 
 
 # T2b (ii): the RAP-16 double tile (8-byte elements only)
@@ -177,16 +222,6 @@ def test_transpose_rap16_strided(rap, oracle):
 def test_transpose_rap16_rejects_32bit(rap):
     with pytest.raises(rap.RapError, match="UNSUPPORTED"):
         rap.transpose(torch.zeros((64, 64), device="cuda"), layout="rap16")
-
-
-def test_transpose_rap16_cfg4_16384_f64(rap, oracle):
-    # cfg4 at full size through the RAP-16 ablation (the launch bench.py --workload cfg4 times)
-    x = workloads.random_bits(16384, 16384, torch.float64, seed=0, device="cuda")
-    y = rap.transpose(x, layout="rap16", seed=0)
-    torch.cuda.synchronize()
-    _band_check(oracle, x, y, n_bands=4, band=40, seed=3)
-    ref = rap.transpose(x, layout="rap", seed=0)
-    assert torch.equal(y.view(torch.int64), ref.view(torch.int64))
 
 
 def test_transpose_cfg1_tile(rap, oracle):
@@ -434,12 +469,8 @@ def test_sharded_transpose_emulated_on_one_gpu(rap, oracle, dtype, G, M):
 
 
 def _cfg5_check(oracle, A, got, seed):
-    """32768^2 check on sampled bands: output rows (= input columns) and output columns (= input
-    rows) both go through the oracle, plus the first/last 33 of each."""
-    _band_check(oracle, A, got, n_bands=3, band=40, seed=seed)
-    N = A.shape[1]
-    for c0 in (0, 12345, N - 33):
-        assert np.array_equal(bits(got[c0:c0 + 33]), oracle.transpose(bits(A[:, c0:c0 + 33]))), c0
+    """32768^2 check of every element: the oracle transposes the whole 4 GiB matrix."""
+    _full_check(oracle, A, got)
 
 
 @pytest.mark.parametrize("G", [2, 4, 8])

@@ -20,15 +20,15 @@ for dt in (torch.float32, torch.float64):
     for (r, c) in ((33, 65), (96, 200), (256, 256)):
         x = workloads.random_bits(r, c, dt, seed=1).to(dev)
         for lay in rap.LAYOUTS:
-            if lay == "rap16" and dt == torch.float32:
+            if lay in ("rap16", "rap2p") and dt == torch.float32:
                 continue
             y = rap.transpose(x, layout=lay, seed=3)
             assert torch.equal(y.cpu().view(torch.int32 if dt == torch.float32 else torch.int64),
                                x.cpu().t().contiguous().view(torch.int32 if dt == torch.float32 else torch.int64))
     xs = workloads.random_bits(100, 64, dt, seed=2).to(dev)[:, 1:60]
     rap.transpose(xs, layout="rap")
-rap.perm_gen(seed=1, count=100, w=32)
-rap.perm_gen(seed=1, count=10, w=7)
+rap.perm_gen_batch(seed=1, count=100, w=32)
+rap.perm_gen_batch(seed=1, count=10, w=7)
 rap.congestion_sweep(5000, seed=1)
 rap.congestion_sweep(5000, seed=1, schemes=("raw", "ras", "rap", "pad", "xor"))
 rap.congestion_sweep(3000, seed=1, w=7, schemes=("raw", "ras", "rap", "pad"))
