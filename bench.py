@@ -1,23 +1,33 @@
 """bench.py -- RAP hot path on B200: one JSON line per run (driver contract).
 
-A step is one pass of the whole hot path over one batch of synthetic input:
-  T0-T3  RAP transpose of the BASELINE cfg3 matrix (8192 x 8192 float32, out-of-place; input
-         and output are 256 MiB each, larger than the 126 MB L2, so no flush between steps),
-  C1-C4  one batch of the cfg2 congestion sweep (w = 32, 5 patterns x RAW/RAS/RAP,
-         --sweep-trials per rank per step; counter-based, so batches are disjoint trial ranges
-         that continue across steps), and on N > 1 ranks the NCCL all-reduce of the histogram.
-`value` is the headline transpose throughput (GB/s, whole job): algorithmic bytes (read once +
-write once) of all ranks / the transpose device time inside the timed steps (CUDA events on
-the launching stream, max over ranks).  The sweep is reported beside it (`sweep`).
+Default step (BASELINE configs; DESIGN.md §7 "Measurement"): one pass of the whole hot path --
+  T0-T3  RAP transpose of the cfg4 matrix: 16384 x 16384 float64 (the paper's 64-bit doubles,
+         P:L855-866), out-of-place, RAP = the w = 32 map on 8-byte tile slots; input and output
+         are 2 GiB each (> the 126 MB L2: no flush between steps);
+  C1-C4  a slice of the cfg2 congestion sweep (w = 32, 5 patterns x RAW/RAS/RAP, seed 1): the K
+         timed steps sweep trials [0, 10^9) between them, so the run's histogram is the full
+         cfg2 result and is compared with the oracle's stored 10^9-trial histogram
+         (tests/golden/sweep_w32_1e9_seed1.txt, written from oracle/ only);
+  (N > 1) the NCCL all-reduce of each step's sweep histogram.
+`value` = the cfg4 transpose (GB/s, whole job): algorithmic bytes (read once + write once) of all
+ranks / mean transpose device time per step (CUDA events on the launching stream, max over
+ranks); `roofline` is that kernel's, on the same mean.  Sub-objects timed in the same run:
+  `sweep`       the 10^9-trial cfg2 sweep (trials/s, ALU roofline, parity with the golden file);
+  `cfg3_layouts` cfg3 8192^2 float32 under RAW / PAD / XOR / RAS / RAP (back-to-back launches);
+  `cfg4_layouts` cfg4 under every 64-bit layout (8-byte slots, RAP2P two planes, RAP-16);
+each with its roofline and `cpu_baseline` (the oracle, all cores and one core, same sample
+definition as the reference arm).
 
---workload picks another timed step: sweep (cfg2 only; value = trials/s), cfg4 (16384^2
-float64 transpose), tile (cfg1 32 x 32), layouts (cfg3 under raw/pad/xor/ras/rap; value =
-RAP), dist (cfg5: 32768^2 float32 row-block-sharded over the ranks, NCCL all-to-all).
+--workload picks another timed step: cfg3 (the round-1 default: cfg3 transpose + a sweep
+batch), sweep (cfg2 only; value = trials/s), cfg4 (cfg4 alone with the 64-bit ablations), tile
+(cfg1 32 x 32), layouts (cfg3 under the five layouts), dist / dist_fused (cfg5 32768^2 float32
+row-block-sharded over the ranks: NCCL all-to-all / fused peer stores), trace (access traces).
 --impl reference times the CPU oracle (the only reference this paper has: it publishes no
 code) on a bounded sample of the same workload on the host cores; rank 0 only.
 
-N > 1 (torchrun, one process per GPU): every rank transposes its own cfg3 matrix (replicas,
-weak scaling) and sweeps its own trial batch; `dist` shards one matrix (strong scaling).
+N > 1 (torchrun, one process per GPU): every rank transposes its own cfg4 matrix (replicas,
+weak scaling) and sweeps its slice of each step's trial batch (the 10^9 trials are split over
+the ranks; one all-reduce per step); `dist` shards one matrix (strong scaling).
 """
 from __future__ import annotations
 
@@ -36,6 +46,11 @@ METRIC = "RAP transpose GB/s vs HBM peak; smem wavefronts/request; congestion tr
 ALL_PAT = ["contiguous", "stride", "diagonal", "random", "malicious"]
 SCH = ["raw", "ras", "rap"]
 NVLINK_GBS = 770.0   # measured peer copy per direction (B200_PROFILING.md); 900 nominal
+SWEEP_TOTAL = 10 ** 9          # cfg2: trials swept by the default run's timed steps
+SWEEP_SEED = 1
+CFG3_LAYOUTS = ["raw", "pad", "xor", "ras", "rap"]
+CFG4_LAYOUTS = ["raw", "pad", "xor", "ras", "rap", "rap2p", "rap16"]
+ORACLE_BAND_BYTES = 32 << 20   # the oracle's transpose sample: one row band of this many bytes
 
 
 # The JSON line goes to the process's original stdout; everything else that native code prints
@@ -62,17 +77,15 @@ def route_native_stdout_to_stderr():
 def parse(argv=None):
     p = argparse.ArgumentParser()
     p.add_argument("--gpus", type=int, default=1)
-    p.add_argument("--steps", type=int, default=50)
+    p.add_argument("--steps", type=int, default=20)
     p.add_argument("--warmup", type=int, default=5)
     p.add_argument("--impl", default="mine", choices=["mine", "reference"])
     p.add_argument("--workload", default="default",
-                   choices=["default", "sweep", "trace", "cfg4", "tile", "layouts", "dist", "dist_fused"])
-    # default workload: one batch of 32 trials for every resident warp of the sweep kernel on a
-    # B200 (148 SMs x 8 CTAs x 4 warps), so the cfg3 transpose stays the larger share of the step
-    # (the step's `value` and `roofline` are the transpose's).  One batch per warp runs the sweep
-    # below its steady rate (launch ramp and tail of a single wave).  `--workload sweep` (cfg2)
-    # defaults to 64 batches per warp (9.7 M trials, ~3 ms per step): the steady rate, as the
-    # 10^9-trial cfg2 run sees it.
+                   choices=["default", "cfg3", "sweep", "trace", "cfg4", "tile", "layouts", "dist", "dist_fused"])
+    # --workload cfg3: one batch of 32 trials for every resident warp of the sweep kernel on a
+    # B200 (148 SMs x 8 CTAs x 4 warps) per step.  `--workload sweep` (cfg2) defaults to 64
+    # batches per warp (9.7 M trials, ~3 ms per step): the steady rate.  The default workload
+    # sweeps ceil(10^9 / steps) trials per step instead.
     p.add_argument("--sweep-trials", type=int, default=None)
     # --workload trace: each of the 4096 trace warps evaluated under this many trials per step
     # (2048: a 0.6 ms launch, past the launch ramp; 256 trials run at ~80 % of that rate)
@@ -83,7 +96,10 @@ def parse(argv=None):
     p.add_argument("--no-cpu", action="store_true")
     a = p.parse_args(argv)
     if a.sweep_trials is None:
-        a.sweep_trials = 148 * 8 * 4 * 32 * (64 if a.workload == "sweep" else 1)
+        if a.workload == "default":
+            a.sweep_trials = -(-SWEEP_TOTAL // max(a.steps, 1))
+        else:
+            a.sweep_trials = 148 * 8 * 4 * 32 * (64 if a.workload == "sweep" else 1)
     return a
 
 
@@ -106,6 +122,23 @@ def load_profile(kernel_key: str):
     if not os.path.exists(path):
         return None
     return json.load(open(path)).get("kernels", {}).get(kernel_key)
+
+
+def host_cpu() -> dict:
+    """The host the oracle runs on: model name, logical CPUs, CPUs this process may use."""
+    model = None
+    try:
+        for ln in open("/proc/cpuinfo"):
+            if ln.startswith("model name"):
+                model = ln.split(":", 1)[1].strip()
+                break
+    except OSError:
+        pass
+    try:
+        usable = len(os.sched_getaffinity(0))
+    except AttributeError:
+        usable = os.cpu_count()
+    return {"cpu_model": model, "nproc": usable, "logical_cpus": os.cpu_count()}
 
 
 class Clocks:
@@ -154,9 +187,20 @@ class Clocks:
                        "samples": len(sm), "window": "timed steps + 0.3 s of identical untimed steps each side"}
 
 
+def clocks_bad(c: dict) -> bool:
+    """A timed region that saw thermal / hardware slowdown, or SM clocks well below max with no
+    reason given (a leftover clock lock), is measured once more."""
+    bad = bool(set(c.get("reasons") or []) & {"hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown"})
+    return bad or bool(c.get("sm_mhz") and c.get("sm_max_mhz") and not c.get("reasons")
+                       and c["sm_mhz"] < 0.85 * c["sm_max_mhz"])
+
+
 # ---------------------------------------------------------------------------- workload config
-DESC = {"default": "cfg3 8192x8192 float32 RAP transpose + cfg2 w=32 sweep batch",
-        "cfg4": "cfg4 16384x16384 float64 RAP transpose (two 32-bit RAP planes)",
+DESC = {"default": "cfg4 16384x16384 float64 RAP transpose (w=32 map on 8-byte tile slots) + cfg2 w=32 "
+                   "sweep slice per step (10^9 trials over the timed steps); sub-objects: cfg2 sweep, "
+                   "cfg3 8192x8192 float32 under raw/pad/xor/ras/rap, cfg4 under every 64-bit layout",
+        "cfg3": "cfg3 8192x8192 float32 RAP transpose + cfg2 w=32 sweep batch",
+        "cfg4": "cfg4 16384x16384 float64 RAP transpose (w=32 map on 8-byte tile slots)",
         "tile": "cfg1 32x32 float32 RAP tile (latency case)",
         "layouts": "cfg3 8192x8192 float32 transpose under 5 smem layouts",
         "dist": "cfg5 32768x32768 float32 row-block-sharded transpose over {world} GPU(s), NCCL all-to-all",
@@ -167,6 +211,17 @@ DESC = {"default": "cfg3 8192x8192 float32 RAP transpose + cfg2 w=32 sweep batch
                  "anti-diagonal / permutation / random) under RAW, RAS, RAP, PAD, XOR"}
 
 
+def transpose_shape(wl: str, world: int):
+    """(rows per rank, cols, elem_bytes) of the workload's timed transpose."""
+    if wl in ("default", "cfg4"):
+        return 16384, 16384, 8
+    if wl == "tile":
+        return 32, 32, 4
+    if wl in ("dist", "dist_fused"):
+        return 32768 // world, 32768, 4
+    return 8192, 8192, 4
+
+
 def arm_config(args, world: int) -> dict:
     """The `config` object of the JSON line for args.workload -- one definition for both arms."""
     wl = args.workload
@@ -175,10 +230,8 @@ def arm_config(args, world: int) -> dict:
                 "parallelism": f"trial ranges x{world} + NCCL all-reduce" if world > 1 else "single GPU"}
     if wl == "trace":
         return {"workload": DESC[wl], "trials_per_step": args.trace_trials, "warps": 4096, "schemes": 5}
-    n = {"cfg4": 16384, "tile": 32, "dist": 32768, "dist_fused": 32768}.get(wl, 8192)
-    eb = 8 if wl == "cfg4" else 4
-    lay = "rap" if wl in ("layouts", "cfg4") else args.layout
-    rows_rank = n // world if wl in ("dist", "dist_fused") else n
+    rows_rank, n, eb = transpose_shape(wl, world)
+    lay = "rap" if wl in ("layouts", "cfg4", "default") else args.layout
     nbytes = 2 * rows_rank * n * eb
     cfg = {"workload": DESC[wl].format(world=world), "rows": n, "cols": n, "elem_bytes": eb, "layout": lay,
            "parallelism": (f"row blocks + NCCL all-to-all, {world} ranks" if wl == "dist"
@@ -187,9 +240,85 @@ def arm_config(args, world: int) -> dict:
            "l2": ("inputs larger than L2 (no flush)" if nbytes // 2 > 126e6
                   else "input fits in L2 (no flush; latency case)"),
            "algorithmic_bytes_per_step_per_rank": nbytes}
-    if wl == "default":
+    if wl == "cfg3":
         cfg["sweep_trials_per_step"] = args.sweep_trials * world
+    if wl == "default":
+        cfg["sweep_trials_per_step"] = args.sweep_trials
+        cfg["sweep_trials_total"] = min(SWEEP_TOTAL, args.sweep_trials * args.steps)
+        cfg["sweep_seed"] = SWEEP_SEED
     return cfg
+
+
+# ---------------------------------------------------------------------------- oracle timing
+def oracle_band(rows: int, cols: int, eb: int) -> int:
+    """Rows of the oracle's transpose sample: one band of ORACLE_BAND_BYTES (both arms)."""
+    return max(1, min(rows, ORACLE_BAND_BYTES // (cols * eb)))
+
+
+def oracle_transpose_sample(rows: int, cols: int, dt):
+    import workloads
+    band = oracle_band(rows, cols, workloads_eb(dt))
+    return workloads.as_bits_numpy(workloads.random_bits(band, cols, dt, seed=0)), band
+
+
+def workloads_eb(dt) -> int:
+    import torch
+    return torch.empty((), dtype=dt).element_size()
+
+
+def rate_for(fn, work: float, seconds: float):
+    """Calls fn() for `seconds` (after one untimed call); returns (work per second, calls, elapsed)."""
+    fn()
+    reps, t0 = 0, time.perf_counter()
+    while True:
+        fn()
+        reps += 1
+        el = time.perf_counter() - t0
+        if el >= seconds:
+            return work * reps / el, reps, el
+
+
+def cpu_baseline_transpose(rows, cols, dt, seconds: float = 3.0):
+    """The oracle's naive transpose on one row band of the matrix: all cores (value) and one core."""
+    import oracle
+    threads = oracle.max_threads()
+    x, band = oracle_transpose_sample(rows, cols, dt)
+    gb = 2 * x.nbytes / 1e9
+    v_all, n_all, t_all = rate_for(lambda: oracle.transpose(x, threads=threads), gb, seconds)
+    v_one, n_one, t_one = rate_for(lambda: oracle.transpose(x, threads=1), gb, seconds)
+    return dict({"value": v_all, "unit": "GB/s", "cores": threads, "kind": "oracle",
+                 "sample": f"{band} x {cols} row band ({x.nbytes >> 20} MiB) of the {rows}x{cols} "
+                           f"{str(dt)[6:]} matrix, naive oracle transpose; {n_all} calls in {t_all:.1f} s "
+                           f"on {threads} threads, {n_one} in {t_one:.1f} s on 1",
+                 "value_single_thread": v_one}, **host_cpu())
+
+
+def cpu_baseline_tile(seconds: float = 1.0):
+    """cfg1: the oracle transposing one 32 x 32 float32 tile (per-call time, one thread)."""
+    import oracle
+    import torch
+    import workloads
+    x = workloads.as_bits_numpy(workloads.random_bits(32, 32, torch.float32, seed=0))
+    v, n, el = rate_for(lambda: oracle.transpose(x, threads=1), 1.0, seconds)
+    return {"us_per_tile": 1e6 / v, "cores": 1, "kind": "oracle",
+            "sample": f"32x32 float32 tile, {n} oracle calls in {el:.1f} s (includes the ctypes call)"}
+
+
+def cpu_baseline_sweep(seconds: float = 3.0):
+    import oracle
+    threads = oracle.max_threads()
+    n = 20000
+    k = [0]
+
+    def run(th):
+        oracle.sweep(32, ALL_PAT, SCH, SWEEP_SEED, k[0] * n, n, threads=th)
+        k[0] += 1
+    v_all, n_all, t_all = rate_for(lambda: run(threads), n, seconds)
+    v_one, n_one, t_one = rate_for(lambda: run(1), n, seconds)
+    return dict({"value": v_all, "unit": "trials/s", "cores": threads, "kind": "oracle",
+                 "sample": f"w=32 sweep (5 patterns x RAW/RAS/RAP), {n}-trial chunks: {n_all} in {t_all:.1f} s "
+                           f"on {threads} threads, {n_one} in {t_one:.1f} s on 1",
+                 "value_single_thread": v_one}, **host_cpu())
 
 
 # ---------------------------------------------------------------------------- reference arm
@@ -201,14 +330,13 @@ def run_reference(args):
     import torch
 
     import oracle
-    import workloads
     threads = oracle.max_threads()
     wl = args.workload
     cfg = arm_config(args, world)          # the same workload / config as our arm's line
     n_sw = 20000                           # oracle sweep sample: trials per step
 
     def sweep_sample(k):
-        oracle.sweep(32, ALL_PAT, SCH, 1, k * n_sw, n_sw, threads=threads)
+        oracle.sweep(32, ALL_PAT, SCH, SWEEP_SEED, k * n_sw, n_sw, threads=threads)
 
     sweep_s = 0.0
     if wl == "sweep":
@@ -218,21 +346,20 @@ def run_reference(args):
         fn, work, what = oracle_trace_sample()
         unit = "warp-evaluations/s"
     else:
-        rows, cols, dt = {"cfg4": (16384, 16384, torch.float64), "dist": (32768, 32768, torch.float32),
-                          "dist_fused": (32768, 32768, torch.float32),
-                          "tile": (32, 32, torch.float32)}.get(wl, (8192, 8192, torch.float32))
-        band = min(rows, 512)
-        x = workloads.as_bits_numpy(workloads.random_bits(band, cols, dt, seed=0))
+        rows_rank, cols, eb = transpose_shape(wl, 1)
+        dt = torch.float64 if eb == 8 else torch.float32
+        x, band = oracle_transpose_sample(rows_rank, cols, dt)
         unit = "GB/s"
-        what = f"{band} x {cols} row band of the {rows}x{cols} {str(dt)[6:]} matrix per step, naive oracle transpose"
-        if wl == "default":
+        what = (f"{band} x {cols} row band ({x.nbytes >> 20} MiB) of the {rows_rank}x{cols} {str(dt)[6:]} matrix "
+                f"per step, naive oracle transpose on {threads} threads")
+        if wl in ("default", "cfg3"):
             what += f"; plus {n_sw} oracle sweep trials per step, timed apart (`sweep`)"
         work = 2 * x.nbytes / 1e9
 
         def fn(k):
             nonlocal sweep_s
             oracle.transpose(x, threads=threads)
-            if wl == "default":                  # the step's second half, timed apart like our arm's
+            if wl in ("default", "cfg3"):        # the step's second half, timed apart like our arm's
                 t = time.perf_counter()
                 sweep_sample(k)
                 sweep_s += time.perf_counter() - t
@@ -247,31 +374,14 @@ def run_reference(args):
     line = {"impl": "reference", "metric": METRIC, "value": value, "unit": unit, "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": el / args.steps * 1e3,
             "higher_is_better": True, "scaling": "strong" if wl in ("dist", "dist_fused") else "weak",
-            "vs_baseline": None, "dtype": "u64" if wl == "cfg4" else "u32", "data": "synthetic", "config": cfg,
-            "cpu_baseline": {"value": value, "unit": unit, "cores": 1 if wl == "trace" else threads, "kind": "oracle",
-                             "sample": what},
+            "vs_baseline": None, "dtype": "u64" if wl in ("cfg4", "default") else "u32", "data": "synthetic",
+            "config": cfg,
+            "cpu_baseline": dict({"value": value, "unit": unit, "cores": 1 if wl == "trace" else threads,
+                                  "kind": "oracle", "sample": what}, **host_cpu()),
             "e2e": {"value": value, "unit": unit, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
-    if wl == "default":
+    if wl in ("default", "cfg3"):
         line["sweep"] = {"trials_per_s": n_sw * args.steps / sweep_s, "trials_per_step": n_sw}
     emit(line)
-
-
-# ---------------------------------------------------------------------------- helpers
-def cpu_baseline_transpose(rows, cols, dt):
-    import oracle
-    import workloads
-    threads = oracle.max_threads()
-    band = min(rows, 1024)
-    x = workloads.as_bits_numpy(workloads.random_bits(band, cols, dt, seed=0))
-    oracle.transpose(x, threads=threads)
-    reps, t0 = 0, time.perf_counter()
-    while time.perf_counter() - t0 < 3.0:
-        oracle.transpose(x, threads=threads)
-        reps += 1
-    el = time.perf_counter() - t0
-    return {"value": 2 * x.nbytes * reps / el / 1e9, "unit": "GB/s", "cores": threads, "kind": "oracle",
-            "sample": f"{band} x {cols} row band of the {rows}x{cols} matrix, naive oracle transpose, "
-                      f"{reps} reps in {el:.1f} s"}
 
 
 def oracle_trace_sample():
@@ -294,26 +404,15 @@ def oracle_trace_sample():
 
 def cpu_baseline_trace():
     fn, work, what = oracle_trace_sample()
-    fn(0)
-    reps, t0 = 0, time.perf_counter()
-    while time.perf_counter() - t0 < 3.0:
-        fn(reps)
-        reps += 1
-    el = time.perf_counter() - t0
-    return {"value": work * reps / el, "unit": "warp-evaluations/s", "cores": 1, "kind": "oracle",
-            "sample": f"{what}; {reps} calls in {el:.1f} s (single thread: one ctypes call per evaluation)"}
+    k = [0]
 
-
-def cpu_baseline_sweep():
-    import oracle
-    threads = oracle.max_threads()
-    n, reps, t0 = 20000, 0, time.perf_counter()
-    while time.perf_counter() - t0 < 3.0:
-        oracle.sweep(32, ALL_PAT, SCH, 1, reps * n, n, threads=threads)
-        reps += 1
-    el = time.perf_counter() - t0
-    return {"value": n * reps / el, "unit": "trials/s", "cores": threads, "kind": "oracle",
-            "sample": f"{n * reps} trials of the w=32 sweep (5 patterns x RAW/RAS/RAP) in {el:.1f} s"}
+    def call():
+        fn(k[0])
+        k[0] += 1
+    v, reps, el = rate_for(call, work, 3.0)
+    return dict({"value": v, "unit": "warp-evaluations/s", "cores": 1, "kind": "oracle",
+                 "sample": f"{what}; {reps} calls in {el:.1f} s (single thread: one ctypes call per evaluation)"},
+                **host_cpu())
 
 
 def sweep_roofline(tps: float, clocks: dict):
@@ -340,7 +439,7 @@ def sweep_roofline(tps: float, clocks: dict):
 
 def trace_roofline(eps: float, clocks: dict):
     """ALU roofline of the trace evaluator (same pipe model as the sweep): achieved = ALU-pipe
-    warp-instructions per warp-evaluation (ncu capture of trace_kernel<32>) x evaluations/s."""
+    warp-instructions per warp-evaluation (ncu capture of trace32_kernel) x evaluations/s."""
     prof = load_profile("trace_w32") or {}
     ape = prof.get("alu_warp_instructions_per_evaluation")
     ipe = prof.get("warp_instructions_per_evaluation")
@@ -355,6 +454,18 @@ def trace_roofline(eps: float, clocks: dict):
             "profile": prof.get("source")}
 
 
+def hbm_roofline(nbytes: int, ms: float, peak: float, peak_src: str, kkey: str) -> dict:
+    """HBM roofline of one transpose launch: algorithmic bytes / mean launch time."""
+    prof = load_profile(kkey) or {}
+    ach = nbytes / (ms * 1e-3) / 1e9
+    return {"bound": "hbm", "achieved": ach, "peak": peak, "unit": "GB/s", "frac": ach / peak,
+            "traffic": prof.get("dram_bytes_per_launch_steady", prof.get("dram_bytes_per_launch")),
+            "peak_source": peak_src, "frac_of_8TBs_nominal": ach / 8000.0, "kernel": kkey,
+            "kernel_name": prof.get("kernel"), "kernel_ms_mean": ms, "algorithmic_bytes_per_launch": nbytes,
+            "smem_wavefronts_per_request": prof.get("smem_wavefronts_per_request"),
+            "profile": prof.get("source")}
+
+
 def reduce_over_ranks(x: float, world: int, dev, op: str) -> float:
     if world == 1:
         return x
@@ -365,12 +476,256 @@ def reduce_over_ranks(x: float, world: int, dev, op: str) -> float:
     return float(t.item())
 
 
-# ---------------------------------------------------------------------------- our arm
-def main():
-    args = parse()
-    route_native_stdout_to_stderr()
-    if args.impl == "reference":
-        return run_reference(args)
+def golden_sweep_1e9(seed: int):
+    """The oracle's stored 10^9-trial cfg2 histogram [5][3][33] (tests/golden, written by
+    tools/oracle_golden_1e9.py from oracle/ only), or None."""
+    import numpy as np
+    path = os.path.join(ROOT, "tests", "golden", f"sweep_w32_1e9_seed{seed}.txt")
+    if not os.path.exists(path):
+        return None
+    rows = [ln.split() for ln in open(path) if ln.strip() and not ln.startswith("#")]
+    h = np.array([[int(v) for v in r[2:]] for r in rows], dtype=np.uint64)
+    return h.reshape(5, 3, 33)
+
+
+# ---------------------------------------------------------------------------- our arm: default
+def init_dist(world: int, dev, force: bool = False):
+    """One process per GPU over NCCL; RAP_BENCH_BACKEND=gloo lets several ranks share one GPU to
+    exercise the multi-rank code paths on a single-GPU box (NCCL refuses duplicate devices)."""
+    import torch.distributed as dist
+    if world > 1 or force:
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        os.environ.setdefault("MASTER_PORT", "29571")
+        os.environ.setdefault("RANK", "0")
+        os.environ.setdefault("WORLD_SIZE", "1")
+        backend = os.environ.get("RAP_BENCH_BACKEND", "nccl")
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(backend)
+
+
+def all_reduce_hist(h, world: int):
+    """Sum a histogram over the ranks (NCCL on device; gloo via host memory)."""
+    if world == 1:
+        return
+    import torch.distributed as dist
+    if dist.get_backend() == "nccl":
+        dist.all_reduce(h)
+    else:
+        hc = h.cpu()
+        dist.all_reduce(hc)
+        h.copy_(hc)
+
+
+def timed_back_to_back(fn, warmup: int, steps: int, stream, world: int, dev, barrier):
+    """Mean device time of one fn() over `steps` back-to-back launches between one event pair
+    (max over ranks), with the clocks sampled over them."""
+    import torch
+    for _ in range(warmup):
+        fn()
+    torch.cuda.synchronize()
+    barrier()
+    with Clocks(dev.index) as clk:
+        t0 = time.perf_counter()
+        while time.perf_counter() - t0 < 0.2:     # soak, so every clock sample is under load
+            fn()
+            torch.cuda.synchronize()
+        st, en = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        st.record(stream)
+        for _ in range(steps):
+            fn()
+        en.record(stream)
+        torch.cuda.synchronize()
+    return reduce_over_ranks(st.elapsed_time(en), world, dev, "max") / steps, clk.result
+
+
+def run_default(args):
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    import __graft_entry__
+    __graft_entry__.build()
+    import paper_conf_icppw_nakanomi14_b200 as rap
+    import workloads
+
+    world, rank, local = dist_env()
+    dev = torch.device("cuda", local % torch.cuda.device_count())
+    torch.cuda.set_device(dev)
+    init_dist(world, dev)
+    stream = torch.cuda.current_stream()
+    peak, peak_src = load_peaks()
+    barrier = (lambda: dist.barrier()) if world > 1 else (lambda: None)
+    rmax = lambda v: reduce_over_ranks(v, world, dev, "max")
+    K, W = args.steps, args.warmup
+
+    # ---------------- cfg4 headline + cfg2 sweep slices
+    rows = cols = 16384
+    dt = torch.float64
+    nbytes = 2 * rows * cols * 8                     # per rank per step
+    x = workloads.random_bits(rows, cols, dt, seed=rank, device=dev)
+    y = torch.empty((cols, rows), dtype=dt, device=dev)
+    S = args.sweep_trials                            # trials per step (all ranks together)
+    total = min(SWEEP_TOTAL, S * K)
+    hist = torch.zeros((5, 3, 33), dtype=torch.int64, device=dev)
+    hstep = torch.zeros_like(hist)
+    scratch = torch.zeros_like(hist)
+
+    def sweep_slice(first: int, n: int, out):
+        """This rank's part of trials [first, first + n) into `out` (+ the all-reduce at N > 1)."""
+        lo = first + n * rank // world
+        hi = first + n * (rank + 1) // world
+        if world == 1:
+            rap.congestion_sweep(hi - lo, seed=SWEEP_SEED, first_trial=lo, out=out)
+            return 1
+        hstep.zero_()
+        rap.congestion_sweep(hi - lo, seed=SWEEP_SEED, first_trial=lo, out=hstep)
+        all_reduce_hist(hstep, world)                # the sweep's one exchange
+        out.add_(hstep)
+        return 1
+
+    def soak(seconds, k0):
+        t0, k = time.perf_counter(), 0
+        while time.perf_counter() - t0 < seconds:
+            rap.transpose(x, layout="rap", seed=0, out=y)
+            sweep_slice((1 << 40) + (k0 + k) * S, S, scratch)    # far trial range, scratch histogram
+            k += 1
+            torch.cuda.synchronize()
+
+    for k in range(W):
+        rap.transpose(x, layout="rap", seed=0, out=y)
+        sweep_slice((1 << 41) + k * S, S, scratch)
+    torch.cuda.synchronize()
+    first_clocks = None
+    for attempt in range(2):
+        hist.zero_()
+        launches, ev = 0, []
+        barrier()
+        torch.cuda.synchronize()
+        with Clocks(dev.index) as clk:
+            soak(0.3, 0)
+            barrier()
+            start = torch.cuda.Event(enable_timing=True)
+            end = torch.cuda.Event(enable_timing=True)
+            start.record(stream)
+            for k in range(K):
+                e = [torch.cuda.Event(enable_timing=True) for _ in range(4)]
+                e[0].record(stream)
+                rap.transpose(x, layout="rap", seed=0, out=y)          # T0-T3
+                launches += 1
+                e[1].record(stream)
+                e[2].record(stream)
+                n = min(S, total - k * S)
+                if n > 0:
+                    launches += sweep_slice(k * S, n, hist)             # C1-C4
+                e[3].record(stream)
+                ev.append(e)
+            end.record(stream)
+            torch.cuda.synchronize()
+            barrier()
+            soak(0.3, 1000)
+        t_ms = [e[0].elapsed_time(e[1]) for e in ev]
+        s_ms = [e[2].elapsed_time(e[3]) for e in ev]
+        c = clk.result
+        if attempt == 0 and rmax(1.0 if clocks_bad(c) else 0.0) > 0:
+            first_clocks = c
+            continue
+        if first_clocks is not None:
+            c = dict(c, remeasured=True, first_attempt=first_clocks)
+        break
+    total_ms, t_sum, s_sum = rmax(start.elapsed_time(end)), rmax(sum(t_ms)), rmax(sum(s_ms))
+    kern_ms = t_sum / K                                           # mean transpose launch
+    line = {"metric": METRIC, "n_gpus": world, "steps": K, "warmup": W, "ms_per_step": total_ms / K,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64",
+            "data": "synthetic (seeded random bit patterns; sweep trials are counters)",
+            "value": nbytes * world / (kern_ms * 1e-3) / 1e9, "unit": "GB/s",
+            "config": arm_config(args, world)}
+    line["roofline"] = hbm_roofline(nbytes, kern_ms, peak, peak_src, "transpose_b64_rap")
+    line["roofline"]["kernel_ms_median"] = rmax(statistics.median(t_ms))
+
+    # sweep sub-object: the 10^9 trials of cfg2 swept by the K timed steps
+    h = hist.cpu().numpy().astype(np.uint64)
+    cc = np.arange(33)
+    E = lambda a: float((a * cc).sum() / a.sum())
+    assert (h.sum(-1) == total).all(), "histogram does not hold every timed trial once"
+    tps = total / (s_sum * 1e-3)
+    gold = golden_sweep_1e9(SWEEP_SEED) if total == SWEEP_TOTAL else None
+    line["sweep"] = {"trials_per_s": tps, "unit": "trials/s", "trials": total, "w": 32, "seed": SWEEP_SEED,
+                     "trials_per_step": S, "scaling": "strong (the trials of each step are split over the ranks)",
+                     "E_ras_stride": E(h[1, 1]), "E_rap_diagonal": E(h[2, 2]), "E_random": E(h[3, 2]),
+                     "E_raw_malicious": E(h[4, 0]), "E_rap_stride": E(h[1, 2]),
+                     "kernel_ms_mean": s_sum / K,
+                     "bit_identical_to_oracle_1e9": (bool(np.array_equal(h, gold)) if gold is not None else None),
+                     "oracle_reference": "tests/golden/sweep_w32_1e9_seed1.txt (oracle/, 10^9 trials)",
+                     "roofline": sweep_roofline(tps / world, c)}
+    if gold is not None:
+        assert np.array_equal(h, gold), "10^9-trial histogram differs from the oracle's"
+    line["kernel_time_share"] = {"transpose": t_sum / (t_sum + s_sum), "sweep": s_sum / (t_sum + s_sum)}
+    line["clocks"] = c
+    line["gpu_launches"] = int(reduce_over_ranks(launches, world, dev, "sum"))
+
+    # ---------------- cfg3 under the five layouts, cfg4 under every 64-bit layout
+    subs = {}
+    x3 = workloads.random_bits(8192, 8192, torch.float32, seed=rank, device=dev)
+    y3 = torch.empty_like(x3)
+    for name, xx, yy, lays in (("cfg3_layouts", x3, y3, CFG3_LAYOUTS), ("cfg4_layouts", x, y, CFG4_LAYOUTS)):
+        eb = xx.element_size()
+        nb = 2 * xx.numel() * eb
+        res = {}
+        for lay in lays:
+            ms, ck = timed_back_to_back(lambda: rap.transpose(xx, layout=lay, seed=0, out=yy), W, K, stream,
+                                        world, dev, barrier)
+            r = hbm_roofline(nb, ms, peak, peak_src, f"transpose_b{eb * 8}_{lay}")
+            res[lay] = {"value": nb * world / (ms * 1e-3) / 1e9, "unit": "GB/s", "frac": r["frac"],
+                        "kernel_ms_mean": ms, "smem_wavefronts_per_request": r["smem_wavefronts_per_request"],
+                        "traffic": r["traffic"], "kernel_name": r["kernel_name"], "sm_mhz": ck.get("sm_mhz"),
+                        "reasons": ck.get("reasons")}
+        sub = {"workload": ("cfg3 8192x8192 float32" if eb == 4 else "cfg4 16384x16384 float64"),
+               "timing": f"{K} back-to-back launches per layout between one event pair (after {W} warm-ups)",
+               "algorithmic_bytes_per_launch": nb, "layouts": res,
+               "roofline": hbm_roofline(nb, res["rap"]["kernel_ms_mean"], peak, peak_src, f"transpose_b{eb * 8}_rap")}
+        subs[name] = sub
+    del x3, y3
+    line.update(subs)
+
+    # ---------------- e2e through the public API with pinned host buffers
+    if not args.no_e2e:
+        KE = max(3, min(K, 10))
+        hx = x.cpu().pin_memory()
+        hy = torch.empty((cols, rows), dtype=dt).pin_memory()
+        for _ in range(2):
+            rap.transpose_host(hx, out=hy, layout="rap", seed=0, device=dev)
+        barrier()
+        st = torch.cuda.Event(enable_timing=True)
+        en = torch.cuda.Event(enable_timing=True)
+        st.record(stream)
+        for _ in range(KE):
+            rap.transpose_host(hx, out=hy, layout="rap", seed=0, device=dev)
+        en.record(stream)
+        torch.cuda.synchronize()
+        ms = rmax(st.elapsed_time(en)) / KE
+        rap.transpose(x, layout="rap", seed=0, out=y)
+        assert torch.equal(hy.view(torch.int64), y.cpu().view(torch.int64)), "e2e result differs from the device result"
+        line["e2e"] = {"value": nbytes * world / (ms * 1e-3) / 1e9, "unit": "GB/s",
+                       "h2d_bytes_per_step": hx.numel() * 8 * world, "d2h_bytes_per_step": hy.numel() * 8 * world,
+                       "ms_per_step": ms, "steps": KE,
+                       "note": "rap_transpose_host: pinned host cfg4 matrix in, pinned host transpose out; "
+                               "upload / RAP transpose / download of row bands (128 MiB workspace) overlapped"}
+        del hx, hy
+    if rank == 0 and not args.no_cpu and world == 1:
+        line["cpu_baseline"] = cpu_baseline_transpose(rows, cols, dt)
+        line["sweep"]["cpu_baseline"] = cpu_baseline_sweep()
+        line["cfg3_layouts"]["cpu_baseline"] = cpu_baseline_transpose(8192, 8192, torch.float32)
+        line["cfg1_tile_cpu_baseline"] = cpu_baseline_tile()
+    if rank == 0:
+        emit(line)
+    if dist.is_initialized():
+        dist.destroy_process_group()
+
+
+# ---------------------------------------------------------------------------- our arm: other workloads
+def run_workload(args):
     import numpy as np
     import torch
     import torch.distributed as dist
@@ -382,20 +737,9 @@ def main():
     import workloads
 
     world, rank, local = dist_env()
-    # one process per GPU; RAP_BENCH_BACKEND=gloo lets several ranks share one GPU to exercise
-    # the multi-rank code paths on a single-GPU box (NCCL refuses duplicate devices)
-    backend = os.environ.get("RAP_BENCH_BACKEND", "nccl")
     dev = torch.device("cuda", local % torch.cuda.device_count())
     torch.cuda.set_device(dev)
-    if world > 1 or args.workload == "dist_fused":
-        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
-        os.environ.setdefault("MASTER_PORT", "29571")
-        os.environ.setdefault("RANK", "0")
-        os.environ.setdefault("WORLD_SIZE", "1")
-        if backend == "nccl":
-            dist.init_process_group("nccl", device_id=dev)
-        else:
-            dist.init_process_group(backend)
+    init_dist(world, dev, force=args.workload == "dist_fused")
     stream = torch.cuda.current_stream()
     peak, peak_src = load_peaks()
     wl = args.workload
@@ -416,7 +760,7 @@ def main():
         rows = cols = 8192
         dt = torch.float32
     do_t = wl not in ("sweep", "trace")
-    do_s = wl in ("default", "sweep", "trace")
+    do_s = wl in ("cfg3", "sweep", "trace")
     layouts = (["raw", "pad", "xor", "ras", "rap"] if wl == "layouts"
                else ["rap16", "rap2p", "rap"] if wl == "cfg4" and args.layout == "rap"     # T2b ablations beside the 8-byte-slot RAP
                else [args.layout])
@@ -465,7 +809,7 @@ def main():
         # to the run total (all-reducing the running total itself would count earlier steps again)
         hstep.zero_()
         rap.congestion_sweep(S, seed=1, first_trial=(k * world + rank) * S, out=hstep, algo=args.sweep_algo)
-        dist.all_reduce(hstep)
+        all_reduce_hist(hstep, world)
         hist.add_(hstep)
         return 1
 
@@ -532,10 +876,7 @@ def main():
             # a timed region that saw thermal / hardware slowdown, or SM clocks well below max with
             # no reason given, is measured once more (every rank agrees through the max)
             c = clk.result
-            bad = bool(set(c.get("reasons") or []) & {"hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown"})
-            bad = bad or bool(c.get("sm_mhz") and c.get("sm_max_mhz") and not c.get("reasons")
-                              and c["sm_mhz"] < 0.85 * c["sm_max_mhz"])
-            if attempt == 0 and rmax(1.0 if bad else 0.0) > 0:
+            if attempt == 0 and rmax(1.0 if clocks_bad(c) else 0.0) > 0:
                 first_clocks = c
                 continue
             if first_clocks is not None:
@@ -550,7 +891,7 @@ def main():
             "dtype": "u64" if eb == 8 else "u32", "data": "synthetic (seeded random bit patterns)"}
     if do_t:
         gbs = nbytes * world * args.steps / (r["t_sum"] * 1e-3) / 1e9
-        kern_ms = statistics.median(r["t_ms"])
+        kern_ms = r["t_sum"] / args.steps                # mean launch (the statistic of `value`)
         line.update(value=gbs, unit="GB/s")
         line["config"] = arm_config(args, world)
         assert line["config"]["layout"] == lay and line["config"]["algorithmic_bytes_per_step_per_rank"] == nbytes
@@ -563,15 +904,7 @@ def main():
                                 "peak_source": "B200_PROFILING.md measured peer copy per direction",
                                 "note": "bytes each rank sends over NVLink per step / step time"}
         else:
-            ach = nbytes / (kern_ms * 1e-3) / 1e9
-            line["roofline"] = {"bound": "hbm", "achieved": ach, "peak": peak, "unit": "GB/s",
-                                "frac": ach / peak,
-                                "traffic": prof.get("dram_bytes_per_launch_steady", prof.get("dram_bytes_per_launch")),
-                                "peak_source": peak_src, "frac_of_8TBs_nominal": ach / 8000.0,
-                                "kernel": kkey, "kernel_ms_median": kern_ms,
-                                "algorithmic_bytes_per_launch": nbytes,
-                                "smem_wavefronts_per_request": prof.get("smem_wavefronts_per_request"),
-                                "profile": prof.get("source")}
+            line["roofline"] = hbm_roofline(nbytes, kern_ms, peak, peak_src, kkey)
         if wl in ("layouts", "cfg4") and len(results) > 1:
             line["layouts_gbs"] = {l: nbytes * world * args.steps / (v["t_sum"] * 1e-3) / 1e9
                                    for l, v in results.items()}
@@ -599,12 +932,12 @@ def main():
                          "trials_in_histogram": int(h[0, 0].sum()),
                          "E_ras_stride": E(h[1, 1]), "E_rap_diagonal": E(h[2, 2]), "E_random": E(h[3, 2]),
                          "E_raw_malicious": E(h[4, 0]), "E_rap_stride": E(h[1, 2]),
-                         "kernel_ms_median": statistics.median(r["s_ms"]),
+                         "kernel_ms_mean": r["s_sum"] / args.steps,
                          "roofline": sweep_roofline(tps / world, r["clocks"])}
         if do_t and S <= 148 * 8 * 4 * 32:
             line["sweep"]["note"] = ("one batch of 32 trials per resident warp per step: a single wave, below the "
                                      "kernel's steady rate (launch ramp and tail); `--workload sweep` times 64 "
-                                     "batches per warp per launch (profiles/r01_bench_sweep.json)")
+                                     "batches per warp per launch; the default workload sweeps 10^9 trials")
         if not do_t:
             line.update(value=tps, unit="trials/s",
                         config=arm_config(args, world))
@@ -742,6 +1075,16 @@ def main():
         emit(line)
     if dist.is_initialized():
         dist.destroy_process_group()
+
+
+def main():
+    args = parse()
+    route_native_stdout_to_stderr()
+    if args.impl == "reference":
+        return run_reference(args)
+    if args.workload == "default":
+        return run_default(args)
+    return run_workload(args)
 
 
 if __name__ == "__main__":

@@ -24,22 +24,25 @@ def _run(*argv, env=None):
     return [json.loads(l) for l in out.stdout.splitlines() if l.startswith("{")]
 
 
-def _args(workload):
-    return bench.parse(["--workload", workload])
+def _args(workload, *extra):
+    return bench.parse(["--workload", workload, *extra])
 
 
-@pytest.mark.parametrize("workload,unit", [("default", "GB/s"), ("sweep", "trials/s"),
+@pytest.mark.parametrize("workload,unit", [("default", "GB/s"), ("cfg3", "GB/s"), ("sweep", "trials/s"),
                                            ("trace", "warp-evaluations/s"), ("tile", "GB/s")])
 def test_reference_line(workload, unit):
     (line,) = _run("--workload", workload, "--steps", "1", "--warmup", "1")
     assert line["impl"] == "reference" and line["metric"] == bench.METRIC
     assert line["unit"] == unit and line["value"] > 0 and line["higher_is_better"] is True
-    assert line["config"] == bench.arm_config(_args(workload), 1)
+    assert line["config"] == bench.arm_config(_args(workload, "--steps", "1", "--warmup", "1"), 1)
     cb = line["cpu_baseline"]
     assert cb["kind"] == "oracle" and cb["value"] == line["value"] and cb["cores"] >= 1 and cb["sample"]
+    assert cb["nproc"] >= 1 and "cpu_model" in cb
     assert line["e2e"] == {"value": line["value"], "unit": unit, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}
-    if workload == "default":
+    if workload in ("default", "cfg3"):
         assert line["sweep"]["trials_per_s"] > 0
+    if workload == "default":
+        assert line["dtype"] == "u64" and line["config"]["rows"] == 16384 and line["config"]["elem_bytes"] == 8
 
 
 def test_reference_only_rank0_prints():
@@ -47,10 +50,29 @@ def test_reference_only_rank0_prints():
     assert _run("--steps", "1", "--warmup", "1", env={"WORLD_SIZE": "2", "RANK": "1", "LOCAL_RANK": "1"}) == []
 
 
-@pytest.mark.parametrize("workload", ["default", "cfg4", "dist", "dist_fused", "layouts"])
+@pytest.mark.parametrize("workload", ["default", "cfg3", "cfg4", "dist", "dist_fused", "layouts"])
 def test_arm_config_bytes(workload):
     cfg = bench.arm_config(_args(workload), 4)
     n, eb = cfg["rows"], cfg["elem_bytes"]
     rows_rank = n // 4 if workload.startswith("dist") else n
     assert cfg["algorithmic_bytes_per_step_per_rank"] == 2 * rows_rank * n * eb
     assert ("4 GPU" in cfg["workload"]) == workload.startswith("dist")
+
+
+def test_default_sweeps_1e9_trials_over_the_timed_steps():
+    # the default run's timed steps cover cfg2's 10^9 trials exactly, whatever --steps is
+    for k in (1, 3, 7, 20, 50):
+        a = _args("default", "--steps", str(k))
+        assert a.sweep_trials * k >= bench.SWEEP_TOTAL > a.sweep_trials * (k - 1)
+        assert bench.arm_config(a, 1)["sweep_trials_total"] == bench.SWEEP_TOTAL
+
+
+def test_oracle_band_is_one_definition():
+    # both arms time the oracle on the same row band of the matrix
+    assert bench.oracle_band(16384, 16384, 8) == 256 and bench.oracle_band(8192, 8192, 4) == 1024
+    assert bench.oracle_band(32, 32, 4) == 32
+
+
+def test_golden_1e9_histogram_loads():
+    h = bench.golden_sweep_1e9(1)
+    assert h.shape == (5, 3, 33) and (h.sum(-1) == 10 ** 9).all()
