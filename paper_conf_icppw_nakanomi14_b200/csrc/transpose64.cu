@@ -38,6 +38,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <type_traits>
+
 #include "rap_internal.h"
 #include "rap_rng.cuh"
 
@@ -64,7 +66,16 @@ __device__ __forceinline__ uint4 ldg_nc_v4(const void *p) {
     return r;
 }
 
-template <int L, bool VEC, int SR, int MINB>
+__device__ __forceinline__ uint2 ldg_nc_v2(const void *p) {
+    uint2 r;
+    asm volatile("ld.global.nc.L1::no_allocate.v2.u32 {%0,%1}, [%2];" : "=r"(r.x), "=r"(r.y) : "l"(p));
+    return r;
+}
+
+// ROWS = true: T1 with one LDG.64 per tile row (lane j reads double j, 256 B per instruction,
+// 32 per tile) and one STS.64 per row: lanes j = 0..15 of row i hit bank pairs (j + P[i]) mod 16,
+// distinct for any P -- the row write needs no grouping.  ROWS = false: the LDG.128 grouping above.
+template <int L, bool VEC, int SR, int MINB, bool ROWS>
 __global__ void __launch_bounds__(SR * 32, MINB)
 transpose64_kernel(const uint2 *__restrict__ src, uint2 *__restrict__ dst, int64_t rows, int64_t cols,
                    int64_t ld_src, int64_t ld_dst, const TileShifts ts, uint32_t tiles_r, uint32_t tiles_c) {
@@ -82,13 +93,22 @@ transpose64_kernel(const uint2 *__restrict__ src, uint2 *__restrict__ dst, int64
     // group; rsel picks the row (RAP: a = P^-1(2g) with P even, b = P^-1(2g+1) with P odd)
     const uint32_t rsel = (lane >> 3) & 1u;
     const uint32_t q = ((lane >> 4) << 3) | (lane & 7u);
-    uint32_t row_g[16], a_g[16];
+    constexpr int NG = ROWS ? 1 : 16;                   // (ROWS: unused)
+    uint32_t row_g[NG], a_g[NG];
 #pragma unroll
-    for (int g = 0; g < 16; ++g) {
+    for (int g = 0; g < NG; ++g) {
         const uint32_t rr = 2u * g + rsel;
         row_g[g] = RAP ? __shfl_sync(kFull, inv_lane, rr) : rr;
         const uint32_t shg = RAP ? rr : (L == RAP_LAYOUT_RAS ? __shfl_sync(kFull, sh_lane, rr) : 0u);
         a_g[g] = slot64<L>(row_g[g], 2u * q, shg);          // double 2q; double 2q+1 follows
+    }
+    // ROWS: lane j writes double j of row r at st_off[r] (RAS / RAP: r*RP + j + sh[r])
+    constexpr int NR = ROWS ? 32 : 1;
+    uint32_t st_off[NR];
+#pragma unroll
+    for (int r = 0; r < NR; ++r) {
+        const uint32_t shr = (RAP || L == RAP_LAYOUT_RAS) ? __shfl_sync(kFull, sh_lane, r) : 0u;
+        st_off[r] = slot64<L>((uint32_t)r, lane, shr);
     }
     // T2 lane geometry: lane l drains row rho = P^-1(l) (RAP) or l; column c at drain_base + c
     const uint32_t rho = inv_lane;
@@ -102,7 +122,25 @@ transpose64_kernel(const uint2 *__restrict__ src, uint2 *__restrict__ dst, int64
         return ti < tiles_r;
     };
 
-    auto load = [&](uint4 (&v)[16], uint32_t ti, uint32_t tj) {
+    using Buf = typename std::conditional<ROWS, uint2[32], uint4[16]>::type;
+    auto load_rows = [&](uint2 (&v)[32], uint32_t ti, uint32_t tj) {
+        const int64_t r0 = (int64_t)ti * 32, c0 = (int64_t)tj * 32;
+        const uint2 *p = src + r0 * ld_src + c0 + lane;
+        if (r0 + 32 <= rows && c0 + 32 <= cols) {
+#pragma unroll
+            for (int r = 0; r < 32; ++r) v[r] = ldg_nc_v2(p + (int64_t)r * ld_src);
+        } else {
+            const bool cok = c0 + lane < cols;
+#pragma unroll
+            for (int r = 0; r < 32; ++r)
+                v[r] = (cok && r0 + r < rows) ? __ldg(p + (int64_t)r * ld_src) : make_uint2(0u, 0u);
+        }
+    };
+    auto store_rows = [&](const uint2 (&v)[32]) {
+#pragma unroll
+        for (int r = 0; r < 32; ++r) tile[st_off[r]] = v[r];
+    };
+    auto load_groups = [&](uint4 (&v)[16], uint32_t ti, uint32_t tj) {
         const int64_t r0 = (int64_t)ti * 32, c0 = (int64_t)tj * 32;
         if (VEC && r0 + 32 <= rows && c0 + 32 <= cols) {
             const uint2 *base = src + r0 * ld_src + c0 + 2 * q;
@@ -121,7 +159,7 @@ transpose64_kernel(const uint2 *__restrict__ src, uint2 *__restrict__ dst, int64
     };
 
     // T1: the contiguous write into the tile, two STS.64 per chunk
-    auto store_tile = [&](const uint4 (&v)[16]) {
+    auto store_groups = [&](const uint4 (&v)[16]) {
 #pragma unroll
         for (int g = 0; g < 16; ++g) {
             if (L == RAP_LAYOUT_XOR) {
@@ -158,9 +196,16 @@ transpose64_kernel(const uint2 *__restrict__ src, uint2 *__restrict__ dst, int64
         }
     };
 
+    auto load = [&](Buf &v, uint32_t ti, uint32_t tj) {
+        if constexpr (ROWS) load_rows(v, ti, tj); else load_groups(v, ti, tj);
+    };
+    auto store_tile = [&](const Buf &v) {
+        if constexpr (ROWS) store_rows(v); else store_groups(v);
+    };
+
     uint32_t st = blockIdx.x, ti = 0, tj = 0;
     bool act = st < nst && coords(st, ti, tj);
-    uint4 v[16];
+    Buf v;
     if (act) load(v, ti, tj);
     while (st < nst) {
         const uint32_t cti = ti, ctj = tj;
@@ -184,11 +229,14 @@ transpose64_kernel(const uint2 *__restrict__ src, uint2 *__restrict__ dst, int64
 #ifndef RAP64_MINB
 #define RAP64_MINB 1
 #endif
+#ifndef RAP64_ROWS
+#define RAP64_ROWS 1
+#endif
 
-template <int L, bool VEC, int SR, int MINB>
+template <int L, bool VEC, int SR, int MINB, bool ROWS = RAP64_ROWS>
 static cudaError_t launch64_one(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
                                 int64_t ld_dst, uint64_t seed, cudaStream_t st) {
-    auto k = transpose64_kernel<L, VEC, SR, MINB>;
+    auto k = transpose64_kernel<L, VEC, SR, MINB, ROWS>;
     static ShapeCache cache;
     const size_t smem = sizeof(uint2) * 32 * Geom64<L>::RP * SR;
     const uint32_t tiles_r = (uint32_t)((rows + 31) / 32), tiles_c = (uint32_t)((cols + 31) / 32);

@@ -23,6 +23,32 @@ from . import transpose_to_peers as _to_peers
 from . import unpack_blocks as _unpack
 
 
+def _staged(t: torch.Tensor, group) -> bool:
+    """gloo has no device collectives for these calls: stage CUDA tensors through host memory
+    (the 1-GPU multi-process tests run gloo ranks that share one device)."""
+    return t.is_cuda and dist.get_backend(group) != "nccl"
+
+
+def all_reduce_sum(h: torch.Tensor, group=None) -> torch.Tensor:
+    if _staged(h, group):
+        hc = h.cpu()
+        dist.all_reduce(hc, op=dist.ReduceOp.SUM, group=group)
+        h.copy_(hc)
+    else:
+        dist.all_reduce(h, op=dist.ReduceOp.SUM, group=group)
+    return h
+
+
+def all_to_all(recv: torch.Tensor, send: torch.Tensor, group=None) -> torch.Tensor:
+    if _staged(send, group):
+        rc = torch.empty(recv.shape, dtype=recv.dtype)
+        dist.all_to_all_single(rc, send.cpu(), group=group)
+        recv.copy_(rc)
+    else:
+        dist.all_to_all_single(recv, send, group=group)
+    return recv
+
+
 def trial_slice(n_trials: int, rank: int, world: int, first_trial: int = 0):
     lo = first_trial + n_trials * rank // world
     hi = first_trial + n_trials * (rank + 1) // world
@@ -42,7 +68,7 @@ def congestion_sweep(n_trials: int, seed: int, group=None, first_trial: int = 0,
     fn = local if local is not None else _sweep
     h = fn(count, seed, first_trial=first, **kw)          # zero-initialised by the callee
     if world > 1:
-        dist.all_reduce(h, op=dist.ReduceOp.SUM, group=group)
+        all_reduce_sum(h, group)
     if out is not None:
         out.add_(h)
         return out
@@ -76,36 +102,71 @@ def transpose_sharded(shard: torch.Tensor, group=None, layout: str = "rap", seed
         work["recv"] = torch.empty_like(send)
     recv = work["recv"]
     tr(shard, send)                                   # T1-T3: local RAP transpose, M x N -> N x M
-    dist.all_to_all_single(recv, send, group=group)   # T4: M x M blocks, NCCL over NVLink
+    all_to_all(recv, send, group)                     # T4: M x M blocks, NCCL over NVLink
     up(recv, out, world)                              # T4: place the blocks
     return out
 
 
 class FusedTranspose:
     """NEXT-2: the sharded transpose as ONE kernel per rank writing over NVLink into the peers'
-    output shards (torch symmetric memory maps every rank's output buffer into every process).
-    No send/receive buffers, no all-to-all, no unpack: each element is read once from local HBM
-    and written once, over NVLink when it belongs to another rank.
+    output shards.  No send/receive buffers, no all-to-all, no unpack: each element is read once
+    from local HBM and written once, over NVLink when it belongs to another rank.
 
         ft = FusedTranspose((M, N), torch.float32, group)
-        out = ft(shard)          # [M, N] symmetric tensor, rows rank*M.. of A^T, valid on return
+        out = ft(shard)          # [M, N] tensor, rows rank*M.. of A^T, valid on return
+
+    transport (how every rank's output buffer is mapped into every process):
+      "symm"  torch symmetric memory; the two cross-rank barriers run on the device
+              (default under NCCL);
+      "ipc"   CUDA IPC handles of plain torch allocations (cudaIpcGetMemHandle /
+              cudaIpcOpenMemHandle through torch's storage sharing), exchanged with
+              all_gather_object; the barriers are device sync + dist.barrier() (default under
+              gloo: works between processes that share one GPU, and between GPUs with P2P).
     """
 
-    def __init__(self, shape, dtype, group=None, layout: str = "rap", seed: int = 0):
-        from torch.distributed import _symmetric_memory as symm
+    def __init__(self, shape, dtype, group=None, layout: str = "rap", seed: int = 0, transport: str | None = None):
         self.group = group if group is not None else dist.group.WORLD
         self.rank, self.world = dist.get_rank(self.group), dist.get_world_size(self.group)
         M, N = shape
         if N != self.world * M or M % 32:
             raise ValueError("fused transpose needs N = world * M and M a multiple of 32")
-        self.out = symm.empty((M, N), dtype=dtype, device=torch.device("cuda", torch.cuda.current_device()))
-        self.handle = symm.rendezvous(self.out, self.group)
-        self.ptrs = [int(p) for p in self.handle.buffer_ptrs]
+        dev = torch.device("cuda", torch.cuda.current_device())
+        if transport is None:
+            transport = "symm" if dist.get_backend(self.group) == "nccl" else "ipc"
+        self.transport = transport
+        if transport == "symm":
+            from torch.distributed import _symmetric_memory as symm
+            self.out = symm.empty((M, N), dtype=dtype, device=dev)
+            self.handle = symm.rendezvous(self.out, self.group)
+            self.ptrs = [int(p) for p in self.handle.buffer_ptrs]
+        elif transport == "ipc":
+            self.out = torch.empty((M, N), dtype=dtype, device=dev)
+            mine = (self.out.untyped_storage()._share_cuda_(), self.out.storage_offset() * self.out.element_size())
+            allh = [None] * self.world
+            dist.all_gather_object(allh, mine, group=self.group)
+            self._mapped = []                  # keeps the opened peer mappings alive
+            self.ptrs = []
+            for r, (h, off) in enumerate(allh):
+                if r == self.rank:
+                    self.ptrs.append(self.out.data_ptr())
+                    continue
+                st = torch.UntypedStorage._new_shared_cuda(*h)
+                self._mapped.append(st)
+                self.ptrs.append(st.data_ptr() + off)
+        else:
+            raise ValueError(f"unknown transport {transport!r}")
         self.layout, self.seed = layout, seed
+
+    def _barrier(self):
+        if self.transport == "symm":
+            self.handle.barrier(channel=0)
+        else:
+            torch.cuda.current_stream().synchronize()
+            dist.barrier(group=self.group)
 
     def __call__(self, shard: torch.Tensor) -> torch.Tensor:
         # every rank must be done reading its shard's previous contents before peers overwrite it
-        self.handle.barrier(channel=0)
+        self._barrier()
         _to_peers(shard, self.ptrs, self.rank, layout=self.layout, seed=self.seed)
-        self.handle.barrier(channel=0)      # all peers' stores into this shard have landed
+        self._barrier()                     # all peers' stores into this shard have landed
         return self.out
