@@ -2,7 +2,7 @@
 
 Default step (BASELINE configs; DESIGN.md §7 "Measurement"): one pass of the whole hot path --
   T0-T3  RAP transpose of the cfg4 matrix: 16384 x 16384 float64 (the paper's 64-bit doubles,
-         P:L855-866), out-of-place, RAP = the w = 32 map on 8-byte tile slots; input and output
+         P:L855-866), out-of-place, RAP = the w = 32 map on two 32-bit planes; input and output
          are 2 GiB each (> the 126 MB L2: no flush between steps);
   C1-C4  a slice of the cfg2 congestion sweep (w = 32, 5 patterns x RAW/RAS/RAP, seed 1): the K
          timed steps sweep trials [0, 10^9) between them, so the run's histogram is the full
@@ -14,7 +14,7 @@ ranks / mean transpose device time per step (CUDA events on the launching stream
 ranks); `roofline` is that kernel's, on the same mean.  Sub-objects timed in the same run:
   `sweep`       the 10^9-trial cfg2 sweep (trials/s, ALU roofline, parity with the golden file);
   `cfg3_layouts` cfg3 8192^2 float32 under RAW / PAD / XOR / RAS / RAP (back-to-back launches);
-  `cfg4_layouts` cfg4 under every 64-bit layout (8-byte slots, RAP2P two planes, RAP-16);
+  `cfg4_layouts` cfg4 under every 64-bit layout (two 32-bit planes; RAP64 8-byte slots; RAP-16);
 each with its roofline and `cpu_baseline` (the oracle, all cores and one core, same sample
 definition as the reference arm).
 
@@ -49,7 +49,7 @@ NVLINK_GBS = 770.0   # measured peer copy per direction (B200_PROFILING.md); 900
 SWEEP_TOTAL = 10 ** 9          # cfg2: trials swept by the default run's timed steps
 SWEEP_SEED = 1
 CFG3_LAYOUTS = ["raw", "pad", "xor", "ras", "rap"]
-CFG4_LAYOUTS = ["raw", "pad", "xor", "ras", "rap", "rap2p", "rap16"]
+CFG4_LAYOUTS = ["raw", "pad", "xor", "ras", "rap", "rap64", "rap16"]
 ORACLE_BAND_BYTES = 32 << 20   # the oracle's transpose sample: one row band of this many bytes
 
 
@@ -196,11 +196,11 @@ def clocks_bad(c: dict) -> bool:
 
 
 # ---------------------------------------------------------------------------- workload config
-DESC = {"default": "cfg4 16384x16384 float64 RAP transpose (w=32 map on 8-byte tile slots) + cfg2 w=32 "
+DESC = {"default": "cfg4 16384x16384 float64 RAP transpose (w=32 map, two 32-bit planes) + cfg2 w=32 "
                    "sweep slice per step (10^9 trials over the timed steps); sub-objects: cfg2 sweep, "
                    "cfg3 8192x8192 float32 under raw/pad/xor/ras/rap, cfg4 under every 64-bit layout",
         "cfg3": "cfg3 8192x8192 float32 RAP transpose + cfg2 w=32 sweep batch",
-        "cfg4": "cfg4 16384x16384 float64 RAP transpose (w=32 map on 8-byte tile slots)",
+        "cfg4": "cfg4 16384x16384 float64 RAP transpose (w=32 map, two 32-bit planes)",
         "tile": "cfg1 32x32 float32 RAP tile (latency case)",
         "layouts": "cfg3 8192x8192 float32 transpose under 5 smem layouts",
         "dist": "cfg5 32768x32768 float32 row-block-sharded transpose over {world} GPU(s), NCCL all-to-all",
@@ -762,7 +762,7 @@ def run_workload(args):
     do_t = wl not in ("sweep", "trace")
     do_s = wl in ("cfg3", "sweep", "trace")
     layouts = (["raw", "pad", "xor", "ras", "rap"] if wl == "layouts"
-               else ["rap16", "rap2p", "rap"] if wl == "cfg4" and args.layout == "rap"     # T2b ablations beside the 8-byte-slot RAP
+               else ["rap16", "rap64", "rap"] if wl == "cfg4" and args.layout == "rap"     # T2b encodings beside the two-plane RAP
                else [args.layout])
     eb = torch.empty((), dtype=dt).element_size()
     nbytes = 2 * rows * cols * eb                     # per rank per step

@@ -68,15 +68,17 @@ typedef enum {
                          /* w = 16 applied to each half row: every half-warp of a 64-bit */
                          /* row or column access hits 16 distinct bank pairs (P:L860,    */
                          /* L1005-1023, DESIGN reading xiv)            */
-    RAP_LAYOUT_RAP2P = 6 /* 64-bit elements only: the w = 32 RAP map on two 32-bit planes */
-                         /* (low words, high words), every smem access 4 bytes wide      */
-                         /* (the round-1 default, kept as an ablation)   */
+    RAP_LAYOUT_RAP64 = 6 /* 64-bit elements only: the paper's map a[i][(j + P[i]) mod 32] */
+                         /* with ONE double per 8-byte tile slot, as the paper's arrays of */
+                         /* doubles (where a bank held one double).  B200 banks */
+                         /* are 4 bytes, so a 64-bit access is served per half-warp (16     */
+                         /* doubles); the kernel assigns rows to lanes so that every half-  */
+                         /* warp of the row write and of the column read hits 16 distinct  */
+                         /* bank pairs (DESIGN reading xv)                                 */
 } rap_layout_t;
-/* With elem_bytes == 8, RAW..RAP keep ONE 8-byte element per tile slot: RAP is the paper's map
- * a[i][(j + P[i]) mod 32] on doubles, P = perm(seed, 0, 32) (where a
- * bank held one double).  B200 banks are 4 bytes, so a 64-bit access is served per half-warp
- * (16 doubles = 128 B per wavefront); the kernel assigns rows to lanes so that every half-warp
- * of the row write and of the column read hits 16 distinct bank pairs (DESIGN reading xv). */
+/* With elem_bytes == 8, RAW..RAP split each 64-bit element into two 32-bit planes (low words,
+ * high words) with identical addressing, so every shared-memory access is a 32-lane 4-byte access
+ * under the w = 32 map of the layout (DESIGN reading viii). */
 
 /* Address maps of the DMM congestion evaluator (physical address of logical cell (i,j)). */
 typedef enum {
@@ -145,8 +147,8 @@ rap_status_t rap_perm_gen_batch(uint64_t seed, uint64_t first_index, uint64_t co
  * by RAW/PAD/XOR.  rows == 0 or cols == 0 is a
  * no-op.  Overlapping src/dst -> RAP_ERR_ALIAS.  16-byte aligned src with ld_src a
  * multiple of 16/elem_bytes takes 128-bit loads; anything else takes 32/64-bit loads
- * (still on the GPU).  RAP_LAYOUT_RAP16 and RAP_LAYOUT_RAP2P (elem_bytes 8 only) are the
- * 64-bit-element ablations of T2b. */
+ * (still on the GPU).  RAP_LAYOUT_RAP16 and RAP_LAYOUT_RAP64 (elem_bytes 8 only) are the
+ * other 64-bit encodings of T2b. */
 rap_status_t rap_transpose(const void *src, void *dst, int64_t rows, int64_t cols,
                            int64_t ld_src, int64_t ld_dst, uint32_t elem_bytes,
                            rap_layout_t layout, uint64_t seed, void *stream);
@@ -174,8 +176,8 @@ rap_status_t rap_transpose_host(const void *h_src, void *h_dst, int64_t rows, in
  * buffers for a one-GPU emulation); ld_dst >= N; G <= 16.  One HBM read and one NVLink write
  * per element; no send/receive buffers, no unpack.  Enqueue only: the caller must make every
  * rank's kernel complete (a cross-rank barrier) before reading its output shard.
- * layout RAW..RAP (RAP16 / RAP2P -> RAP_ERR_UNSUPPORTED); 64-bit elements are staged as two
- * 32-bit planes here. */
+ * layout RAW..RAP (RAP16 / RAP64 -> RAP_ERR_UNSUPPORTED); 64-bit elements are staged as two
+ * 32-bit planes. */
 rap_status_t rap_transpose_to_peers(const void *src, int64_t M, int64_t N, int64_t ld_src,
                                     void *const *peer_dst, uint32_t G, uint32_t rank, int64_t ld_dst,
                                     uint32_t elem_bytes, rap_layout_t layout, uint64_t seed, void *stream);

@@ -27,7 +27,7 @@ __all__ = ["perm_gen", "perm_gen_batch", "transpose", "transpose_host", "transpo
            "LAYOUTS", "SCHEMES", "PATTERNS", "SWEEP_ALGOS", "SMEM_ALGORITHMS", "SCHEMES4", "PATTERNS4",
            "RapError", "lib", "library_path"]
 
-LAYOUTS = {"raw": 0, "pad": 1, "xor": 2, "ras": 3, "rap": 4, "rap16": 5, "rap2p": 6}   # rap16/rap2p: 8-byte only
+LAYOUTS = {"raw": 0, "pad": 1, "xor": 2, "ras": 3, "rap": 4, "rap16": 5, "rap64": 6}   # rap16/rap64: 8-byte only
 SCHEMES = {"raw": 0, "ras": 1, "rap": 2, "pad": 3, "xor": 4}
 SWEEP_ALGOS = {"default": 0, "match": 1}
 PATTERNS = {"contiguous": 0, "stride": 1, "diagonal": 2, "random": 3, "malicious": 4}

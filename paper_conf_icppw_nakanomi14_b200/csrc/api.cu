@@ -72,8 +72,8 @@ rap_status_t rap_transpose(const void *src, void *dst, int64_t rows, int64_t col
                            int64_t ld_dst, uint32_t elem_bytes, rap_layout_t layout, uint64_t seed,
                            void *stream) {
     if (elem_bytes != 4 && elem_bytes != 8) return RAP_ERR_INVALID_ARG;
-    if ((int)layout < RAP_LAYOUT_RAW || (int)layout > RAP_LAYOUT_RAP2P) return RAP_ERR_INVALID_ARG;
-    if ((layout == RAP_LAYOUT_RAP16 || layout == RAP_LAYOUT_RAP2P) && elem_bytes != 8) return RAP_ERR_UNSUPPORTED;
+    if ((int)layout < RAP_LAYOUT_RAW || (int)layout > RAP_LAYOUT_RAP64) return RAP_ERR_INVALID_ARG;
+    if ((layout == RAP_LAYOUT_RAP16 || layout == RAP_LAYOUT_RAP64) && elem_bytes != 8) return RAP_ERR_UNSUPPORTED;
     if (rows < 0 || cols < 0) return RAP_ERR_INVALID_ARG;
     if (rows == 0 || cols == 0) return RAP_OK;
     if (!src || !dst) return RAP_ERR_INVALID_ARG;
@@ -94,8 +94,8 @@ rap_status_t rap_transpose_host(const void *h_src, void *h_dst, int64_t rows, in
                                 int64_t ld_dst, uint32_t elem_bytes, rap_layout_t layout, uint64_t seed,
                                 void *d_workspace, size_t workspace_bytes, void *stream) {
     if (elem_bytes != 4 && elem_bytes != 8) return RAP_ERR_INVALID_ARG;
-    if ((int)layout < RAP_LAYOUT_RAW || (int)layout > RAP_LAYOUT_RAP2P) return RAP_ERR_INVALID_ARG;
-    if ((layout == RAP_LAYOUT_RAP16 || layout == RAP_LAYOUT_RAP2P) && elem_bytes != 8) return RAP_ERR_UNSUPPORTED;
+    if ((int)layout < RAP_LAYOUT_RAW || (int)layout > RAP_LAYOUT_RAP64) return RAP_ERR_INVALID_ARG;
+    if ((layout == RAP_LAYOUT_RAP16 || layout == RAP_LAYOUT_RAP64) && elem_bytes != 8) return RAP_ERR_UNSUPPORTED;
     if (rows < 0 || cols < 0) return RAP_ERR_INVALID_ARG;
     if (rows == 0 || cols == 0) return RAP_OK;
     if (!h_src || !h_dst || !d_workspace) return RAP_ERR_INVALID_ARG;
@@ -114,8 +114,8 @@ rap_status_t rap_transpose_to_peers(const void *src, int64_t M, int64_t N, int64
                                     void *const *peer_dst, uint32_t G, uint32_t rank, int64_t ld_dst,
                                     uint32_t elem_bytes, rap_layout_t layout, uint64_t seed, void *stream) {
     if (elem_bytes != 4 && elem_bytes != 8) return RAP_ERR_INVALID_ARG;
-    if ((int)layout < RAP_LAYOUT_RAW || (int)layout > RAP_LAYOUT_RAP2P) return RAP_ERR_INVALID_ARG;
-    if (layout == RAP_LAYOUT_RAP16 || layout == RAP_LAYOUT_RAP2P) return RAP_ERR_UNSUPPORTED;
+    if ((int)layout < RAP_LAYOUT_RAW || (int)layout > RAP_LAYOUT_RAP64) return RAP_ERR_INVALID_ARG;
+    if (layout == RAP_LAYOUT_RAP16 || layout == RAP_LAYOUT_RAP64) return RAP_ERR_UNSUPPORTED;
     if (G < 1 || G > (uint32_t)rapk::kMaxPeers || rank >= G || !peer_dst) return RAP_ERR_INVALID_ARG;
     if (M <= 0 || M % 32 != 0) return RAP_ERR_INVALID_ARG;
     int64_t gm;

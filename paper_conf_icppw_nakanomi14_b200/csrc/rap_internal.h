@@ -58,18 +58,31 @@ struct TransposeTuning {
     bool vst = false;     // 128-bit output stores (shuffle-transposed) instead of 32/64-bit rows
     bool tma_store = false;  // drain into a dense staging tile, one TMA bulk tensor store per super-tile
     int cl = 1;           // thread-block cluster of cl CTAs stacked along the input rows, drains in lockstep
-    bool force_planes = false;  // 64-bit elements through the two-plane kernel for every layout (tuning A/B)
+    bool slots64 = false;  // 64-bit elements on 8-byte tile slots (transpose64.cu) for every layout (A/B)
 };
 // fp32: 4 x 2 warps per CTA, clusters of 4 CTAs (a 16 x 2-tile cluster super-tile);
 // fp64: 12 x 1 warps, no cluster (profiles/r01_tune_transpose*.txt, r01_probe_transpose.txt)
-constexpr int kDefaultSR32 = 4, kDefaultSC32 = 2, kDefaultSR64 = 12, kDefaultSC64 = 1;
-constexpr int kDefaultCL32 = 4, kDefaultCL64 = 1;
+// (RAP32_SR / RAP32_SC / RAP32_CL / RAP32_MINB override the fp32 shape in tuning builds)
+#ifndef RAP32_SR
+#define RAP32_SR 4
+#endif
+#ifndef RAP32_SC
+#define RAP32_SC 2
+#endif
+#ifndef RAP32_CL
+#define RAP32_CL 4
+#endif
+#ifndef RAP32_MINB
+#define RAP32_MINB 2
+#endif
+constexpr int kDefaultSR32 = RAP32_SR, kDefaultSC32 = RAP32_SC, kDefaultSR64 = 12, kDefaultSC64 = 1;
+constexpr int kDefaultCL32 = RAP32_CL, kDefaultCL64 = 1;
 // fused sharded transpose (peer stores): 8 x 2 warps, no cluster
 constexpr int kPeerSR32 = 8, kPeerSC32 = 2;
 // up to this many 32 x 32 tiles: one single-warp CTA per tile
 constexpr int64_t kSmallTiles = 8;
 // measured on B200 (tools/tune_transpose.cu, profiles/r01_tune_transpose.txt)
-constexpr int kDefaultMinB32 = 2, kDefaultMinB64 = 1;   // fp32: 2 CTAs of 8 warps per SM (128 registers)
+constexpr int kDefaultMinB32 = RAP32_MINB, kDefaultMinB64 = 1;   // fp32: 2 CTAs of 8 warps per SM (128 registers)
 constexpr int kDefaultDepth32 = 1, kDefaultDepth64 = 1;
 constexpr int kDefaultCtas32 = 0, kDefaultCtas64 = 0;
 constexpr bool kDefaultVst32 = false, kDefaultVst64 = false;
@@ -95,6 +108,53 @@ cudaError_t launch_transpose_peers(const void *src, int64_t M, int64_t N, int64_
 
 cudaError_t launch_perm_gen(uint64_t seed, uint64_t first, uint64_t count, uint32_t w, uint8_t *out,
                             cudaStream_t st);
+
+// Programmatic dependent launch (RAP_PDL, default on): the transposes are launched with
+// cudaLaunchAttributeProgrammaticStreamSerialization, trigger their dependents at entry and
+// wait (griddepcontrol.wait) for the previous grid in the stream -- its completion and memory
+// flush -- before their first global access.  A following launch's CTAs are then scheduled and
+// run their prologue while this grid drains, instead of after it; the data dependence is kept.
+#ifndef RAP_PDL
+#define RAP_PDL 1
+#endif
+__device__ __forceinline__ void pdl_wait() {
+#if RAP_PDL
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+#endif
+}
+__device__ __forceinline__ void pdl_trigger() {
+#if RAP_PDL
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+#endif
+}
+
+// cudaLaunchKernelEx with an optional cluster dimension and the PDL attribute
+template <typename K, typename... Args>
+cudaError_t launch_ex(K kernel, int grid, int block, size_t smem, cudaStream_t st, int cluster, Args... args) {
+    cudaLaunchConfig_t cfg = {};
+    cudaLaunchAttribute attr[2];
+    int na = 0;
+    if (cluster > 1) {
+        attr[na].id = cudaLaunchAttributeClusterDimension;
+        attr[na].val.clusterDim.x = (unsigned)cluster;
+        attr[na].val.clusterDim.y = 1;
+        attr[na].val.clusterDim.z = 1;
+        ++na;
+    }
+#if RAP_PDL
+    attr[na].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[na].val.programmaticStreamSerializationAllowed = 1;
+    ++na;
+#endif
+    cfg.gridDim = dim3((unsigned)grid);
+    cfg.blockDim = dim3((unsigned)block);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cfg.attrs = attr;
+    cfg.numAttrs = na;
+    const cudaError_t e = cudaLaunchKernelEx(&cfg, kernel, args...);
+    return e != cudaSuccess ? e : cudaGetLastError();
+}
 
 // occupancy-capped persistent grid for `want` work units (ShapeCache above)
 template <typename K>

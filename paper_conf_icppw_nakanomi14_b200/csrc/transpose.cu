@@ -20,7 +20,9 @@
 //           coalesced STG.32 of output row c (or a staging tile + TMA store, TMAS).
 // 64-bit elements: 32 banks of 4 bytes (the paper assumed one double per bank word,
 // P:L278-283, L860), so a tile of doubles is split into two 32-bit RAP planes (low / high
-// words) with identical addressing; every smem access stays a 32-lane 4-byte access.
+// words) with identical addressing; every smem access stays a 32-lane 4-byte access.  (The
+// other encodings: one double per 8-byte slot, transpose64.cu / RAP_LAYOUT_RAP64; RAP over 16
+// double banks, transpose_rap16.cu / RAP_LAYOUT_RAP16.)
 #include <cuda.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
@@ -59,12 +61,21 @@ __device__ __forceinline__ uint32_t word_of(uint32_t row, uint32_t col, uint32_t
     return row * RP + col;
 }
 
+// RAP32_LDG_NA = 1: 128-bit loads with L1::no_allocate; 0 (default): plain read-only loads
+// (LDG.E.128.CONSTANT) -- +4-5 % on cfg3 in interleaved A/B runs (profiles/r02_ab32.txt)
+#ifndef RAP32_LDG_NA
+#define RAP32_LDG_NA 0
+#endif
 __device__ __forceinline__ uint4 ldg_stream128(const void *p) {
+#if RAP32_LDG_NA
     uint4 r;
     // (an L2::256B prefetch hint measured no different, profiles/r01_tune_transpose_tma.txt)
     asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
                  : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
     return r;
+#else
+    return __ldg(reinterpret_cast<const uint4 *>(p));
+#endif
 }
 
 // Load geometry: a 128-bit load carries NE = 4/EW elements, LPR = 32/NE lanes cover one tile
@@ -285,6 +296,8 @@ transpose_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, i
 
     uint32_t st = st_first, ti = 0, tj = 0;
     bool act = st < nst && coords(st, ti, tj);
+    pdl_trigger();
+    pdl_wait();                                          // the previous grid's writes are visible
     if (TMAS) {
         uint4 v[G];
         if (act) load(v, ti, tj);
@@ -360,7 +373,7 @@ TileShifts tile_shifts(int layout, uint64_t seed) {
     uint32_t a[32];
     memset(&t, 0, sizeof(t));
     const uint32_t w = layout == RAP_LAYOUT_RAP16 ? 16u : 32u;
-    if (layout == RAP_LAYOUT_RAP || layout == RAP_LAYOUT_RAP2P || layout == RAP_LAYOUT_RAP16) {
+    if (layout == RAP_LAYOUT_RAP || layout == RAP_LAYOUT_RAP64 || layout == RAP_LAYOUT_RAP16) {
         perm_serial(seed, 0, w, a);
         for (uint32_t i = 0; i < w; ++i) {
             t.sh[i / 4] |= a[i] << (8 * (i % 4));
@@ -428,17 +441,6 @@ static cudaError_t launch_clustered(K kernel, ShapeCache &cache, int cl, int thr
     cudaError_t e = cudaGetDevice(&dev);
     if (e != cudaSuccess) return e;
     if (dev < 0 || dev >= kMaxDevices) return cudaErrorInvalidDevice;
-    cudaLaunchConfig_t cfg = {};
-    cudaLaunchAttribute attr[1];
-    attr[0].id = cudaLaunchAttributeClusterDimension;
-    attr[0].val.clusterDim.x = (unsigned)cl;
-    attr[0].val.clusterDim.y = 1;
-    attr[0].val.clusterDim.z = 1;
-    cfg.blockDim = dim3((unsigned)threads);
-    cfg.dynamicSmemBytes = smem;
-    cfg.stream = st;
-    cfg.attrs = attr;
-    cfg.numAttrs = 1;
     int ncl = cache.occ[dev].load(std::memory_order_acquire);   // here: co-resident clusters
     if (ncl == 0) {
         e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -446,6 +448,16 @@ static cudaError_t launch_clustered(K kernel, ShapeCache &cache, int cl, int thr
         int sms = 0;
         e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
         if (e != cudaSuccess) return e;
+        cudaLaunchConfig_t cfg = {};
+        cudaLaunchAttribute attr[1];
+        attr[0].id = cudaLaunchAttributeClusterDimension;
+        attr[0].val.clusterDim.x = (unsigned)cl;
+        attr[0].val.clusterDim.y = 1;
+        attr[0].val.clusterDim.z = 1;
+        cfg.blockDim = dim3((unsigned)threads);
+        cfg.dynamicSmemBytes = smem;
+        cfg.attrs = attr;
+        cfg.numAttrs = 1;
         cfg.gridDim = dim3((unsigned)(sms * cl));
         e = cudaOccupancyMaxActiveClusters(&ncl, kernel, &cfg);
         if (e != cudaSuccess) return e;
@@ -453,11 +465,8 @@ static cudaError_t launch_clustered(K kernel, ShapeCache &cache, int cl, int thr
         cache.occ[dev].store(ncl, std::memory_order_release);
     }
     const int64_t nclusters = nst < ncl ? nst : ncl;
-    cfg.gridDim = dim3((unsigned)(nclusters * cl));
-    e = cudaLaunchKernelEx(&cfg, kernel, src, dst, rows, cols, ld_src, ld_dst, ts, tiles_r, tiles_c, vst_ok,
-                           peers, tmap);
-    if (e != cudaSuccess) return e;
-    return cudaGetLastError();
+    return launch_ex(kernel, (int)(nclusters * cl), threads, smem, st, cl, src, dst, rows, cols, ld_src, ld_dst, ts,
+                     tiles_r, tiles_c, vst_ok, peers, tmap);
 }
 
 template <int L, int EW, bool VEC, int DEPTH, int MINB, bool VST, int SR, int SC, bool PEERS = false,
@@ -488,9 +497,8 @@ static cudaError_t launch_one(const void *src, void *dst, int64_t rows, int64_t 
     int grid = 0;
     const cudaError_t e = cached_grid(k, cache, SR * SC * 32, smem, nst, tu.ctas_per_sm, &grid);
     if (e != cudaSuccess) return e;
-    k<<<grid, SR * SC * 32, smem, st>>>((const uint32_t *)src, (uint32_t *)dst, rows, cols, ld_src,
-                                        ld_dst, ts, tiles_r, tiles_c, vst_ok, peers, tmap);
-    return cudaGetLastError();
+    return launch_ex(k, grid, SR * SC * 32, smem, st, 1, (const uint32_t *)src, (uint32_t *)dst, rows, cols, ld_src,
+                     ld_dst, ts, tiles_r, tiles_c, vst_ok, peers, tmap);
 }
 
 template <int L, int EW, bool VEC>
@@ -534,11 +542,11 @@ template <bool VEC>
 static cudaError_t dispatch(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
                             int64_t ld_dst, uint32_t eb, int layout, uint64_t seed,
                             const TransposeTuning &tu, cudaStream_t st) {
-    // 64-bit elements: one element per 8 bytes of the tile (transpose64.cu) for RAW..RAP; the
-    // round-1 design, two 32-bit planes under the w = 32 RAP map, is layout RAP2P
-    if (eb == 8 && layout == RAP_LAYOUT_RAP2P)
-        return launch_shape<RAP_LAYOUT_RAP, 2, VEC>(src, dst, rows, cols, ld_src, ld_dst, seed, tu, st);
-    if (eb == 8 && !tu.force_planes)
+    // 64-bit elements: RAW..RAP on two 32-bit planes (this kernel, EW = 2); RAP64 keeps one
+    // element per 8-byte slot (transpose64.cu, which also serves RAW..RAS with tu.slots64)
+    if (eb == 8 && layout == RAP_LAYOUT_RAP64)
+        return launch_transpose64(src, dst, rows, cols, ld_src, ld_dst, RAP_LAYOUT_RAP, seed, st);
+    if (eb == 8 && tu.slots64)
         return launch_transpose64(src, dst, rows, cols, ld_src, ld_dst, layout, seed, st);
 #define RAPK_CASE(LAY)                                                                             \
     case LAY:                                                                                      \

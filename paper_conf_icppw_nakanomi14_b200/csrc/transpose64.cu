@@ -23,7 +23,7 @@
 //          fills the 8 pairs of parity e, row b the 8 of parity 1-e -> 16 distinct per half-warp.
 // So every shared-memory request of the RAP tile takes the minimum 2 wavefronts, with the paper's
 // w = 32 map, and a tile costs 16 LDG.128 + 32 STS.64 + 32 LDS.64 + 32 STG.64 (112 memory
-// instructions; the two-plane RAP2P kernel needs 176, RAP-16 128).
+// instructions; the two-plane kernel of transpose.cu needs 176, RAP-16 128).  Layout RAP64.
 // The same kernel serves RAW / PAD ([32][33]) / XOR ([i][j ^ i]) / RAS on 8-byte slots as the
 // baselines (rows in natural order, lane l drains row l).
 //
@@ -59,17 +59,30 @@ __device__ __forceinline__ uint32_t slot64(uint32_t row, uint32_t col, uint32_t 
     return row * RP + col;
 }
 
+// RAP64_LDG_NA = 1: the loads carry L1::no_allocate; 0 (default): plain read-only loads
+// (LDG.E.64 / .128 .CONSTANT), measured faster on cfg4 (profiles/r02_ab64.txt)
+#ifndef RAP64_LDG_NA
+#define RAP64_LDG_NA 0
+#endif
 __device__ __forceinline__ uint4 ldg_nc_v4(const void *p) {
+#if RAP64_LDG_NA
     uint4 r;
     asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
                  : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
     return r;
+#else
+    return __ldg(reinterpret_cast<const uint4 *>(p));
+#endif
 }
 
 __device__ __forceinline__ uint2 ldg_nc_v2(const void *p) {
+#if RAP64_LDG_NA
     uint2 r;
     asm volatile("ld.global.nc.L1::no_allocate.v2.u32 {%0,%1}, [%2];" : "=r"(r.x), "=r"(r.y) : "l"(p));
     return r;
+#else
+    return __ldg(reinterpret_cast<const uint2 *>(p));
+#endif
 }
 
 // ROWS = true: T1 with one LDG.64 per tile row (lane j reads double j, 256 B per instruction,
@@ -107,12 +120,21 @@ transpose64_kernel(const uint2 *__restrict__ src, uint2 *__restrict__ dst, int64
     uint32_t st_off[NR];
 #pragma unroll
     for (int r = 0; r < NR; ++r) {
-        const uint32_t shr = (RAP || L == RAP_LAYOUT_RAS) ? __shfl_sync(kFull, sh_lane, r) : 0u;
+        // sh[r] read straight from the kernel parameter (r is a compile-time constant): a
+        // warp-uniform value, so the row base r*RP + sh[r] can live in a uniform register
+        const uint32_t shr = (RAP || L == RAP_LAYOUT_RAS) ? (ts.sh[r >> 2] >> (8 * (r & 3))) & 0xffu : 0u;
         st_off[r] = slot64<L>((uint32_t)r, lane, shr);
     }
     // T2 lane geometry: lane l drains row rho = P^-1(l) (RAP) or l; column c at drain_base + c
+    // (RAP64_NATURAL_DRAIN: lane l drains row l under RAP too -- an ablation with ~2-way
+    // conflicted LDS.64, to measure what the permuted output lanes cost)
+#ifdef RAP64_NATURAL_DRAIN
+    const uint32_t rho = lane;
+    const uint32_t drain_base = slot64<L>(lane, 0, sh_lane);
+#else
     const uint32_t rho = inv_lane;
     const uint32_t drain_base = RAP ? rho * RP + lane : slot64<L>(lane, 0, sh_lane);
+#endif
 
     const uint32_t nst = ((tiles_r + SR - 1) / SR) * tiles_c;
     auto coords = [&](uint32_t st, uint32_t &ti, uint32_t &tj) -> bool {
@@ -206,6 +228,8 @@ transpose64_kernel(const uint2 *__restrict__ src, uint2 *__restrict__ dst, int64
     uint32_t st = blockIdx.x, ti = 0, tj = 0;
     bool act = st < nst && coords(st, ti, tj);
     Buf v;
+    pdl_trigger();
+    pdl_wait();                                      // the previous grid's writes are visible
     if (act) load(v, ti, tj);
     while (st < nst) {
         const uint32_t cti = ti, ctj = tj;
@@ -242,12 +266,17 @@ static cudaError_t launch64_one(const void *src, void *dst, int64_t rows, int64_
     const uint32_t tiles_r = (uint32_t)((rows + 31) / 32), tiles_c = (uint32_t)((cols + 31) / 32);
     const int64_t nst = (int64_t)((tiles_r + SR - 1) / SR) * tiles_c;
     int grid = 0;
+#ifdef RAP64_CARVEOUT
+    static bool carve = [&] {
+        return cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, RAP64_CARVEOUT) == cudaSuccess;
+    }();
+    (void)carve;
+#endif
     const cudaError_t e = cached_grid(k, cache, SR * 32, smem, nst, 0, &grid);
     if (e != cudaSuccess) return e;
     const TileShifts ts = tile_shifts(L, seed);
-    k<<<grid, SR * 32, smem, st>>>((const uint2 *)src, (uint2 *)dst, rows, cols, ld_src, ld_dst, ts, tiles_r,
-                                   tiles_c);
-    return cudaGetLastError();
+    return launch_ex(k, grid, SR * 32, smem, st, 1, (const uint2 *)src, (uint2 *)dst, rows, cols, ld_src, ld_dst, ts,
+                     tiles_r, tiles_c);
 }
 
 template <int L, bool VEC>

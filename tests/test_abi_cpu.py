@@ -54,7 +54,7 @@ def test_transpose_validation(L):
     assert L.rap_transpose(a, b, 4, 4, 4, 4, 3, 4, 0, s) == INVALID      # elem_bytes
     assert L.rap_transpose(a, b, 4, 4, 4, 4, 4, 9, 0, s) == INVALID      # layout
     assert L.rap_transpose(a, b, 4, 4, 4, 4, 4, 7, 0, s) == INVALID      # layout
-    assert L.rap_transpose(a, b, 4, 4, 4, 4, 4, 6, 0, s) == UNSUPPORTED  # RAP2P needs 8-byte elements
+    assert L.rap_transpose(a, b, 4, 4, 4, 4, 4, 6, 0, s) == UNSUPPORTED  # RAP64 needs 8-byte elements
     assert L.rap_transpose(a, b, 4, 4, 4, 4, 4, 5, 0, s) == UNSUPPORTED  # RAP16 needs 8-byte elements
     assert L.rap_transpose(a, b, -1, 4, 4, 4, 4, 4, 0, s) == INVALID     # rows < 0
     assert L.rap_transpose(a, b, 4, 8, 4, 4, 4, 4, 0, s) == INVALID      # ld_src < cols

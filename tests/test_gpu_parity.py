@@ -154,11 +154,11 @@ def test_transpose_extreme_aspect(rap, oracle, shape):
     assert np.array_equal(bits(y), oracle.transpose(bits(x), threads=oracle.max_threads()))
 
 
-@pytest.mark.parametrize("layout", ["rap", "rap2p", "rap16"])
+@pytest.mark.parametrize("layout", ["rap", "rap64", "rap16"])
 def test_transpose_cfg4_16384_f64(rap, oracle, layout):
     # BASELINE cfg4 at full size, in the launch configuration bench.py times: all 2^28 doubles
-    # compared with the oracle (rap: the paper's w = 32 map on 8-byte slots, the headline;
-    # rap2p: two 32-bit planes; rap16: RAP over 16 double banks)
+    # compared with the oracle (rap: the w = 32 map on two 32-bit planes, the headline; rap64:
+    # the w = 32 map on 8-byte slots; rap16: RAP over 16 double banks)
     x = workloads.random_bits(16384, 16384, torch.float64, seed=0, device="cuda")
     y = rap.transpose(x, layout=layout, seed=0)
     torch.cuda.synchronize()
@@ -169,7 +169,7 @@ def test_transpose_cfg4_16384_f64(rap, oracle, layout):
 
 @pytest.mark.parametrize("layout", ["raw", "pad", "xor", "ras"])
 def test_transpose_cfg4_16384_f64_baselines(rap, layout):
-    # the baseline layouts on 8-byte slots at cfg4 size: equal to the RAP result (itself
+    # the baseline layouts (two 32-bit planes) at cfg4 size: equal to the RAP result (itself
     # checked in full against the oracle above) and an involution
     x = workloads.random_bits(16384, 16384, torch.float64, seed=0, device="cuda")
     ref = rap.transpose(x, layout="rap", seed=0)
@@ -178,24 +178,24 @@ def test_transpose_cfg4_16384_f64_baselines(rap, layout):
 
 
 def test_transpose64_seeds_and_ragged(rap, oracle):
-    # the 8-byte-slot kernel under many P (the P^-1 row grouping and drain lanes depend on P)
-    # on ragged shapes spanning several 12-warp super-tiles
+    # the 8-byte-slot kernel under many P (the P^-1 drain lanes depend on P) on ragged shapes
+    # spanning several 12-warp super-tiles
     for i, (r, c) in enumerate([(385, 33), (31, 1025), (800, 417), (1024, 96)]):
         x = workloads.random_bits(r, c, torch.float64, seed=200 + i)
         for seed in (0, 1, 2, 3, 12345, 2 ** 64 - 1):
-            y = rap.transpose(x.cuda(), layout="rap", seed=seed)
+            y = rap.transpose(x.cuda(), layout="rap64", seed=seed)
             torch.cuda.synchronize()
             assert np.array_equal(bits(y), oracle.transpose(bits(x))), (r, c, seed)
 
 
-def test_transpose_rap2p_shapes(rap, oracle):
+def test_transpose_rap64_shapes(rap, oracle):
     for i, (r, c) in enumerate(SHAPES + [(384, 64), (385, 33)]):
         x = workloads.random_bits(r, c, torch.float64, seed=300 + i)
-        y = rap.transpose(x.cuda(), layout="rap2p", seed=i)
+        y = rap.transpose(x.cuda(), layout="rap64", seed=i)
         torch.cuda.synchronize()
         assert np.array_equal(bits(y), oracle.transpose(bits(x))), (r, c)
     with pytest.raises(rap.RapError, match="UNSUPPORTED"):
-        rap.transpose(torch.zeros((64, 64), device="cuda"), layout="rap2p")
+        rap.transpose(torch.zeros((64, 64), device="cuda"), layout="rap64")
 
 
 # T2b (ii): the RAP-16 double tile (8-byte elements only)

@@ -19,7 +19,7 @@ import torch  # noqa: E402
 
 import workloads  # noqa: E402
 
-LAYOUTS = {"raw": 0, "pad": 1, "xor": 2, "ras": 3, "rap": 4, "rap16": 5, "rap2p": 6}
+LAYOUTS = {"raw": 0, "pad": 1, "xor": 2, "ras": 3, "rap": 4, "rap16": 5, "rap64": 6}
 
 
 def load(path):
@@ -60,6 +60,10 @@ def main():
         if ref is None:
             ref = bits
         assert torch.equal(bits, ref), spec
+    import subprocess
+    smi = subprocess.Popen(["nvidia-smi", "-i", str(torch.cuda.current_device()),
+                            "--query-gpu=clocks.sm,clocks.mem,power.draw,temperature.gpu,clocks_event_reasons.active",
+                            "--format=csv,noheader,nounits", "-lms", "250"], stdout=subprocess.PIPE, text=True)
     res = {spec: [] for spec, _, _ in arms}
     nb = 2 * a.n * a.n * eb
     for r in range(a.rounds):
@@ -74,6 +78,13 @@ def main():
             torch.cuda.synchronize()
             res[spec].append(nb * a.launches / (s.elapsed_time(e) * 1e-3) / 1e9)
         print(f"round {r}: " + "  ".join(f"{k}={v[-1]:.0f}" for k, v in res.items()), flush=True)
+    smi.terminate()
+    samples = [ln.split(", ") for ln in smi.communicate()[0].strip().splitlines()]
+    if samples:
+        col = lambda i: sorted(float(x[i]) for x in samples if len(x) > 4)
+        sm, mem, pw, tc = col(0), col(1), col(2), col(3)
+        print(f"clocks: sm {sm[0]:.0f}..{sm[-1]:.0f} MHz (median {sm[len(sm) // 2]:.0f}), mem {mem[len(mem) // 2]:.0f} MHz, "
+              f"power max {pw[-1]:.0f} W, temp max {tc[-1]:.0f} C, reasons {sorted(set(x[4] for x in samples if len(x) > 4))}")
     for k, v in res.items():
         print(f"{k:40s} median {statistics.median(v):7.1f} GB/s  min {min(v):7.1f}  max {max(v):7.1f}")
 

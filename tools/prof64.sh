@@ -1,6 +1,6 @@
 #!/bin/bash
 # ncu captures of the cfg4 (16384^2 float64) transpose kernels: the 8-byte-slot RAP kernel
-# (transpose64_kernel), RAP-16 and the two-plane RAP2P; full sets + steady-state DRAM bytes.
+# (transpose64_kernel, layout rap64), RAP-16 and the two-plane RAP; full sets + steady-state DRAM bytes.
 set -u
 OUT=${1:-gpurun_out}
 mkdir -p "$OUT"
