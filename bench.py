@@ -280,16 +280,19 @@ def rate_for(fn, work: float, seconds: float):
 
 def cpu_baseline_transpose(rows, cols, dt, seconds: float = 3.0):
     """The oracle's naive transpose on one row band of the matrix: all cores (value) and one core."""
+    import numpy as np
+
     import oracle
     threads = oracle.max_threads()
     x, band = oracle_transpose_sample(rows, cols, dt)
+    out = np.empty((x.shape[1], x.shape[0]), dtype=x.dtype)
     gb = 2 * x.nbytes / 1e9
-    v_all, n_all, t_all = rate_for(lambda: oracle.transpose(x, threads=threads), gb, seconds)
-    v_one, n_one, t_one = rate_for(lambda: oracle.transpose(x, threads=1), gb, seconds)
+    v_all, n_all, t_all = rate_for(lambda: oracle.transpose(x, threads=threads, out=out), gb, seconds)
+    v_one, n_one, t_one = rate_for(lambda: oracle.transpose(x, threads=1, out=out), gb, seconds)
     return dict({"value": v_all, "unit": "GB/s", "cores": threads, "kind": "oracle",
                  "sample": f"{band} x {cols} row band ({x.nbytes >> 20} MiB) of the {rows}x{cols} "
-                           f"{str(dt)[6:]} matrix, naive oracle transpose; {n_all} calls in {t_all:.1f} s "
-                           f"on {threads} threads, {n_one} in {t_one:.1f} s on 1",
+                           f"{str(dt)[6:]} matrix, naive oracle transpose into a reused output array; "
+                           f"{n_all} calls in {t_all:.1f} s on {threads} threads, {n_one} in {t_one:.1f} s on 1",
                  "value_single_thread": v_one}, **host_cpu())
 
 
@@ -327,6 +330,7 @@ def run_reference(args):
     world, rank, _ = dist_env()
     if world > 1 and rank != 0:
         return
+    import numpy as np
     import torch
 
     import oracle
@@ -349,16 +353,17 @@ def run_reference(args):
         rows_rank, cols, eb = transpose_shape(wl, 1)
         dt = torch.float64 if eb == 8 else torch.float32
         x, band = oracle_transpose_sample(rows_rank, cols, dt)
+        out = np.empty((x.shape[1], x.shape[0]), dtype=x.dtype)
         unit = "GB/s"
         what = (f"{band} x {cols} row band ({x.nbytes >> 20} MiB) of the {rows_rank}x{cols} {str(dt)[6:]} matrix "
-                f"per step, naive oracle transpose on {threads} threads")
+                f"per step, naive oracle transpose on {threads} threads into a reused output array")
         if wl in ("default", "cfg3"):
             what += f"; plus {n_sw} oracle sweep trials per step, timed apart (`sweep`)"
         work = 2 * x.nbytes / 1e9
 
         def fn(k):
             nonlocal sweep_s
-            oracle.transpose(x, threads=threads)
+            oracle.transpose(x, threads=threads, out=out)
             if wl in ("default", "cfg3"):        # the step's second half, timed apart like our arm's
                 t = time.perf_counter()
                 sweep_sample(k)

@@ -180,15 +180,21 @@ def sweep(w: int, patterns, schemes, seed: int, first: int, n_trials: int,
     return hist
 
 
-def transpose(src: np.ndarray, threads: int = 1) -> np.ndarray:
-    """Plain definition: dst[c][r] = src[r][c] on the raw bits of a 2-D array."""
+def transpose(src: np.ndarray, threads: int = 1, out: np.ndarray | None = None) -> np.ndarray:
+    """Plain definition: dst[c][r] = src[r][c] on the raw bits of a 2-D array.  `out`: an optional
+    preallocated contiguous [cols, rows] array of src's dtype (the timing harness reuses one, so
+    that a measurement is not dominated by first-touch page faults of a fresh result array)."""
     assert src.ndim == 2
     s = src
     if s.strides[1] != s.itemsize or s.strides[0] % s.itemsize:
         s = np.ascontiguousarray(s)
     rows, cols = s.shape
     ld_src = s.strides[0] // s.itemsize if rows else cols
-    dst = np.empty((cols, rows), dtype=s.dtype)
+    if out is not None:
+        assert out.shape == (cols, rows) and out.dtype == s.dtype and out.flags.c_contiguous
+        dst = out
+    else:
+        dst = np.empty((cols, rows), dtype=s.dtype)
     _check(lib().oracle_transpose(_ptr(s), _ptr(dst), rows, cols, max(ld_src, cols),
                                   max(rows, 0), s.itemsize, threads), "transpose")
     return dst

@@ -327,7 +327,7 @@ __device__ __forceinline__ uint32_t lane_bits(int b) {
 
 struct BankMask { uint32_t b[5]; };
 
-__device__ __forceinline__ BankMask masks_ballot(uint32_t bank) {   // bank < 32
+__device__ __forceinline__ BankMask masks_ballot(uint32_t bank) {   // bits 0..4 of bank (bank mod 32)
     BankMask B;
     ballot_planes5(bank, B.b);
     return B;
@@ -366,10 +366,7 @@ __device__ __forceinline__ BankMask masks_add(const BankMask &X, const BankMask 
 }
 
 __device__ __forceinline__ uint32_t max_load(const BankMask &B, uint32_t counted, const LaneSel &ls) {
-    uint32_t m = counted;
-#pragma unroll
-    for (int k = 0; k < 5; ++k) m &= B.b[k] ^ ls.nsel[k];
-    return __reduce_max_sync(kFull, __popc(m));
+    return __reduce_max_sync(kFull, __popc(lanes_equal(B.b, counted, ls)));
 }
 
 // Per-lane constants of the two rewritten evaluators below (lane v):
@@ -535,12 +532,14 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
                             c = max_load_add_lane(isp ? Pm : Rm, le);       // bank t + shift[t]
                             goto counted;
                         }
+                        // (the ballots read bits 0..4 only: `packed` carries rcol in those bits,
+                        // and packed + shift has (rcol + shift) mod 32 there -- the "mod w")
                         if (s == RAP_SCHEME_RAW) {
                             B = (pp == RAP_PAT_STRIDE) ? masks_const(0)
-                              : (pp == RAP_PAT_RANDOM) ? masks_ballot(rcol) : masks_lane();
+                              : (pp == RAP_PAT_RANDOM) ? masks_ballot(packed) : masks_lane();
                         } else if (s == RAP_SCHEME_RAS || s == RAP_SCHEME_RAP) {
                             if (pp == RAP_PAT_STRIDE) B = isp ? Pm : Rm;
-                            else B = masks_ballot((rcol + (isp ? Pr : rr)) & 31u);
+                            else B = masks_ballot(packed + (isp ? Pr : rr));
                         } else {                                    // PAD / XOR: per-lane bank
                             uint32_t row, col;
                             switch (pp) {

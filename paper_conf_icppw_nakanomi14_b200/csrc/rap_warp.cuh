@@ -24,7 +24,7 @@ __device__ __forceinline__ uint32_t ballot_bit(uint32_t x) {
     return v;
 }
 
-// B[k] = ballot(bit k of x), k = 0..4 (x < 32)
+// B[k] = ballot(bit k of x), k = 0..4 (only bits 0..4 of x are read: x mod 32)
 __device__ __forceinline__ void ballot_planes5(uint32_t x, uint32_t (&B)[5]) {
     B[0] = ballot_bit<1u>(x);
     B[1] = ballot_bit<2u>(x);
@@ -42,21 +42,52 @@ __device__ __forceinline__ uint32_t ballot_zero(uint32_t x, uint32_t m) {
     return v;
 }
 
+// RAP_FMA_XOR (default 1): x ^ nsel_k, with nsel_k all-zero or all-one per lane, is evaluated as
+// the integer multiply-add x * (nsel_k | 1) + nsel_k -- x when nsel_k = 0, -x - 1 = ~x when
+// nsel_k = ~0 -- i.e. an IMAD on the FMA pipe; the evaluators are bound by the ALU pipe (LOP3),
+// and the remaining ANDs then take three operands per LOP3.
+#ifndef RAP_FMA_XOR
+#define RAP_FMA_XOR 1
+#endif
+
 struct LaneSel {
     uint32_t nsel[5];        // bit k of lane ? 0 : ~0
+    uint32_t flip[5];        // nsel | 1: +1 or -1
     __device__ __forceinline__ explicit LaneSel(uint32_t lane) {
 #pragma unroll
-        for (int k = 0; k < 5; ++k) nsel[k] = ((lane >> k) & 1u) ? 0u : 0xffffffffu;
+        for (int k = 0; k < 5; ++k) {
+            nsel[k] = ((lane >> k) & 1u) ? 0u : 0xffffffffu;
+            flip[k] = nsel[k] | 1u;
+        }
+    }
+    // x ^ nsel[k]
+    __device__ __forceinline__ uint32_t sel(uint32_t x, int k) const {
+#if RAP_FMA_XOR
+        return x * flip[k] + nsel[k];
+#else
+        return x ^ nsel[k];
+#endif
     }
 };
+
+// counted AND_k (B_k ^ nsel_k): lanes whose bank (bit planes B) equals this lane's index
+__device__ __forceinline__ uint32_t lanes_equal(const uint32_t (&B)[5], uint32_t counted, const LaneSel &ls) {
+#if RAP_FMA_XOR
+    const uint32_t t0 = ls.sel(B[0], 0), t1 = ls.sel(B[1], 1), t2 = ls.sel(B[2], 2), t3 = ls.sel(B[3], 3),
+                   t4 = ls.sel(B[4], 4);
+    return ((counted & t0 & t1) & t2 & t3) & t4;
+#else
+    uint32_t m = counted;
+#pragma unroll
+    for (int k = 0; k < 5; ++k) m &= B[k] ^ ls.nsel[k];
+    return m;
+#endif
+}
 
 __device__ __forceinline__ uint32_t max_bank_load(uint32_t bank, uint32_t counted, const LaneSel &ls) {
     uint32_t B[5];
     ballot_planes5(bank, B);
-    uint32_t m = counted;
-#pragma unroll
-    for (int k = 0; k < 5; ++k) m &= B[k] ^ ls.nsel[k];
-    return __reduce_max_sync(kFull, __popc(m));
+    return __reduce_max_sync(kFull, __popc(lanes_equal(B, counted, ls)));
 }
 
 // Merged requests: lanes of `active` that carry the first occurrence of their
