@@ -466,7 +466,7 @@ def hbm_roofline(nbytes: int, ms: float, peak: float, peak_src: str, kkey: str) 
     return {"bound": "hbm", "achieved": ach, "peak": peak, "unit": "GB/s", "frac": ach / peak,
             "traffic": prof.get("dram_bytes_per_launch_steady", prof.get("dram_bytes_per_launch")),
             "peak_source": peak_src, "frac_of_8TBs_nominal": ach / 8000.0, "kernel": kkey,
-            "kernel_name": prof.get("kernel"), "kernel_ms_mean": ms, "algorithmic_bytes_per_launch": nbytes,
+            "kernel_name": prof.get("kernel_name"), "kernel_ms_mean": ms, "algorithmic_bytes_per_launch": nbytes,
             "smem_wavefronts_per_request": prof.get("smem_wavefronts_per_request"),
             "profile": prof.get("source")}
 

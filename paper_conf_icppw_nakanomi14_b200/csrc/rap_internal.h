@@ -25,9 +25,17 @@ struct TileShifts {
 // byte i (< 32) of a packed TileShifts vector: uniform constant-bank words + a per-lane select
 // (a dynamic index into a kernel parameter would copy the struct to local memory)
 __device__ __forceinline__ uint32_t shift_byte(const uint32_t (&w)[8], uint32_t i) {
-    uint32_t x = w[0];
+    // the words are first moved into registers through opaque movs: otherwise the compiler
+    // recognises the select chain as an indexed parameter access and lowers THAT to a
+    // predicated walk over the whole struct, once per use
+    uint32_t r[8];
 #pragma unroll
-    for (int k = 1; k < 8; ++k) x = ((i >> 2) == (uint32_t)k) ? w[k] : x;
+    for (int k = 0; k < 8; ++k) asm("mov.b32 %0, %1;" : "=r"(r[k]) : "r"(w[k]));
+    const uint32_t q = i >> 2;
+    const uint32_t a = (q & 1u) ? r[1] : r[0], b = (q & 1u) ? r[3] : r[2];
+    const uint32_t c = (q & 1u) ? r[5] : r[4], d = (q & 1u) ? r[7] : r[6];
+    const uint32_t ab = (q & 2u) ? b : a, cd = (q & 2u) ? d : c;
+    const uint32_t x = (q & 4u) ? cd : ab;
     return (x >> (8u * (i & 3u))) & 0xffu;
 }
 TileShifts tile_shifts(int layout, uint64_t seed);

@@ -34,3 +34,16 @@ steady steady_t64_rap64 "transpose64_kernel" --workload cfg4 --steps 4 --warmup 
 steady steady_t64_rap16 "transpose_rap16_kernel" --workload cfg4 --steps 4 --warmup 3
 steady steady_t32 "^transpose_kernel" --workload cfg3 --steps 4 --warmup 3 --sweep-trials 1024
 ls -la "$OUT"
+# export the pages the summary reads, keep compressed reports of the key kernels only (gpurun
+# brings back at most 64 MiB)
+for rep in "$OUT"/*.ncu-rep; do
+  stem=${rep%.ncu-rep}
+  ncu -i "$rep" --page raw --csv > "$stem.raw.csv" 2>/dev/null
+  ncu -i "$rep" --page source --csv --print-source sass > "$stem.source.csv" 2>/dev/null
+  case $(basename "$stem") in
+    prof_t64_rap|prof_t32_rap|prof_sweep|prof_trace) gzip -9 -f "$rep" ;;
+    *) rm -f "$rep" ;;
+  esac
+done
+gzip -9 -f "$OUT"/*.source.csv
+du -sh "$OUT"

@@ -15,7 +15,7 @@ CAPTURES = {
     "transpose_b32_rap": "prof_t32_rap", "transpose_b32_raw": "prof_t32_raw",
     "transpose_b32_pad": "prof_t32_pad", "transpose_b32_xor": "prof_t32_xor",
     "transpose_b32_ras": "prof_t32_ras", "transpose_b64_rap": "prof_t64_rap",
-    "transpose_b64_rap16": "prof_t64_rap16",
+    "transpose_b64_rap16": "prof_t64_rap16", "transpose_b64_rap64": "prof_t64_rap64",
     "sweep_w32": "prof_sweep", "sweep_w32_match": "prof_sweep_match", "trace_w32": "prof_trace",
 }
 
@@ -25,7 +25,8 @@ UNITS = {"sweep_w32": ("trials", 8388608), "sweep_w32_match": ("trials", 4194304
          "transpose_b32_rap": ("bytes", 2 * 8192 * 8192 * 4), "transpose_b32_raw": ("bytes", 2 * 8192 * 8192 * 4),
          "transpose_b32_pad": ("bytes", 2 * 8192 * 8192 * 4), "transpose_b32_xor": ("bytes", 2 * 8192 * 8192 * 4),
          "transpose_b32_ras": ("bytes", 2 * 8192 * 8192 * 4), "transpose_b64_rap": ("bytes", 2 * 16384 * 16384 * 8),
-         "transpose_b64_rap16": ("bytes", 2 * 16384 * 16384 * 8)}
+         "transpose_b64_rap16": ("bytes", 2 * 16384 * 16384 * 8),
+         "transpose_b64_rap64": ("bytes", 2 * 16384 * 16384 * 8)}
 
 WANT = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum",
         "l1tex__data_pipe_lsu_wavefronts_mem_shared_op_ld.sum",
@@ -49,8 +50,22 @@ SCALE = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "ns": 1e-9, "us": 
          "msecond": 1e-3, "second": 1.0}
 
 
+def _page(rep, page):
+    """ncu's CSV export of a capture: <stem>.<page>.csv written on the GPU box (tools/ncu_export.sh),
+    else ncu -i on the .ncu-rep here."""
+    stem = rep[:-len(".ncu-rep")] if rep.endswith(".ncu-rep") else rep
+    csv_path = f"{stem}.{page}.csv"
+    if os.path.exists(csv_path):
+        return open(csv_path).read()
+    if os.path.exists(csv_path + ".gz"):
+        import gzip
+        return gzip.open(csv_path + ".gz", "rt").read()
+    args = ["ncu", "-i", rep, "--page", page, "--csv"] + (["--print-source", "sass"] if page == "source" else [])
+    return subprocess.run(args, capture_output=True, text=True).stdout
+
+
 def raw_metrics(rep):
-    out = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    out = _page(rep, "raw")
     rows = list(csv.reader(io.StringIO(out)))
     head, units, vals = rows[0], rows[1], rows[2]
     d = {}
@@ -67,8 +82,7 @@ def raw_metrics(rep):
 
 def source_smem(rep):
     """Per-instruction shared-memory wavefronts from the source page: (ld_wf, ld_inst, st_wf, st_inst, excessive)."""
-    out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "sass"],
-                         capture_output=True, text=True).stdout
+    out = _page(rep, "source")
     rows = list(csv.reader(io.StringIO(out)))
     if len(rows) < 3:
         return None
@@ -99,10 +113,13 @@ def source_smem(rep):
 def main(src_dir, dst, tag):
     kernels = {}
     for key, stem in CAPTURES.items():
-        rep = os.path.join(src_dir, stem + ".ncu-rep")
-        if not os.path.exists(rep):                     # committed copies: profiles/<tag>_<stem>
-            rep = os.path.join(src_dir, f"{tag}_{stem}.ncu-rep")
-        if not os.path.exists(rep):
+        rep = None
+        for cand in (stem, f"{tag}_{stem}"):            # committed copies: profiles/<tag>_<stem>
+            base = os.path.join(src_dir, cand)
+            if os.path.exists(base + ".ncu-rep") or os.path.exists(base + ".raw.csv"):
+                rep = base + ".ncu-rep"
+                break
+        if rep is None:
             continue
         m = raw_metrics(rep)
         ld_w = m.get("l1tex__data_pipe_lsu_wavefronts_mem_shared_op_ld.sum")
@@ -111,7 +128,7 @@ def main(src_dir, dst, tag):
         st_i = m.get("smsp__sass_inst_executed_op_shared_st.sum")
         dram = (m.get("dram__bytes_read.sum") or 0) + (m.get("dram__bytes_write.sum") or 0)
         kernels[key] = {
-            "source": f"profiles/{tag}_{stem}.ncu-rep (ncu --set full --clock-control none)",
+            "source": f"profiles/{tag}_{stem}.ncu-rep[.gz] / .raw.csv / .source.csv (ncu --set full --clock-control none)",
             "kernel_name": m.get("kernel_name"),
             "duration_us_cold": m.get("gpu__time_duration.sum", 0) * 1e6,
             "dram_bytes_read": m.get("dram__bytes_read.sum"), "dram_bytes_write": m.get("dram__bytes_write.sum"),
@@ -149,7 +166,7 @@ def main(src_dir, dst, tag):
     # a launch leaves in L2 are written back during the next one, so per-launch read + write
     # bytes here are the true cost (the --set full captures flush caches between replays)
     for key, stem in (("transpose_b32_rap", "steady_t32"), ("transpose_b64_rap", "steady_t64"),
-                       ("transpose_b64_rap16", "steady_t64_rap16")):
+                       ("transpose_b64_rap16", "steady_t64_rap16"), ("transpose_b64_rap64", "steady_t64_rap64")):
         path = os.path.join(src_dir, stem + ".csv")
         if not os.path.exists(path):
             path = os.path.join(src_dir, f"{tag}_steady_dram_{stem[7:]}.csv")
