@@ -51,6 +51,7 @@ SWEEP_SEED = 1
 CFG3_LAYOUTS = ["raw", "pad", "xor", "ras", "rap"]
 CFG4_LAYOUTS = ["raw", "pad", "xor", "ras", "rap", "rap64", "rap16"]
 ORACLE_BAND_BYTES = 32 << 20   # the oracle's transpose sample: one row band of this many bytes
+E2E_WS = 512 << 20             # device workspace of the cfg4 host-to-host transpose (4 band buffers)
 
 
 # The JSON line goes to the process's original stdout; everything else that native code prints
@@ -420,6 +421,19 @@ def cpu_baseline_trace():
                 **host_cpu())
 
 
+def _pipe_frac(prof: dict, pipe: str):
+    """ncu's sm__inst_executed_pipe_<pipe> active fraction of the committed capture, if exported."""
+    src = (prof or {}).get("source", "")
+    path = os.path.join(ROOT, src.split()[0].replace(".ncu-rep[.gz]", ".raw.csv")) if src else ""
+    if not path.endswith(".raw.csv") or not os.path.exists(path):
+        return None
+    import csv
+    rows = list(csv.reader(open(path)))
+    h, v = rows[0], rows[2]
+    key = f"sm__inst_executed_pipe_{pipe}.avg.pct_of_peak_sustained_active"
+    return float(v[h.index(key)].replace(",", "")) / 100 if key in h else None
+
+
 def sweep_roofline(tps: float, clocks: dict):
     """ALU roofline of the sweep.  The binding unit is the ALU pipe (LOP3 / SHF / ISETP / IADD3 ...),
     which accepts one warp-instruction every 2 cycles per SMSP (B300_MICROARCH.md "Pipe rates"):
@@ -439,7 +453,10 @@ def sweep_roofline(tps: float, clocks: dict):
             "issue_frac": ipt * tps / issue_peak if ipt else None,
             "peak_source": "148 SMs x 4 SMSPs x 0.5 ALU warp-instr/clk (B300_MICROARCH.md pipe rates) x sm_max_mhz",
             "profile": prof.get("source"), "alu_pipe_active_frac_ncu": prof.get("alu_pipe_active_frac"),
-            "issue_active_frac_ncu": prof.get("issue_active_frac")}
+            "adu_pipe_active_frac_ncu": _pipe_frac(prof, "adu"),
+            "issue_active_frac_ncu": prof.get("issue_active_frac"),
+            "note": "integer kernel co-limited by the ALU pipe (LOP3/SHF/VOTE-free work) and the ADU pipe "
+                    "(VOTE ballots, CREDUX reductions, R2P): both ~74% active in the ncu capture"}
 
 
 def trace_roofline(eps: float, clocks: dict):
@@ -700,13 +717,13 @@ def run_default(args):
         hx = x.cpu().pin_memory()
         hy = torch.empty((cols, rows), dtype=dt).pin_memory()
         for _ in range(2):
-            rap.transpose_host(hx, out=hy, layout="rap", seed=0, device=dev)
+            rap.transpose_host(hx, out=hy, layout="rap", seed=0, device=dev, workspace_bytes=E2E_WS)
         barrier()
         st = torch.cuda.Event(enable_timing=True)
         en = torch.cuda.Event(enable_timing=True)
         st.record(stream)
         for _ in range(KE):
-            rap.transpose_host(hx, out=hy, layout="rap", seed=0, device=dev)
+            rap.transpose_host(hx, out=hy, layout="rap", seed=0, device=dev, workspace_bytes=E2E_WS)
         en.record(stream)
         torch.cuda.synchronize()
         ms = rmax(st.elapsed_time(en)) / KE
@@ -716,7 +733,8 @@ def run_default(args):
                        "h2d_bytes_per_step": hx.numel() * 8 * world, "d2h_bytes_per_step": hy.numel() * 8 * world,
                        "ms_per_step": ms, "steps": KE,
                        "note": "rap_transpose_host: pinned host cfg4 matrix in, pinned host transpose out; "
-                               "upload / RAP transpose / download of row bands (128 MiB workspace) overlapped"}
+                               f"upload / RAP transpose / download of row bands ({E2E_WS >> 20} MiB workspace) "
+                               "overlapped"}
         del hx, hy
     if rank == 0 and not args.no_cpu and world == 1:
         line["cpu_baseline"] = cpu_baseline_transpose(rows, cols, dt)

@@ -26,7 +26,7 @@ for (r, c, dt) in ((8192, 8192, torch.float32), (16384, 16384, torch.float64)):
     x = workloads.random_bits(r, c, dt, seed=0).pin_memory()
     y = torch.empty((c, r), dtype=dt).pin_memory()
     nbytes = 2 * x.numel() * x.element_size()
-    for ws in (16 << 20, 32 << 20, 64 << 20, 128 << 20, 256 << 20):
+    for ws in (64 << 20, 128 << 20, 256 << 20, 512 << 20, 1024 << 20):
         el = t_of(lambda: rap.transpose_host(x, out=y, workspace_bytes=ws))
         print(r, c, str(dt)[6:], 'ws MiB', ws >> 20, f'{nbytes / el / 1e9:.1f} GB/s', f'{el * 1e3:.2f} ms', flush=True)
     d = x.cuda()
