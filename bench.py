@@ -51,7 +51,7 @@ SWEEP_SEED = 1
 CFG3_LAYOUTS = ["raw", "pad", "xor", "ras", "rap"]
 CFG4_LAYOUTS = ["raw", "pad", "xor", "ras", "rap", "rap64", "rap16"]
 ORACLE_BAND_BYTES = 32 << 20   # the oracle's transpose sample: one row band of this many bytes
-E2E_WS = 512 << 20             # device workspace of the cfg4 host-to-host transpose (4 band buffers)
+E2E_WS = 128 << 20             # device workspace of the cfg4 host-to-host transpose (4 band buffers)
 
 
 # The JSON line goes to the process's original stdout; everything else that native code prints
@@ -331,13 +331,20 @@ def run_reference(args):
     world, rank, _ = dist_env()
     if world > 1 and rank != 0:
         return
+    emit(oracle_arm(args, world))
+
+
+def oracle_arm(args, world: int, threads: int | None = None, workload: str | None = None) -> dict:
+    """The reference arm's measurement (K steps of the workload's oracle sample after W warm-ups),
+    as the JSON line `--impl reference` prints.  Our arm's `cpu_baseline` objects call the same
+    function (same sample, same step structure), so the two agree up to box noise."""
     import numpy as np
     import torch
 
     import oracle
-    threads = oracle.max_threads()
-    wl = args.workload
-    cfg = arm_config(args, world)          # the same workload / config as our arm's line
+    threads = oracle.max_threads() if threads is None else threads
+    wl = args.workload if workload is None else workload
+    cfg = arm_config(args if workload is None else argparse.Namespace(**dict(vars(args), workload=wl)), world)
     n_sw = 20000                           # oracle sweep sample: trials per step
 
     def sweep_sample(k):
@@ -387,7 +394,7 @@ def run_reference(args):
             "e2e": {"value": value, "unit": unit, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     if wl in ("default", "cfg3"):
         line["sweep"] = {"trials_per_s": n_sw * args.steps / sweep_s, "trials_per_step": n_sw}
-    emit(line)
+    return line
 
 
 def oracle_trace_sample():
@@ -737,9 +744,22 @@ def run_default(args):
                                "overlapped"}
         del hx, hy
     if rank == 0 and not args.no_cpu and world == 1:
-        line["cpu_baseline"] = cpu_baseline_transpose(rows, cols, dt)
-        line["sweep"]["cpu_baseline"] = cpu_baseline_sweep()
-        line["cfg3_layouts"]["cpu_baseline"] = cpu_baseline_transpose(8192, 8192, torch.float32)
+        # the reference arm's own measurement (oracle_arm), all host cores, plus one core
+        ref = oracle_arm(args, 1)
+        one = oracle_arm(args, 1, threads=1)
+        cb = dict(ref["cpu_baseline"], value_single_thread=one["value"],
+                  sample=ref["cpu_baseline"]["sample"] + f"; {args.steps} steps after {args.warmup} warm-ups "
+                         "(the --impl reference measurement); value_single_thread: the same on 1 thread")
+        line["cpu_baseline"] = cb
+        line["sweep"]["cpu_baseline"] = dict({"value": ref["sweep"]["trials_per_s"], "unit": "trials/s",
+                                               "cores": cb["cores"], "kind": "oracle",
+                                               "value_single_thread": one["sweep"]["trials_per_s"],
+                                               "sample": f"{ref['sweep']['trials_per_step']} oracle trials of the "
+                                                         "w=32 sweep per step (the --impl reference step)"},
+                                              **host_cpu())
+        c3 = oracle_arm(args, 1, workload="cfg3")
+        line["cfg3_layouts"]["cpu_baseline"] = dict(c3["cpu_baseline"], value_single_thread=oracle_arm(
+            args, 1, threads=1, workload="cfg3")["value"])
         line["cfg1_tile_cpu_baseline"] = cpu_baseline_tile()
     if rank == 0:
         emit(line)
