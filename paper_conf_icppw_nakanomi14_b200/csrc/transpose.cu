@@ -43,9 +43,16 @@ namespace rapk {
 //          RAW / XOR: 32 words; PAD: 33 words (the [32][33] baseline).
 //   EW   : 4-byte words per element (1: 32-bit, 2: 64-bit split into lo / hi planes, each a
 //          full 32 x RP array, so both planes see the 32-bit bank function).
+// RAP32_WRAP (tuning, default 0): RAP / RAS rows 32 words wide with the rotation wrapped in the
+// address arithmetic, (j + sh[i]) & 31 -- half the shared memory per tile, two more ALU
+// operations per shared access
+#ifndef RAP32_WRAP
+#define RAP32_WRAP 0
+#endif
 template <int L>
 struct Geom {
-    static constexpr int RP = (L == RAP_LAYOUT_RAP || L == RAP_LAYOUT_RAS) ? 64
+    static constexpr bool WRAP = RAP32_WRAP && (L == RAP_LAYOUT_RAP || L == RAP_LAYOUT_RAS);
+    static constexpr int RP = WRAP ? 32 : (L == RAP_LAYOUT_RAP || L == RAP_LAYOUT_RAS) ? 64
                             : (L == RAP_LAYOUT_PAD) ? 33 : 32;
 };
 
@@ -57,6 +64,7 @@ template <int L>
 __device__ __forceinline__ uint32_t word_of(uint32_t row, uint32_t col, uint32_t sh) {
     constexpr int RP = Geom<L>::RP;
     if (L == RAP_LAYOUT_XOR) return row * RP + (col ^ row);
+    if (Geom<L>::WRAP) return row * RP + ((col + sh) & 31u);
     if (L == RAP_LAYOUT_RAS || L == RAP_LAYOUT_RAP) return row * RP + col + sh;
     return row * RP + col;
 }
@@ -137,14 +145,20 @@ transpose_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, i
     // RAP: the R rows of group g are P^-1(R*g + 0..R-1) -- one row per residue of P mod R --
     // so each STS of the group hits 32 distinct banks.
     const uint32_t q = lane % LPR, c_in = lane / LPR;
-    uint32_t row_g[G], a_g[G];
+    constexpr bool WRAP = Geom<L>::WRAP;
+    uint32_t row_g[G], a_g[G], rot_g[WRAP ? G : 1];
     const uint32_t pinv = (L == RAP_LAYOUT_RAP) ? shift_byte(ts.inv, lane) : lane;
 #pragma unroll
     for (int g = 0; g < G; ++g) {
         const uint32_t rr = (uint32_t)(R * g) + c_in;
         row_g[g] = (L == RAP_LAYOUT_RAP) ? __shfl_sync(kFull, pinv, rr) : rr;
         const uint32_t shg = (L == RAP_LAYOUT_RAP) ? rr : __shfl_sync(kFull, sh_lane, rr);
-        a_g[g] = word_of<L>(row_g[g], NE * q, shg);     // first element of the chunk
+        if constexpr (WRAP) {
+            a_g[g] = row_g[g] * Geom<L>::RP;            // row base; column (NE*q + e + sh) & 31
+            rot_g[g] = NE * q + shg;
+        } else {
+            a_g[g] = word_of<L>(row_g[g], NE * q, shg);  // first element of the chunk
+        }
     }
     const uint32_t drain_base = word_of<L>(lane, 0, sh_lane);
 
@@ -200,6 +214,7 @@ transpose_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, i
                 const uint32_t e = k / EW, plane = k % EW;     // element of the chunk, lo/hi word
                 uint32_t off;
                 if (L == RAP_LAYOUT_XOR) off = word_of<L>(row_g[g], NE * q + e, 0);
+                else if constexpr (WRAP) off = a_g[g] + ((rot_g[g] + e) & 31u);
                 else off = a_g[g] + e;
                 tile[plane * PW + off] = w4[k];
             }
@@ -233,7 +248,7 @@ transpose_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, i
                 if (EW == 1) {
 #pragma unroll
                     for (int m = 0; m < 4; ++m) {
-                        const uint32_t off = (L == RAP_LAYOUT_XOR) ? word_of<L>(lane, 4 * cg + m, 0) : drain_base + 4 * cg + m;
+                        const uint32_t off = (L == RAP_LAYOUT_XOR || WRAP) ? word_of<L>(lane, 4 * cg + m, sh_lane) : drain_base + 4 * cg + m;
                         r[m] = tile[off];
                     }
                     const bool b0 = lane & 1u, b1 = lane & 2u;
@@ -248,7 +263,7 @@ transpose_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, i
                 } else {
 #pragma unroll
                     for (int m = 0; m < 2; ++m) {
-                        const uint32_t off = (L == RAP_LAYOUT_XOR) ? word_of<L>(lane, 2 * cg + m, 0) : drain_base + 2 * cg + m;
+                        const uint32_t off = (L == RAP_LAYOUT_XOR || WRAP) ? word_of<L>(lane, 2 * cg + m, sh_lane) : drain_base + 2 * cg + m;
                         r[2 * m] = tile[off];
                         r[2 * m + 1] = tile[PW + off];
                     }
@@ -263,7 +278,7 @@ transpose_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, i
         } else if ((r0 + 32 <= rows) && (c0 + 32 <= cols)) {
 #pragma unroll
             for (int c = 0; c < 32; ++c) {
-                const uint32_t off = (L == RAP_LAYOUT_XOR) ? word_of<L>(lane, c, 0) : drain_base + c;
+                const uint32_t off = (L == RAP_LAYOUT_XOR || WRAP) ? word_of<L>(lane, c, sh_lane) : drain_base + c;
                 if (EW == 1) *o = tile[off];
                 else *reinterpret_cast<uint2 *>(o) = make_uint2(tile[off], tile[PW + off]);
                 o += ostride;
@@ -272,7 +287,7 @@ transpose_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, i
             const bool rok = r0 + lane < rows;
             const int cmax = (int)min((int64_t)32, cols - c0);
             for (int c = 0; c < cmax; ++c) {
-                const uint32_t off = (L == RAP_LAYOUT_XOR) ? word_of<L>(lane, c, 0) : drain_base + c;
+                const uint32_t off = (L == RAP_LAYOUT_XOR || WRAP) ? word_of<L>(lane, c, sh_lane) : drain_base + c;
                 if (rok) {
                     if (EW == 1) *o = tile[off];
                     else *reinterpret_cast<uint2 *>(o) = make_uint2(tile[off], tile[PW + off]);
@@ -287,7 +302,7 @@ transpose_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, i
         constexpr int SW = SR * 32;                                // staging row length (elements)
 #pragma unroll
         for (int c = 0; c < 32; ++c) {
-            const uint32_t off = (L == RAP_LAYOUT_XOR) ? word_of<L>(lane, c, 0) : drain_base + c;
+            const uint32_t off = (L == RAP_LAYOUT_XOR || WRAP) ? word_of<L>(lane, c, sh_lane) : drain_base + c;
             const uint32_t e = (wc * 32 + c) * SW + wr * 32 + lane;
             if (EW == 1) staging[e] = tile[off];
             else *reinterpret_cast<uint2 *>(staging + 2 * e) = make_uint2(tile[off], tile[PW + off]);
