@@ -51,7 +51,8 @@ SWEEP_SEED = 1
 CFG3_LAYOUTS = ["raw", "pad", "xor", "ras", "rap"]
 CFG4_LAYOUTS = ["raw", "pad", "xor", "ras", "rap", "rap64", "rap16"]
 ORACLE_BAND_BYTES = 32 << 20   # the oracle's transpose sample: one row band of this many bytes
-E2E_WS = 128 << 20             # device workspace of the cfg4 host-to-host transpose (4 band buffers)
+E2E_WS = 64 << 20              # device workspace of the cfg4 host-to-host transpose: 4 band buffers of
+                               # 128 rows (profiles/r02_e2e_bands.txt: the fastest band plan for cfg4)
 
 
 # The JSON line goes to the process's original stdout; everything else that native code prints

@@ -408,6 +408,23 @@ __device__ __forceinline__ uint32_t max_load_add_lane(const BankMask &Y, const L
     return __reduce_max_sync(kFull, __popc(S[0] & S[1] & S[2] & S[3] & S[4]));
 }
 
+// RAP_SWEEP_SMEM_BANKS (default 1): the accesses whose banks are data-dependent per lane -- RAS
+// stride (bank r[t]), RAS diagonal (t + r[t]), and the random cells under RAW / RAS / RAP -- are
+// counted with shared-memory atomics instead of ballots: each counted lane adds 1 to its bank's
+// counter (a [32] array per evaluation and warp, conflict-free across distinct banks) and gets
+// the previous count back; the congestion is the warp maximum of (previous + 1), i.e. the final
+// count of the fullest bank.  That replaces 5 VOTE + 1 R2P (the ADU pipe, which co-limits the
+// kernel with the ALU pipe) and the mask algebra by one ATOMS (the MIO / shared-memory pipe)
+// per access; the counters are cleared after the trial (one STS per lane and evaluation).
+#ifndef RAP_SWEEP_SMEM_BANKS
+#define RAP_SWEEP_SMEM_BANKS 1
+#endif
+constexpr int kSmemBankEvals = 5;      // RAS stride, RAS diagonal, random RAW / RAS / RAP
+
+__device__ __forceinline__ uint32_t count_in_bank(uint32_t *cnt, uint32_t bank, bool counted) {
+    return counted ? atomicAdd(cnt + (bank & 31u), 1u) + 1u : 0u;
+}
+
 template <uint32_t PM, uint32_t SM>
 __global__ void __launch_bounds__(kSweepWarpsV2 * 32, RAP_SWEEP_MINB)
 sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint64_t n_trials,
@@ -420,6 +437,7 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
     __shared__ uint32_t sh_hist[nbins];
     __shared__ uint32_t sh_tr[kSweepWarpsV2][32 * 33];
     __shared__ uint32_t sh_res[kSweepWarpsV2][32];
+    __shared__ uint32_t sh_cnt[RAP_SWEEP_SMEM_BANKS ? kSweepWarpsV2 : 1][kSmemBankEvals][32];
     const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
     for (uint32_t b = threadIdx.x; b < nbins; b += blockDim.x) sh_hist[b] = 0;
     __syncthreads();
@@ -428,6 +446,13 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
     const uint32_t lt_mask = (1u << lane) - 1u;
     uint32_t *tr = sh_tr[warp];
     uint32_t *res = sh_res[warp];
+    uint32_t *cnt = &sh_cnt[RAP_SWEEP_SMEM_BANKS ? warp : 0][0][0];
+    constexpr bool kSB = RAP_SWEEP_SMEM_BANKS != 0;
+    if (kSB) {
+#pragma unroll
+        for (int e = 0; e < kSmemBankEvals; ++e) cnt[e * 32 + lane] = 0u;
+        __syncwarp();
+    }
 
     // Accesses whose banks do not depend on the trial's draws -- every non-random pattern under
     // the deterministic maps RAW / PAD / XOR -- have the same congestion in every trial:
@@ -490,7 +515,7 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
             const uint32_t packed = tr[lane * 33 + m];
             const uint32_t rt = packed >> 10;
             BankMask Rm;
-            if (need_r) Rm = masks_ballot(rt);                      // bit t = bit b of r[t]
+            if (need_r && !kSB) Rm = masks_ballot(rt);              // bit t = bit b of r[t]
             uint32_t rrow = 0, rcol = 0, Pr = 0, rr = 0, leaders = kFull;
             if (any_random) {
                 const uint32_t cell = packed & 1023u;
@@ -525,6 +550,18 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
                                : (s == RAP_SCHEME_PAD) ? -1 : RAP_PAT_DIAGONAL) : p;
                         BankMask B;
                         const bool isp = (s == RAP_SCHEME_RAP);
+                        if (kSB && ((s == RAP_SCHEME_RAS && (pp == RAP_PAT_STRIDE || pp == RAP_PAT_DIAGONAL)) ||
+                                    pp == RAP_PAT_RANDOM)) {
+                            // shared-memory bank counters (slot: RAS stride 0, RAS diagonal 1,
+                            // random RAW / RAS / RAP 2 / 3 / 4); packed carries rcol in bits 0..4
+                            const int slot = pp == RAP_PAT_STRIDE ? 0 : pp == RAP_PAT_DIAGONAL ? 1
+                                           : s == RAP_SCHEME_RAW ? 2 : s == RAP_SCHEME_RAS ? 3 : 4;
+                            const uint32_t bank = pp == RAP_PAT_STRIDE ? rt : pp == RAP_PAT_DIAGONAL ? lane + rt
+                                                : packed + (s == RAP_SCHEME_RAW ? 0u : isp ? Pr : rr);
+                            const bool counted = pp != RAP_PAT_RANDOM || ((leaders >> lane) & 1u);
+                            c = __reduce_max_sync(kFull, count_in_bank(cnt + slot * 32, bank, counted));
+                            goto counted;
+                        }
                         if ((s == RAP_SCHEME_RAS || s == RAP_SCHEME_RAP) && pp == RAP_PAT_CONTIGUOUS) {
                             c = max_load_rot(isp ? P0 : r0, le);            // bank t + shift[0]
                             goto counted;
@@ -563,6 +600,10 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
             }
             __syncwarp();
             if (lane < e) atomicAdd(&sh_hist[lane * (w + 1) + res[lane]], 1u);
+            if (kSB) {                                                  // clear the bank counters
+#pragma unroll
+                for (int k = 0; k < kSmemBankEvals; ++k) cnt[k * 32 + lane] = 0u;
+            }
             __syncwarp();
         }
         __syncwarp();

@@ -63,10 +63,15 @@ size_t host_band_rows(int64_t rows, int64_t cols, uint32_t eb, size_t work_bytes
 #define RAP_HOST_RAMP_DIV 4    // smallest ramp band = rb / RAP_HOST_RAMP_DIV (0: no ramp); narrower bands
                                // make the strided download slow (256 B of each 32 KiB row: 32 GB/s)
 #endif
-static std::vector<int64_t> band_plan(int64_t rows, int64_t rb) {
+static std::vector<int64_t> band_plan(int64_t rows, int64_t rb, uint32_t eb) {
     std::vector<int64_t> head;
     int64_t ramp = 0;
-    const int64_t s0 = RAP_HOST_RAMP_DIV ? rb / RAP_HOST_RAMP_DIV / 32 * 32 : rb;
+    int64_t s0 = RAP_HOST_RAMP_DIV ? rb / RAP_HOST_RAMP_DIV / 32 * 32 : rb;
+    // a band of s rows downloads as `cols` segments of s * eb bytes; ramp bands below 1 KiB
+    // segments cost more than the shorter fill saves (cfg4 at a 64 MiB workspace: 91 GB/s without
+    // the 256 / 512-byte ramp bands, 85 with them; profiles/r02_e2e_bands.txt)
+    const int64_t min_rows = (1024 / eb + 31) / 32 * 32;
+    if (s0 < min_rows) s0 = min_rows;
     for (int64_t s = s0 < 32 ? 32 : s0; s < rb; s *= 2) {
         head.push_back(s);
         ramp += s;
@@ -109,7 +114,7 @@ cudaError_t transpose_host(const void *h_src, void *h_dst, int64_t rows, int64_t
     const size_t band_bytes = rb * (size_t)cols * eb;
     uint8_t *din[2] = {(uint8_t *)d_work, (uint8_t *)d_work + band_bytes};
     uint8_t *dout[2] = {(uint8_t *)d_work + 2 * band_bytes, (uint8_t *)d_work + 3 * band_bytes};
-    const std::vector<int64_t> plan = band_plan(rows, (int64_t)rb);
+    const std::vector<int64_t> plan = band_plan(rows, (int64_t)rb, eb);
     const int64_t nb = (int64_t)plan.size();
     int64_t r0 = 0;
     for (int64_t b = 0; b < nb && e == cudaSuccess; r0 += plan[b], ++b) {
