@@ -419,7 +419,7 @@ __device__ __forceinline__ uint32_t max_load_add_lane(const BankMask &Y, const L
 #ifndef RAP_SWEEP_SMEM_BANKS
 #define RAP_SWEEP_SMEM_BANKS 1
 #endif
-constexpr int kSmemBankEvals = 5;      // RAS stride, RAS diagonal, random RAW / RAS / RAP
+constexpr int kSmemBankEvals = 7;      // RAS stride, RAS diagonal, random under each of the 5 schemes
 
 __device__ __forceinline__ uint32_t count_in_bank(uint32_t *cnt, uint32_t bank, bool counted) {
     return counted ? atomicAdd(cnt + (bank & 31u), 1u) + 1u : 0u;
@@ -448,6 +448,11 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
     uint32_t *res = sh_res[warp];
     uint32_t *cnt = &sh_cnt[RAP_SWEEP_SMEM_BANKS ? warp : 0][0][0];
     constexpr bool kSB = RAP_SWEEP_SMEM_BANKS != 0;
+    // counter slots in use: 0 RAS stride, 1 RAS diagonal (and malicious, which reuses them), 2 + s
+    // the random access under scheme s
+    constexpr uint32_t kSlots = (((SM >> RAP_SCHEME_RAS) & 1u) && ((PM >> RAP_PAT_STRIDE) & 1u) ? 1u : 0u) |
+                                (((SM >> RAP_SCHEME_RAS) & 1u) && ((PM >> RAP_PAT_DIAGONAL) & 1u) ? 2u : 0u) |
+                                (((PM >> RAP_PAT_RANDOM) & 1u) ? (SM << 2) : 0u);
     if (kSB) {
 #pragma unroll
         for (int e = 0; e < kSmemBankEvals; ++e) cnt[e * 32 + lane] = 0u;
@@ -553,11 +558,14 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
                         if (kSB && ((s == RAP_SCHEME_RAS && (pp == RAP_PAT_STRIDE || pp == RAP_PAT_DIAGONAL)) ||
                                     pp == RAP_PAT_RANDOM)) {
                             // shared-memory bank counters (slot: RAS stride 0, RAS diagonal 1,
-                            // random RAW / RAS / RAP 2 / 3 / 4); packed carries rcol in bits 0..4
-                            const int slot = pp == RAP_PAT_STRIDE ? 0 : pp == RAP_PAT_DIAGONAL ? 1
-                                           : s == RAP_SCHEME_RAW ? 2 : s == RAP_SCHEME_RAS ? 3 : 4;
+                            // random under scheme s 2 + s); packed carries rcol in bits 0..4, and
+                            // count_in_bank reduces the bank mod 32
+                            const int slot = pp == RAP_PAT_STRIDE ? 0 : pp == RAP_PAT_DIAGONAL ? 1 : 2 + s;
                             const uint32_t bank = pp == RAP_PAT_STRIDE ? rt : pp == RAP_PAT_DIAGONAL ? lane + rt
-                                                : packed + (s == RAP_SCHEME_RAW ? 0u : isp ? Pr : rr);
+                                                : s == RAP_SCHEME_RAW ? packed
+                                                : s == RAP_SCHEME_PAD ? rrow + rcol
+                                                : s == RAP_SCHEME_XOR ? (rcol ^ rrow)
+                                                : packed + (isp ? Pr : rr);
                             const bool counted = pp != RAP_PAT_RANDOM || ((leaders >> lane) & 1u);
                             c = __reduce_max_sync(kFull, count_in_bank(cnt + slot * 32, bank, counted));
                             goto counted;
@@ -602,7 +610,8 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
             if (lane < e) atomicAdd(&sh_hist[lane * (w + 1) + res[lane]], 1u);
             if (kSB) {                                                  // clear the bank counters
 #pragma unroll
-                for (int k = 0; k < kSmemBankEvals; ++k) cnt[k * 32 + lane] = 0u;
+                for (int k = 0; k < kSmemBankEvals; ++k)
+                    if ((kSlots >> k) & 1u) cnt[k * 32 + lane] = 0u;
             }
             __syncwarp();
         }
@@ -774,6 +783,9 @@ __device__ __forceinline__ bool lane_active(uint32_t w) { return W == 32 || (thr
 template <int W>
 __device__ __forceinline__ uint32_t wrap_w(uint32_t x, uint32_t w) { return W == 32 ? x : (x >= w ? x - w : x); }
 
+#ifndef RAP_TRACE_SMEM_BANKS
+#define RAP_TRACE_SMEM_BANKS 1
+#endif
 // W = 32: compile-time w (cells split by shift / mask, the ballots' bits 0..4 are the "mod 32");
 // W = 0: runtime w < 32 (lanes >= w idle, explicit mod w, w + 1 bins per scheme).
 template <int W, uint32_t SM>
@@ -786,6 +798,10 @@ trace32_kernel(uint32_t w_rt, uint64_t n_warps, const uint32_t *__restrict__ cel
     constexpr uint32_t nsch = __builtin_popcount(SM);
     constexpr bool need_p = (SM >> RAP_SCHEME_RAP) & 1u, need_r = (SM >> RAP_SCHEME_RAS) & 1u;
     __shared__ uint8_t shP[kTraceTB][32], shR[kTraceTB][32];
+    // RAP_TRACE_SMEM_BANKS: per-trial RAS / RAP evaluations count the lanes of each bank with
+    // shared-memory atomics (see RAP_SWEEP_SMEM_BANKS) -- four counter sets per warp, one per
+    // trial of the unrolled loop, cleared after use
+    __shared__ uint32_t sh_tcnt[RAP_TRACE_SMEM_BANKS ? kTraceWarps : 1][4][32];
     const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
     const LaneSel ls(lane);
     const uint32_t lt_mask = (1u << lane) - 1u;
@@ -793,6 +809,11 @@ trace32_kernel(uint32_t w_rt, uint64_t n_warps, const uint32_t *__restrict__ cel
 #pragma unroll
     for (uint32_t e = 0; e < nsch; ++e) hc[e] = 0;
     uint32_t hbad = 0;                                      // evaluations of warps with a bad cell
+    if (RAP_TRACE_SMEM_BANKS && W == 32) {
+#pragma unroll
+        for (int k = 0; k < 4; ++k) sh_tcnt[RAP_TRACE_SMEM_BANKS ? warp : 0][k][lane] = 0u;
+        __syncwarp();
+    }
     const uint64_t nkc = (n_warps + kTraceTK - 1) / kTraceTK;
     const uint64_t ntb = (n_trials + kTraceTB - 1) / kTraceTB;
     for (uint64_t unit = blockIdx.x; unit < ntb * nkc; unit += gridDim.x) {
@@ -825,6 +846,19 @@ trace32_kernel(uint32_t w_rt, uint64_t n_warps, const uint32_t *__restrict__ cel
                     const uint32_t bank = s == RAP_SCHEME_RAW ? col : s == RAP_SCHEME_PAD ? wrap_w<W>(row + col, w) : (col ^ row);
                     const uint32_t c = max_bank_load(bank, leaders, ls);
                     hc[e] += (c == lane + 1u) ? tcnt : 0u;
+                } else if (RAP_TRACE_SMEM_BANKS && W == 32) {
+                    const uint8_t *sh = s == RAP_SCHEME_RAP ? &shP[0][0] : &shR[0][0];
+                    uint32_t *cnt = &sh_tcnt[RAP_TRACE_SMEM_BANKS ? warp : 0][0][0];
+                    const bool lead = (leaders >> lane) & 1u;
+#pragma unroll 4
+                    for (uint32_t t = 0; t < tcnt; ++t) {
+                        uint32_t *ct = cnt + (t & 3u) * 32;
+                        const uint32_t c = __reduce_max_sync(kFull, count_in_bank(ct, col + sh[t * 32 + row], lead));
+                        __syncwarp();
+                        ct[lane] = 0u;                     // every lane's increment has returned
+                        hc[e] += (c == lane + 1u) ? 1u : 0u;
+                    }
+                    __syncwarp();
                 } else {
                     const uint8_t *sh = s == RAP_SCHEME_RAP ? &shP[0][0] : &shR[0][0];
 #pragma unroll 4
