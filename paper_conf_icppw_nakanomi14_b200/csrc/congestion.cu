@@ -422,7 +422,9 @@ __device__ __forceinline__ uint32_t max_load_add_lane(const BankMask &Y, const L
 constexpr int kSmemBankEvals = 7;      // RAS stride, RAS diagonal, random under each of the 5 schemes
 
 __device__ __forceinline__ uint32_t count_in_bank(uint32_t *cnt, uint32_t bank, bool counted) {
-    return counted ? atomicAdd(cnt + (bank & 31u), 1u) + 1u : 0u;
+    // every lane issues the atomic (a merged duplicate adds 0 to its leader's bank): no branch
+    const uint32_t one = counted ? 1u : 0u;
+    return (atomicAdd(cnt + (bank & 31u), one) + 1u) * one;
 }
 
 template <uint32_t PM, uint32_t SM>
@@ -483,6 +485,25 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
             cfix[p][s] = max_load(masks_ballot(bank), kFull, ls);
         }
     }
+    // evaluation slots of the trial-invariant accesses (bit e) and, for lane e, its congestion:
+    // they are counted once per batch (+nvalid) instead of once per trial
+    uint32_t fixed_slots = 0, fix_lane = 0;
+    {
+        uint32_t e = 0;
+#pragma unroll
+        for (int p = 0; p < 5; ++p) {
+#pragma unroll
+            for (int s = 0; s < 5; ++s) {
+                if (!((PM >> p) & 1u) || !((SM >> s) & 1u)) continue;
+                if (p != RAP_PAT_RANDOM && (s == RAP_SCHEME_RAW || s == RAP_SCHEME_PAD || s == RAP_SCHEME_XOR)) {
+                    fixed_slots |= 1u << e;
+                    if (lane == e) fix_lane = cfix[p][s];
+                }
+                ++e;
+            }
+        }
+    }
+    const bool lane_fixed = (fixed_slots >> lane) & 1u;
 
     const uint64_t nbatch = (n_trials + 31) / 32;
     const uint64_t stride = (uint64_t)gridDim.x * kSweepWarpsV2;
@@ -602,12 +623,12 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
                 counted:
                     if (p == RAP_PAT_STRIDE) c_stride[s] = c;
                     if (p == RAP_PAT_DIAGONAL) c_diag[s] = c;
-                    if (lane == 0) res[e] = c;                      // C4: result slot e
+                    if (lane == 0 && !((fixed_slots >> e) & 1u)) res[e] = c;   // C4: result slot e
                     ++e;
                 }
             }
             __syncwarp();
-            if (lane < e) atomicAdd(&sh_hist[lane * (w + 1) + res[lane]], 1u);
+            if (lane < e && !lane_fixed) atomicAdd(&sh_hist[lane * (w + 1) + res[lane]], 1u);
             if (kSB) {                                                  // clear the bank counters
 #pragma unroll
                 for (int k = 0; k < kSmemBankEvals; ++k)
@@ -615,6 +636,7 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
             }
             __syncwarp();
         }
+        if (lane_fixed) atomicAdd(&sh_hist[lane * (w + 1) + fix_lane], nvalid);   // trial-invariant slots
         __syncwarp();
     }
     __syncthreads();
