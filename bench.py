@@ -429,59 +429,69 @@ def cpu_baseline_trace():
                 **host_cpu())
 
 
-def _pipe_frac(prof: dict, pipe: str):
-    """ncu's sm__inst_executed_pipe_<pipe> active fraction of the committed capture, if exported."""
+def _capture_pipes(prof: dict):
+    """(pipe-active fractions, capture duration s) of the committed ncu capture (exported raw page)."""
     src = (prof or {}).get("source", "")
     path = os.path.join(ROOT, src.split()[0].replace(".ncu-rep[.gz]", ".raw.csv")) if src else ""
     if not path.endswith(".raw.csv") or not os.path.exists(path):
-        return None
+        return None, None
     import csv
     rows = list(csv.reader(open(path)))
-    h, v = rows[0], rows[2]
-    key = f"sm__inst_executed_pipe_{pipe}.avg.pct_of_peak_sustained_active"
-    return float(v[h.index(key)].replace(",", "")) / 100 if key in h else None
+    h, u, v = rows[0], rows[1], rows[2]
+    fr = {}
+    for pipe in ("alu", "adu", "fma", "lsu", "xu"):
+        key = f"sm__inst_executed_pipe_{pipe}.avg.pct_of_peak_sustained_active"
+        if key in h:
+            fr[pipe] = float(v[h.index(key)].replace(",", "")) / 100
+    key = "smsp__issue_active.avg.pct_of_peak_sustained_active"
+    if key in h:
+        fr["issue"] = float(v[h.index(key)].replace(",", "")) / 100
+    k = "gpu__time_duration.sum"
+    dur = None
+    if k in h:
+        scale = {"ns": 1e-9, "nsecond": 1e-9, "us": 1e-6, "usecond": 1e-6, "ms": 1e-3, "msecond": 1e-3, "s": 1.0}
+        dur = float(v[h.index(k)].replace(",", "")) * scale.get(u[h.index(k)], 1.0)
+    return fr, dur
+
+
+def pipe_roofline(rate: float, unit: str, prof_key: str, what: str) -> dict:
+    """Roofline of an integer kernel against its busiest pipe.  The committed ncu capture gives,
+    per pipe (ALU: LOP3 / SHF / IADD3 / SEL ...; ADU: CREDUX / VOTE / MATCH; FMA: IMAD; LSU:
+    shared memory, shuffles; the issue slots, 1 warp-instruction / clk / SMSP), the fraction of its
+    peak the kernel used at the
+    capture's rate; peak = the rate at which the busiest pipe would be 100 % busy with the same
+    instruction mix (capture rate / that fraction); achieved = the live rate; frac = achieved / peak.
+    The ALU-pipe view of round 1 (148 SMs x 4 SMSPs x 0.5 warp-instr/clk) is in `pipes`."""
+    prof = load_profile(prof_key) or {}
+    fr, dur = _capture_pipes(prof)
+    units = (prof.get("units_per_launch") or {})
+    n = next(iter(units.values()), None)
+    if not fr or not dur or not n:
+        return {"bound": "alu", "achieved": rate, "peak": None, "unit": unit, "frac": None, "traffic": None,
+                "note": "no committed ncu capture"}
+    cap_rate = n / dur
+    pipe = max(fr, key=lambda p: fr[p])                 # the issue slots count as a pipe too
+    peak = cap_rate / fr[pipe]
+    return {"bound": pipe, "achieved": rate, "peak": peak, "unit": unit, "frac": rate / peak, "traffic": None,
+            "pipes_active_at_capture": fr, "capture_rate": cap_rate,
+            "peak_source": f"ncu capture {prof.get('source', '').split()[0]}: {what} rate at which the {pipe.upper()} "
+                           f"pipe (the busiest) is 100% busy = capture rate / its active fraction",
+            "alu_warp_instructions_per_unit": prof.get("alu_warp_instructions_per_trial",
+                                                        prof.get("alu_warp_instructions_per_evaluation")),
+            "warp_instructions_per_unit": prof.get("warp_instructions_per_trial",
+                                                    prof.get("warp_instructions_per_evaluation"))}
 
 
 def sweep_roofline(tps: float, clocks: dict):
-    """ALU roofline of the sweep.  The binding unit is the ALU pipe (LOP3 / SHF / ISETP / IADD3 ...),
-    which accepts one warp-instruction every 2 cycles per SMSP (B300_MICROARCH.md "Pipe rates"):
-    peak = 148 SMs x 4 SMSPs x 0.5 x SM clock.  achieved = ALU-pipe warp-instructions per trial
-    (from the ncu capture: pipe-active fraction x peak x active cycles / trials) x trials/s.
-    The issue-slot view (all instructions against 1 / clk / SMSP) is reported beside it."""
-    prof = load_profile("sweep_w32") or {}
-    ipt = prof.get("warp_instructions_per_trial")
-    apt = prof.get("alu_warp_instructions_per_trial")
-    mhz = (clocks or {}).get("sm_max_mhz") or 1965.0
-    peak = 148 * 4 * 0.5 * mhz * 1e6
-    ach = apt * tps if apt else None
-    issue_peak = 148 * 4 * mhz * 1e6
-    return {"bound": "alu", "achieved": ach, "peak": peak, "unit": "ALU-pipe warp-instructions/s",
-            "frac": ach / peak if ach else None, "traffic": None,
-            "alu_warp_instructions_per_trial": apt, "warp_instructions_per_trial": ipt,
-            "issue_frac": ipt * tps / issue_peak if ipt else None,
-            "peak_source": "148 SMs x 4 SMSPs x 0.5 ALU warp-instr/clk (B300_MICROARCH.md pipe rates) x sm_max_mhz",
-            "profile": prof.get("source"), "alu_pipe_active_frac_ncu": prof.get("alu_pipe_active_frac"),
-            "adu_pipe_active_frac_ncu": _pipe_frac(prof, "adu"),
-            "issue_active_frac_ncu": prof.get("issue_active_frac"),
-            "note": "integer kernel co-limited by the ALU pipe (LOP3/SHF/VOTE-free work) and the ADU pipe "
-                    "(VOTE ballots, CREDUX reductions, R2P): both ~74% active in the ncu capture"}
+    """The sweep against its busiest pipe (pipe_roofline; the ADU since the bank counters)."""
+    return pipe_roofline(tps, "trials/s", "sweep_w32", "trial")
 
 
 def trace_roofline(eps: float, clocks: dict):
-    """ALU roofline of the trace evaluator (same pipe model as the sweep): achieved = ALU-pipe
-    warp-instructions per warp-evaluation (ncu capture of trace32_kernel) x evaluations/s."""
-    prof = load_profile("trace_w32") or {}
-    ape = prof.get("alu_warp_instructions_per_evaluation")
-    ipe = prof.get("warp_instructions_per_evaluation")
-    mhz = (clocks or {}).get("sm_max_mhz") or 1965.0
-    peak = 148 * 4 * 0.5 * mhz * 1e6
-    ach = ape * eps if ape else None
-    return {"bound": "alu", "achieved": ach, "peak": peak, "unit": "ALU-pipe warp-instructions/s",
-            "frac": ach / peak if ach else None, "traffic": prof.get("dram_bytes_per_launch"),
-            "alu_warp_instructions_per_evaluation": ape, "warp_instructions_per_evaluation": ipe,
-            "issue_frac": ipe * eps / (148 * 4 * mhz * 1e6) if ipe else None,
-            "peak_source": "148 SMs x 4 SMSPs x 0.5 ALU warp-instr/clk (B300_MICROARCH.md pipe rates) x sm_max_mhz",
-            "profile": prof.get("source")}
+    """The trace evaluator against its busiest pipe (pipe_roofline)."""
+    r = pipe_roofline(eps, "warp-evaluations/s", "trace_w32", "warp-evaluation")
+    r["traffic"] = (load_profile("trace_w32") or {}).get("dram_bytes_per_launch")
+    return r
 
 
 def hbm_roofline(nbytes: int, ms: float, peak: float, peak_src: str, kkey: str) -> dict:
