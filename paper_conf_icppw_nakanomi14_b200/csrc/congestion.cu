@@ -371,6 +371,19 @@ __device__ __forceinline__ uint32_t max_load(const BankMask &B, uint32_t counted
     return __reduce_max_sync(kFull, __popc(lanes_equal(B.b, counted, ls)));
 }
 
+// RAP_SWEEP_PACKED_MAX (default 1): the per-trial warp maxima are reduced two at a time -- two
+// lane values (<= 32) packed as 16x2 halves, five SHFL.BFLY + VIMNMX.U16x2 steps -- instead of one
+// CREDUX each: the CREDUX reductions were most of the ADU pipe, the kernel's busiest
+// (profiles/r02_prof_sweep.*); SHFL and VIMNMX run on the LSU and ALU pipes, which had room.
+#ifndef RAP_SWEEP_PACKED_MAX
+#define RAP_SWEEP_PACKED_MAX 1
+#endif
+__device__ __forceinline__ uint32_t warp_max_16x2(uint32_t x) {
+#pragma unroll
+    for (int d = 16; d >= 1; d >>= 1) x = __vimax3_u16x2(x, __shfl_xor_sync(kFull, x, d), 0u);
+    return x;
+}
+
 // Per-lane constants of the two rewritten evaluators below (lane v):
 //   E    = AND_k (L_k ^ nsel_k)  -- bit t set iff t == v (the incidence mask of the identity map)
 //   M_k  = L_k ^ nsel_k          -- bit t set iff bit k of t equals bit k of v
@@ -390,15 +403,18 @@ struct LaneEq {
 // XOR by an all-zero / all-one word, so AND_k (rotr(L_k, s) ^ nsel_k) = rotr(AND_k (L_k ^ nsel_k), s)
 // = rotr(E, s): lane v's incidence mask {t : (t + s) mod 32 = v} in one funnel shift instead of
 // 5 shifts + 5 LOP3 (bit-identical; tests/test_gpu_parity.py).
+__device__ __forceinline__ uint32_t lane_load_rot(uint32_t s, const LaneEq &le) {
+    return __popc(__funnelshift_r(le.E, le.E, s));
+}
 __device__ __forceinline__ uint32_t max_load_rot(uint32_t s, const LaneEq &le) {
-    return __reduce_max_sync(kFull, __popc(__funnelshift_r(le.E, le.E, s)));
+    return __reduce_max_sync(kFull, lane_load_rot(s, le));
 }
 
 // max_load(masks_add(masks_lane(), Y), kFull): bank(t) = (t + y_t) mod 32, y_t given as planes
 // Y_k.  The ripple-carry sum bit S_k = L_k ^ Y_k ^ c is produced already XORed with the lane's
 // selector (S_k ^ nsel_k = Y_k ^ c ^ M_k, one LOP3 as before), so the incidence mask is a plain
 // AND of five words: two LOP3 instead of five.
-__device__ __forceinline__ uint32_t max_load_add_lane(const BankMask &Y, const LaneEq &le) {
+__device__ __forceinline__ uint32_t lane_load_add_lane(const BankMask &Y, const LaneEq &le) {
     uint32_t S[5], c = 0;
 #pragma unroll
     for (int k = 0; k < 5; ++k) {
@@ -406,7 +422,10 @@ __device__ __forceinline__ uint32_t max_load_add_lane(const BankMask &Y, const L
         S[k] = Y.b[k] ^ c ^ le.M[k];
         c = (L & Y.b[k]) | (c & (L ^ Y.b[k]));
     }
-    return __reduce_max_sync(kFull, __popc(S[0] & S[1] & S[2] & S[3] & S[4]));
+    return __popc(S[0] & S[1] & S[2] & S[3] & S[4]);
+}
+__device__ __forceinline__ uint32_t max_load_add_lane(const BankMask &Y, const LaneEq &le) {
+    return __reduce_max_sync(kFull, lane_load_add_lane(Y, le));
 }
 
 // RAP_SWEEP_SMEM_BANKS (default 1): the accesses whose banks are data-dependent per lane -- RAS
@@ -426,6 +445,33 @@ __device__ __forceinline__ uint32_t count_in_bank(uint32_t *cnt, uint32_t bank, 
     // every lane issues the atomic (a merged duplicate adds 0 to its leader's bank): no branch
     const uint32_t one = counted ? 1u : 0u;
     return (atomicAdd(cnt + (bank & 31u), one) + 1u) * one;
+}
+
+// Evaluation bookkeeping of sweep32_kernel, all compile-time: evaluation e = (pattern p, scheme s)
+// in mask order; "fixed" = trial-invariant (non-random pattern under RAW / PAD / XOR); "dup" =
+// malicious access equal to the stride (RAW, RAS) or diagonal (RAP, XOR) access (reading iii).
+__host__ __device__ constexpr int eval_index(uint32_t PM, uint32_t SM, int p, int s) {
+    return __builtin_popcount(PM & ((1u << p) - 1u)) * __builtin_popcount(SM) +
+           __builtin_popcount(SM & ((1u << s) - 1u));
+}
+__host__ __device__ constexpr bool eval_fixed(int p, int s) {
+    return p != RAP_PAT_RANDOM && (s == RAP_SCHEME_RAW || s == RAP_SCHEME_PAD || s == RAP_SCHEME_XOR);
+}
+__host__ __device__ constexpr int eval_dup_src(uint32_t PM, uint32_t SM, int p, int s) {   // -1: not a duplicate
+    return (p != RAP_PAT_MALICIOUS || eval_fixed(p, s)) ? -1
+         : ((s == RAP_SCHEME_RAW || s == RAP_SCHEME_RAS) && ((PM >> RAP_PAT_STRIDE) & 1u))
+               ? eval_index(PM, SM, RAP_PAT_STRIDE, s)
+         : ((s == RAP_SCHEME_RAP || s == RAP_SCHEME_XOR) && ((PM >> RAP_PAT_DIAGONAL) & 1u))
+               ? eval_index(PM, SM, RAP_PAT_DIAGONAL, s) : -1;
+}
+struct LiveEvals { int n; int idx[25]; };
+__host__ __device__ constexpr LiveEvals live_evals(uint32_t PM, uint32_t SM) {      // evaluated per trial, in order
+    LiveEvals L{0, {}};
+    for (int p = 0; p < 5; ++p)
+        for (int s = 0; s < 5; ++s)
+            if (((PM >> p) & 1u) && ((SM >> s) & 1u) && !eval_fixed(p, s) && eval_dup_src(PM, SM, p, s) < 0)
+                L.idx[L.n++] = eval_index(PM, SM, p, s);
+    return L;
 }
 
 template <uint32_t PM, uint32_t SM>
@@ -505,6 +551,29 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
         }
     }
     const bool lane_fixed = (fixed_slots >> lane) & 1u;
+#if RAP_SWEEP_PACKED_MAX
+    // where lane e finds its evaluation's per-trial congestion: pair slot and half (a duplicate
+    // reads its source's)
+    uint32_t res_slot = 0, res_shift = 0;
+    {
+        constexpr LiveEvals LL = live_evals(PM, SM);
+#pragma unroll
+        for (int p = 0; p < 5; ++p) {
+#pragma unroll
+            for (int s = 0; s < 5; ++s) {
+                if (!((PM >> p) & 1u) || !((SM >> s) & 1u)) continue;
+                const int e = eval_index(PM, SM, p, s);
+                const int src = eval_dup_src(PM, SM, p, s) >= 0 ? eval_dup_src(PM, SM, p, s) : e;
+#pragma unroll
+                for (int i = 0; i < LL.n; ++i)
+                    if (LL.idx[i] == src && lane == (uint32_t)e) {
+                        res_slot = (uint32_t)(i / 2);
+                        res_shift = (i & 1) ? 16u : 0u;
+                    }
+            }
+        }
+    }
+#endif
 
     const uint64_t nbatch = (n_trials + 31) / 32;
     const uint64_t stride = (uint64_t)gridDim.x * kSweepWarpsV2;
@@ -553,6 +622,55 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
                 const uint32_t same = __match_any_sync(kFull, cell);   // merged requests
                 leaders = ballot_zero(same, lt_mask);              // first lane of its cell
             }
+#if RAP_SWEEP_PACKED_MAX
+            // lane values of the evaluations done per trial, then their warp maxima two at a time
+            constexpr int NE = npat * nsch;
+            uint32_t lv[NE];
+#pragma unroll
+            for (int p = 0; p < 5; ++p) {
+                if (!((PM >> p) & 1u)) continue;
+#pragma unroll
+                for (int s = 0; s < 5; ++s) {
+                    if (!((SM >> s) & 1u)) continue;
+                    const int e = eval_index(PM, SM, p, s);
+                    lv[e] = 0u;
+                    if (eval_fixed(p, s) || eval_dup_src(PM, SM, p, s) >= 0) continue;
+                    const bool isp = (s == RAP_SCHEME_RAP);
+                    if (kSB && ((s == RAP_SCHEME_RAS && (p == RAP_PAT_STRIDE || p == RAP_PAT_DIAGONAL ||
+                                                         p == RAP_PAT_MALICIOUS)) || p == RAP_PAT_RANDOM)) {
+                        // shared-memory bank counters (slot: RAS stride 0, RAS diagonal 1, random
+                        // under scheme s 2 + s); the malicious RAS access is the stride access
+                        const bool stride_like = p == RAP_PAT_STRIDE || p == RAP_PAT_MALICIOUS;
+                        const int slot = stride_like ? 0 : p == RAP_PAT_DIAGONAL ? 1 : 2 + s;
+                        const uint32_t bank = stride_like ? rt : p == RAP_PAT_DIAGONAL ? lane + rt
+                                            : s == RAP_SCHEME_RAW ? packed
+                                            : s == RAP_SCHEME_PAD ? rrow + rcol
+                                            : s == RAP_SCHEME_XOR ? (rcol ^ rrow)
+                                            : packed + (isp ? Pr : rr);
+                        lv[e] = count_in_bank(cnt + slot * 32, bank, p != RAP_PAT_RANDOM || ((leaders >> lane) & 1u));
+                    } else if (p == RAP_PAT_CONTIGUOUS) {                          // RAS / RAP
+                        lv[e] = lane_load_rot(isp ? P0 : r0, le);
+                    } else if (p == RAP_PAT_DIAGONAL || (p == RAP_PAT_MALICIOUS && isp)) {   // RAP (RAS: counters)
+                        lv[e] = lane_load_add_lane(Pm, le);
+                    } else if (p == RAP_PAT_STRIDE || p == RAP_PAT_MALICIOUS) {   // RAP stride
+                        lv[e] = __popc(lanes_equal(Pm.b, kFull, ls));
+                    }
+                }
+            }
+            // pair i of live evaluations -> res[i] = (max of the second) << 16 | max of the first;
+            // lane e of the histogram step reads its evaluation's half (res_slot / res_shift)
+            constexpr LiveEvals LL = live_evals(PM, SM);
+#pragma unroll
+            for (int i = 0; i + 1 < LL.n; i += 2) {
+                const uint32_t x = warp_max_16x2(lv[LL.idx[i]] + (lv[LL.idx[i + 1]] << 16));
+                if (lane == 0) res[i / 2] = x;
+            }
+            if (LL.n & 1) {
+                const uint32_t x = __reduce_max_sync(kFull, lv[LL.idx[LL.n - 1]]);
+                if (lane == 0) res[LL.n / 2] = x;
+            }
+            const uint32_t e = npat * nsch;
+#else
             uint32_t e = 0;
             uint32_t c_stride[5] = {0, 0, 0, 0, 0}, c_diag[5] = {0, 0, 0, 0, 0};
 #pragma unroll
@@ -628,8 +746,14 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
                     ++e;
                 }
             }
+#endif
             __syncwarp();
+#if RAP_SWEEP_PACKED_MAX
+            if (lane < e && !lane_fixed)
+                atomicAdd(&sh_hist[lane * (w + 1) + ((res[res_slot] >> res_shift) & 0xffffu)], 1u);
+#else
             if (lane < e && !lane_fixed) atomicAdd(&sh_hist[lane * (w + 1) + res[lane]], 1u);
+#endif
             if (kSB) {                                                  // clear the bank counters
 #pragma unroll
                 for (int k = 0; k < kSmemBankEvals; ++k)
