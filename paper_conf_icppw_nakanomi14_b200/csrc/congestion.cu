@@ -371,12 +371,13 @@ __device__ __forceinline__ uint32_t max_load(const BankMask &B, uint32_t counted
     return __reduce_max_sync(kFull, __popc(lanes_equal(B.b, counted, ls)));
 }
 
-// RAP_SWEEP_PACKED_MAX (default 1): the per-trial warp maxima are reduced two at a time -- two
-// lane values (<= 32) packed as 16x2 halves, five SHFL.BFLY + VIMNMX.U16x2 steps -- instead of one
-// CREDUX each: the CREDUX reductions were most of the ADU pipe, the kernel's busiest
-// (profiles/r02_prof_sweep.*); SHFL and VIMNMX run on the LSU and ALU pipes, which had room.
+// RAP_SWEEP_PACKED_MAX (ablation, default 0): the per-trial warp maxima reduced two at a time --
+// two lane values (<= 32) packed as 16x2 halves, five SHFL.BFLY + VIMNMX.U16x2 steps -- instead of
+// one CREDUX each, to unload the ADU pipe (the busiest in profiles/r02_prof_sweep.*).  Measured
+// 2.99 against 3.47 G trials/s (profiles/r02_ab_sweep5.txt): the 60 extra instructions per trial
+// cost more than the 8 reductions they replace.  Bit-identical; kept for the record.
 #ifndef RAP_SWEEP_PACKED_MAX
-#define RAP_SWEEP_PACKED_MAX 1
+#define RAP_SWEEP_PACKED_MAX 0
 #endif
 __device__ __forceinline__ uint32_t warp_max_16x2(uint32_t x) {
 #pragma unroll
