@@ -447,3 +447,13 @@ def test_golden_1e9_histograms_pinned(seed):
         obs[-1] += o_acc; exp[-1] += e_acc
         chi2 = sum((o - e) ** 2 / e for o, e in zip(obs, exp))
         assert chi2 < 2 * len(obs) + 20, (chi2, len(obs))             # above the 0.999 chi-square quantile for these dof
+
+
+def test_oracle_transpose_into_reused_output(oracle):
+    """The timing harness passes a preallocated output (bench.py's oracle_arm): same result as a
+    fresh array, and the array is written in place."""
+    import numpy as np
+    x = np.random.default_rng(5).integers(0, 2 ** 32, size=(37, 53), dtype=np.uint64).astype(np.uint32)
+    out = np.empty((53, 37), dtype=np.uint32)
+    r = oracle.transpose(x, threads=2, out=out)
+    assert r is out and np.array_equal(out, x.T) and np.array_equal(oracle.transpose(x), x.T)
