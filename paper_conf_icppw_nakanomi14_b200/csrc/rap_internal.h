@@ -83,14 +83,24 @@ struct TransposeTuning {
 #ifndef RAP32_MINB
 #define RAP32_MINB 2
 #endif
-constexpr int kDefaultSR32 = RAP32_SR, kDefaultSC32 = RAP32_SC, kDefaultSR64 = 12, kDefaultSC64 = 1;
-constexpr int kDefaultCL32 = RAP32_CL, kDefaultCL64 = 1;
+// (RAP64P_SR / RAP64P_CL / RAP64P_MINB: the two-plane fp64 shape in tuning builds)
+#ifndef RAP64P_SR
+#define RAP64P_SR 12
+#endif
+#ifndef RAP64P_CL
+#define RAP64P_CL 1
+#endif
+#ifndef RAP64P_MINB
+#define RAP64P_MINB 1
+#endif
+constexpr int kDefaultSR32 = RAP32_SR, kDefaultSC32 = RAP32_SC, kDefaultSR64 = RAP64P_SR, kDefaultSC64 = 1;
+constexpr int kDefaultCL32 = RAP32_CL, kDefaultCL64 = RAP64P_CL;
 // fused sharded transpose (peer stores): 8 x 2 warps, no cluster
 constexpr int kPeerSR32 = 8, kPeerSC32 = 2;
 // up to this many 32 x 32 tiles: one single-warp CTA per tile
 constexpr int64_t kSmallTiles = 8;
 // measured on B200 (tools/tune_transpose.cu, profiles/r01_tune_transpose.txt)
-constexpr int kDefaultMinB32 = RAP32_MINB, kDefaultMinB64 = 1;   // fp32: 2 CTAs of 8 warps per SM (128 registers)
+constexpr int kDefaultMinB32 = RAP32_MINB, kDefaultMinB64 = RAP64P_MINB;   // fp32: 2 CTAs of 8 warps per SM (128 registers)
 constexpr int kDefaultDepth32 = 1, kDefaultDepth64 = 1;
 constexpr int kDefaultCtas32 = 0, kDefaultCtas64 = 0;
 constexpr bool kDefaultVst32 = false, kDefaultVst64 = false;

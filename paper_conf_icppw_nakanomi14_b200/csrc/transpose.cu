@@ -549,8 +549,8 @@ static cudaError_t launch_shape(const void *src, void *dst, int64_t rows, int64_
                           false, false, kDefaultCL32>(src, dst, rows, cols, ld_src, ld_dst, seed, tu, st);
     if (EW == 1)      // the round-1 shape without cluster (8 x 2 warps), kept selectable for A/B runs
         return launch_one<L, EW, VEC, 1, 1, false, 8, 2>(src, dst, rows, cols, ld_src, ld_dst, seed, tu, st);
-    return launch_one<L, EW, VEC, kDefaultDepth64, kDefaultMinB64, kDefaultVst64, kDefaultSR64, kDefaultSC64>(
-        src, dst, rows, cols, ld_src, ld_dst, seed, tu, st);
+    return launch_one<L, EW, VEC, kDefaultDepth64, kDefaultMinB64, kDefaultVst64, kDefaultSR64, kDefaultSC64,
+                      false, false, kDefaultCL64>(src, dst, rows, cols, ld_src, ld_dst, seed, tu, st);
 }
 
 template <bool VEC>
