@@ -4,17 +4,21 @@ Default step (BASELINE configs; DESIGN.md §7 "Measurement"): one pass of the wh
   T0-T3  RAP transpose of the cfg4 matrix: 16384 x 16384 float64 (the paper's 64-bit doubles,
          P:L855-866), out-of-place, RAP = the w = 32 map on two 32-bit planes; input and output
          are 2 GiB each (> the 126 MB L2: no flush between steps);
-  C1-C4  a slice of the cfg2 congestion sweep (w = 32, 5 patterns x RAW/RAS/RAP, seed 1): the K
-         timed steps sweep trials [0, 10^9) between them, so the run's histogram is the full
-         cfg2 result and is compared with the oracle's stored 10^9-trial histogram
-         (tests/golden/sweep_w32_1e9_seed1.txt, written from oracle/ only);
+  C1-C4  a slice of the cfg2 congestion sweep (w = 32, 5 patterns x RAW/RAS/RAP, seed 1): step k
+         sweeps trials [k*S, (k+1)*S), S = 2^20 (~0.3 ms, so the transpose stays the step's
+         dominant kernel); after the timed steps one timed sweep call covers the rest of
+         [0, 10^9), so the run's histogram is the full cfg2 result and is compared with the
+         oracle's stored 10^9-trial histogram (tests/golden/sweep_w32_1e9_seed1.txt, written from
+         oracle/ only);
   (N > 1) the NCCL all-reduce of each step's sweep histogram.
 `value` = the cfg4 transpose (GB/s, whole job): algorithmic bytes (read once + write once) of all
 ranks / mean transpose device time per step (CUDA events on the launching stream, max over
 ranks); `roofline` is that kernel's, on the same mean.  Sub-objects timed in the same run:
-  `sweep`       the 10^9-trial cfg2 sweep (trials/s, ALU roofline, parity with the golden file);
+  `sweep`       the 10^9-trial cfg2 sweep (trials/s, pipe roofline, parity with the golden file);
   `cfg3_layouts` cfg3 8192^2 float32 under RAW / PAD / XOR / RAS / RAP (back-to-back launches);
   `cfg4_layouts` cfg4 under every 64-bit layout (two 32-bit planes; RAP64 8-byte slots; RAP-16);
+  `cfg1_tile`    cfg1's single 32 x 32 tile (latency, CUDA-graph replay);
+  `cfg5_single_gpu` the 32768^2 float32 transpose on one GPU (N = 1);
 each with its roofline and `cpu_baseline` (the oracle, all cores and one core, same sample
 definition as the reference arm).
 
@@ -46,7 +50,9 @@ METRIC = "RAP transpose GB/s vs HBM peak; smem wavefronts/request; congestion tr
 ALL_PAT = ["contiguous", "stride", "diagonal", "random", "malicious"]
 SCH = ["raw", "ras", "rap"]
 NVLINK_GBS = 770.0   # measured peer copy per direction (B200_PROFILING.md); 900 nominal
-SWEEP_TOTAL = 10 ** 9          # cfg2: trials swept by the default run's timed steps
+SWEEP_TOTAL = 10 ** 9          # cfg2: trials swept by the default run (timed steps + the sweep sub-run)
+STEP_SWEEP_TRIALS = 1 << 20    # default step's sweep slice: ~0.3 ms, so the cfg4 transpose stays the
+                               # step's dominant kernel (its roofline is the line's `roofline`)
 SWEEP_SEED = 1
 CFG3_LAYOUTS = ["raw", "pad", "xor", "ras", "rap"]
 CFG4_LAYOUTS = ["raw", "pad", "xor", "ras", "rap", "rap64", "rap16"]
@@ -99,7 +105,7 @@ def parse(argv=None):
     a = p.parse_args(argv)
     if a.sweep_trials is None:
         if a.workload == "default":
-            a.sweep_trials = -(-SWEEP_TOTAL // max(a.steps, 1))
+            a.sweep_trials = STEP_SWEEP_TRIALS
         else:
             a.sweep_trials = 148 * 8 * 4 * 32 * (64 if a.workload == "sweep" else 1)
     return a
@@ -246,7 +252,7 @@ def arm_config(args, world: int) -> dict:
         cfg["sweep_trials_per_step"] = args.sweep_trials * world
     if wl == "default":
         cfg["sweep_trials_per_step"] = args.sweep_trials
-        cfg["sweep_trials_total"] = min(SWEEP_TOTAL, args.sweep_trials * args.steps)
+        cfg["sweep_trials_total"] = SWEEP_TOTAL
         cfg["sweep_seed"] = SWEEP_SEED
     return cfg
 
@@ -607,7 +613,8 @@ def run_default(args):
     x = workloads.random_bits(rows, cols, dt, seed=rank, device=dev)
     y = torch.empty((cols, rows), dtype=dt, device=dev)
     S = args.sweep_trials                            # trials per step (all ranks together)
-    total = min(SWEEP_TOTAL, S * K)
+    total = min(SWEEP_TOTAL, S * K)                  # swept by the timed steps; the rest of the 10^9
+                                                     # in the timed sweep sub-run below
     hist = torch.zeros((5, 3, 33), dtype=torch.int64, device=dev)
     hstep = torch.zeros_like(hist)
     scratch = torch.zeros_like(hist)
@@ -684,26 +691,42 @@ def run_default(args):
     line["roofline"] = hbm_roofline(nbytes, kern_ms, peak, peak_src, "transpose_b64_rap")
     line["roofline"]["kernel_ms_median"] = rmax(statistics.median(t_ms))
 
-    # sweep sub-object: the 10^9 trials of cfg2 swept by the K timed steps
-    h = hist.cpu().numpy().astype(np.uint64)
-    cc = np.arange(33)
-    E = lambda a: float((a * cc).sum() / a.sum())
-    assert (h.sum(-1) == total).all(), "histogram does not hold every timed trial once"
-    tps = total / (s_sum * 1e-3)
-    gold = golden_sweep_1e9(SWEEP_SEED) if total == SWEEP_TOTAL else None
-    line["sweep"] = {"trials_per_s": tps, "unit": "trials/s", "trials": total, "w": 32, "seed": SWEEP_SEED,
-                     "trials_per_step": S, "scaling": "strong (the trials of each step are split over the ranks)",
-                     "E_ras_stride": E(h[1, 1]), "E_rap_diagonal": E(h[2, 2]), "E_random": E(h[3, 2]),
-                     "E_raw_malicious": E(h[4, 0]), "E_rap_stride": E(h[1, 2]),
-                     "kernel_ms_mean": s_sum / K,
-                     "bit_identical_to_oracle_1e9": (bool(np.array_equal(h, gold)) if gold is not None else None),
-                     "oracle_reference": "tests/golden/sweep_w32_1e9_seed1.txt (oracle/, 10^9 trials)",
-                     "roofline": sweep_roofline(tps / world, c)}
-    if gold is not None:
-        assert np.array_equal(h, gold), "10^9-trial histogram differs from the oracle's"
     line["kernel_time_share"] = {"transpose": t_sum / (t_sum + s_sum), "sweep": s_sum / (t_sum + s_sum)}
     line["clocks"] = c
     line["gpu_launches"] = int(reduce_over_ranks(launches, world, dev, "sum"))
+
+    # ---------------- sweep sub-object: the rest of cfg2's 10^9 trials (the steps swept
+    # [0, K*S)), timed as one sweep of [K*S, 10^9) into the same histogram, then the whole
+    # 10^9-trial histogram against the oracle's stored one
+    rest = SWEEP_TOTAL - total
+    barrier()
+    torch.cuda.synchronize()
+    with Clocks(dev.index) as sclk:
+        st_, en_ = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        st_.record(stream)
+        if rest > 0:
+            sweep_slice(total, rest, hist)
+        en_.record(stream)
+        torch.cuda.synchronize()
+    rest_ms = rmax(st_.elapsed_time(en_))
+    h = hist.cpu().numpy().astype(np.uint64)
+    cc = np.arange(33)
+    E = lambda a: float((a * cc).sum() / a.sum())
+    assert (h.sum(-1) == SWEEP_TOTAL).all(), "histogram does not hold every trial once"
+    tps = rest / (rest_ms * 1e-3) if rest > 0 else total / (s_sum * 1e-3)
+    gold = golden_sweep_1e9(SWEEP_SEED)
+    line["sweep"] = {"trials_per_s": tps, "unit": "trials/s", "trials": SWEEP_TOTAL, "w": 32, "seed": SWEEP_SEED,
+                     "timing": f"trials [0, {total}) in the {K} timed steps ({S} per step), [{total}, 10^9) in one "
+                               "timed sweep call; trials_per_s is the latter's",
+                     "trials_per_s_in_steps": total / (s_sum * 1e-3), "sub_run_ms": rest_ms,
+                     "scaling": "strong (every call's trial range is split over the ranks)",
+                     "E_ras_stride": E(h[1, 1]), "E_rap_diagonal": E(h[2, 2]), "E_random": E(h[3, 2]),
+                     "E_raw_malicious": E(h[4, 0]), "E_rap_stride": E(h[1, 2]),
+                     "bit_identical_to_oracle_1e9": (bool(np.array_equal(h, gold)) if gold is not None else None),
+                     "oracle_reference": "tests/golden/sweep_w32_1e9_seed1.txt (oracle/, 10^9 trials)",
+                     "clocks": sclk.result, "roofline": sweep_roofline(tps / world, sclk.result)}
+    if gold is not None:
+        assert np.array_equal(h, gold), "10^9-trial histogram differs from the oracle's"
 
     # ---------------- cfg3 under the five layouts, cfg4 under every 64-bit layout
     subs = {}
@@ -728,6 +751,51 @@ def run_default(args):
         subs[name] = sub
     del x3, y3
     line.update(subs)
+
+    # ---------------- cfg1: one 32 x 32 float32 tile (latency case: CUDA-graph replay of 256 launches)
+    x1 = workloads.random_bits(32, 32, torch.float32, seed=rank, device=dev)
+    y1 = torch.empty_like(x1)
+    g = torch.cuda.CUDAGraph()
+    cs = torch.cuda.Stream()
+    cs.wait_stream(stream)
+    with torch.cuda.stream(cs):
+        rap.transpose(x1, layout="rap", seed=0, out=y1)
+        torch.cuda.synchronize()
+        with torch.cuda.graph(g, stream=cs):
+            for _ in range(256):
+                rap.transpose(x1, layout="rap", seed=0, out=y1)
+    g.replay()
+    torch.cuda.synchronize()
+    gs, ge = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    gs.record(stream)
+    for _ in range(10):
+        g.replay()
+    ge.record(stream)
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    for _ in range(200):
+        rap.transpose(x1, layout="rap", seed=0, out=y1)
+    torch.cuda.synchronize()
+    line["cfg1_tile"] = {"us_per_transpose_cuda_graph": rmax(gs.elapsed_time(ge)) * 1e3 / 2560,
+                         "us_per_call_python": (time.perf_counter() - t0) / 200 * 1e6,
+                         "note": "latency case, no roofline: one single-warp CTA, P from the host call"}
+
+    # ---------------- cfg5 on one GPU: the 32768^2 float32 transpose the sharded path splits
+    if world == 1:
+        del x, y
+        x5 = workloads.random_bits(32768, 32768, torch.float32, seed=rank, device=dev)
+        y5 = torch.empty_like(x5)
+        nb5 = 2 * x5.numel() * 4
+        ms5, ck5 = timed_back_to_back(lambda: rap.transpose(x5, layout="rap", seed=0, out=y5), W, K, stream,
+                                      world, dev, barrier)
+        r5 = hbm_roofline(nb5, ms5, peak, peak_src, "transpose_b32_rap")
+        line["cfg5_single_gpu"] = {"value": nb5 / (ms5 * 1e-3) / 1e9, "unit": "GB/s", "frac": r5["frac"],
+                                   "kernel_ms_mean": ms5, "algorithmic_bytes_per_launch": nb5,
+                                   "note": "32768^2 float32 RAP transpose on one GPU, back to back (the sharded "
+                                           "cfg5 runs with --workload dist / dist_fused under torchrun)"}
+        del x5, y5
+        x = workloads.random_bits(rows, cols, dt, seed=rank, device=dev)
+        y = torch.empty((cols, rows), dtype=dt, device=dev)
 
     # ---------------- e2e through the public API with pinned host buffers
     if not args.no_e2e:
