@@ -10,7 +10,7 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "librap.so")
 SOURCES = ["api.cu", "transpose.cu", "congestion.cu", "exchange.cu", "smem_bench.cu", "sweep_wide.cu", "sweep4.cu", "host_pipeline.cu", "transpose_rap16.cu",
-           "transpose64.cu"]
+           "transpose64.cu", "pdl_registry.cu"]
 HEADERS = ["rap_rng.cuh", "rap_warp.cuh", "rap_internal.h"]
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 

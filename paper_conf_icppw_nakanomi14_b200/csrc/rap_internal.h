@@ -20,6 +20,8 @@ constexpr int kMaxPeers = 16;
 struct TileShifts {
     uint32_t sh[8];    // byte i of the 32-byte vector = sh[i / 4] >> (8 * (i % 4))
     uint32_t inv[8];
+    uint32_t early = 0;  // 1: the grid may load its source before the previous grid completes
+                         // (pdl_early_loads); it still waits before its first global store
 };
 
 // byte i (< 32) of a packed TileShifts vector: uniform constant-bank words + a per-lane select
@@ -145,6 +147,22 @@ __device__ __forceinline__ void pdl_trigger() {
     asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
 #endif
 }
+
+// Early loads under programmatic dependent launch.  A transpose grid waits for its predecessor
+// in the stream (griddepcontrol.wait) before its first global STORE always (write-after-read and
+// write-after-write on the previous grid's buffers), and before its first LOAD unless the library
+// knows the predecessor: when the previous kernel in this stream was one of these transposes and
+// its destination does not overlap this launch's source, nothing this grid reads is being written,
+// so its first tiles are loaded while the previous grid drains.  (A kernel of anyone else in
+// between is not PDL-aware: this grid then starts after it completes, which covers that case.)
+// A grid triggers its dependents (launch_dependents) only after its own wait has returned, so when
+// a dependent starts, every grid before this one has completed and only this one may still be
+// running: comparing against the previous launch's destination is enough.
+// pdl_early_loads() answers for a launch and records its destination for the next one;
+// pdl_forget() marks a stream's last kernel as unknown (the fused peer-store transpose).
+bool pdl_early_loads(cudaStream_t st, const void *src, int64_t rows, int64_t cols, int64_t ld_src, const void *dst,
+                     int64_t drows, int64_t dcols, int64_t ld_dst, uint32_t eb);
+void pdl_forget(cudaStream_t st);
 
 // cudaLaunchKernelEx with an optional cluster dimension and the PDL attribute
 template <typename K, typename... Args>

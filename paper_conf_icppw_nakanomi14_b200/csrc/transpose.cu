@@ -311,11 +311,11 @@ transpose_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, i
 
     uint32_t st = st_first, ti = 0, tj = 0;
     bool act = st < nst && coords(st, ti, tj);
-    pdl_trigger();
-    pdl_wait();                                          // the previous grid's writes are visible
+    if (!ts.early) pdl_wait(), pdl_trigger();                           // the previous grid's writes are visible
     if (TMAS) {
         uint4 v[G];
         if (act) load(v, ti, tj);
+        if (ts.early) pdl_wait(), pdl_trigger();        // before the first global store
         while (st < nst) {
             const uint32_t si = st / stc, sj = st - si * stc;
             const bool cact = act;
@@ -336,6 +336,7 @@ transpose_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, i
     } else if (DEPTH == 1) {
         uint4 v[G];
         if (act) load(v, ti, tj);
+        if (ts.early) pdl_wait(), pdl_trigger();        // before the first global store
         while (st < nst) {
             const uint32_t cti = ti, ctj = tj;
             const bool cact = act;
@@ -355,6 +356,7 @@ transpose_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, i
         if (act) load(va, ti, tj);
         bool act2 = st + gridDim.x < nst && coords(st + gridDim.x, ti2, tj2);
         if (act2) load(vb, ti2, tj2);
+        if (ts.early) pdl_wait(), pdl_trigger();        // before the first global store
         while (st < nst) {
             uint32_t cti = ti, ctj = tj;
             bool cact = act;
@@ -505,7 +507,9 @@ static cudaError_t launch_one(const void *src, void *dst, int64_t rows, int64_t 
     }
     const size_t smem = sizeof(uint32_t) * (warp_smem_words<L, EW>() * SR * SC +
                                             (TMAS ? (size_t)SR * 32 * SC * 32 * EW : 0));
-    const TileShifts ts = tile_shifts(L, seed);
+    TileShifts ts = tile_shifts(L, seed);
+    if (PEERS) pdl_forget(st);
+    else ts.early = pdl_early_loads(st, src, rows, cols, ld_src, dst, cols, rows, ld_dst, 4u * EW) ? 1u : 0u;
     if (CL > 1)
         return launch_clustered(k, cache, CL, SR * SC * 32, smem, nst, st, (const uint32_t *)src, (uint32_t *)dst,
                                 rows, cols, ld_src, ld_dst, ts, tiles_r, tiles_c, vst_ok, peers, tmap);

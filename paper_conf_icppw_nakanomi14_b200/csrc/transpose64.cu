@@ -228,9 +228,9 @@ transpose64_kernel(const uint2 *__restrict__ src, uint2 *__restrict__ dst, int64
     uint32_t st = blockIdx.x, ti = 0, tj = 0;
     bool act = st < nst && coords(st, ti, tj);
     Buf v;
-    pdl_trigger();
-    pdl_wait();                                      // the previous grid's writes are visible
+    if (!ts.early) pdl_wait(), pdl_trigger();                       // the previous grid's writes are visible
     if (act) load(v, ti, tj);
+    if (ts.early) pdl_wait(), pdl_trigger();        // before the first global store
     while (st < nst) {
         const uint32_t cti = ti, ctj = tj;
         const bool cact = act;
@@ -274,7 +274,8 @@ static cudaError_t launch64_one(const void *src, void *dst, int64_t rows, int64_
 #endif
     const cudaError_t e = cached_grid(k, cache, SR * 32, smem, nst, 0, &grid);
     if (e != cudaSuccess) return e;
-    const TileShifts ts = tile_shifts(L, seed);
+    TileShifts ts = tile_shifts(L, seed);
+    ts.early = pdl_early_loads(st, src, rows, cols, ld_src, dst, cols, rows, ld_dst, 8u) ? 1u : 0u;
     return launch_ex(k, grid, SR * 32, smem, st, 1, (const uint2 *)src, (uint2 *)dst, rows, cols, ld_src, ld_dst, ts,
                      tiles_r, tiles_c);
 }

@@ -93,9 +93,9 @@ transpose_rap16_kernel(const uint2 *__restrict__ src, uint2 *__restrict__ dst, i
     uint32_t st = blockIdx.x, ti = 0, tj = 0;
     bool act = st < nst && coords(st, ti, tj);
     uint2 v[32];
-    pdl_trigger();
-    pdl_wait();                                      // the previous grid's writes are visible
+    if (!ts.early) pdl_wait(), pdl_trigger();                       // the previous grid's writes are visible
     if (act) load(v, ti, tj);
+    if (ts.early) pdl_wait(), pdl_trigger();        // before the first global store
     while (st < nst) {
         const uint32_t cti = ti, ctj = tj;
         const bool cact = act;
@@ -121,7 +121,8 @@ cudaError_t launch_transpose_rap16(const void *src, void *dst, int64_t rows, int
     int grid = 0;
     const cudaError_t e = cached_grid(k, cache, SR * 32, smem, nst, 0, &grid);
     if (e != cudaSuccess) return e;
-    const TileShifts ts = tile_shifts(RAP_LAYOUT_RAP16, seed);
+    TileShifts ts = tile_shifts(RAP_LAYOUT_RAP16, seed);
+    ts.early = pdl_early_loads(st, src, rows, cols, ld_src, dst, cols, rows, ld_dst, 8u) ? 1u : 0u;
     return launch_ex(k, grid, SR * 32, smem, st, 1, (const uint2 *)src, (uint2 *)dst, rows, cols, ld_src, ld_dst, ts,
                      tiles_r, tiles_c);
 }

@@ -725,3 +725,32 @@ def test_transpose_randomized_geometry(rap, oracle):
         assert np.array_equal(bits(out_big[:, :rows]), oracle.transpose(bits(xs))), (k, rows, cols, layout)
         if pad_d:
             assert not bits(out_big[:, rows:]).any()
+
+
+# ------------------------------------------------------------------ programmatic dependent launch
+@pytest.mark.parametrize("dtype,layout", [(torch.float32, "rap"), (torch.float64, "rap"), (torch.float64, "rap64"),
+                                          (torch.float64, "rap16"), (torch.float32, "raw")])
+def test_transpose_chains_under_pdl(rap, dtype, layout):
+    """Back-to-back transposes on one stream, no host sync in between: a grid may load its source
+    before its predecessor completes only when that source is not the predecessor's destination
+    (pdl_early_loads).  Chains that read what the previous and the one-before-previous launches
+    wrote, and a torch kernel rewriting a source in between, must all see finished data."""
+    n = 4096
+    bd = torch.int32 if dtype == torch.float32 else torch.int64
+    xs = [workloads.random_bits(n, n, dtype, seed=40 + i, device="cuda") for i in range(6)]
+    ys = [torch.empty_like(x) for x in xs]
+    for _ in range(3):
+        for x, y in zip(xs, ys):                       # independent launches: early loads
+            rap.transpose(x, layout=layout, seed=1, out=y)
+        z = rap.transpose(ys[3], layout=layout, seed=2)   # reads the output of 3 launches ago
+        w = rap.transpose(z, layout=layout, seed=3)       # reads its predecessor's output
+        u = rap.transpose(ys[5], layout=layout, seed=4)   # reads the output of 3 launches ago
+        xs[0].view(bd).add_(1)                            # a torch kernel rewrites a source ...
+        v = rap.transpose(xs[0], layout=layout, seed=5)   # ... that the next launch reads
+        torch.cuda.synchronize()
+        assert torch.equal(z.view(bd), xs[3].view(bd))
+        assert torch.equal(w.view(bd), ys[3].view(bd))
+        assert torch.equal(u.view(bd), xs[5].view(bd))
+        assert torch.equal(v.view(bd), xs[0].t().contiguous().view(bd))
+        for x, y in zip(xs[1:], ys[1:]):
+            assert torch.equal(y.view(bd), x.t().contiguous().view(bd))
