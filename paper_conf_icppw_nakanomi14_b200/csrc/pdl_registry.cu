@@ -36,8 +36,14 @@ Entry *find(int dev, cudaStream_t st) {
 
 }  // namespace
 
+// RAP_PDL_EARLY = 0 (tuning / A/B): never load before the predecessor completes
+#ifndef RAP_PDL_EARLY
+#define RAP_PDL_EARLY 1
+#endif
+
 bool pdl_early_loads(cudaStream_t st, const void *src, int64_t rows, int64_t cols, int64_t ld_src, const void *dst,
                      int64_t drows, int64_t dcols, int64_t ld_dst, uint32_t eb) {
+    if (!RAP_PDL || !RAP_PDL_EARLY) return false;
     int dev = 0;
     if (cudaGetDevice(&dev) != cudaSuccess) return false;
     uintptr_t s_lo, s_hi, d_lo, d_hi;
