@@ -36,9 +36,12 @@ Entry *find(int dev, cudaStream_t st) {
 
 }  // namespace
 
-// RAP_PDL_EARLY = 0 (tuning / A/B): never load before the predecessor completes
+// RAP_PDL_EARLY (default 0): whether early loads are used at all.  The registry knows the last
+// transpose launched in a stream, not the last kernel: a third-party kernel launched in between
+// with programmatic dependent launch of its own (CUTLASS / GEMM libraries trigger early) could
+// still be writing this launch's source -- so early loads stay off unless a build opts in.
 #ifndef RAP_PDL_EARLY
-#define RAP_PDL_EARLY 1
+#define RAP_PDL_EARLY 0
 #endif
 
 bool pdl_early_loads(cudaStream_t st, const void *src, int64_t rows, int64_t cols, int64_t ld_src, const void *dst,
