@@ -129,13 +129,16 @@ cudaError_t launch_transpose_peers(const void *src, int64_t M, int64_t N, int64_
 cudaError_t launch_perm_gen(uint64_t seed, uint64_t first, uint64_t count, uint32_t w, uint8_t *out,
                             cudaStream_t st);
 
-// Programmatic dependent launch (RAP_PDL, default on): the transposes are launched with
-// cudaLaunchAttributeProgrammaticStreamSerialization, trigger their dependents at entry and
-// wait (griddepcontrol.wait) for the previous grid in the stream -- its completion and memory
-// flush -- before their first global access.  A following launch's CTAs are then scheduled and
-// run their prologue while this grid drains, instead of after it; the data dependence is kept.
+// Programmatic dependent launch (RAP_PDL, default OFF): the transposes can be launched with
+// cudaLaunchAttributeProgrammaticStreamSerialization; they then wait (griddepcontrol.wait) for the
+// previous grid in the stream -- its completion and memory flush -- before their first global
+// access and trigger their own dependents after that wait, so a following launch's CTAs are
+// scheduled and run their prologue while this grid drains; the data dependence is kept.  Measured
+// over 21 interleaved rounds (profiles/r02_ab_pdl32b.txt, r02_ab_pdl64b.txt): -4 to -5 % on
+// back-to-back cfg3 fp32 launches (clustered grids, much wider spread) and +0.4 % on cfg4 fp64
+// (noise) -- so it is off; the kernels' wait / trigger instructions are no-ops without it.
 #ifndef RAP_PDL
-#define RAP_PDL 1
+#define RAP_PDL 0
 #endif
 __device__ __forceinline__ void pdl_wait() {
 #if RAP_PDL
