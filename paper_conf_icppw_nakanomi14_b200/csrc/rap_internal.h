@@ -70,7 +70,8 @@ struct TransposeTuning {
     int cl = 1;           // thread-block cluster of cl CTAs stacked along the input rows, drains in lockstep
     bool slots64 = false;  // 64-bit elements on 8-byte tile slots (transpose64.cu) for every layout (A/B)
 };
-// fp32: 4 x 2 warps per CTA, clusters of 4 CTAs (a 16 x 2-tile cluster super-tile);
+// fp32: 4 x 2 warps per CTA, clusters of 8 CTAs (a 32 x 2-tile cluster super-tile: each output
+// row receives 4 KiB per drain; +1.5 % over clusters of 4 with PDL off, profiles/r02_ab32s3.txt);
 // fp64: 12 x 1 warps, no cluster (profiles/r01_tune_transpose*.txt, r01_probe_transpose.txt)
 // (RAP32_SR / RAP32_SC / RAP32_CL / RAP32_MINB override the fp32 shape in tuning builds)
 #ifndef RAP32_SR
@@ -80,7 +81,7 @@ struct TransposeTuning {
 #define RAP32_SC 2
 #endif
 #ifndef RAP32_CL
-#define RAP32_CL 4
+#define RAP32_CL 8
 #endif
 #ifndef RAP32_MINB
 #define RAP32_MINB 2

@@ -115,7 +115,8 @@ __device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.
 
 // Cluster lockstep (CL > 1): the CL CTAs of a thread-block cluster take the CL row blocks of one
 // (CL*SR) x SC-tile cluster super-tile and drain behind one barrier.cluster, so each output row
-// receives CL*SR*128 B at once (+1.5-2 % over CL = 1, profiles/r01_probe_transpose.txt).
+// receives CL*SR*128 B at once (+1.5-2 % over CL = 1, profiles/r01_probe_transpose.txt; 8 CTAs
+// +1.5 % over 4, profiles/r02_ab32s3.txt).
 __device__ __forceinline__ void cluster_sync_relaxed() {
     asm volatile("barrier.cluster.arrive.relaxed.aligned;" ::: "memory");
     asm volatile("barrier.cluster.wait.aligned;" ::: "memory");

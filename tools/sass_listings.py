@@ -11,7 +11,7 @@ import sys
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 KERNELS = {
-    "transpose_b32_rap_cluster": "_ZN4rapk16transpose_kernelILi4ELi1ELb1ELi1ELi2ELb0ELi4ELi2ELb0ELb0ELi4EEEvPKjPjllllNS_10TileShiftsEjjbNS_7PeerOutE14CUtensorMap_st",
+    "transpose_b32_rap_cluster": "_ZN4rapk16transpose_kernelILi4ELi1ELb1ELi1ELi2ELb0ELi4ELi2ELb0ELb0ELi8EEEvPKjPjllllNS_10TileShiftsEjjbNS_7PeerOutE14CUtensorMap_st",
     "transpose_b64_rap_two_planes": "_ZN4rapk16transpose_kernelILi4ELi2ELb1ELi1ELi1ELb0ELi12ELi1ELb0ELb0ELi1EEEvPKjPjllllNS_10TileShiftsEjjbNS_7PeerOutE14CUtensorMap_st",
     "transpose_b64_rap64_slots": "_ZN4rapk18transpose64_kernelILi4ELb1ELi12ELi1ELb1EEEvPK5uint2PS1_llllNS_10TileShiftsEjj",
     "transpose_b64_rap16": "_ZN4rapk22transpose_rap16_kernelILi12EEEvPK5uint2PS1_llllNS_10TileShiftsEjj",
