@@ -6,9 +6,11 @@ mkdir -p "$OUT"
 python -c "import __graft_entry__ as g; g.build(); g.smoke()" > "$OUT/r02_smoke.log" 2>&1
 timeout 2400 python -m pytest tests -m gpu -q -x > "$OUT/r02_pytest_gpu.log" 2>&1
 tail -2 "$OUT/r02_pytest_gpu.log"
-bash tools/ab_trace.sh "$OUT" > "$OUT/ab_trace.log" 2>&1
 python -c "import __graft_entry__ as g; g.build()"
 timeout 900 python bench.py > "$OUT/r02_bench_default.json" 2> "$OUT/r02_bench_default.err"
 timeout 900 python bench.py --impl reference > "$OUT/r02_bench_ref.json" 2> "$OUT/r02_bench_ref.err"
 timeout 600 python bench.py --workload sweep > "$OUT/r02_bench_sweep.json" 2> "$OUT/r02_bench_sweep.err"
 timeout 600 python bench.py --workload trace > "$OUT/r02_bench_trace.json" 2> "$OUT/r02_bench_trace.err"
+bash tools/gpu_profile_r02.sh "$OUT/p02" > "$OUT/p02.log" 2>&1
+bash tools/sanitize.sh "$OUT/r02_sanitizer.txt" > "$OUT/san.log" 2>&1
+du -sh "$OUT"
