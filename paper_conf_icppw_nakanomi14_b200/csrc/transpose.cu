@@ -113,6 +113,20 @@ __device__ __forceinline__ void tma_wait_read() { asm volatile("cp.async.bulk.wa
 __device__ __forceinline__ void tma_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
 __device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 
+// RAP32_KP: 32-bit transposes through the row-pair-plane form (KP above) -- tuning flag
+#ifndef RAP32_KP
+#define RAP32_KP 0
+#endif
+#ifndef RAP32_KP_SR
+#define RAP32_KP_SR 12
+#endif
+#ifndef RAP32_KP_MINB
+#define RAP32_KP_MINB 1
+#endif
+#ifndef RAP32_KP_CL
+#define RAP32_KP_CL 1
+#endif
+
 // Cluster lockstep (CL > 1): the CL CTAs of a thread-block cluster take the CL row blocks of one
 // (CL*SR) x SC-tile cluster super-tile and drain behind one barrier.cluster, so each output row
 // receives CL*SR*128 B at once (+1.5-2 % over CL = 1, profiles/r01_probe_transpose.txt; 8 CTAs
@@ -122,14 +136,25 @@ __device__ __forceinline__ void cluster_sync_relaxed() {
     asm volatile("barrier.cluster.wait.aligned;" ::: "memory");
 }
 
+// KP (row-pair planes, 32-bit elements): the kernel runs its EW = 2 form on a matrix of virtual
+// 8-byte elements v(i, j) = (src[2i][j], src[2i+1][j]): plane 0 of a tile holds input row 2i,
+// plane 1 input row 2i+1, both under the tile's RAP map, and the transpose of the virtual matrix
+// IS the 32-bit transpose -- output element v(j, i) = (out[j][2i], out[j][2i+1]) is contiguous.
+// So a warp moves a 64 x 32 block of 32-bit elements per tile (8 KiB) and the drain writes each
+// output row as one 256-byte STG.64 instead of a 128-byte STG.32, like the 64-bit kernel.  Loads:
+// one LDG.128 = 4 elements of one input row; instruction g (16 per tile) takes plane g & 1 of the
+// 4 virtual rows P^-1(4 (g >> 1) + 0..3) -- one per residue of P mod 4 -- so each STS.32 is
+// conflict-free as in the 32-bit kernel.  Here `rows` counts virtual rows (input rows / 2) and
+// ld_dst is in 8-byte units; ld_src stays in 32-bit words.
 template <int L, int EW, bool VEC, int DEPTH, int MINB, bool VST, int SR, int SC, bool PEERS, bool TMAS,
-          int CL = 1>
+          int CL = 1, bool KP = false>
 __global__ void __launch_bounds__(SR * SC * 32, MINB)
 transpose_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, int64_t rows,
                  int64_t cols, int64_t ld_src, int64_t ld_dst, const TileShifts ts, uint32_t tiles_r,
                  uint32_t tiles_c, bool vst_ok, PeerOut peers, const __grid_constant__ CUtensorMap tmap) {
     static_assert(!TMAS || (DEPTH == 1 && !PEERS && SR * 32 <= 256), "TMA store: depth 1, box <= 256");
     static_assert(CL == 1 || (DEPTH == 1 && !TMAS), "cluster lockstep: depth 1, no TMA store");
+    static_assert(!KP || (EW == 2 && VEC && DEPTH == 1 && !VST && !PEERS && !TMAS), "row-pair planes: EW 2 form");
     using C = TileCfg<L, EW>;
     constexpr int NE = C::NE, R = C::R, G = C::G, LPR = C::LPR;
     constexpr int PW = 32 * Geom<L>::RP;            // plane size in words
@@ -162,6 +187,19 @@ transpose_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, i
         }
     }
     const uint32_t drain_base = word_of<L>(lane, 0, sh_lane);
+    if constexpr (KP) {          // row-pair planes: chunk kq of 4 elements, virtual row set kc
+        const uint32_t kq = lane & 7u, kc = lane >> 3;
+#pragma unroll
+        for (int g = 0; g < G; ++g) {
+            const uint32_t p = (uint32_t)g & 1u, rr = 4u * (uint32_t)(g >> 1) + kc;
+            const uint32_t vr = (L == RAP_LAYOUT_RAP) ? __shfl_sync(kFull, pinv, rr) : rr;
+            const uint32_t shv = (L == RAP_LAYOUT_RAP) ? rr
+                               : (L == RAP_LAYOUT_RAS) ? __shfl_sync(kFull, sh_lane, rr) : 0u;
+            row_g[g] = 2u * vr + p;                               // input row within the 64-row block
+            a_g[g] = p * PW + ((L == RAP_LAYOUT_XOR) ? vr * Geom<L>::RP + ((4u * kq) ^ vr)
+                                                     : word_of<L>(vr, 4u * kq, shv));
+        }
+    }
 
     // super-tile s -> this warp's tile (ti, tj); false when it falls outside the matrix.  With
     // clusters, s counts cluster super-tiles and CTA rank `crank` takes row block crank of it.
@@ -184,7 +222,24 @@ transpose_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, i
     auto load = [&](uint4 (&v)[G], uint32_t ti, uint32_t tj) {
         const int64_t r0 = (int64_t)ti * 32, c0 = (int64_t)tj * 32;
         const bool full = (r0 + 32 <= rows) && (c0 + 32 <= cols);
-        if (VEC && full) {
+        if constexpr (KP) {
+            const uint32_t *base = src + 2 * r0 * ld_src + c0 + 4 * (lane & 7u);
+            if (full) {
+#pragma unroll
+                for (int g = 0; g < G; ++g) v[g] = ldg_stream128(base + (int64_t)row_g[g] * ld_src);
+            } else {
+                const int64_t prow_end = 2 * rows, cc = c0 + 4 * (lane & 7u);
+#pragma unroll
+                for (int g = 0; g < G; ++g) {
+                    const int64_t r = 2 * r0 + row_g[g];
+                    const uint32_t *pp = base + (int64_t)row_g[g] * ld_src;
+                    uint32_t w4[4];
+#pragma unroll
+                    for (int k = 0; k < 4; ++k) w4[k] = (r < prow_end && cc + k < cols) ? __ldg(pp + k) : 0u;
+                    v[g] = make_uint4(w4[0], w4[1], w4[2], w4[3]);
+                }
+            }
+        } else if (VEC && full) {
             const uint32_t *base = src + (r0 * ld_src + c0 + NE * q) * EW;
 #pragma unroll
             for (int g = 0; g < G; ++g) v[g] = ldg_stream128(base + (int64_t)row_g[g] * ld_src * EW);
@@ -207,17 +262,27 @@ transpose_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, i
 
     // T1: contiguous (row-wise) write into the RAP tile -- every address is a_g + immediate
     auto store_tile = [&](const uint4 (&v)[G]) {
+        if constexpr (KP) {      // 4 consecutive elements of one input row into its plane
 #pragma unroll
-        for (int g = 0; g < G; ++g) {
-            const uint32_t w4[4] = {v[g].x, v[g].y, v[g].z, v[g].w};
+            for (int g = 0; g < G; ++g) {
+                const uint32_t w4[4] = {v[g].x, v[g].y, v[g].z, v[g].w};
 #pragma unroll
-            for (int k = 0; k < 4; ++k) {
-                const uint32_t e = k / EW, plane = k % EW;     // element of the chunk, lo/hi word
-                uint32_t off;
-                if (L == RAP_LAYOUT_XOR) off = word_of<L>(row_g[g], NE * q + e, 0);
-                else if constexpr (WRAP) off = a_g[g] + ((rot_g[g] + e) & 31u);
-                else off = a_g[g] + e;
-                tile[plane * PW + off] = w4[k];
+                for (int k = 0; k < 4; ++k)
+                    tile[(L == RAP_LAYOUT_XOR) ? (a_g[g] ^ (uint32_t)k) : a_g[g] + k] = w4[k];
+            }
+        } else {
+#pragma unroll
+            for (int g = 0; g < G; ++g) {
+                const uint32_t w4[4] = {v[g].x, v[g].y, v[g].z, v[g].w};
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    const uint32_t e = k / EW, plane = k % EW;     // element of the chunk, lo/hi word
+                    uint32_t off;
+                    if (L == RAP_LAYOUT_XOR) off = word_of<L>(row_g[g], NE * q + e, 0);
+                    else if constexpr (WRAP) off = a_g[g] + ((rot_g[g] + e) & 31u);
+                    else off = a_g[g] + e;
+                    tile[plane * PW + off] = w4[k];
+                }
             }
         }
     };
@@ -492,7 +557,7 @@ static cudaError_t launch_clustered(K kernel, ShapeCache &cache, int cl, int thr
 }
 
 template <int L, int EW, bool VEC, int DEPTH, int MINB, bool VST, int SR, int SC, bool PEERS = false,
-          bool TMAS = false, int CL = 1>
+          bool TMAS = false, int CL = 1, bool KP = false>
 static cudaError_t launch_one(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
                               int64_t ld_dst, uint64_t seed, const TransposeTuning &tu, cudaStream_t st,
                               const PeerOut &peers = PeerOut{}) {
@@ -503,7 +568,7 @@ static cudaError_t launch_one(const void *src, void *dst, int64_t rows, int64_t 
                                                                              ld_dst, seed, tu, st, peers);
     const uint32_t tiles_r = (uint32_t)((rows + 31) / 32), tiles_c = (uint32_t)((cols + 31) / 32);
     const int64_t nst = (int64_t)((tiles_r + SR * CL - 1) / (SR * CL)) * ((tiles_c + SC - 1) / SC);
-    auto k = transpose_kernel<L, EW, VEC, DEPTH, MINB, VST, SR, SC, PEERS, TMAS, CL>;
+    auto k = transpose_kernel<L, EW, VEC, DEPTH, MINB, VST, SR, SC, PEERS, TMAS, CL, KP>;
     static ShapeCache cache;
     bool vst_ok = ((uintptr_t)dst % 16 == 0) && ((ld_dst * EW * 4) % 16 == 0);
     if (PEERS) {
@@ -513,7 +578,7 @@ static cudaError_t launch_one(const void *src, void *dst, int64_t rows, int64_t 
     const size_t smem = sizeof(uint32_t) * (warp_smem_words<L, EW>() * SR * SC +
                                             (TMAS ? (size_t)SR * 32 * SC * 32 * EW : 0));
     TileShifts ts = tile_shifts(L, seed);
-    if (PEERS) pdl_forget(st);
+    if (PEERS || KP) pdl_forget(st);
     else ts.early = pdl_early_loads(st, src, rows, cols, ld_src, dst, cols, rows, ld_dst, 4u * EW) ? 1u : 0u;
     if (CL > 1)
         return launch_clustered(k, cache, CL, SR * SC * 32, smem, nst, st, (const uint32_t *)src, (uint32_t *)dst,
@@ -553,6 +618,12 @@ static cudaError_t launch_shape(const void *src, void *dst, int64_t rows, int64_
     // cluster, no idle warps of a super-tile computing P, the cheapest launch
     if (((rows + 31) / 32) * ((cols + 31) / 32) <= kSmallTiles)
         return launch_one<L, EW, VEC, 1, 1, false, 1, 1>(src, dst, rows, cols, ld_src, ld_dst, seed, tu, st);
+    // row-pair planes (KP): 32-bit elements as virtual 8-byte elements, the 64-bit kernel's shape
+    if constexpr (EW == 1 && VEC) {
+        if (RAP32_KP && tu.cl == kDefaultCL32 && rows % 2 == 0 && ld_dst % 2 == 0 && (uintptr_t)dst % 8 == 0)
+            return launch_one<L, 2, true, 1, RAP32_KP_MINB, false, RAP32_KP_SR, 1, false, false, RAP32_KP_CL, true>(
+                src, dst, rows / 2, cols, ld_src, ld_dst / 2, seed, tu, st);
+    }
     if (EW == 1 && tu.cl == kDefaultCL32)
         return launch_one<L, EW, VEC, kDefaultDepth32, kDefaultMinB32, kDefaultVst32, kDefaultSR32, kDefaultSC32,
                           false, false, kDefaultCL32>(src, dst, rows, cols, ld_src, ld_dst, seed, tu, st);
