@@ -113,7 +113,9 @@ __device__ __forceinline__ void tma_wait_read() { asm volatile("cp.async.bulk.wa
 __device__ __forceinline__ void tma_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
 __device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 
-// RAP32_KP: 32-bit transposes through the row-pair-plane form (KP above) -- tuning flag
+// RAP32_KP: 32-bit transposes through the row-pair-plane form (KP above) -- tuning flag, off:
+// measured 5.85 against 6.08 TB/s for the default at 8192^2 and 6.05 against 6.16 at 16384^2
+// (profiles/r02_ab_kp*.txt), so 256-byte output rows are not what the 32-bit kernel lacks
 #ifndef RAP32_KP
 #define RAP32_KP 0
 #endif

@@ -20,12 +20,15 @@ NB = 2 * x.nbytes
 K = 20
 
 
+LAYOUT = sys.argv[1] if len(sys.argv) > 1 else "rap"
+
+
 def bracketed(neigh):
     evs = []
     for k in range(K + 3):
         e = [torch.cuda.Event(enable_timing=True) for _ in range(2)]
         e[0].record()
-        rap.transpose(x, layout="rap", out=y)
+        rap.transpose(x, layout=LAYOUT, out=y)
         e[1].record()
         if neigh == "sweep":
             rap.congestion_sweep(50_000_000, seed=1, first_trial=k * 50_000_000, out=hist)
@@ -41,16 +44,17 @@ def bracketed(neigh):
 
 def back_to_back():
     for _ in range(3):
-        rap.transpose(x, layout="rap", out=y)
+        rap.transpose(x, layout=LAYOUT, out=y)
     s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     s.record()
     for _ in range(K):
-        rap.transpose(x, layout="rap", out=y)
+        rap.transpose(x, layout=LAYOUT, out=y)
     e.record()
     torch.cuda.synchronize()
     return s.elapsed_time(e) * 1e-3 / K
 
 
+print("layout", LAYOUT)
 for rnd in range(3):
     r = {"back_to_back": back_to_back(), "bracketed_alone": bracketed(None), "bracketed_tiny": bracketed("tiny"),
          "bracketed_sweep_small": bracketed("sweep_small"), "bracketed_sweep_5e7": bracketed("sweep")}
