@@ -17,7 +17,8 @@
  *     rap_transpose) are DEVICE pointers on the current CUDA device.  The library keeps no
  *     memory allocation and no shared mutable state; calls are thread-safe.  (Cached per
  *     kernel: the launch shape; per calling thread and device: rap_transpose_host's three
- *     streams and their events, created on first use and destroyed at thread exit.)
+ *     streams and their events, created on first use and destroyed at thread exit; in builds
+ *     with RAP_PDL_EARLY only, a mutex-guarded table of the last transpose per stream.)
  *   - Asynchrony: device work is enqueued on `stream` (a cudaStream_t passed as void*;
  *     NULL = the legacy default stream) and returns immediately; results are valid once
  *     the stream is synchronised.
