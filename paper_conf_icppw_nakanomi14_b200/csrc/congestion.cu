@@ -442,6 +442,16 @@ __device__ __forceinline__ uint32_t max_load_add_lane(const BankMask &Y, const L
 #endif
 constexpr int kSmemBankEvals = 7;      // RAS stride, RAS diagonal, random under each of the 5 schemes
 
+#ifndef RAP_SWEEP_HIST_SA
+#define RAP_SWEEP_HIST_SA 1
+#endif
+// += 1 on a shared-memory u32 given its shared-window address (computed once per kernel: the
+// generic-to-shared conversion of a generic atomicAdd re-reads the CTA window base per use,
+// an S2UR + ULEA that was 17 % of the sweep's stall samples)
+__device__ __forceinline__ void smem_inc(uint32_t saddr) {
+    asm volatile("red.shared.add.u32 [%0], 1;" :: "r"(saddr) : "memory");
+}
+
 __device__ __forceinline__ uint32_t count_in_bank(uint32_t *cnt, uint32_t bank, bool counted) {
     // every lane issues the atomic (a merged duplicate adds 0 to its leader's bank): no branch
     const uint32_t one = counted ? 1u : 0u;
@@ -497,6 +507,8 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
     uint32_t *tr = sh_tr[warp];
     uint32_t *res = sh_res[warp];
     uint32_t *cnt = &sh_cnt[RAP_SWEEP_SMEM_BANKS ? warp : 0][0][0];
+    uint32_t hist_sa;                 // opaque to the compiler: kept, not rematerialised per trial
+    asm volatile("mov.u32 %0, %1;" : "=r"(hist_sa) : "r"((uint32_t)__cvta_generic_to_shared(sh_hist)));
     constexpr bool kSB = RAP_SWEEP_SMEM_BANKS != 0;
     // counter slots in use: 0 RAS stride, 1 RAS diagonal (and malicious, which reuses them), 2 + s
     // the random access under scheme s
@@ -753,7 +765,11 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
             if (lane < e && !lane_fixed)
                 atomicAdd(&sh_hist[lane * (w + 1) + ((res[res_slot] >> res_shift) & 0xffffu)], 1u);
 #else
+#if RAP_SWEEP_HIST_SA
+            if (lane < e && !lane_fixed) smem_inc(hist_sa + 4u * (lane * (w + 1) + res[lane]));
+#else
             if (lane < e && !lane_fixed) atomicAdd(&sh_hist[lane * (w + 1) + res[lane]], 1u);
+#endif
 #endif
             if (kSB) {                                                  // clear the bank counters
 #pragma unroll
