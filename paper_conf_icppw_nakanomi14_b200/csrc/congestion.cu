@@ -442,12 +442,15 @@ __device__ __forceinline__ uint32_t max_load_add_lane(const BankMask &Y, const L
 #endif
 constexpr int kSmemBankEvals = 7;      // RAS stride, RAS diagonal, random under each of the 5 schemes
 
+// RAP_SWEEP_HIST_SA (ablation, default 0): histogram increments through a shared-window address
+// kept in a register instead of atomicAdd on a generic pointer (whose conversion re-reads the CTA
+// window base per trial, an S2UR + ULEA carrying 17 % of the stall samples).  Measured 3.445
+// against 3.466 G trials/s (profiles/r02_ab_sweep6.txt): the extra live register costs more than
+// the conversion -- the stall samples only marked where the warps waited.
 #ifndef RAP_SWEEP_HIST_SA
-#define RAP_SWEEP_HIST_SA 1
+#define RAP_SWEEP_HIST_SA 0
 #endif
-// += 1 on a shared-memory u32 given its shared-window address (computed once per kernel: the
-// generic-to-shared conversion of a generic atomicAdd re-reads the CTA window base per use,
-// an S2UR + ULEA that was 17 % of the sweep's stall samples)
+// += 1 on a shared-memory u32 given its shared-window address
 __device__ __forceinline__ void smem_inc(uint32_t saddr) {
     asm volatile("red.shared.add.u32 [%0], 1;" :: "r"(saddr) : "memory");
 }
@@ -507,8 +510,10 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
     uint32_t *tr = sh_tr[warp];
     uint32_t *res = sh_res[warp];
     uint32_t *cnt = &sh_cnt[RAP_SWEEP_SMEM_BANKS ? warp : 0][0][0];
+#if RAP_SWEEP_HIST_SA
     uint32_t hist_sa;                 // opaque to the compiler: kept, not rematerialised per trial
     asm volatile("mov.u32 %0, %1;" : "=r"(hist_sa) : "r"((uint32_t)__cvta_generic_to_shared(sh_hist)));
+#endif
     constexpr bool kSB = RAP_SWEEP_SMEM_BANKS != 0;
     // counter slots in use: 0 RAS stride, 1 RAS diagonal (and malicious, which reuses them), 2 + s
     // the random access under scheme s
