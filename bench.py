@@ -17,6 +17,7 @@ ranks); `roofline` is that kernel's, on the same mean.  Sub-objects timed in the
   `sweep`       the 10^9-trial cfg2 sweep (trials/s, pipe roofline, parity with the golden file);
   `cfg3_layouts` cfg3 8192^2 float32 under RAW / PAD / XOR / RAS / RAP (back-to-back launches);
   `cfg4_layouts` cfg4 under every 64-bit layout (two 32-bit planes; RAP64 8-byte slots; RAP-16);
+  `trace`        the access-trace evaluator (4096 synthetic trace warps x 2048 trials x 5 schemes);
   `cfg1_tile`    cfg1's single 32 x 32 tile (latency, CUDA-graph replay);
   `cfg5_single_gpu` the 32768^2 float32 transpose on one GPU (N = 1);
 each with its roofline and `cpu_baseline` (the oracle, all cores and one core, same sample
@@ -766,6 +767,28 @@ def run_default(args):
         subs[name] = sub
     del x3, y3
     line.update(subs)
+
+    # ---------------- access traces (north star: "synthetic matrices and access traces"): 4096
+    # trace warps of the paper's pattern families, each evaluated under 2048 trials and 5 schemes
+    # per launch; K back-to-back launches over disjoint trial ranges
+    cells = workloads.trace_cells(4096, 32, seed=rank, device=dev)
+    th = torch.zeros((5, 33), dtype=torch.int64, device=dev)
+    sch5 = ("raw", "ras", "rap", "pad", "xor")
+    tk = [0]
+
+    def trace_launch():
+        rap.congestion_trace(cells, 2048, seed=1, schemes=sch5, first_trial=tk[0] * 2048, out=th)
+        tk[0] += 1
+    ms_t, ck_t = timed_back_to_back(trace_launch, W, K, stream, world, dev, barrier)
+    evs = 4096 * 2048 * 5 / (ms_t * 1e-3)
+    thc = th.cpu().numpy()
+    cc33 = np.arange(33)
+    line["trace"] = {"warp_evaluations_per_s": evs * world, "unit": "warp-evaluations/s",
+                     "ras_rap_evaluations_per_s": evs * world * 2 / 5, "kernel_ms_mean": ms_t,
+                     "per_launch": "4096 trace warps x 2048 trials x 5 schemes",
+                     "E_by_scheme": {n: float((thc[i] * cc33).sum() / thc[i].sum()) for i, n in enumerate(sch5)},
+                     "roofline": trace_roofline(evs, ck_t)}
+    del cells, th
 
     # ---------------- cfg1: one 32 x 32 float32 tile (latency case: CUDA-graph replay of 256 launches)
     x1 = workloads.random_bits(32, 32, torch.float32, seed=rank, device=dev)
