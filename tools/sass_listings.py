@@ -11,8 +11,8 @@ import sys
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 KERNELS = {
-    "transpose_b32_rap_cluster": "_ZN4rapk16transpose_kernelILi4ELi1ELb1ELi1ELi2ELb0ELi4ELi2ELb0ELb0ELi8EEEvPKjPjllllNS_10TileShiftsEjjbNS_7PeerOutE14CUtensorMap_st",
-    "transpose_b64_rap_two_planes": "_ZN4rapk16transpose_kernelILi4ELi2ELb1ELi1ELi1ELb0ELi12ELi1ELb0ELb0ELi1EEEvPKjPjllllNS_10TileShiftsEjjbNS_7PeerOutE14CUtensorMap_st",
+    "transpose_b32_rap_cluster": "_ZN4rapk16transpose_kernelILi4ELi1ELb1ELi1ELi2ELb0ELi4ELi2ELb0ELb0ELi8ELb0EEEvPKjPjllllNS_10TileShiftsEjjbNS_7PeerOutE14CUtensorMap_st",
+    "transpose_b64_rap_two_planes": "_ZN4rapk16transpose_kernelILi4ELi2ELb1ELi1ELi1ELb0ELi12ELi1ELb0ELb0ELi1ELb0EEEvPKjPjllllNS_10TileShiftsEjjbNS_7PeerOutE14CUtensorMap_st",
     "transpose_b64_rap64_slots": "_ZN4rapk18transpose64_kernelILi4ELb1ELi12ELi1ELb1EEEvPK5uint2PS1_llllNS_10TileShiftsEjj",
     "transpose_b64_rap16": "_ZN4rapk22transpose_rap16_kernelILi12EEEvPK5uint2PS1_llllNS_10TileShiftsEjj",
     "sweep32_w32_5pat_3sch": "_ZN4rapk14sweep32_kernelILj31ELj7EEEvjjjmmmPm",
@@ -31,6 +31,8 @@ def main(lib, out_dir):
             if m:
                 op = re.sub(r"^@!?U?P[0-9T] ", "", m.group(1)).split()[0]
                 ops[op] += 1
+        if not ops:
+            sys.exit(f"{name}: no SASS for {fn} in {lib} (template signature changed?)")
         with open(os.path.join(out_dir, f"{name}.sass"), "w") as f:
             f.write(f"// cuobjdump -sass -fun {fn} {os.path.relpath(lib, ROOT)}\n")
             f.write("// opcode histogram (static): " + ", ".join(f"{k} {v}" for k, v in ops.most_common()) + "\n")
