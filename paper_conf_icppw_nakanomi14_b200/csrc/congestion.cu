@@ -488,6 +488,68 @@ __host__ __device__ constexpr LiveEvals live_evals(uint32_t PM, uint32_t SM) {  
     return L;
 }
 
+// RAP_SWEEP_ONEHOT (ablation, default 0): the per-trial warp maxima of all live evaluations in
+// two reductions instead of one CREDUX.MAX each (9 for the cfg2 sweep), to unload the ADU pipe
+// (the kernel's busiest, 78 % in profiles/r02_prof_sweep.*).  Measured 3.390 against 3.470 G
+// trials/s (profiles/r02_ab_sweep_onehot.txt): with no CREDUX left on the fast path the ADU pipe
+// still reads 81 % (profiles/r02_prof_sweep_onehot.raw.csv) -- its load follows the instruction
+// count, not the reductions -- and the one-hot words cost 10 instructions per trial more.
+// Bit-identical (every sweep parity test, profiles/r02_pytest_sweep_onehot.log).  Lane v's count c_i(v) of
+// live evaluation i sets bit  min(c_i(v), width_i - 1)  of field i of a 64-bit word pair
+// (u0, u1); __reduce_or_sync of each word over the warp leaves in field i exactly the set of
+// counts that occur, and its highest bit is the maximum -- the congestion -- unless it is the
+// field's top bit, which only says "at least width_i - 1": then (a warp-uniform branch, rare)
+// the exact maxima are taken with one CREDUX.MAX per evaluation as before.  The histogram is
+// therefore the same for every trial, whatever the widths.  Fields: one byte (counts 0..6 exact,
+// top bit ">= 7"; a max load >= 7 has probability ~1e-3 for w = 32) per evaluation, one nibble
+// (0..2, ">= 3") for the accesses a rotation or Theorem 2 makes conflict-free (contiguous under
+// RAS / RAP, stride under RAP: count 1 in every trial), two nibbles per byte -- 8 bytes for the
+// cfg2 sweep.  Lane e then reads its field in three operations: PRMT brings the field's byte of
+// (u0, u1) to byte 3, an AND keeps the field's bits, FLO finds the highest (the count plus the
+// field's bit offset 24 or 28, folded into the histogram row base).  Sets that need more than 8
+// bytes keep the exact reductions.
+#ifndef RAP_SWEEP_ONEHOT
+#define RAP_SWEEP_ONEHOT 0
+#endif
+// RAP_SWEEP_RES_VEC: lane 0 stores the per-trial result slots with STS.128 (4 slots per
+// instruction) instead of one predicated STS per evaluation
+#ifndef RAP_SWEEP_RES_VEC
+#define RAP_SWEEP_RES_VEC 0
+#endif
+__host__ __device__ constexpr bool eval_narrow(int p, int s) {
+    return (p == RAP_PAT_CONTIGUOUS && (s == RAP_SCHEME_RAS || s == RAP_SCHEME_RAP)) ||
+           (p == RAP_PAT_STRIDE && s == RAP_SCHEME_RAP);
+}
+struct OneHotLayout {
+    bool fits;                                       // <= 8 bytes: two words
+    int bit[kMaxEval], width[kMaxEval];              // per live evaluation i: first bit (0..63), 8 or 4
+    uint32_t sat0, sat1;                             // top bits of the fields of u0 / u1
+};
+__host__ __device__ constexpr OneHotLayout onehot_layout(uint32_t PM, uint32_t SM) {
+    OneHotLayout O{false, {}, {}, 0u, 0u};
+    int nbyte = 0, half = -1, i = 0;                 // half: byte whose high nibble is free
+    for (int p = 0; p < 5; ++p)
+        for (int s = 0; s < 5; ++s) {
+            if (!(((PM >> p) & 1u) && ((SM >> s) & 1u)) || eval_fixed(p, s) || eval_dup_src(PM, SM, p, s) >= 0)
+                continue;
+            if (eval_narrow(p, s)) {
+                O.width[i] = 4;
+                if (half >= 0) { O.bit[i] = 8 * half + 4; half = -1; }
+                else { half = nbyte++; O.bit[i] = 8 * half; }
+            } else {
+                O.width[i] = 8;
+                O.bit[i] = 8 * nbyte++;
+            }
+            if (nbyte <= 8) {
+                const int top = O.bit[i] + O.width[i] - 1;
+                if (top < 32) O.sat0 |= 1u << top; else O.sat1 |= 1u << (top - 32);
+            }
+            ++i;
+        }
+    O.fits = nbyte <= 8;
+    return O;
+}
+
 template <uint32_t PM, uint32_t SM>
 __global__ void __launch_bounds__(kSweepWarpsV2 * 32, RAP_SWEEP_MINB)
 sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint64_t n_trials,
@@ -499,7 +561,7 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
     constexpr bool need_r = (SM >> RAP_SCHEME_RAS) & 1u;
     __shared__ uint32_t sh_hist[nbins];
     __shared__ uint32_t sh_tr[kSweepWarpsV2][32 * 33];
-    __shared__ uint32_t sh_res[kSweepWarpsV2][32];
+    __shared__ __align__(16) uint32_t sh_res[kSweepWarpsV2][32];
     __shared__ uint32_t sh_cnt[RAP_SWEEP_SMEM_BANKS ? kSweepWarpsV2 : 1][kSmemBankEvals][32];
     const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
     for (uint32_t b = threadIdx.x; b < nbins; b += blockDim.x) sh_hist[b] = 0;
@@ -591,6 +653,36 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
             }
         }
     }
+#elif RAP_SWEEP_ONEHOT
+    static_assert(RAP_SWEEP_SMEM_BANKS, "one-hot maxima: lane values from the bank counters");
+    // lane e's evaluation (a duplicate: its source's): live index oh_i; oh_info = the PRMT
+    // selector that brings its field's byte to byte 3 (bits 12..14) | the field's bits there
+    // (bits 24..31, PRMT reads bits 0..15 only); oh_base = its histogram row - the FLO offset
+    uint32_t oh_i = 0, oh_info = 0, oh_base = 0;
+    {
+        constexpr LiveEvals LL = live_evals(PM, SM);
+        constexpr OneHotLayout O = onehot_layout(PM, SM);
+#pragma unroll
+        for (int p = 0; p < 5; ++p) {
+#pragma unroll
+            for (int s = 0; s < 5; ++s) {
+                if (!((PM >> p) & 1u) || !((SM >> s) & 1u)) continue;
+                const int e = eval_index(PM, SM, p, s);
+                const int src = eval_dup_src(PM, SM, p, s) >= 0 ? eval_dup_src(PM, SM, p, s) : e;
+#pragma unroll
+                for (int i = 0; i < LL.n; ++i)
+                    if (LL.idx[i] == src && lane == (uint32_t)e) {
+                        const uint32_t nib = (uint32_t)(O.bit[i] & 7), off = 24u + nib;
+                        oh_i = (uint32_t)i;
+                        oh_info = ((uint32_t)(O.bit[i] >> 3) << 12) | ((((1u << O.width[i]) - 1u) << off));
+                        oh_base = lane * (w + 1) - off;
+                    }
+            }
+        }
+        // opaque: kept in registers, not rematerialised per trial from the lane index
+        asm volatile("mov.b32 %0, %0;" : "+r"(oh_info));
+        asm volatile("mov.b32 %0, %0;" : "+r"(oh_base));
+    }
 #endif
 
     const uint64_t nbatch = (n_trials + 31) / 32;
@@ -640,8 +732,9 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
                 const uint32_t same = __match_any_sync(kFull, cell);   // merged requests
                 leaders = ballot_zero(same, lt_mask);              // first lane of its cell
             }
-#if RAP_SWEEP_PACKED_MAX
-            // lane values of the evaluations done per trial, then their warp maxima two at a time
+#if RAP_SWEEP_PACKED_MAX || RAP_SWEEP_ONEHOT
+            // lane values of the evaluations done per trial, then their warp maxima (two at a
+            // time, or every one of them through the one-hot words)
             constexpr int NE = npat * nsch;
             uint32_t lv[NE];
 #pragma unroll
@@ -675,9 +768,10 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
                     }
                 }
             }
+            constexpr LiveEvals LL = live_evals(PM, SM);
+#if RAP_SWEEP_PACKED_MAX
             // pair i of live evaluations -> res[i] = (max of the second) << 16 | max of the first;
             // lane e of the histogram step reads its evaluation's half (res_slot / res_shift)
-            constexpr LiveEvals LL = live_evals(PM, SM);
 #pragma unroll
             for (int i = 0; i + 1 < LL.n; i += 2) {
                 const uint32_t x = warp_max_16x2(lv[LL.idx[i]] + (lv[LL.idx[i + 1]] << 16));
@@ -687,10 +781,43 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
                 const uint32_t x = __reduce_max_sync(kFull, lv[LL.idx[LL.n - 1]]);
                 if (lane == 0) res[LL.n / 2] = x;
             }
+#else
+            // one-hot fields (RAP_SWEEP_ONEHOT): bit min(c, width - 1) of field i, OR over the warp
+            constexpr OneHotLayout O = onehot_layout(PM, SM);
+            uint32_t hidx;                                 // this lane's histogram bin
+            uint32_t u0 = 0, u1 = 0;
+            bool sat = !O.fits;
+            if constexpr (O.fits) {
+#pragma unroll
+                for (int i = 0; i < LL.n; ++i) {
+                    const uint32_t bitv = (1u << (O.bit[i] & 31)) << min(lv[LL.idx[i]], (uint32_t)(O.width[i] - 1));
+                    if (O.bit[i] < 32) u0 |= bitv; else u1 |= bitv;
+                }
+                u0 = __reduce_or_sync(kFull, u0);
+                if (O.sat1) u1 = __reduce_or_sync(kFull, u1);
+                sat = ((u0 & O.sat0) | (u1 & O.sat1)) != 0u;
+            }
+            if (sat) {                                     // a top bit: exact maxima (warp-uniform)
+#pragma unroll
+                for (int i = 0; i < LL.n; ++i) {
+                    const uint32_t x = __reduce_max_sync(kFull, lv[LL.idx[i]]);
+                    if (lane == 0) res[i] = x;
+                }
+                __syncwarp();
+                hidx = lane * (w + 1) + res[oh_i];
+            } else {
+                hidx = oh_base + (31u - __clz(__byte_perm(u0, u1, oh_info) & oh_info));
+            }
+#endif
             const uint32_t e = npat * nsch;
 #else
             uint32_t e = 0;
             uint32_t c_stride[5] = {0, 0, 0, 0, 0}, c_diag[5] = {0, 0, 0, 0, 0};
+#if RAP_SWEEP_RES_VEC
+            uint32_t cres[(npat * nsch + 3) & ~3u];        // result slots, stored 4 at a time
+#pragma unroll
+            for (uint32_t k = 0; k < ((npat * nsch + 3) & ~3u); ++k) cres[k] = 0u;
+#endif
 #pragma unroll
             for (int p = 0; p < 5; ++p) {
                 if (!((PM >> p) & 1u)) continue;
@@ -760,15 +887,28 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
                 counted:
                     if (p == RAP_PAT_STRIDE) c_stride[s] = c;
                     if (p == RAP_PAT_DIAGONAL) c_diag[s] = c;
+#if RAP_SWEEP_RES_VEC
+                    if (!((fixed_slots >> e) & 1u)) cres[e] = c;
+#else
                     if (lane == 0 && !((fixed_slots >> e) & 1u)) res[e] = c;   // C4: result slot e
+#endif
                     ++e;
                 }
             }
+#if RAP_SWEEP_RES_VEC
+            if (lane == 0) {                                   // C4: the result slots, STS.128
+#pragma unroll
+                for (uint32_t k = 0; k < ((npat * nsch + 3) & ~3u); k += 4)
+                    *reinterpret_cast<uint4 *>(res + k) = make_uint4(cres[k], cres[k + 1], cres[k + 2], cres[k + 3]);
+            }
+#endif
 #endif
             __syncwarp();
 #if RAP_SWEEP_PACKED_MAX
             if (lane < e && !lane_fixed)
                 atomicAdd(&sh_hist[lane * (w + 1) + ((res[res_slot] >> res_shift) & 0xffffu)], 1u);
+#elif RAP_SWEEP_ONEHOT
+            if (lane < e && !lane_fixed) atomicAdd(&sh_hist[hidx], 1u);
 #else
 #if RAP_SWEEP_HIST_SA
             if (lane < e && !lane_fixed) smem_inc(hist_sa + 4u * (lane * (w + 1) + res[lane]));

@@ -157,8 +157,8 @@ def test_transpose_extreme_aspect(rap, oracle, shape):
 @pytest.mark.parametrize("layout", ["rap", "rap64", "rap16"])
 def test_transpose_cfg4_16384_f64(rap, oracle, layout):
     # BASELINE cfg4 at full size, in the launch configuration bench.py times: all 2^28 doubles
-    # compared with the oracle (rap: the w = 32 map on two 32-bit planes, the headline; rap64:
-    # the w = 32 map on 8-byte slots; rap16: RAP over 16 double banks)
+    # compared with the oracle (rap64: the w = 32 map on 8-byte slots, the headline; rap: the
+    # w = 32 map on two 32-bit planes; rap16: RAP over 16 double banks)
     x = workloads.random_bits(16384, 16384, torch.float64, seed=0, device="cuda")
     y = rap.transpose(x, layout=layout, seed=0)
     torch.cuda.synchronize()
