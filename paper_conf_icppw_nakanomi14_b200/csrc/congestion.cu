@@ -186,6 +186,12 @@ __device__ __forceinline__ uint32_t plane_value(const uint32_t (&q)[5], uint32_t
     for (int b = 0; b < 5; ++b) v |= ((q[b] >> i) & 1u) << b;
     return v;
 }
+__device__ __forceinline__ uint32_t plane_value4(const uint32_t (&q)[5], uint32_t i) {   // 4 * value
+    uint32_t v = 0;
+#pragma unroll
+    for (int b = 0; b < 5; ++b) v |= ((q[b] >> i) & 1u) << (b + 2);
+    return v;
+}
 
 // (x mod w) for x < 2w; a mask when w is a compile-time power of two
 template <int W>
@@ -461,6 +467,26 @@ __device__ __forceinline__ uint32_t count_in_bank(uint32_t *cnt, uint32_t bank, 
     return (atomicAdd(cnt + (bank & 31u), one) + 1u) * one;
 }
 
+// RAP_SWEEP_BANK4 (default 1): the sweep's data-dependent banks are carried pre-multiplied by 4
+// (the byte offset of the bank's counter): the transpose buffer holds r << 12 | cell << 2, P[row]
+// is assembled in bits 2..6, and a bank-counter address is one LOP3 -- (bank4 & 0x7c) | slot
+// base, the slots 128-byte aligned -- instead of shift, mask and add.  Junk below bit 2 (from
+// the shifts) never carries into the bank bits: every operand added to it has bits 0..1 clear.
+// 8 fewer instructions per trial; +0.5 % with the STS.128 result slots (3.613 vs 3.594 G
+// trials/s, profiles/r02_ab_sweep_bank4.txt), -0.3 % without them.
+#ifndef RAP_SWEEP_BANK4
+#define RAP_SWEEP_BANK4 1
+#endif
+__device__ __forceinline__ uint32_t count_in_bank4(uint32_t cnt_sa, int slot, uint32_t bank4, bool counted) {
+    const uint32_t one = counted ? 1u : 0u;
+    uint32_t a, old;
+    // one LOP3: cnt_sa | (bank4 & 0x7c) (written out: the compiler otherwise emits AND + IADD);
+    // the slot offset folds into the ATOMS address immediate
+    asm("lop3.b32 %0, %1, 0x7c, %2, 0xf8;" : "=r"(a) : "r"(cnt_sa), "r"(bank4));
+    asm volatile("atom.shared.add.u32 %0, [%1], %2;" : "=r"(old) : "r"(a + 128u * (uint32_t)slot), "r"(one) : "memory");
+    return (old + 1u) * one;
+}
+
 // Evaluation bookkeeping of sweep32_kernel, all compile-time: evaluation e = (pattern p, scheme s)
 // in mask order; "fixed" = trial-invariant (non-random pattern under RAW / PAD / XOR); "dup" =
 // malicious access equal to the stride (RAW, RAS) or diagonal (RAP, XOR) access (reading iii).
@@ -511,10 +537,24 @@ __host__ __device__ constexpr LiveEvals live_evals(uint32_t PM, uint32_t SM) {  
 #ifndef RAP_SWEEP_ONEHOT
 #define RAP_SWEEP_ONEHOT 0
 #endif
-// RAP_SWEEP_RES_VEC: lane 0 stores the per-trial result slots with STS.128 (4 slots per
-// instruction) instead of one predicated STS per evaluation
+// RAP_SWEEP_PLANES_SMEM (default 1): the lane-mode phase leaves each trial's permutation planes,
+// P[0] and r[0] in shared memory (two 16-byte rows per trial) and the warp-mode phase reads trial
+// m's with two broadcast LDS.128 instead of seven SHFL; RAP_SWEEP_CLEAR_VEC (default 1): the bank
+// counters of a trial are cleared with STS.128 spread over the lanes (2 instructions for the 5
+// slots of the cfg2 sweep) instead of one STS per slot.  Both cut MIO-pipe instructions, as the
+// result-slot stores below did: 3.613 -> 3.816 G trials/s together (planes +5.0 %, clears +0.5 %;
+// profiles/r02_ab_sweep_planes.txt).
+#ifndef RAP_SWEEP_PLANES_SMEM
+#define RAP_SWEEP_PLANES_SMEM 1
+#endif
+#ifndef RAP_SWEEP_CLEAR_VEC
+#define RAP_SWEEP_CLEAR_VEC 1
+#endif
+// RAP_SWEEP_RES_VEC (default 1): lane 0 stores the per-trial result slots with STS.128 (4 slots
+// per instruction) instead of one predicated STS per evaluation: 3.467 -> 3.591 G trials/s
+// (profiles/r02_ab_sweep_resvec.txt) -- a predicated one-lane STS still takes a full MIO slot
 #ifndef RAP_SWEEP_RES_VEC
-#define RAP_SWEEP_RES_VEC 0
+#define RAP_SWEEP_RES_VEC 1
 #endif
 __host__ __device__ constexpr bool eval_narrow(int p, int s) {
     return (p == RAP_PAT_CONTIGUOUS && (s == RAP_SCHEME_RAS || s == RAP_SCHEME_RAP)) ||
@@ -562,7 +602,8 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
     __shared__ uint32_t sh_hist[nbins];
     __shared__ uint32_t sh_tr[kSweepWarpsV2][32 * 33];
     __shared__ __align__(16) uint32_t sh_res[kSweepWarpsV2][32];
-    __shared__ uint32_t sh_cnt[RAP_SWEEP_SMEM_BANKS ? kSweepWarpsV2 : 1][kSmemBankEvals][32];
+    __shared__ __align__(128) uint32_t sh_cnt[RAP_SWEEP_SMEM_BANKS ? kSweepWarpsV2 : 1][kSmemBankEvals][32];
+    __shared__ __align__(16) uint32_t sh_pl[RAP_SWEEP_PLANES_SMEM ? kSweepWarpsV2 : 1][RAP_SWEEP_PLANES_SMEM ? 32 : 1][8];
     const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
     for (uint32_t b = threadIdx.x; b < nbins; b += blockDim.x) sh_hist[b] = 0;
     __syncthreads();
@@ -572,6 +613,8 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
     uint32_t *tr = sh_tr[warp];
     uint32_t *res = sh_res[warp];
     uint32_t *cnt = &sh_cnt[RAP_SWEEP_SMEM_BANKS ? warp : 0][0][0];
+    constexpr bool kB4 = RAP_SWEEP_BANK4 && RAP_SWEEP_SMEM_BANKS && !RAP_SWEEP_PACKED_MAX && !RAP_SWEEP_ONEHOT;
+    const uint32_t cnt_sa = (uint32_t)__cvta_generic_to_shared(cnt);   // 128-byte aligned slots
 #if RAP_SWEEP_HIST_SA
     uint32_t hist_sa;                 // opaque to the compiler: kept, not rematerialised per trial
     asm volatile("mov.u32 %0, %1;" : "=r"(hist_sa) : "r"((uint32_t)__cvta_generic_to_shared(sh_hist)));
@@ -706,29 +749,40 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
                 for (int i = 0; i < 4; ++i) {
                     const uint32_t r = ur[i] >> 27, cell = uc[i] >> 22;   // floor(u*32/2^32), floor(u*1024/2^32)
                     if (blk == 0 && i == 0) r0_lane = r;
-                    tr[(4 * blk + i) * 33 + lane] = (r << 10) | cell;
+                    tr[(4 * blk + i) * 33 + lane] = kB4 ? (r << 12) | (cell << 2) : (r << 10) | cell;
                 }
             }
         }
+#if RAP_SWEEP_PLANES_SMEM
+        *reinterpret_cast<uint4 *>(&sh_pl[warp][lane][0]) = make_uint4(pl[0], pl[1], pl[2], pl[3]);
+        *reinterpret_cast<uint4 *>(&sh_pl[warp][lane][4]) = make_uint4(pl[4], p0_lane, r0_lane, 0u);
+#endif
         __syncwarp();
         // ---- warp mode: lane t is DMM thread t of trial n0 + m
         for (uint32_t m = 0; m < nvalid; ++m) {
             BankMask Pm;                                           // bit t = bit b of P[t]
+#if RAP_SWEEP_PLANES_SMEM
+            const uint4 qa = *reinterpret_cast<const uint4 *>(&sh_pl[warp][m][0]);   // broadcast reads
+            const uint4 qb = *reinterpret_cast<const uint4 *>(&sh_pl[warp][m][4]);
+            Pm.b[0] = qa.x; Pm.b[1] = qa.y; Pm.b[2] = qa.z; Pm.b[3] = qa.w; Pm.b[4] = qb.x;
+            const uint32_t P0 = qb.y, r0 = qb.z;
+#else
 #pragma unroll
             for (int b = 0; b < 5; ++b) Pm.b[b] = __shfl_sync(kFull, pl[b], m);
             const uint32_t P0 = __shfl_sync(kFull, p0_lane, m);
             const uint32_t r0 = __shfl_sync(kFull, r0_lane, m);
+#endif
             const uint32_t packed = tr[lane * 33 + m];
-            const uint32_t rt = packed >> 10;
+            const uint32_t rt = packed >> 10;                      // kB4: 4 r[t] (+ junk in bits 0..1)
             BankMask Rm;
             if (need_r && !kSB) Rm = masks_ballot(rt);              // bit t = bit b of r[t]
             uint32_t rrow = 0, rcol = 0, Pr = 0, rr = 0, leaders = kFull;
             if (any_random) {
-                const uint32_t cell = packed & 1023u;
-                rrow = cell >> 5;
-                rcol = cell & 31u;
-                Pr = plane_value(Pm.b, rrow);                      // P[row_t]
-                rr = __shfl_sync(kFull, rt, rrow);                 // r[row_t]
+                const uint32_t cell = kB4 ? packed & 0xffcu : packed & 1023u;
+                rrow = kB4 ? cell >> 7 : cell >> 5;
+                rcol = kB4 ? cell & 0x7cu : cell & 31u;            // kB4: 4 col
+                Pr = kB4 ? plane_value4(Pm.b, rrow) : plane_value(Pm.b, rrow);   // (4) P[row_t]
+                rr = __shfl_sync(kFull, rt, rrow);                 // (4) r[row_t]
                 const uint32_t same = __match_any_sync(kFull, cell);   // merged requests
                 leaders = ballot_zero(same, lt_mask);              // first lane of its cell
             }
@@ -846,12 +900,22 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
                             // random under scheme s 2 + s); packed carries rcol in bits 0..4, and
                             // count_in_bank reduces the bank mod 32
                             const int slot = pp == RAP_PAT_STRIDE ? 0 : pp == RAP_PAT_DIAGONAL ? 1 : 2 + s;
+                            const bool counted = pp != RAP_PAT_RANDOM || ((leaders >> lane) & 1u);
+                            if (kB4) {                             // banks as 4 x bank (counter byte offsets)
+                                const uint32_t bank4 = pp == RAP_PAT_STRIDE ? rt
+                                                     : pp == RAP_PAT_DIAGONAL ? (lane << 2) + rt
+                                                     : s == RAP_SCHEME_RAW ? packed
+                                                     : s == RAP_SCHEME_PAD ? packed + (packed >> 5)
+                                                     : s == RAP_SCHEME_XOR ? packed ^ (packed >> 5)
+                                                     : packed + (isp ? Pr : rr);
+                                c = __reduce_max_sync(kFull, count_in_bank4(cnt_sa, slot, bank4, counted));
+                                goto counted;
+                            }
                             const uint32_t bank = pp == RAP_PAT_STRIDE ? rt : pp == RAP_PAT_DIAGONAL ? lane + rt
                                                 : s == RAP_SCHEME_RAW ? packed
                                                 : s == RAP_SCHEME_PAD ? rrow + rcol
                                                 : s == RAP_SCHEME_XOR ? (rcol ^ rrow)
                                                 : packed + (isp ? Pr : rr);
-                            const bool counted = pp != RAP_PAT_RANDOM || ((leaders >> lane) & 1u);
                             c = __reduce_max_sync(kFull, count_in_bank(cnt + slot * 32, bank, counted));
                             goto counted;
                         }
@@ -917,9 +981,18 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
 #endif
 #endif
             if (kSB) {                                                  // clear the bank counters
+#if RAP_SWEEP_CLEAR_VEC
+                // every slot up to the highest in use, 16 bytes per lane (unused slots stay 0)
+                constexpr uint32_t n4 = kSlots ? 8u * (32u - __builtin_clz(kSlots)) : 0u;
+#pragma unroll
+                for (uint32_t i = 0; i < n4; i += 32)
+                    if (i + 32 <= n4 || i + lane < n4)
+                        reinterpret_cast<uint4 *>(cnt)[i + lane] = make_uint4(0u, 0u, 0u, 0u);
+#else
 #pragma unroll
                 for (int k = 0; k < kSmemBankEvals; ++k)
                     if ((kSlots >> k) & 1u) cnt[k * 32 + lane] = 0u;
+#endif
             }
             __syncwarp();
         }
