@@ -556,6 +556,38 @@ __host__ __device__ constexpr LiveEvals live_evals(uint32_t PM, uint32_t SM) {  
 #ifndef RAP_SWEEP_RES_VEC
 #define RAP_SWEEP_RES_VEC 1
 #endif
+// RAP_SWEEP_UNROLL_M (tuning): unroll factor of the per-trial warp-mode loop (1: none).  Measured
+// with the default 8 CTAs of 64 registers per SM: unroll 2 3.797 vs 3.839 G trials/s, and 7 / 6
+// CTAs per SM with more registers 3.786 / 3.746 (profiles/r02c_ab_sweep_unroll.txt)
+#ifndef RAP_SWEEP_UNROLL_M
+#define RAP_SWEEP_UNROLL_M 1
+#endif
+constexpr int kSweepUnrollM = RAP_SWEEP_UNROLL_M;
+// RAP_SWEEP_LEAD_LANE (default 1): with the bank counters every merged-request test reads only the
+// lane's own leader bit, so the lane tests its own __match_any_sync word ((same & lanes below) ==
+// 0) instead of gathering every lane's bit with a ballot: one VOTE fewer per trial; 3.800 -> 3.819
+// G trials/s (+0.5 %, profiles/r02c_ab_sweep_pred.txt).
+#ifndef RAP_SWEEP_LEAD_LANE
+#define RAP_SWEEP_LEAD_LANE 1
+#endif
+// RAP_SWEEP_HIST_PRED (ablation, default 0): a branch-free per-trial histogram step -- the result
+// slots stored by a predicated STS.128, every lane adding 0 or 1 with one red.shared -- instead of
+// a branch around the 11 incrementing lanes (BSSY, BRA, two BSYNC, WARPSYNC per trial).  The loop
+// loses those 5 control instructions (the ADU pipe's, 86 % busy in profiles/r02_prof_sweep.*),
+// yet ran 0.3 % slower (3.788 vs 3.800 G trials/s) and ncu still shows the ADU pipe 85 % busy
+// (profiles/r02c_prof_sweep_pred.raw.csv): the branch was not what loaded it.  Bit-identical.
+#ifndef RAP_SWEEP_HIST_PRED
+#define RAP_SWEEP_HIST_PRED 0
+#endif
+__device__ __forceinline__ void smem_add(uint32_t saddr, uint32_t v) {
+    asm volatile("red.shared.add.u32 [%0], %1;" :: "r"(saddr), "r"(v) : "memory");
+}
+// 16-byte shared store executed only where `on` (a predicate in PTX, not a branch around it)
+__device__ __forceinline__ void sts128_if(uint32_t saddr, uint32_t a, uint32_t b, uint32_t c, uint32_t d, bool on) {
+    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %5, 0;\n\t@p st.shared.v4.u32 [%0], {%1, %2, %3, %4};\n\t}"
+                 :: "r"(saddr), "r"(a), "r"(b), "r"(c), "r"(d), "r"((uint32_t)on) : "memory");
+}
+
 __host__ __device__ constexpr bool eval_narrow(int p, int s) {
     return (p == RAP_PAT_CONTIGUOUS && (s == RAP_SCHEME_RAS || s == RAP_SCHEME_RAP)) ||
            (p == RAP_PAT_STRIDE && s == RAP_SCHEME_RAP);
@@ -606,6 +638,7 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
     __shared__ __align__(16) uint32_t sh_pl[RAP_SWEEP_PLANES_SMEM ? kSweepWarpsV2 : 1][RAP_SWEEP_PLANES_SMEM ? 32 : 1][8];
     const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
     for (uint32_t b = threadIdx.x; b < nbins; b += blockDim.x) sh_hist[b] = 0;
+    sh_res[warp][lane] = 0u;                      // slots no evaluation writes stay in range
     __syncthreads();
     const LaneSel ls(lane);
     const LaneEq le(ls);
@@ -615,6 +648,8 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
     uint32_t *cnt = &sh_cnt[RAP_SWEEP_SMEM_BANKS ? warp : 0][0][0];
     constexpr bool kB4 = RAP_SWEEP_BANK4 && RAP_SWEEP_SMEM_BANKS && !RAP_SWEEP_PACKED_MAX && !RAP_SWEEP_ONEHOT;
     const uint32_t cnt_sa = (uint32_t)__cvta_generic_to_shared(cnt);   // 128-byte aligned slots
+    const uint32_t hist_sa0 = (uint32_t)__cvta_generic_to_shared(sh_hist);
+    static_assert(nbins >= 32, "HIST_PRED: idle lanes add 0 to word `lane` of the histogram");
 #if RAP_SWEEP_HIST_SA
     uint32_t hist_sa;                 // opaque to the compiler: kept, not rematerialised per trial
     asm volatile("mov.u32 %0, %1;" : "=r"(hist_sa) : "r"((uint32_t)__cvta_generic_to_shared(sh_hist)));
@@ -759,6 +794,7 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
 #endif
         __syncwarp();
         // ---- warp mode: lane t is DMM thread t of trial n0 + m
+#pragma unroll kSweepUnrollM
         for (uint32_t m = 0; m < nvalid; ++m) {
             BankMask Pm;                                           // bit t = bit b of P[t]
 #if RAP_SWEEP_PLANES_SMEM
@@ -777,6 +813,7 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
             BankMask Rm;
             if (need_r && !kSB) Rm = masks_ballot(rt);              // bit t = bit b of r[t]
             uint32_t rrow = 0, rcol = 0, Pr = 0, rr = 0, leaders = kFull;
+            bool lead_me = true;                                   // this lane leads its cell
             if (any_random) {
                 const uint32_t cell = kB4 ? packed & 0xffcu : packed & 1023u;
                 rrow = kB4 ? cell >> 7 : cell >> 5;
@@ -784,7 +821,12 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
                 Pr = kB4 ? plane_value4(Pm.b, rrow) : plane_value(Pm.b, rrow);   // (4) P[row_t]
                 rr = __shfl_sync(kFull, rt, rrow);                 // (4) r[row_t]
                 const uint32_t same = __match_any_sync(kFull, cell);   // merged requests
-                leaders = ballot_zero(same, lt_mask);              // first lane of its cell
+                if (kSB && RAP_SWEEP_LEAD_LANE) {
+                    lead_me = (same & lt_mask) == 0u;              // first lane of its cell
+                } else {
+                    leaders = ballot_zero(same, lt_mask);          // first lane of its cell
+                    lead_me = (leaders >> lane) & 1u;
+                }
             }
 #if RAP_SWEEP_PACKED_MAX || RAP_SWEEP_ONEHOT
             // lane values of the evaluations done per trial, then their warp maxima (two at a
@@ -812,7 +854,7 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
                                             : s == RAP_SCHEME_PAD ? rrow + rcol
                                             : s == RAP_SCHEME_XOR ? (rcol ^ rrow)
                                             : packed + (isp ? Pr : rr);
-                        lv[e] = count_in_bank(cnt + slot * 32, bank, p != RAP_PAT_RANDOM || ((leaders >> lane) & 1u));
+                        lv[e] = count_in_bank(cnt + slot * 32, bank, p != RAP_PAT_RANDOM || lead_me);
                     } else if (p == RAP_PAT_CONTIGUOUS) {                          // RAS / RAP
                         lv[e] = lane_load_rot(isp ? P0 : r0, le);
                     } else if (p == RAP_PAT_DIAGONAL || (p == RAP_PAT_MALICIOUS && isp)) {   // RAP (RAS: counters)
@@ -900,7 +942,7 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
                             // random under scheme s 2 + s); packed carries rcol in bits 0..4, and
                             // count_in_bank reduces the bank mod 32
                             const int slot = pp == RAP_PAT_STRIDE ? 0 : pp == RAP_PAT_DIAGONAL ? 1 : 2 + s;
-                            const bool counted = pp != RAP_PAT_RANDOM || ((leaders >> lane) & 1u);
+                            const bool counted = pp != RAP_PAT_RANDOM || lead_me;
                             if (kB4) {                             // banks as 4 x bank (counter byte offsets)
                                 const uint32_t bank4 = pp == RAP_PAT_STRIDE ? rt
                                                      : pp == RAP_PAT_DIAGONAL ? (lane << 2) + rt
@@ -960,11 +1002,20 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
                 }
             }
 #if RAP_SWEEP_RES_VEC
+#if RAP_SWEEP_HIST_PRED
+            {                                                  // C4: the result slots, STS.128,
+                const uint32_t rsa = (uint32_t)__cvta_generic_to_shared(res);   // predicated on lane 0
+#pragma unroll
+                for (uint32_t k = 0; k < ((npat * nsch + 3) & ~3u); k += 4)
+                    sts128_if(rsa + 4u * k, cres[k], cres[k + 1], cres[k + 2], cres[k + 3], lane == 0);
+            }
+#else
             if (lane == 0) {                                   // C4: the result slots, STS.128
 #pragma unroll
                 for (uint32_t k = 0; k < ((npat * nsch + 3) & ~3u); k += 4)
                     *reinterpret_cast<uint4 *>(res + k) = make_uint4(cres[k], cres[k + 1], cres[k + 2], cres[k + 3]);
             }
+#endif
 #endif
 #endif
             __syncwarp();
@@ -976,6 +1027,14 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
 #else
 #if RAP_SWEEP_HIST_SA
             if (lane < e && !lane_fixed) smem_inc(hist_sa + 4u * (lane * (w + 1) + res[lane]));
+#elif RAP_SWEEP_HIST_PRED
+            // every lane adds: lane e of a live evaluation 1 to its bin, the others 0 to word `lane`
+            // of the histogram (in range, distinct banks) -- no branch, no predicate to if-convert
+            {
+                const bool on = lane < e && !lane_fixed;
+                const uint32_t bin = on ? lane * (w + 1) + res[lane] : lane;
+                smem_add(hist_sa0 + 4u * bin, on ? 1u : 0u);
+            }
 #else
             if (lane < e && !lane_fixed) atomicAdd(&sh_hist[lane * (w + 1) + res[lane]], 1u);
 #endif

@@ -124,6 +124,10 @@ cudaError_t launch_transpose_rap16(const void *src, void *dst, int64_t rows, int
 cudaError_t launch_transpose64(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
                                int64_t ld_dst, int layout, uint64_t seed, cudaStream_t st);
 
+// 32-bit elements as column-pair 8-byte slots (transpose64.cu; tuning path RAP32_PAIR of transpose.cu)
+cudaError_t launch_transpose_pair32(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
+                                    int64_t ld_dst, int layout, uint64_t seed, cudaStream_t st);
+
 cudaError_t launch_transpose_peers(const void *src, int64_t M, int64_t N, int64_t ld_src, const PeerOut &pe,
                                    int64_t ld_dst, uint32_t elem_bytes, int layout, uint64_t seed, cudaStream_t st);
 

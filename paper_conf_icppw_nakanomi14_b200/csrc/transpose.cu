@@ -119,6 +119,11 @@ __device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.
 #ifndef RAP32_KP
 #define RAP32_KP 0
 #endif
+// RAP32_PAIR: 32-bit transposes through column-pair 8-byte slots (transpose64.cu's P32 form) --
+// tuning flag, off
+#ifndef RAP32_PAIR
+#define RAP32_PAIR 0
+#endif
 #ifndef RAP32_KP_SR
 #define RAP32_KP_SR 12
 #endif
@@ -620,6 +625,12 @@ static cudaError_t launch_shape(const void *src, void *dst, int64_t rows, int64_
     // cluster, no idle warps of a super-tile computing P, the cheapest launch
     if (((rows + 31) / 32) * ((cols + 31) / 32) <= kSmallTiles)
         return launch_one<L, EW, VEC, 1, 1, false, 1, 1>(src, dst, rows, cols, ld_src, ld_dst, seed, tu, st);
+    // column-pair slots (RAP32_PAIR): 32-bit elements as virtual 8-byte elements (a[i][2k], a[i][2k+1])
+    // through the one-double-per-slot kernel (transpose64.cu)
+    if constexpr (EW == 1 && VEC) {
+        if (RAP32_PAIR && tu.cl == kDefaultCL32 && cols % 2 == 0 && ld_src % 2 == 0)
+            return launch_transpose_pair32(src, dst, rows, cols, ld_src, ld_dst, L, seed, st);
+    }
     // row-pair planes (KP): 32-bit elements as virtual 8-byte elements, the 64-bit kernel's shape
     if constexpr (EW == 1 && VEC) {
         if (RAP32_KP && tu.cl == kDefaultCL32 && rows % 2 == 0 && ld_dst % 2 == 0 && (uintptr_t)dst % 8 == 0)

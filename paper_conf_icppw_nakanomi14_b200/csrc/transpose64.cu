@@ -88,7 +88,12 @@ __device__ __forceinline__ uint2 ldg_nc_v2(const void *p) {
 // ROWS = true: T1 with one LDG.64 per tile row (lane j reads double j, 256 B per instruction,
 // 32 per tile) and one STS.64 per row: lanes j = 0..15 of row i hit bank pairs (j + P[i]) mod 16,
 // distinct for any P -- the row write needs no grouping.  ROWS = false: the LDG.128 grouping above.
-template <int L, bool VEC, int SR, int MINB, bool ROWS>
+// P32 (tuning, RAP32_PAIR): the same kernel moves a 32-bit matrix as a matrix of virtual 8-byte
+// elements v(i, k) = (a[i][2k], a[i][2k+1]) -- column pairs, so `cols` / `ld_src` count pairs and
+// `ld_dst` counts 32-bit words.  A tile is 32 rows x 64 words (256-byte input rows, one LDG.64
+// per row); the drain's slot (rho, c) holds output elements (2c, rho) and (2c+1, rho), stored by
+// two STG.32 into two 128-byte output row segments.
+template <int L, bool VEC, int SR, int MINB, bool ROWS, bool P32 = false>
 __global__ void __launch_bounds__(SR * 32, MINB)
 transpose64_kernel(const uint2 *__restrict__ src, uint2 *__restrict__ dst, int64_t rows, int64_t cols,
                    int64_t ld_src, int64_t ld_dst, const TileShifts ts, uint32_t tiles_r, uint32_t tiles_c) {
@@ -197,6 +202,32 @@ transpose64_kernel(const uint2 *__restrict__ src, uint2 *__restrict__ dst, int64
     // T2: the stride (column) read and 256-byte output rows
     auto drain = [&](uint32_t ti, uint32_t tj) {
         const int64_t r0 = (int64_t)ti * 32, c0 = (int64_t)tj * 32;
+        if constexpr (P32) {
+            uint32_t *o = reinterpret_cast<uint32_t *>(dst) + 2 * c0 * ld_dst + r0 + rho;
+            const bool rok = r0 + rho < rows;
+            const int cmax = (int)min((int64_t)32, cols - c0);
+            if (r0 + 32 <= rows && cmax == 32) {
+#pragma unroll
+                for (int c = 0; c < 32; ++c) {
+                    const uint32_t off = (L == RAP_LAYOUT_XOR) ? drain_base ^ (uint32_t)c : drain_base + c;
+                    const uint2 x = tile[off];
+                    o[0] = x.x;
+                    o[ld_dst] = x.y;
+                    o += 2 * ld_dst;
+                }
+            } else {
+                for (int c = 0; c < cmax; ++c) {
+                    const uint32_t off = (L == RAP_LAYOUT_XOR) ? drain_base ^ (uint32_t)c : drain_base + c;
+                    if (rok) {
+                        const uint2 x = tile[off];
+                        o[0] = x.x;
+                        o[ld_dst] = x.y;
+                    }
+                    o += 2 * ld_dst;
+                }
+            }
+            return;
+        }
         uint2 *o = dst + c0 * ld_dst + r0 + rho;
         if (r0 + 32 <= rows && c0 + 32 <= cols) {
 #pragma unroll
@@ -257,10 +288,10 @@ transpose64_kernel(const uint2 *__restrict__ src, uint2 *__restrict__ dst, int64
 #define RAP64_ROWS 1
 #endif
 
-template <int L, bool VEC, int SR, int MINB, bool ROWS = RAP64_ROWS>
+template <int L, bool VEC, int SR, int MINB, bool ROWS = RAP64_ROWS, bool P32 = false>
 static cudaError_t launch64_one(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
                                 int64_t ld_dst, uint64_t seed, cudaStream_t st) {
-    auto k = transpose64_kernel<L, VEC, SR, MINB, ROWS>;
+    auto k = transpose64_kernel<L, VEC, SR, MINB, ROWS, P32>;
     static ShapeCache cache;
     const size_t smem = sizeof(uint2) * 32 * Geom64<L>::RP * SR;
     const uint32_t tiles_r = (uint32_t)((rows + 31) / 32), tiles_c = (uint32_t)((cols + 31) / 32);
@@ -275,7 +306,8 @@ static cudaError_t launch64_one(const void *src, void *dst, int64_t rows, int64_
     const cudaError_t e = cached_grid(k, cache, SR * 32, smem, nst, 0, &grid);
     if (e != cudaSuccess) return e;
     TileShifts ts = tile_shifts(L, seed);
-    ts.early = pdl_early_loads(st, src, rows, cols, ld_src, dst, cols, rows, ld_dst, 8u) ? 1u : 0u;
+    if (P32) pdl_forget(st);
+    else ts.early = pdl_early_loads(st, src, rows, cols, ld_src, dst, cols, rows, ld_dst, 8u) ? 1u : 0u;
     return launch_ex(k, grid, SR * 32, smem, st, 1, (const uint2 *)src, (uint2 *)dst, rows, cols, ld_src, ld_dst, ts,
                      tiles_r, tiles_c);
 }
@@ -304,6 +336,31 @@ cudaError_t launch_transpose64(const void *src, void *dst, int64_t rows, int64_t
         RAPK64_CASE(RAP_LAYOUT_RAP)
     }
 #undef RAPK64_CASE
+    return cudaErrorInvalidValue;
+}
+
+#ifndef RAP32_PAIR_SR
+#define RAP32_PAIR_SR 12
+#endif
+#ifndef RAP32_PAIR_MINB
+#define RAP32_PAIR_MINB 1
+#endif
+// 32-bit transposes through column-pair 8-byte slots (RAP32_PAIR tuning path of transpose.cu):
+// requires an even `cols`, an even `ld_src` and an 8-byte aligned source (the caller checks)
+cudaError_t launch_transpose_pair32(const void *src, void *dst, int64_t rows, int64_t cols, int64_t ld_src,
+                                    int64_t ld_dst, int layout, uint64_t seed, cudaStream_t st) {
+#define RAPK32P_CASE(LAY)                                                                            \
+    case LAY:                                                                                        \
+        return launch64_one<LAY, true, RAP32_PAIR_SR, RAP32_PAIR_MINB, true, true>(src, dst, rows, cols / 2, \
+                                                                               ld_src / 2, ld_dst, seed, st);
+    switch (layout) {
+        RAPK32P_CASE(RAP_LAYOUT_RAW)
+        RAPK32P_CASE(RAP_LAYOUT_PAD)
+        RAPK32P_CASE(RAP_LAYOUT_XOR)
+        RAPK32P_CASE(RAP_LAYOUT_RAS)
+        RAPK32P_CASE(RAP_LAYOUT_RAP)
+    }
+#undef RAPK32P_CASE
     return cudaErrorInvalidValue;
 }
 

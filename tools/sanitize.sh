@@ -1,4 +1,5 @@
 #!/bin/bash
+# NOTE: compute-sanitizer is closed on the GPU pool (profiles/r02c_sanitizer_refused.txt); kept for other machines
 # compute-sanitizer memcheck / racecheck / synccheck over tools/sanitize.py (small calls of every kernel)
 OUT=${1:-gpurun_out/r02_sanitizer.txt}
 python -c "import __graft_entry__ as g; g.build()"
