@@ -1203,8 +1203,12 @@ trace_kernel(uint32_t w_rt, uint64_t n_warps, const uint32_t *__restrict__ cells
 #ifndef RAP_TRACE_TB
 #define RAP_TRACE_TB 32
 #endif
+// trace warps per unit: the per-trial P / r draws of a unit are shared by its TK trace warps.
+// Measured with the BANK4 counters (4096 trace warps x 2048 trials): TK 64 105.1, 128 111.9,
+// 192 112.3, 256 105.4 G warp-evaluations/s (fewer units than 2 waves), TB 16 x TK 128 101.2
+// (profiles/r02c_ab_trace*.txt)
 #ifndef RAP_TRACE_TK
-#define RAP_TRACE_TK 64
+#define RAP_TRACE_TK 128
 #endif
 #ifndef RAP_TRACE_WARPS
 #define RAP_TRACE_WARPS 8
@@ -1227,6 +1231,12 @@ __device__ __forceinline__ uint32_t wrap_w(uint32_t x, uint32_t w) { return W ==
 #ifndef RAP_TRACE_SMEM_BANKS
 #define RAP_TRACE_SMEM_BANKS 1
 #endif
+// RAP_TRACE_BANK4 (default 1): as RAP_SWEEP_BANK4 -- the shifts are kept as 4 x shift (a byte:
+// <= 124) and the lane's column as 4 x col, so a counter address is (4 col + 4 shift) & 0x7c
+// OR'ed into the counter set's 128-byte-aligned base: one LOP3 instead of mask, shift and add
+#ifndef RAP_TRACE_BANK4
+#define RAP_TRACE_BANK4 1
+#endif
 // W = 32: compile-time w (cells split by shift / mask, the ballots' bits 0..4 are the "mod 32");
 // W = 0: runtime w < 32 (lanes >= w idle, explicit mod w, w + 1 bins per scheme).
 template <int W, uint32_t SM>
@@ -1242,7 +1252,8 @@ trace32_kernel(uint32_t w_rt, uint64_t n_warps, const uint32_t *__restrict__ cel
     // RAP_TRACE_SMEM_BANKS: per-trial RAS / RAP evaluations count the lanes of each bank with
     // shared-memory atomics (see RAP_SWEEP_SMEM_BANKS) -- four counter sets per warp, one per
     // trial of the unrolled loop, cleared after use
-    __shared__ uint32_t sh_tcnt[RAP_TRACE_SMEM_BANKS ? kTraceWarps : 1][4][32];
+    __shared__ __align__(128) uint32_t sh_tcnt[RAP_TRACE_SMEM_BANKS ? kTraceWarps : 1][4][32];
+    constexpr bool kTB4 = RAP_TRACE_BANK4 && RAP_TRACE_SMEM_BANKS && W == 32;
     const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
     const LaneSel ls(lane);
     const uint32_t lt_mask = (1u << lane) - 1u;
@@ -1263,8 +1274,8 @@ trace32_kernel(uint32_t w_rt, uint64_t n_warps, const uint32_t *__restrict__ cel
         const uint32_t tcnt = (uint32_t)min((uint64_t)kTraceTB, n_trials - t0);
         __syncthreads();                                    // the previous unit is done with shP / shR
         for (uint32_t t = warp; t < tcnt; t += kTraceWarps) {
-            if (need_p) shP[t][lane] = (uint8_t)warp_perm<W>(seed, first + t0 + t, lane, w);
-            if (need_r) shR[t][lane] = (uint8_t)warp_ras_shift(seed, first + t0 + t, lane, w);
+            if (need_p) shP[t][lane] = (uint8_t)(warp_perm<W>(seed, first + t0 + t, lane, w) << (kTB4 ? 2 : 0));
+            if (need_r) shR[t][lane] = (uint8_t)(warp_ras_shift(seed, first + t0 + t, lane, w) << (kTB4 ? 2 : 0));
         }
         __syncthreads();
         const uint64_t k_end = min(n_warps, (kc + 1) * kTraceTK);
@@ -1291,6 +1302,17 @@ trace32_kernel(uint32_t w_rt, uint64_t n_warps, const uint32_t *__restrict__ cel
                     const uint8_t *sh = s == RAP_SCHEME_RAP ? &shP[0][0] : &shR[0][0];
                     uint32_t *cnt = &sh_tcnt[RAP_TRACE_SMEM_BANKS ? warp : 0][0][0];
                     const bool lead = (leaders >> lane) & 1u;
+                    if constexpr (kTB4) {
+                        const uint32_t cnt_sa = (uint32_t)__cvta_generic_to_shared(cnt), col4 = col << 2;
+#pragma unroll 4
+                        for (uint32_t t = 0; t < tcnt; ++t) {
+                            const uint32_t c = __reduce_max_sync(
+                                kFull, count_in_bank4(cnt_sa, (int)(t & 3u), col4 + sh[t * 32 + row], lead));
+                            __syncwarp();
+                            cnt[(t & 3u) * 32 + lane] = 0u;   // every lane's increment has returned
+                            hc[e] += (c == lane + 1u) ? 1u : 0u;
+                        }
+                    } else {
 #pragma unroll 4
                     for (uint32_t t = 0; t < tcnt; ++t) {
                         uint32_t *ct = cnt + (t & 3u) * 32;
@@ -1298,6 +1320,7 @@ trace32_kernel(uint32_t w_rt, uint64_t n_warps, const uint32_t *__restrict__ cel
                         __syncwarp();
                         ct[lane] = 0u;                     // every lane's increment has returned
                         hc[e] += (c == lane + 1u) ? 1u : 0u;
+                    }
                     }
                     __syncwarp();
                 } else {
