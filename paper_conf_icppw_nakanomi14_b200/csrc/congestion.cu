@@ -446,7 +446,20 @@ __device__ __forceinline__ uint32_t max_load_add_lane(const BankMask &Y, const L
 #ifndef RAP_SWEEP_SMEM_BANKS
 #define RAP_SWEEP_SMEM_BANKS 1
 #endif
-constexpr int kSmemBankEvals = 7;      // RAS stride, RAS diagonal, random under each of the 5 schemes
+// RAP_SWEEP_DEDUP_SMEM (default 1): the merged requests of the random access (equal cells)
+// are found with a 1024-bit shared-memory bitmap of the warp's cells instead of __match_any_sync:
+// each lane sets its cell's bit with one atom.shared.or and leads its cell iff the bit was clear
+// (lanes of one instruction to the same word are serialised, so exactly one lane per distinct cell
+// finds it clear -- any one representative per cell gives the same count per bank).  MATCH.ANY's
+// result latency held 29 % of the sweep's stall samples (profiles/r02_prof_sweep.source.csv.gz),
+// and MATCH.ANY was what loaded the "ADU" pipe (86 % busy with it, 0.6 % without).  The bitmap is
+// slot 7 of the warp's counter block and is cleared with the counters.  3.837 -> 4.571 G trials/s
+// (+19 %), 4.765 with RAP_SWEEP_BATCH_HIST (profiles/r02c_ab_sweep_dedup.txt); bit-identical.
+#ifndef RAP_SWEEP_DEDUP_SMEM
+#define RAP_SWEEP_DEDUP_SMEM 1
+#endif
+constexpr int kSmemBankEvals = RAP_SWEEP_DEDUP_SMEM ? 8 : 7;   // RAS stride, RAS diagonal, random
+                                                                 // under each of the 5 schemes (+ bitmap)
 
 // RAP_SWEEP_HIST_SA (ablation, default 0): histogram increments through a shared-window address
 // kept in a register instead of atomicAdd on a generic pointer (whose conversion re-reads the CTA
@@ -556,6 +569,18 @@ __host__ __device__ constexpr LiveEvals live_evals(uint32_t PM, uint32_t SM) {  
 #ifndef RAP_SWEEP_RES_VEC
 #define RAP_SWEEP_RES_VEC 1
 #endif
+// RAP_SWEEP_BATCH_HIST (default 1): the per-trial congestions of a batch of 32 trials are kept in
+// shared memory (lane 0's STS.128 result slots, one 64-byte row per trial) and counted into the
+// histogram once per batch -- lane e walks the 32 rows of its evaluation -- instead of one LDS +
+// atomic (and the rematerialised shared-window address of the histogram, 19 % of the stall
+// samples in profiles/r02_prof_sweep.source.csv.gz) per trial.  The room comes from the lane-mode
+// transpose buffer, now 16-bit (r << 10 | cell: 15 bits, rows of 34 halves: still conflict-free);
+// the buffer and the 32 result rows fit the 4224 bytes the 32-bit buffer took.  For up to 16
+// evaluations (the cfg2 sweep has 15).  +4.2 % (4.571 -> 4.765 G trials/s with the bitmap dedupe,
+// profiles/r02c_ab_sweep_dedup.txt).
+#ifndef RAP_SWEEP_BATCH_HIST
+#define RAP_SWEEP_BATCH_HIST 1
+#endif
 // RAP_SWEEP_UNROLL_M (tuning): unroll factor of the per-trial warp-mode loop (1: none).  Measured
 // with the default 8 CTAs of 64 registers per SM: unroll 2 3.797 vs 3.839 G trials/s, and 7 / 6
 // CTAs per SM with more registers 3.786 / 3.746 (profiles/r02c_ab_sweep_unroll.txt)
@@ -632,7 +657,7 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
     constexpr bool any_random = (PM >> RAP_PAT_RANDOM) & 1u;
     constexpr bool need_r = (SM >> RAP_SCHEME_RAS) & 1u;
     __shared__ uint32_t sh_hist[nbins];
-    __shared__ uint32_t sh_tr[kSweepWarpsV2][32 * 33];
+    __shared__ __align__(16) uint32_t sh_tr[kSweepWarpsV2][32 * 33];   // 16: batch result rows take STS.128
     __shared__ __align__(16) uint32_t sh_res[kSweepWarpsV2][32];
     __shared__ __align__(128) uint32_t sh_cnt[RAP_SWEEP_SMEM_BANKS ? kSweepWarpsV2 : 1][kSmemBankEvals][32];
     __shared__ __align__(16) uint32_t sh_pl[RAP_SWEEP_PLANES_SMEM ? kSweepWarpsV2 : 1][RAP_SWEEP_PLANES_SMEM ? 32 : 1][8];
@@ -647,6 +672,14 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
     uint32_t *res = sh_res[warp];
     uint32_t *cnt = &sh_cnt[RAP_SWEEP_SMEM_BANKS ? warp : 0][0][0];
     constexpr bool kB4 = RAP_SWEEP_BANK4 && RAP_SWEEP_SMEM_BANKS && !RAP_SWEEP_PACKED_MAX && !RAP_SWEEP_ONEHOT;
+    constexpr bool kDedup = RAP_SWEEP_DEDUP_SMEM && kB4 && RAP_SWEEP_LEAD_LANE && RAP_SWEEP_CLEAR_VEC;
+    // batch histogram: 16-bit transpose buffer (pitch 34 halves = 17 words: row t starts in bank
+    // 17 t mod 32, distinct, so the column read stays conflict-free) + 32 result rows of 16 slots
+    constexpr bool kBatch = RAP_SWEEP_BATCH_HIST && kB4 && RAP_SWEEP_RES_VEC && !RAP_SWEEP_HIST_PRED &&
+                            !RAP_SWEEP_HIST_SA && npat * nsch <= 16;
+    uint16_t *tr16 = reinterpret_cast<uint16_t *>(sh_tr[warp]);
+    uint32_t *res_b = sh_tr[warp] + 544;                 // byte 2176: after 32 x 34 u16, 16-aligned
+    static_assert(!kBatch || 544 + 32 * 16 <= 32 * 33, "batch result rows fit the transpose buffer");
     const uint32_t cnt_sa = (uint32_t)__cvta_generic_to_shared(cnt);   // 128-byte aligned slots
     const uint32_t hist_sa0 = (uint32_t)__cvta_generic_to_shared(sh_hist);
     static_assert(nbins >= 32, "HIST_PRED: idle lanes add 0 to word `lane` of the histogram");
@@ -784,7 +817,8 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
                 for (int i = 0; i < 4; ++i) {
                     const uint32_t r = ur[i] >> 27, cell = uc[i] >> 22;   // floor(u*32/2^32), floor(u*1024/2^32)
                     if (blk == 0 && i == 0) r0_lane = r;
-                    tr[(4 * blk + i) * 33 + lane] = kB4 ? (r << 12) | (cell << 2) : (r << 10) | cell;
+                    if (kBatch) tr16[(4 * blk + i) * 34 + lane] = (uint16_t)((r << 10) | cell);
+                    else tr[(4 * blk + i) * 33 + lane] = kB4 ? (r << 12) | (cell << 2) : (r << 10) | cell;
                 }
             }
         }
@@ -808,7 +842,7 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
             const uint32_t P0 = __shfl_sync(kFull, p0_lane, m);
             const uint32_t r0 = __shfl_sync(kFull, r0_lane, m);
 #endif
-            const uint32_t packed = tr[lane * 33 + m];
+            const uint32_t packed = kBatch ? (uint32_t)tr16[lane * 34 + m] << 2 : tr[lane * 33 + m];
             const uint32_t rt = packed >> 10;                      // kB4: 4 r[t] (+ junk in bits 0..1)
             BankMask Rm;
             if (need_r && !kSB) Rm = masks_ballot(rt);              // bit t = bit b of r[t]
@@ -820,10 +854,18 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
                 rcol = kB4 ? cell & 0x7cu : cell & 31u;            // kB4: 4 col
                 Pr = kB4 ? plane_value4(Pm.b, rrow) : plane_value(Pm.b, rrow);   // (4) P[row_t]
                 rr = __shfl_sync(kFull, rt, rrow);                 // (4) r[row_t]
-                const uint32_t same = __match_any_sync(kFull, cell);   // merged requests
-                if (kSB && RAP_SWEEP_LEAD_LANE) {
+                if constexpr (kDedup) {                            // merged requests: cell bitmap
+                    // kB4: cell = 4 x (32 row + col); the word of the cell is `row`, its bit `col`
+                    const uint32_t bit = 1u << ((cell >> 2) & 31u);
+                    uint32_t old;
+                    asm volatile("atom.shared.or.b32 %0, [%1], %2;"
+                                 : "=r"(old) : "r"(cnt_sa + 7u * 128u + ((cell >> 5) & 0x7cu)), "r"(bit) : "memory");
+                    lead_me = (old & bit) == 0u;                   // the one lane that set the bit
+                } else if (kSB && RAP_SWEEP_LEAD_LANE) {
+                    const uint32_t same = __match_any_sync(kFull, cell);   // merged requests
                     lead_me = (same & lt_mask) == 0u;              // first lane of its cell
                 } else {
+                    const uint32_t same = __match_any_sync(kFull, cell);   // merged requests
                     leaders = ballot_zero(same, lt_mask);          // first lane of its cell
                     lead_me = (leaders >> lane) & 1u;
                 }
@@ -1011,9 +1053,10 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
             }
 #else
             if (lane == 0) {                                   // C4: the result slots, STS.128
+                uint32_t *rr = kBatch ? res_b + m * 16 : res;   // batch: row m of the batch
 #pragma unroll
                 for (uint32_t k = 0; k < ((npat * nsch + 3) & ~3u); k += 4)
-                    *reinterpret_cast<uint4 *>(res + k) = make_uint4(cres[k], cres[k + 1], cres[k + 2], cres[k + 3]);
+                    *reinterpret_cast<uint4 *>(rr + k) = make_uint4(cres[k], cres[k + 1], cres[k + 2], cres[k + 3]);
             }
 #endif
 #endif
@@ -1036,13 +1079,14 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
                 smem_add(hist_sa0 + 4u * bin, on ? 1u : 0u);
             }
 #else
-            if (lane < e && !lane_fixed) atomicAdd(&sh_hist[lane * (w + 1) + res[lane]], 1u);
+            if (!kBatch && lane < e && !lane_fixed) atomicAdd(&sh_hist[lane * (w + 1) + res[lane]], 1u);
 #endif
 #endif
             if (kSB) {                                                  // clear the bank counters
 #if RAP_SWEEP_CLEAR_VEC
                 // every slot up to the highest in use, 16 bytes per lane (unused slots stay 0)
-                constexpr uint32_t n4 = kSlots ? 8u * (32u - __builtin_clz(kSlots)) : 0u;
+                constexpr uint32_t kClr = (kDedup ? (kSlots | 0x80u) : kSlots);
+                constexpr uint32_t n4 = kClr ? 8u * (32u - __builtin_clz(kClr)) : 0u;
 #pragma unroll
                 for (uint32_t i = 0; i < n4; i += 32)
                     if (i + 32 <= n4 || i + lane < n4)
@@ -1056,6 +1100,11 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
             __syncwarp();
         }
         if (lane_fixed) atomicAdd(&sh_hist[lane * (w + 1) + fix_lane], nvalid);   // trial-invariant slots
+        if (kBatch && lane < npat * nsch && !lane_fixed) {        // C4 of the batch: lane e, row m
+            uint32_t *hrow = &sh_hist[lane * (w + 1)];
+#pragma unroll 4
+            for (uint32_t m = 0; m < nvalid; ++m) atomicAdd(hrow + res_b[m * 16 + lane], 1u);
+        }
         __syncwarp();
     }
     __syncthreads();
