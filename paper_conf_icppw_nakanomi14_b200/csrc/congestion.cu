@@ -131,6 +131,14 @@ __device__ __forceinline__ void flush_hist(uint32_t (*sh)[kMaxBins], int nwarps,
 #endif
 constexpr int kSweepWarpsV2 = RAP_SWEEP_WARPS;
 
+// RAP_SWEEP_SWAP_MULHI (ablation, default 0): in the plane swap, pl >> d on the FMA pipe as
+// umulhi(pl, 2^(32-d)) (IMAD.HI): 3.9 ALU instructions fewer per trial for the ALU-bound sweep,
+// yet 2 % slower (4.689 vs 4.768 G trials/s, profiles/r02c_ab_sweep_mulhi.txt).  d = 0 (j = k, no
+// swap) makes the multiplier 2^32 -> 0 in PTX's shl, so y = pl & mj, and pl ^= y ^ (y * 1)
+// leaves pl unchanged as it must.  Bit-identical.
+#ifndef RAP_SWEEP_SWAP_MULHI
+#define RAP_SWEEP_SWAP_MULHI 0
+#endif
 template <int W>
 __device__ __forceinline__ void swap_planes(uint32_t (&pl)[5], uint32_t k, uint32_t j) {
     // j <= k: y holds bit_j ^ bit_k at position j; flipping bits j and k by y swaps them.
@@ -139,11 +147,23 @@ __device__ __forceinline__ void swap_planes(uint32_t (&pl)[5], uint32_t k, uint3
     const uint32_t d = k - j, mj = 1u << j;
     uint32_t sd;
     asm("shl.b32 %0, %1, %2;" : "=r"(sd) : "r"(1u), "r"(d));
+#if RAP_SWEEP_SWAP_MULHI
+    uint32_t sr;                                          // 2^(32-d); 0 for d = 0 (shl clamps)
+    asm("shl.b32 %0, %1, %2;" : "=r"(sr) : "r"(1u), "r"(32u - d));
+#pragma unroll
+    for (int b = 0; b < 5; ++b) {
+        uint32_t hi;
+        asm("mul.hi.u32 %0, %1, %2;" : "=r"(hi) : "r"(pl[b]), "r"(sr));
+        const uint32_t y = (pl[b] ^ hi) & mj;
+        pl[b] ^= y ^ (y * sd);
+    }
+#else
 #pragma unroll
     for (int b = 0; b < 5; ++b) {
         const uint32_t y = (pl[b] ^ (pl[b] >> d)) & mj;
         pl[b] ^= y ^ (y * sd);
     }
+#endif
 }
 
 // C1+C2 in lane mode: P_n = perm(seed, n, w) as bit planes.
@@ -526,6 +546,16 @@ __host__ __device__ constexpr LiveEvals live_evals(uint32_t PM, uint32_t SM) {  
                 L.idx[L.n++] = eval_index(PM, SM, p, s);
     return L;
 }
+// position of each evaluation among the live evaluations (-1: trial-invariant or a duplicate),
+// as a table built at compile time (indexed with the unrolled evaluation index)
+struct LivePos { int pos[25]; };
+__host__ __device__ constexpr LivePos live_pos_table(uint32_t PM, uint32_t SM) {
+    LivePos T{};
+    for (int e = 0; e < 25; ++e) T.pos[e] = -1;
+    const LiveEvals L = live_evals(PM, SM);
+    for (int i = 0; i < L.n; ++i) T.pos[L.idx[i]] = i;
+    return T;
+}
 
 // RAP_SWEEP_ONEHOT (ablation, default 0): the per-trial warp maxima of all live evaluations in
 // two reductions instead of one CREDUX.MAX each (9 for the cfg2 sweep), to unload the ADU pipe
@@ -580,6 +610,15 @@ __host__ __device__ constexpr LiveEvals live_evals(uint32_t PM, uint32_t SM) {  
 // profiles/r02c_ab_sweep_dedup.txt).
 #ifndef RAP_SWEEP_BATCH_HIST
 #define RAP_SWEEP_BATCH_HIST 1
+#endif
+// RAP_SWEEP_PACK_SLOTS (ablation, default 0; with the batch histogram): a trial's row holds only
+// its live evaluations (9 for the cfg2 sweep: no slot for the trial-invariant RAW / PAD / XOR
+// accesses nor for the malicious accesses that repeat the stride / diagonal ones) -- two STS.128
+// and one STS instead of four STS.128 with zeros to fill; the lane of a duplicate reads its
+// source's slot.  7 zero moves fewer, but ptxas spent 5 more LOP3 on the ALU pipe elsewhere in
+// the loop: 4.672 vs 4.768 G trials/s (profiles/r02c_ab_sweep_mulhi.txt).  Bit-identical.
+#ifndef RAP_SWEEP_PACK_SLOTS
+#define RAP_SWEEP_PACK_SLOTS 0
 #endif
 // RAP_SWEEP_UNROLL_M (tuning): unroll factor of the per-trial warp-mode loop (1: none).  Measured
 // with the default 8 CTAs of 64 registers per SM: unroll 2 3.797 vs 3.839 G trials/s, and 7 / 6
@@ -680,6 +719,22 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
     uint16_t *tr16 = reinterpret_cast<uint16_t *>(sh_tr[warp]);
     uint32_t *res_b = sh_tr[warp] + 544;                 // byte 2176: after 32 x 34 u16, 16-aligned
     static_assert(!kBatch || 544 + 32 * 16 <= 32 * 33, "batch result rows fit the transpose buffer");
+    constexpr bool kPack = kBatch && RAP_SWEEP_PACK_SLOTS;
+    constexpr int kNLive = live_evals(PM, SM).n;
+    constexpr LivePos kPos = live_pos_table(PM, SM);
+    uint32_t my_slot = lane;                             // the row slot lane e reads in the batch flush
+    if (kPack) {
+#pragma unroll
+        for (int p = 0; p < 5; ++p) {
+#pragma unroll
+            for (int s = 0; s < 5; ++s) {
+                if (!((PM >> p) & 1u) || !((SM >> s) & 1u)) continue;
+                const int e = eval_index(PM, SM, p, s), d = eval_dup_src(PM, SM, p, s);
+                const int pos = kPos.pos[d >= 0 ? d : e];
+                if (lane == (uint32_t)e && pos >= 0) my_slot = (uint32_t)pos;
+            }
+        }
+    }
     const uint32_t cnt_sa = (uint32_t)__cvta_generic_to_shared(cnt);   // 128-byte aligned slots
     const uint32_t hist_sa0 = (uint32_t)__cvta_generic_to_shared(sh_hist);
     static_assert(nbins >= 32, "HIST_PRED: idle lanes add 0 to word `lane` of the histogram");
@@ -954,7 +1009,7 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
 #if RAP_SWEEP_RES_VEC
             uint32_t cres[(npat * nsch + 3) & ~3u];        // result slots, stored 4 at a time
 #pragma unroll
-            for (uint32_t k = 0; k < ((npat * nsch + 3) & ~3u); ++k) cres[k] = 0u;
+            for (uint32_t k = (kPack ? kNLive : 0u); k < ((npat * nsch + 3) & ~3u); ++k) cres[k] = 0u;
 #endif
 #pragma unroll
             for (int p = 0; p < 5; ++p) {
@@ -1036,7 +1091,12 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
                     if (p == RAP_PAT_STRIDE) c_stride[s] = c;
                     if (p == RAP_PAT_DIAGONAL) c_diag[s] = c;
 #if RAP_SWEEP_RES_VEC
-                    if (!((fixed_slots >> e) & 1u)) cres[e] = c;
+                    if (kPack) {
+                        const int pos = kPos.pos[eval_index(PM, SM, p, s)];
+                        if (pos >= 0) cres[pos] = c;
+                    } else if (!((fixed_slots >> e) & 1u)) {
+                        cres[e] = c;
+                    }
 #else
                     if (lane == 0 && !((fixed_slots >> e) & 1u)) res[e] = c;   // C4: result slot e
 #endif
@@ -1054,9 +1114,12 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
 #else
             if (lane == 0) {                                   // C4: the result slots, STS.128
                 uint32_t *rr = kBatch ? res_b + m * 16 : res;   // batch: row m of the batch
+                constexpr uint32_t nst = kPack ? (uint32_t)kNLive : (npat * nsch + 3) & ~3u;
 #pragma unroll
-                for (uint32_t k = 0; k < ((npat * nsch + 3) & ~3u); k += 4)
+                for (uint32_t k = 0; k + 4 <= nst; k += 4)
                     *reinterpret_cast<uint4 *>(rr + k) = make_uint4(cres[k], cres[k + 1], cres[k + 2], cres[k + 3]);
+#pragma unroll
+                for (uint32_t k = nst & ~3u; k < nst; ++k) rr[k] = cres[k];   // the packed tail
             }
 #endif
 #endif
@@ -1103,7 +1166,7 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
         if (kBatch && lane < npat * nsch && !lane_fixed) {        // C4 of the batch: lane e, row m
             uint32_t *hrow = &sh_hist[lane * (w + 1)];
 #pragma unroll 4
-            for (uint32_t m = 0; m < nvalid; ++m) atomicAdd(hrow + res_b[m * 16 + lane], 1u);
+            for (uint32_t m = 0; m < nvalid; ++m) atomicAdd(hrow + res_b[m * 16 + my_slot], 1u);
         }
         __syncwarp();
     }
