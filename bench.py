@@ -61,7 +61,8 @@ CFG4_LAYOUTS = ["raw", "pad", "xor", "ras", "rap", "rap64", "rap16"]
 # (DESIGN reading xv; 2.00 wavefronts per 256-byte request, the minimum) -- the two-plane and
 # RAP-16 encodings are timed beside it in `cfg4_layouts`
 HEADLINE64 = "rap64"
-ORACLE_BAND_BYTES = 32 << 20   # the oracle's transpose sample: one row band of this many bytes
+ORACLE_BAND_BYTES = 256 << 20  # the oracle's transpose sample: one row band of this many bytes (32 MiB
+#   bands -- ~2 ms steps -- left the two arms 20-25 % apart on the same box: thread start-up noise)
 E2E_WS = 64 << 20              # device workspace of the cfg4 host-to-host transpose: 4 band buffers of
                                # 128 rows (profiles/r02_e2e_bands.txt: the fastest band plan for cfg4)
 
