@@ -61,8 +61,10 @@ CFG4_LAYOUTS = ["raw", "pad", "xor", "ras", "rap", "rap64", "rap16"]
 # (DESIGN reading xv; 2.00 wavefronts per 256-byte request, the minimum) -- the two-plane and
 # RAP-16 encodings are timed beside it in `cfg4_layouts`
 HEADLINE64 = "rap64"
-ORACLE_BAND_BYTES = 256 << 20  # the oracle's transpose sample: one row band of this many bytes (32 MiB
-#   bands -- ~2 ms steps -- left the two arms 20-25 % apart on the same box: thread start-up noise)
+ORACLE_BAND_BYTES = 32 << 20   # the oracle's transpose sample: one row band of this many bytes,
+ORACLE_PASSES = 8              # transposed this many times per step: one ~2 ms pass per step left the
+#   two arms 20-25 % apart on the same box (thread start-up noise); one 256 MiB band per step measured
+#   the oracle 5x slower (6 vs 32-40 GB/s: its naive column writes then thrash the caches)
 E2E_WS = 64 << 20              # device workspace of the cfg4 host-to-host transpose: 4 band buffers of
                                # 128 rows (profiles/r02_e2e_bands.txt: the fastest band plan for cfg4)
 
@@ -383,16 +385,18 @@ def oracle_arm(args, world: int, threads: int | None = None, workload: str | Non
         x, band = oracle_transpose_sample(rows_rank, cols, dt)
         out = np.empty((x.shape[1], x.shape[0]), dtype=x.dtype)
         unit = "GB/s"
-        what = (f"{band} x {cols} row band ({x.nbytes >> 20} MiB) of the {rows_rank}x{cols} {str(dt)[6:]} matrix "
-                f"per step, naive oracle transpose on {threads} threads into a reused output array")
+        what = (f"{ORACLE_PASSES} passes over a {band} x {cols} row band ({x.nbytes >> 20} MiB) of the "
+                f"{rows_rank}x{cols} {str(dt)[6:]} matrix per step, naive oracle transpose on {threads} threads "
+                f"into a reused output array")
         if wl in ("default", "cfg3"):
             what += f"; plus {n_sw} oracle sweep trials per step, timed apart (`sweep`)"
-        work = 2 * x.nbytes / 1e9
+        work = 2 * x.nbytes * ORACLE_PASSES / 1e9
 
         def fn(k):
             nonlocal sweep_s
             t = time.perf_counter()
-            oracle.transpose(x, threads=threads, out=out)
+            for _ in range(ORACLE_PASSES):
+                oracle.transpose(x, threads=threads, out=out)
             t_steps.append(time.perf_counter() - t)
             if wl in ("default", "cfg3"):        # the step's second half, timed apart like our arm's
                 t = time.perf_counter()

@@ -220,6 +220,12 @@ __device__ __forceinline__ uint32_t mod_w(uint32_t x, uint32_t w) {
     return x >= w ? x - w : x;
 }
 
+// RAP_SWEEP_GENERIC_DEDUP (default 1): the w < 32 kernel finds the merged requests of the random
+// access with a per-warp cell bitmap and one atom.shared.or (as sweep32_kernel's
+// RAP_SWEEP_DEDUP_SMEM) instead of __match_any_sync
+#ifndef RAP_SWEEP_GENERIC_DEDUP
+#define RAP_SWEEP_GENERIC_DEDUP 1
+#endif
 // PM / SM: pattern / scheme masks fixed at compile time (0 = take the runtime masks), so the
 // common configurations evaluate with no mask tests and constant evaluation slots.
 template <int W, uint32_t PM, uint32_t SM>
@@ -230,10 +236,12 @@ sweep_kernel(uint32_t w_rt, uint32_t pmask_rt, uint32_t smask_rt, uint64_t seed,
     const uint32_t pmask = PM ? PM : pmask_rt, smask = SM ? SM : smask_rt;
     __shared__ uint32_t sh_hist[kMaxBins];
     __shared__ uint32_t sh_tr[kSweepWarpsV2][32 * 33];
+    __shared__ uint32_t sh_bm[RAP_SWEEP_GENERIC_DEDUP ? kSweepWarpsV2 : 1][32];   // cell bitmap, row words
     const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
     const uint32_t npat = __popc(pmask), nsch = __popc(smask);
     const uint32_t nbins = npat * nsch * (w + 1);
     for (uint32_t b = threadIdx.x; b < nbins; b += blockDim.x) sh_hist[b] = 0;
+    if (RAP_SWEEP_GENERIC_DEDUP) sh_bm[RAP_SWEEP_GENERIC_DEDUP ? warp : 0][lane] = 0u;
     __syncthreads();
 
     const LaneSel ls(lane);
@@ -284,7 +292,20 @@ sweep_kernel(uint32_t w_rt, uint32_t pmask_rt, uint32_t smask_rt, uint64_t seed,
                 else { rrow = cell / w; rcol = cell - rrow * w; }
                 Pr = plane_value(q, rrow);                     // P[row_t]
                 rr = __shfl_sync(kFull, rt, rrow);             // r[row_t]
+#if RAP_SWEEP_GENERIC_DEDUP
+                {   // merged requests: the lane whose atom.shared.or sets its cell's bit leads
+                    uint32_t *bm = sh_bm[RAP_SWEEP_GENERIC_DEDUP ? warp : 0];
+                    const bool act = W || lane < w;
+                    const uint32_t bit = 1u << rcol;
+                    const bool lead = act && !(atomicOr(&bm[rrow], bit) & bit);
+                    leaders = __ballot_sync(kFull, lead);
+                    __syncwarp();
+                    if (act) bm[rrow] = 0u;                    // cleared for the next trial
+                    __syncwarp();
+                }
+#else
                 leaders = first_occurrences(rrow * 32u + rcol, active, lane);
+#endif
             }
             uint32_t mine = 0, e = 0;
             uint32_t c_stride[5] = {0, 0, 0, 0, 0}, c_diag[5] = {0, 0, 0, 0, 0};

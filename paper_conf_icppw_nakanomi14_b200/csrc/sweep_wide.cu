@@ -147,13 +147,21 @@ sweep_wide_kernel(uint32_t w, uint32_t pmask, uint32_t smask, uint64_t seed, uin
 //     become j_t = floor(u_t (w - t) / 2^32) in jv[], the RAS shifts r[], the random cells stay in
 //     registers;
 //   * Durstenfeld on a[] is one sequential chain (lane 0; k = w-1 .. 1: swap a[k], a[jv[w-1-k]]);
-//   * merged requests: slice by slice, a request leads if it is the lowest lane of
-//     its cell in the slice (__match_any_sync) and the cell's bit in a w*w-bit bitmap is not yet
-//     set by an earlier slice; the bits are cleared again afterwards (O(w) per trial);
+//   * merged requests: slice by slice, a request leads iff its atom.shared.or is the
+//     one that sets its cell's bit in a w*w-bit bitmap (RAP_WIDE_DEDUP_ATOM; formerly the lowest
+//     lane of its cell in the slice by __match_any_sync, bit not yet set by an earlier slice);
+//     the bits are cleared again afterwards (O(w) per trial);
 //   * each (pattern, scheme): every lane adds its requests to the per-bank counters cnt[] with
 //     shared atomics -- congestion = max over requests of the returned count + 1 (= max over
 //     banks), reduce-max over the warp -- then zeroes the counters it touched.
 constexpr int kWideWarps = 8;
+// RAP_WIDE_DEDUP_ATOM (default 1): a request leads iff its atom.shared.or sets the cell's bit in
+// the w*w-bit bitmap (lanes of one instruction to one word are serialised: one leader per distinct
+// cell, across and within slices) -- no __match_any_sync, whose latency dominated the w = 32
+// sweep (DESIGN §6 C, step 4)
+#ifndef RAP_WIDE_DEDUP_ATOM
+#define RAP_WIDE_DEDUP_ATOM 1
+#endif
 #ifndef RAP_WIDE_LANE_FY
 #define RAP_WIDE_LANE_FY 1
 #endif
@@ -250,6 +258,13 @@ sweep_wide_warp_kernel(uint32_t w, uint32_t pmask_rt, uint32_t smask_rt, uint64_
                 const uint32_t t = lane + 32u * q;
                 const bool valid = t < w;
                 const uint32_t c = cellv[q];
+#if RAP_WIDE_DEDUP_ATOM
+                if (valid) {                                  // the one lane that sets the bit leads
+                    const uint32_t bit = 1u << (c & 31u);
+                    if (!(atomicOr(&S.bm[c >> 5], bit) & bit)) lead |= 1u << q;
+                }
+                __syncwarp();
+#else
                 const uint32_t same = __match_any_sync(kFull, valid ? c : (0x80000000u | lane));
                 const bool first_in_slice = (__ffs(same) - 1) == (int)lane;
                 const bool seen = valid && ((S.bm[c >> 5] >> (c & 31u)) & 1u);
@@ -257,6 +272,7 @@ sweep_wide_warp_kernel(uint32_t w, uint32_t pmask_rt, uint32_t smask_rt, uint64_
                 __syncwarp();
                 if (valid) atomicOr(&S.bm[c >> 5], 1u << (c & 31u));
                 __syncwarp();
+#endif
             }
 #pragma unroll
             for (int q = 0; q < NI; ++q)
@@ -411,6 +427,13 @@ sweep_wide_lane_kernel(uint32_t w, uint32_t pmask_rt, uint32_t smask_rt, uint64_
                     const uint32_t t = lane + 32u * q;
                     const bool valid = t < w;
                     const uint32_t c = cellv[q];
+#if RAP_WIDE_DEDUP_ATOM
+                    if (valid) {                              // the one lane that sets the bit leads
+                        const uint32_t bit = 1u << (c & 31u);
+                        if (!(atomicOr(&bm[c >> 5], bit) & bit)) lead |= 1u << q;
+                    }
+                    __syncwarp();
+#else
                     const uint32_t same = __match_any_sync(kFull, valid ? c : (0x80000000u | lane));
                     const bool first_in_slice = (__ffs(same) - 1) == (int)lane;
                     const bool seen = valid && ((bm[c >> 5] >> (c & 31u)) & 1u);
@@ -418,6 +441,7 @@ sweep_wide_lane_kernel(uint32_t w, uint32_t pmask_rt, uint32_t smask_rt, uint64_
                     __syncwarp();
                     if (valid) atomicOr(&bm[c >> 5], 1u << (c & 31u));
                     __syncwarp();
+#endif
                 }
 #pragma unroll
                 for (int q = 0; q < NI; ++q)

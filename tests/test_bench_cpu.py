@@ -70,7 +70,7 @@ def test_default_sweeps_1e9_trials():
 
 def test_oracle_band_is_one_definition():
     # both arms time the oracle on the same row band of the matrix
-    assert bench.oracle_band(16384, 16384, 8) == 2048 and bench.oracle_band(8192, 8192, 4) == 8192
+    assert bench.oracle_band(16384, 16384, 8) == 256 and bench.oracle_band(8192, 8192, 4) == 1024
     assert bench.oracle_band(32, 32, 4) == 32
 
 
