@@ -641,6 +641,18 @@ __host__ __device__ constexpr LivePos live_pos_table(uint32_t PM, uint32_t SM) {
 #ifndef RAP_SWEEP_PACK_SLOTS
 #define RAP_SWEEP_PACK_SLOTS 0
 #endif
+// RAP_SWEEP_PBYTES (default 1, with the bitmap dedupe and the batch histogram, RAW / RAS / RAP
+// schemes): the lane-mode phase turns its trial's permutation planes into a 32-byte table 4 P[t]
+// (t = 0..31; nibble k of plane b spread over 4 bytes by one multiply, (nib * 0x00204081) &
+// 0x01010101) in the 32-byte shared row that held the planes, so that the warp-mode phase reads
+// P[t] and P[row_t] with one LDS.U8 each instead of the 14-instruction bit gather, and counts the
+// RAP stride (bank P[t]) and diagonal (bank t + P[t]) accesses with the shared-memory bank
+// counters (slots 5 and 6) instead of the bit-sliced mask algebra; r[0] comes from the 16-bit
+// transpose buffer.  Warp-mode loop 124 -> 97 instructions, 190 -> 166 per trial in all: 4.763 ->
+// 5.305 G trials/s (+11 %, profiles/r02c_ab_sweep_pbytes.txt); bit-identical.
+#ifndef RAP_SWEEP_PBYTES
+#define RAP_SWEEP_PBYTES 1
+#endif
 // RAP_SWEEP_UNROLL_M (tuning): unroll factor of the per-trial warp-mode loop (1: none).  Measured
 // with the default 8 CTAs of 64 registers per SM: unroll 2 3.797 vs 3.839 G trials/s, and 7 / 6
 // CTAs per SM with more registers 3.786 / 3.746 (profiles/r02c_ab_sweep_unroll.txt)
@@ -740,6 +752,8 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
     uint16_t *tr16 = reinterpret_cast<uint16_t *>(sh_tr[warp]);
     uint32_t *res_b = sh_tr[warp] + 544;                 // byte 2176: after 32 x 34 u16, 16-aligned
     static_assert(!kBatch || 544 + 32 * 16 <= 32 * 33, "batch result rows fit the transpose buffer");
+    constexpr bool kPB = RAP_SWEEP_PBYTES && kDedup && kBatch && RAP_SWEEP_PLANES_SMEM &&
+                         !((SM >> RAP_SCHEME_PAD) & 1u) && !((SM >> RAP_SCHEME_XOR) & 1u);
     constexpr bool kPack = kBatch && RAP_SWEEP_PACK_SLOTS;
     constexpr int kNLive = live_evals(PM, SM).n;
     constexpr LivePos kPos = live_pos_table(PM, SM);
@@ -768,7 +782,10 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
     // the random access under scheme s
     constexpr uint32_t kSlots = (((SM >> RAP_SCHEME_RAS) & 1u) && ((PM >> RAP_PAT_STRIDE) & 1u) ? 1u : 0u) |
                                 (((SM >> RAP_SCHEME_RAS) & 1u) && ((PM >> RAP_PAT_DIAGONAL) & 1u) ? 2u : 0u) |
-                                (((PM >> RAP_PAT_RANDOM) & 1u) ? (SM << 2) : 0u);
+                                (((PM >> RAP_PAT_RANDOM) & 1u) ? (SM << 2) : 0u) |
+                                (RAP_SWEEP_PBYTES && RAP_SWEEP_DEDUP_SMEM && RAP_SWEEP_BATCH_HIST &&
+                                 !((SM >> RAP_SCHEME_PAD) & 1u) && !((SM >> RAP_SCHEME_XOR) & 1u) &&
+                                 ((SM >> RAP_SCHEME_RAP) & 1u) ? 0x60u : 0u);   // PBYTES: RAP stride 5, diagonal 6
     if (kSB) {
 #pragma unroll
         for (int e = 0; e < kSmemBankEvals; ++e) cnt[e * 32 + lane] = 0u;
@@ -899,8 +916,22 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
             }
         }
 #if RAP_SWEEP_PLANES_SMEM
-        *reinterpret_cast<uint4 *>(&sh_pl[warp][lane][0]) = make_uint4(pl[0], pl[1], pl[2], pl[3]);
-        *reinterpret_cast<uint4 *>(&sh_pl[warp][lane][4]) = make_uint4(pl[4], p0_lane, r0_lane, 0u);
+        if constexpr (kPB) {                 // 4 P[t] as bytes: word k holds t = 4k .. 4k+3
+            uint32_t pw[8];
+#pragma unroll
+            for (int k = 0; k < 8; ++k) {
+                uint32_t x = 0;
+#pragma unroll
+                for (int b = 0; b < 5; ++b)
+                    x |= ((((pl[b] >> (4 * k)) & 15u) * 0x00204081u) & 0x01010101u) << (b + 2);
+                pw[k] = x;
+            }
+            *reinterpret_cast<uint4 *>(&sh_pl[warp][lane][0]) = make_uint4(pw[0], pw[1], pw[2], pw[3]);
+            *reinterpret_cast<uint4 *>(&sh_pl[warp][lane][4]) = make_uint4(pw[4], pw[5], pw[6], pw[7]);
+        } else {
+            *reinterpret_cast<uint4 *>(&sh_pl[warp][lane][0]) = make_uint4(pl[0], pl[1], pl[2], pl[3]);
+            *reinterpret_cast<uint4 *>(&sh_pl[warp][lane][4]) = make_uint4(pl[4], p0_lane, r0_lane, 0u);
+        }
 #endif
         __syncwarp();
         // ---- warp mode: lane t is DMM thread t of trial n0 + m
@@ -908,10 +939,20 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
         for (uint32_t m = 0; m < nvalid; ++m) {
             BankMask Pm;                                           // bit t = bit b of P[t]
 #if RAP_SWEEP_PLANES_SMEM
-            const uint4 qa = *reinterpret_cast<const uint4 *>(&sh_pl[warp][m][0]);   // broadcast reads
-            const uint4 qb = *reinterpret_cast<const uint4 *>(&sh_pl[warp][m][4]);
-            Pm.b[0] = qa.x; Pm.b[1] = qa.y; Pm.b[2] = qa.z; Pm.b[3] = qa.w; Pm.b[4] = qb.x;
-            const uint32_t P0 = qb.y, r0 = qb.z;
+            uint32_t P0, r0, Pt4 = 0;                              // Pt4 (kPB): 4 P[t]
+            const uint8_t *pbytes = reinterpret_cast<const uint8_t *>(&sh_pl[warp][m][0]);
+            if constexpr (kPB) {
+                Pt4 = pbytes[lane];
+                P0 = (uint32_t)pbytes[0] >> 2;                     // broadcast
+                r0 = (uint32_t)tr16[m] >> 10;                      // r[0] of trial m (row 0)
+#pragma unroll
+                for (int b = 0; b < 5; ++b) Pm.b[b] = 0u;          // (unused)
+            } else {
+                const uint4 qa = *reinterpret_cast<const uint4 *>(&sh_pl[warp][m][0]);   // broadcast reads
+                const uint4 qb = *reinterpret_cast<const uint4 *>(&sh_pl[warp][m][4]);
+                Pm.b[0] = qa.x; Pm.b[1] = qa.y; Pm.b[2] = qa.z; Pm.b[3] = qa.w; Pm.b[4] = qb.x;
+                P0 = qb.y; r0 = qb.z;
+            }
 #else
 #pragma unroll
             for (int b = 0; b < 5; ++b) Pm.b[b] = __shfl_sync(kFull, pl[b], m);
@@ -928,6 +969,10 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
                 const uint32_t cell = kB4 ? packed & 0xffcu : packed & 1023u;
                 rrow = kB4 ? cell >> 7 : cell >> 5;
                 rcol = kB4 ? cell & 0x7cu : cell & 31u;            // kB4: 4 col
+#if RAP_SWEEP_PLANES_SMEM
+                if constexpr (kPB) Pr = pbytes[rrow];               // 4 P[row_t]
+                else
+#endif
                 Pr = kB4 ? plane_value4(Pm.b, rrow) : plane_value(Pm.b, rrow);   // (4) P[row_t]
                 rr = __shfl_sync(kFull, rt, rrow);                 // (4) r[row_t]
                 if constexpr (kDedup) {                            // merged requests: cell bitmap
@@ -1054,16 +1099,20 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
                                : (s == RAP_SCHEME_PAD) ? -1 : RAP_PAT_DIAGONAL) : p;
                         BankMask B;
                         const bool isp = (s == RAP_SCHEME_RAP);
+                        const bool pb_rap = kPB && isp && (pp == RAP_PAT_STRIDE || pp == RAP_PAT_DIAGONAL);
                         if (kSB && ((s == RAP_SCHEME_RAS && (pp == RAP_PAT_STRIDE || pp == RAP_PAT_DIAGONAL)) ||
-                                    pp == RAP_PAT_RANDOM)) {
+                                    pp == RAP_PAT_RANDOM || pb_rap)) {
                             // shared-memory bank counters (slot: RAS stride 0, RAS diagonal 1,
-                            // random under scheme s 2 + s); packed carries rcol in bits 0..4, and
-                            // count_in_bank reduces the bank mod 32
-                            const int slot = pp == RAP_PAT_STRIDE ? 0 : pp == RAP_PAT_DIAGONAL ? 1 : 2 + s;
+                            // random under scheme s 2 + s, PBYTES: RAP stride 5, RAP diagonal 6);
+                            // packed carries rcol in bits 0..4, and count_in_bank reduces the bank
+                            // mod 32
+                            const int slot = pb_rap ? (pp == RAP_PAT_STRIDE ? 5 : 6)
+                                           : pp == RAP_PAT_STRIDE ? 0 : pp == RAP_PAT_DIAGONAL ? 1 : 2 + s;
                             const bool counted = pp != RAP_PAT_RANDOM || lead_me;
                             if (kB4) {                             // banks as 4 x bank (counter byte offsets)
-                                const uint32_t bank4 = pp == RAP_PAT_STRIDE ? rt
-                                                     : pp == RAP_PAT_DIAGONAL ? (lane << 2) + rt
+                                const uint32_t sh4 = pb_rap ? Pt4 : rt;    // 4 P[t] / 4 r[t]
+                                const uint32_t bank4 = pp == RAP_PAT_STRIDE ? sh4
+                                                     : pp == RAP_PAT_DIAGONAL ? (lane << 2) + sh4
                                                      : s == RAP_SCHEME_RAW ? packed
                                                      : s == RAP_SCHEME_PAD ? packed + (packed >> 5)
                                                      : s == RAP_SCHEME_XOR ? packed ^ (packed >> 5)
