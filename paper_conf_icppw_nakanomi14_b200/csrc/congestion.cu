@@ -632,14 +632,15 @@ __host__ __device__ constexpr LivePos live_pos_table(uint32_t PM, uint32_t SM) {
 #ifndef RAP_SWEEP_BATCH_HIST
 #define RAP_SWEEP_BATCH_HIST 1
 #endif
-// RAP_SWEEP_PACK_SLOTS (ablation, default 0; with the batch histogram): a trial's row holds only
-// its live evaluations (9 for the cfg2 sweep: no slot for the trial-invariant RAW / PAD / XOR
-// accesses nor for the malicious accesses that repeat the stride / diagonal ones) -- two STS.128
-// and one STS instead of four STS.128 with zeros to fill; the lane of a duplicate reads its
-// source's slot.  7 zero moves fewer, but ptxas spent 5 more LOP3 on the ALU pipe elsewhere in
-// the loop: 4.672 vs 4.768 G trials/s (profiles/r02c_ab_sweep_mulhi.txt).  Bit-identical.
+// RAP_SWEEP_PACK_SLOTS (default 1; with the batch histogram): a trial's row holds only its live
+// evaluations (9 for the cfg2 sweep: no slot for the trial-invariant RAW / PAD / XOR accesses nor
+// for the malicious accesses that repeat the stride / diagonal ones) -- two STS.128 and one STS
+// instead of four STS.128 with zeros to fill; the lane of a duplicate reads its source's slot.
+// Before the P table ptxas spent 5 more LOP3 elsewhere in the loop for it (4.672 vs 4.768 G
+// trials/s, profiles/r02c_ab_sweep_mulhi.txt); with the P table the loop is 97 -> 92 instructions
+// and 5.307 -> 5.452 G trials/s (profiles/r02c_ab_sweep_pack2.txt; unroll 2 5.04 / 5.45).
 #ifndef RAP_SWEEP_PACK_SLOTS
-#define RAP_SWEEP_PACK_SLOTS 0
+#define RAP_SWEEP_PACK_SLOTS 1
 #endif
 // RAP_SWEEP_PBYTES (default 1, with the bitmap dedupe and the batch histogram, RAW / RAS / RAP
 // schemes): the lane-mode phase turns its trial's permutation planes into a 32-byte table 4 P[t]
