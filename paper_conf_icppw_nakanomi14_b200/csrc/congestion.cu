@@ -654,6 +654,22 @@ __host__ __device__ constexpr LivePos live_pos_table(uint32_t PM, uint32_t SM) {
 #ifndef RAP_SWEEP_PBYTES
 #define RAP_SWEEP_PBYTES 1
 #endif
+// RAP_SWEEP_FY_BYTES (ablation, default 0; with RAP_SWEEP_PBYTES): the lane-mode Durstenfeld
+// shuffle runs directly on the lane's 32-byte P table in shared memory (a[i] = 4 i; swap a[k],
+// a[j] = two LDS.U8 and two STS.U8) instead of on 5 bit planes that are converted afterwards: ~6
+// instead of ~19 instructions per swap, no conversion.  The table's words are XOR-swizzled by
+// (row >> 2) & 7 so that the step's common index k (the same in every lane) hits 32 distinct
+// banks; the random j costs ~2-3 wavefronts.  161 -> 147 instructions per trial, but issue fell
+// from 77 to 67 % (short scoreboard, MIO throttle: the swap chain's shared-memory round trips):
+// 5.31 vs 5.45 G trials/s, also with the other domains' Philox interleaved into the FY loop
+// (RAP_SWEEP_FY_INTERLEAVE) -- profiles/r02c_ab_sweep_fyb*.txt, r02c_prof_sweep_fyb.raw.csv.
+// Bit-identical.
+#ifndef RAP_SWEEP_FY_BYTES
+#define RAP_SWEEP_FY_BYTES 0
+#endif
+#ifndef RAP_SWEEP_FY_INTERLEAVE
+#define RAP_SWEEP_FY_INTERLEAVE 1
+#endif
 // RAP_SWEEP_UNROLL_M (tuning): unroll factor of the per-trial warp-mode loop (1: none).  Measured
 // with the default 8 CTAs of 64 registers per SM: unroll 2 3.797 vs 3.839 G trials/s, and 7 / 6
 // CTAs per SM with more registers 3.786 / 3.746 (profiles/r02c_ab_sweep_unroll.txt)
@@ -755,6 +771,7 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
     static_assert(!kBatch || 544 + 32 * 16 <= 32 * 33, "batch result rows fit the transpose buffer");
     constexpr bool kPB = RAP_SWEEP_PBYTES && kDedup && kBatch && RAP_SWEEP_PLANES_SMEM &&
                          !((SM >> RAP_SCHEME_PAD) & 1u) && !((SM >> RAP_SCHEME_XOR) & 1u);
+    constexpr bool kFYB = kPB && RAP_SWEEP_FY_BYTES;
     constexpr bool kPack = kBatch && RAP_SWEEP_PACK_SLOTS;
     constexpr int kNLive = live_evals(PM, SM).n;
     constexpr LivePos kPos = live_pos_table(PM, SM);
@@ -896,11 +913,48 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
         const uint64_t n0 = first + bt * 32;
         const uint32_t nvalid = (uint32_t)min((uint64_t)32, n_trials - bt * 32);
         // ---- lane mode: trial n0 + lane
-        uint32_t pl[5];
-        lane_perm_planes<32>(seed, n0 + lane, w, pl);
-        const uint32_t p0_lane = plane_value(pl, 0);              // P[0] of this lane's trial
+        uint32_t pl[5] = {0u, 0u, 0u, 0u, 0u};
+        uint32_t p0_lane = 0;
+        if constexpr (kFYB) {
+            // C2 on the lane's byte table (row `lane` of this warp's P rows, words swizzled)
+            uint8_t *rowb = reinterpret_cast<uint8_t *>(&sh_pl[warp][lane][0]);
+            const uint32_t swz = ((lane >> 2) & 7u) << 2;             // byte-index XOR
+#pragma unroll
+            for (uint32_t q = 0; q < 8; ++q)                            // a[i] = 4 i
+                reinterpret_cast<uint32_t *>(rowb)[q ^ (swz >> 2)] = 0x0C080400u + 0x10101010u * q;
+#pragma unroll
+            for (int blk = 0; blk < 8; ++blk) {
+                const uint4 c = philox_block(seed, n0 + lane, kDomainFY, blk);
+                const uint32_t u[4] = {c.x, c.y, c.z, c.w};
+#if RAP_SWEEP_FY_INTERLEAVE
+                // C1 of the RAS / random domains for the same block here, so that their Philox
+                // arithmetic fills the latency of the swap chain's shared-memory round trips
+                if (need_r || any_random) {
+                    const uint4 cr = need_r ? philox_block(seed, n0 + lane, kDomainRAS, blk) : make_uint4(0, 0, 0, 0);
+                    const uint4 cc = any_random ? philox_block(seed, n0 + lane, kDomainRandom, blk) : make_uint4(0, 0, 0, 0);
+                    const uint32_t ur[4] = {cr.x, cr.y, cr.z, cr.w};
+                    const uint32_t uc[4] = {cc.x, cc.y, cc.z, cc.w};
+#pragma unroll
+                    for (int i = 0; i < 4; ++i)
+                        tr16[(4 * blk + i) * 34 + lane] = (uint16_t)(((ur[i] >> 27) << 10) | (uc[i] >> 22));
+                }
+#endif
+#pragma unroll
+                for (int i = 0; i < 4; ++i) {
+                    const int t = 4 * blk + i;
+                    if (t >= 31) break;
+                    const uint32_t k = 31u - (uint32_t)t, j = mulshift(u[i], k + 1);
+                    const uint8_t ak = rowb[k ^ swz], aj = rowb[j ^ swz];
+                    rowb[k ^ swz] = aj;
+                    rowb[j ^ swz] = ak;
+                }
+            }
+        } else {
+            lane_perm_planes<32>(seed, n0 + lane, w, pl);
+            p0_lane = plane_value(pl, 0);                              // P[0] of this lane's trial
+        }
         uint32_t r0_lane = 0;
-        if (need_r || any_random) {
+        if ((need_r || any_random) && !(kFYB && RAP_SWEEP_FY_INTERLEAVE)) {
 #pragma unroll
             for (int blk = 0; blk < 8; ++blk) {
                 const uint4 cr = need_r ? philox_block(seed, n0 + lane, kDomainRAS, blk) : make_uint4(0, 0, 0, 0);
@@ -917,7 +971,9 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
             }
         }
 #if RAP_SWEEP_PLANES_SMEM
-        if constexpr (kPB) {                 // 4 P[t] as bytes: word k holds t = 4k .. 4k+3
+        if constexpr (kFYB) {
+            // (the table is already in place)
+        } else if constexpr (kPB) {          // 4 P[t] as bytes: word k holds t = 4k .. 4k+3
             uint32_t pw[8];
 #pragma unroll
             for (int k = 0; k < 8; ++k) {
@@ -942,9 +998,10 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
 #if RAP_SWEEP_PLANES_SMEM
             uint32_t P0, r0, Pt4 = 0;                              // Pt4 (kPB): 4 P[t]
             const uint8_t *pbytes = reinterpret_cast<const uint8_t *>(&sh_pl[warp][m][0]);
+            const uint32_t mswz = kFYB ? ((m >> 2) & 7u) << 2 : 0u;  // row m's byte-index XOR
             if constexpr (kPB) {
-                Pt4 = pbytes[lane];
-                P0 = (uint32_t)pbytes[0] >> 2;                     // broadcast
+                Pt4 = pbytes[lane ^ mswz];
+                P0 = (uint32_t)pbytes[mswz] >> 2;                  // broadcast
                 r0 = (uint32_t)tr16[m] >> 10;                      // r[0] of trial m (row 0)
 #pragma unroll
                 for (int b = 0; b < 5; ++b) Pm.b[b] = 0u;          // (unused)
@@ -971,7 +1028,7 @@ sweep32_kernel(uint32_t, uint32_t, uint32_t, uint64_t seed, uint64_t first, uint
                 rrow = kB4 ? cell >> 7 : cell >> 5;
                 rcol = kB4 ? cell & 0x7cu : cell & 31u;            // kB4: 4 col
 #if RAP_SWEEP_PLANES_SMEM
-                if constexpr (kPB) Pr = pbytes[rrow];               // 4 P[row_t]
+                if constexpr (kPB) Pr = pbytes[rrow ^ mswz];        // 4 P[row_t]
                 else
 #endif
                 Pr = kB4 ? plane_value4(Pm.b, rrow) : plane_value(Pm.b, rrow);   // (4) P[row_t]
