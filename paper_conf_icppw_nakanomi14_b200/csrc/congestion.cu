@@ -1477,6 +1477,14 @@ __device__ __forceinline__ uint32_t wrap_w(uint32_t x, uint32_t w) { return W ==
 #ifndef RAP_TRACE_BANK4
 #define RAP_TRACE_BANK4 1
 #endif
+// RAP_TRACE_HIST_SMEM (ablation, default 0; with RAP_TRACE_BANK4): per trial of the RAS / RAP
+// loop, lane t keeps trial t's congestion (one select) instead of every lane testing c == lane + 1
+// and counting (compare, add, select); after the block's trials each lane adds its value to a
+// per-warp shared-memory histogram with one atomic.  59 -> 56 instructions per 4 unrolled trials,
+// no measurable gain (111.73 vs 111.79 G warp-evaluations/s, profiles/r02c_ab_trace3*.txt).
+#ifndef RAP_TRACE_HIST_SMEM
+#define RAP_TRACE_HIST_SMEM 0
+#endif
 // W = 32: compile-time w (cells split by shift / mask, the ballots' bits 0..4 are the "mod 32");
 // W = 0: runtime w < 32 (lanes >= w idle, explicit mod w, w + 1 bins per scheme).
 template <int W, uint32_t SM>
@@ -1494,6 +1502,8 @@ trace32_kernel(uint32_t w_rt, uint64_t n_warps, const uint32_t *__restrict__ cel
     // trial of the unrolled loop, cleared after use
     __shared__ __align__(128) uint32_t sh_tcnt[RAP_TRACE_SMEM_BANKS ? kTraceWarps : 1][4][32];
     constexpr bool kTB4 = RAP_TRACE_BANK4 && RAP_TRACE_SMEM_BANKS && W == 32;
+    constexpr bool kTHS = kTB4 && RAP_TRACE_HIST_SMEM;
+    __shared__ uint32_t sh_th[kTHS ? kTraceWarps : 1][kTHS ? nsch : 1][33];   // RAS / RAP bins per warp
     const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
     const LaneSel ls(lane);
     const uint32_t lt_mask = (1u << lane) - 1u;
@@ -1504,6 +1514,10 @@ trace32_kernel(uint32_t w_rt, uint64_t n_warps, const uint32_t *__restrict__ cel
     if (RAP_TRACE_SMEM_BANKS && W == 32) {
 #pragma unroll
         for (int k = 0; k < 4; ++k) sh_tcnt[RAP_TRACE_SMEM_BANKS ? warp : 0][k][lane] = 0u;
+        __syncwarp();
+    }
+    if constexpr (kTHS) {
+        for (uint32_t i = lane; i < nsch * 33; i += 32) (&sh_th[warp][0][0])[i] = 0u;
         __syncwarp();
     }
     const uint64_t nkc = (n_warps + kTraceTK - 1) / kTraceTK;
@@ -1544,14 +1558,17 @@ trace32_kernel(uint32_t w_rt, uint64_t n_warps, const uint32_t *__restrict__ cel
                     const bool lead = (leaders >> lane) & 1u;
                     if constexpr (kTB4) {
                         const uint32_t cnt_sa = (uint32_t)__cvta_generic_to_shared(cnt), col4 = col << 2;
+                        uint32_t mine = 0;                     // kTHS: trial `lane`'s congestion
 #pragma unroll 4
                         for (uint32_t t = 0; t < tcnt; ++t) {
                             const uint32_t c = __reduce_max_sync(
                                 kFull, count_in_bank4(cnt_sa, (int)(t & 3u), col4 + sh[t * 32 + row], lead));
                             __syncwarp();
                             cnt[(t & 3u) * 32 + lane] = 0u;   // every lane's increment has returned
-                            hc[e] += (c == lane + 1u) ? 1u : 0u;
+                            if (kTHS) mine = (lane == t) ? c : mine;
+                            else hc[e] += (c == lane + 1u) ? 1u : 0u;
                         }
+                        if (kTHS && lane < tcnt) atomicAdd(&sh_th[kTHS ? warp : 0][kTHS ? e : 0][mine], 1u);
                     } else {
 #pragma unroll 4
                     for (uint32_t t = 0; t < tcnt; ++t) {
@@ -1575,9 +1592,11 @@ trace32_kernel(uint32_t w_rt, uint64_t n_warps, const uint32_t *__restrict__ cel
             }
         }
     }
+    if (kTHS) __syncwarp();
 #pragma unroll
     for (uint32_t e = 0; e < nsch; ++e) {
-        if (hc[e]) atomicAdd((unsigned long long *)(hist + e * (w + 1) + lane + 1), (unsigned long long)hc[e]);
+        const uint32_t v = hc[e] + (kTHS ? sh_th[kTHS ? warp : 0][kTHS ? e : 0][lane + 1] : 0u);
+        if (v) atomicAdd((unsigned long long *)(hist + e * (w + 1) + lane + 1), (unsigned long long)v);
         if (lane == 0 && hbad) atomicAdd((unsigned long long *)(hist + e * (w + 1)), (unsigned long long)hbad);
     }
 }
