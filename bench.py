@@ -590,6 +590,26 @@ def all_reduce_hist(h, world: int):
         h.copy_(hc)
 
 
+def soak_for(seconds: float, body, world: int, dev):
+    """Runs body(k) (k = 0, 1, ...) for about `seconds` of wall time with the device synchronised
+    after each call.  At N > 1 every rank runs the SAME number of calls -- the count comes from the
+    first call's duration, max over ranks -- because a body may hold collectives (the sweep's
+    all-reduce, the sharded transpose's all-to-all): a loop on each rank's own clock could leave
+    the ranks a collective apart (a gloo size mismatch, an NCCL hang)."""
+    import math
+    import torch
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    body(0)
+    torch.cuda.synchronize()
+    dt = max(time.perf_counter() - t0, 1e-6)
+    n = max(1, int(math.ceil(seconds / dt)))
+    n = int(reduce_over_ranks(float(n), world, dev, "max"))
+    for k in range(1, n):
+        body(k)
+        torch.cuda.synchronize()
+
+
 def timed_back_to_back(fn, warmup: int, steps: int, stream, world: int, dev, barrier):
     """Mean device time of one fn() over `steps` back-to-back launches between one event pair
     (max over ranks), with the clocks sampled over them."""
@@ -599,10 +619,7 @@ def timed_back_to_back(fn, warmup: int, steps: int, stream, world: int, dev, bar
     torch.cuda.synchronize()
     barrier()
     with Clocks(dev.index) as clk:
-        t0 = time.perf_counter()
-        while time.perf_counter() - t0 < 0.2:     # soak, so every clock sample is under load
-            fn()
-            torch.cuda.synchronize()
+        soak_for(0.2, lambda k: fn(), world, dev)  # soak, so every clock sample is under load
         st, en = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         st.record(stream)
         for _ in range(steps):
@@ -659,12 +676,10 @@ def run_default(args):
         return 1
 
     def soak(seconds, k0):
-        t0, k = time.perf_counter(), 0
-        while time.perf_counter() - t0 < seconds:
+        def body(k):
             rap.transpose(x, layout=HEADLINE64, seed=0, out=y)
             sweep_slice((1 << 40) + (k0 + k) * S, S, scratch)    # far trial range, scratch histogram
-            k += 1
-            torch.cuda.synchronize()
+        soak_for(seconds, body, world, dev)                       # (the same count on every rank)
 
     for k in range(W):
         rap.transpose(x, layout=HEADLINE64, seed=0, out=y)
@@ -987,19 +1002,20 @@ def run_workload(args):
     soak_hist = torch.zeros_like(hist)
 
     def soak(lay, seconds):
-        """Identical untimed steps (scratch histogram, far trial range) for `seconds`."""
-        t0, k = time.perf_counter(), 0
-        while time.perf_counter() - t0 < seconds:
-            if do_t:
-                step_transpose(lay)
-            if do_s and wl == "trace":
-                rap.congestion_trace(trace_cells, TT, seed=1, first_trial=(1 << 40) + k * TT,
-                                     schemes=("raw", "ras", "rap", "pad", "xor"), out=torch.zeros_like(trace_hist))
-            elif do_s:
-                rap.congestion_sweep(S, seed=1, first_trial=(1 << 40) + k * S, out=soak_hist, algo=args.sweep_algo)
-            k += 1
-            if k % 16 == 0:
-                torch.cuda.synchronize()
+        """Identical untimed steps (scratch histogram, far trial range) for `seconds`, in groups of
+        16 between synchronisations; the same number of groups on every rank (soak_for: a step
+        may hold the sharded transpose's all-to-all)."""
+        def group(j):
+            for i in range(16):
+                k = 16 * j + i
+                if do_t:
+                    step_transpose(lay)
+                if do_s and wl == "trace":
+                    rap.congestion_trace(trace_cells, TT, seed=1, first_trial=(1 << 40) + k * TT,
+                                         schemes=("raw", "ras", "rap", "pad", "xor"), out=torch.zeros_like(trace_hist))
+                elif do_s:
+                    rap.congestion_sweep(S, seed=1, first_trial=(1 << 40) + k * S, out=soak_hist, algo=args.sweep_algo)
+        soak_for(seconds, group, world, dev)
 
     results = {}
     for lay in layouts:
